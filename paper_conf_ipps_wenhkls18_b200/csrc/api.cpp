@@ -1,0 +1,348 @@
+// api.cpp -- the C ABI of libgbdt.so (include/gbdt.h): validation, handles, error reporting.
+#include <cmath>
+#include <cstring>
+#include <exception>
+#include <limits>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+
+namespace gbdt {
+
+namespace {
+thread_local std::string g_err;
+}
+
+void fail(gbdt_status st, const std::string& msg) { throw Error{st, msg}; }
+
+void DBuf::alloc(size_t b, cudaStream_t s) {
+  release();
+  st = s;
+  bytes = b ? b : 16;
+  GBDT_CUDA(cudaMallocAsync(&p, bytes, st));
+}
+
+void DBuf::release() {
+  if (p) {
+    cudaFreeAsync(p, st);
+    p = nullptr;
+    bytes = 0;
+  }
+}
+
+int64_t launches_get();
+void comm_unique_id(uint8_t id[128]);
+Comm* comm_init(int rank, int world, const uint8_t id[128], int device);
+void comm_free(Comm* c);
+
+template <class F>
+static gbdt_status guarded(F&& f) {
+  try {
+    g_err.clear();
+    f();
+    return GBDT_OK;
+  } catch (const Error& e) {
+    g_err = e.msg;
+    return e.st;
+  } catch (const std::bad_alloc&) {
+    g_err = "host allocation failed";
+    return GBDT_E_NOMEM;
+  } catch (const std::exception& e) {
+    g_err = e.what();
+    return GBDT_E_CUDA;
+  }
+}
+
+// CSR structure checks shared by load and predict (P:32 sparse rows; indices strictly increasing).
+static void validate_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr, const int32_t* indices,
+                         const float* values, bool require_cols_in_range) {
+  const int64_t kMax = (int64_t(1) << 31) - 1;
+  if (n_rows < 1 || n_rows >= kMax) fail(GBDT_E_INVAL, "n_rows must be in [1, 2^31-1)");
+  if (n_cols < 1 || n_cols >= kMax) fail(GBDT_E_INVAL, "n_cols must be in [1, 2^31-1)");
+  if (!indptr) fail(GBDT_E_INVAL, "indptr is NULL");
+  if (indptr[0] != 0) fail(GBDT_E_INVAL, "indptr[0] must be 0");
+  for (int64_t i = 0; i < n_rows; ++i)
+    if (indptr[i + 1] < indptr[i]) fail(GBDT_E_INVAL, "indptr must be non-decreasing (row " + std::to_string(i) + ")");
+  const int64_t nnz = indptr[n_rows];
+  if (nnz >= kMax) fail(GBDT_E_INVAL, "nnz must be < 2^31-1");
+  if (nnz > 0 && (!indices || !values)) fail(GBDT_E_INVAL, "indices/values NULL with nnz > 0");
+  for (int64_t i = 0; i < n_rows; ++i) {
+    int32_t prev = -1;
+    for (int64_t p = indptr[i]; p < indptr[i + 1]; ++p) {
+      const int32_t a = indices[p];
+      if (a < 0 || (require_cols_in_range && a >= n_cols))
+        fail(GBDT_E_INVAL, "column index out of range in row " + std::to_string(i));
+      if (a <= prev) fail(GBDT_E_INVAL, "column indices must be strictly increasing in row " + std::to_string(i));
+      prev = a;
+    }
+  }
+}
+
+}  // namespace gbdt
+
+using namespace gbdt;
+
+struct gbdt_dataset {
+  Dataset ds;
+};
+struct gbdt_model {
+  Model m;
+};
+struct gbdt_comm {
+  Comm* c = nullptr;
+};
+
+extern "C" {
+
+const char* gbdt_last_error(void) { return g_err.c_str(); }
+
+int64_t gbdt_last_launch_count(void) { return launches_get(); }
+
+gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr, const int32_t* indices,
+                          const float* values, const float* labels, const gbdt_load_opts* opts,
+                          gbdt_dataset** out) {
+  if (out) *out = nullptr;
+  return guarded([&] {
+    if (!out) fail(GBDT_E_INVAL, "out is NULL");
+    validate_csr(n_rows, n_cols, indptr, indices, values, true);
+    if (!labels) fail(GBDT_E_INVAL, "labels is NULL");
+    float lmin = std::numeric_limits<float>::infinity(), lmax = -lmin;
+    for (int64_t i = 0; i < n_rows; ++i) {
+      if (!std::isfinite(labels[i])) fail(GBDT_E_INVAL, "labels must be finite (row " + std::to_string(i) + ")");
+      lmin = std::min(lmin, labels[i]);
+      lmax = std::max(lmax, labels[i]);
+    }
+    gbdt_load_opts o;
+    std::memset(&o, 0, sizeof o);
+    if (opts) o = *opts;
+    if (o.rle < 0 || o.rle > 2) fail(GBDT_E_INVAL, "rle must be OFF, ON or AUTO");
+    int nsh = o.n_shards <= 0 ? 1 : o.n_shards;
+    if (nsh != 1 && nsh != 2 && nsh != 4 && nsh != 8) fail(GBDT_E_RANGE, "n_shards must be 1, 2, 4 or 8");
+    Comm* comm = o.comm ? o.comm->c : nullptr;
+    if (comm && nsh != 1) fail(GBDT_E_RANGE, "n_shards must be 1 with a communicator");
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < 1) fail(GBDT_E_CUDA, "no CUDA device visible");
+    int dev = o.device;
+    if (dev < 0) GBDT_CUDA(cudaGetDevice(&dev));
+    if (dev >= ndev) fail(GBDT_E_RANGE, "device ordinal out of range");
+    if (comm) dev = comm->device;
+    GBDT_CUDA(cudaSetDevice(dev));
+
+    const int64_t nnz = indptr[n_rows];
+    std::vector<int64_t> col_counts(n_cols, 0);
+    for (int64_t p = 0; p < nnz; ++p)
+      if (!std::isnan(values[p])) col_counts[indices[p]]++;
+    bool missing = false;
+    for (int64_t a = 0; a < n_cols; ++a) missing |= col_counts[a] != n_rows;
+
+    auto* h = new gbdt_dataset();
+    Dataset& ds = h->ds;
+    try {
+      ds.n = n_rows;
+      ds.m = n_cols;
+      ds.nnz = nnz;
+      ds.device = dev;
+      ds.stream = (cudaStream_t)o.stream;
+      ds.has_missing = missing;
+      ds.comm = comm;
+      ds.rle = o.rle;
+      ds.h_labels_minmax = {lmin, lmax};
+      const int world = comm ? comm->world : 1;
+      const int P = comm ? world : nsh;
+      ds.n_total_shards = P;
+      // contiguous attribute ranges balanced by stored entries
+      std::vector<int64_t> pre(n_cols + 1, 0);
+      for (int64_t a = 0; a < n_cols; ++a) pre[a + 1] = pre[a] + col_counts[a];
+      std::vector<int32_t> bnd(P + 1, 0);
+      bnd[P] = (int32_t)n_cols;
+      int64_t a = 0;
+      for (int i = 1; i < P; ++i) {
+        const double target = (double)pre[n_cols] * i / P;
+        while (a < n_cols && (double)pre[a] < target) ++a;
+        bnd[i] = (int32_t)std::max<int64_t>(a, bnd[i - 1]);
+      }
+      for (int i = 0; i < P; ++i) {
+        if (comm && i != comm->rank) continue;
+        auto sh = std::make_unique<Shard>();
+        sh->index = i;
+        sh->a_begin = bnd[i];
+        sh->a_end = bnd[i + 1];
+        sh->m = sh->a_end - sh->a_begin;
+        ds.shards.push_back(std::move(sh));
+      }
+      cudaStream_t st = ds.stream;
+      DBuf dptr((size_t)(n_rows + 1) * 8, st), didx((size_t)std::max<int64_t>(nnz, 1) * 4, st),
+          dval((size_t)std::max<int64_t>(nnz, 1) * 4, st);
+      GBDT_CUDA(cudaMemcpyAsync(dptr.p, indptr, (size_t)(n_rows + 1) * 8, cudaMemcpyHostToDevice, st));
+      if (nnz) {
+        GBDT_CUDA(cudaMemcpyAsync(didx.p, indices, (size_t)nnz * 4, cudaMemcpyHostToDevice, st));
+        GBDT_CUDA(cudaMemcpyAsync(dval.p, values, (size_t)nnz * 4, cudaMemcpyHostToDevice, st));
+      }
+      ds.y.alloc((size_t)n_rows * 4, st);
+      GBDT_CUDA(cudaMemcpyAsync(ds.y.p, labels, (size_t)n_rows * 4, cudaMemcpyHostToDevice, st));
+      build_layout(ds, dptr.as<int64_t>(), didx.as<int32_t>(), dval.as<float>(), col_counts, o.rle_min_ratio);
+      dptr.release();
+      didx.release();
+      dval.release();
+      GBDT_CUDA(cudaStreamSynchronize(st));
+    } catch (...) {
+      delete h;
+      throw;
+    }
+    *out = h;
+  });
+}
+
+gbdt_status gbdt_train(gbdt_dataset* dsh, const gbdt_params* p, gbdt_model** out, double* train_margin) {
+  if (out) *out = nullptr;
+  return guarded([&] {
+    if (!dsh || !p || !out) fail(GBDT_E_INVAL, "NULL argument");
+    Dataset& ds = dsh->ds;
+    if (p->max_depth < 1 || p->max_depth > 16) fail(GBDT_E_INVAL, "max_depth must be in [1, 16]");
+    if (p->n_trees < 1) fail(GBDT_E_INVAL, "n_trees must be >= 1");
+    if (!(p->lambda >= 0) || !std::isfinite(p->lambda)) fail(GBDT_E_INVAL, "lambda must be finite and >= 0");
+    if (!(p->gamma >= 0) || !std::isfinite(p->gamma)) fail(GBDT_E_INVAL, "gamma must be finite and >= 0");
+    if (!(p->eta > 0 && p->eta <= 1)) fail(GBDT_E_INVAL, "eta must be in (0, 1]");
+    if (!std::isfinite(p->base_margin)) fail(GBDT_E_INVAL, "base_margin must be finite");
+    if (p->loss != GBDT_LOSS_SQUARED && p->loss != GBDT_LOSS_LOGISTIC) fail(GBDT_E_INVAL, "unknown loss");
+    if (p->loss == GBDT_LOSS_LOGISTIC && (ds.h_labels_minmax[0] < 0 || ds.h_labels_minmax[1] > 1))
+      fail(GBDT_E_INVAL, "logistic loss needs labels in [0, 1]");
+    if (p->lambda == 0 && p->loss == GBDT_LOSS_LOGISTIC) {
+      // H >= 1e-16 * count > 0, so every denominator of Eq. 2 stays positive: allowed
+    }
+    auto* m = new gbdt_model();
+    try {
+      train(ds, *p, m->m, train_margin);
+    } catch (...) {
+      delete m;
+      throw;
+    }
+    *out = m;
+  });
+}
+
+gbdt_status gbdt_predict(const gbdt_model* mh, int64_t n_rows, int64_t n_cols, const int64_t* indptr,
+                         const int32_t* indices, const float* values, int32_t output_margin, double* out) {
+  return guarded([&] {
+    if (!mh || !out) fail(GBDT_E_INVAL, "NULL argument");
+    if (mh->m.n_trees < 1) fail(GBDT_E_STATE, "model has no trees");
+    validate_csr(n_rows, n_cols, indptr, indices, values, false);
+    predict(mh->m, n_rows, n_cols, indptr, indices, values, output_margin, out);
+  });
+}
+
+gbdt_status gbdt_model_num_trees(const gbdt_model* m, int32_t* out) {
+  return guarded([&] {
+    if (!m || !out) fail(GBDT_E_INVAL, "NULL argument");
+    *out = m->m.n_trees;
+  });
+}
+
+gbdt_status gbdt_model_num_nodes(const gbdt_model* m, int32_t tree, int32_t* out) {
+  return guarded([&] {
+    if (!m || !out) fail(GBDT_E_INVAL, "NULL argument");
+    if (tree < 0 || tree >= m->m.n_trees) fail(GBDT_E_RANGE, "tree index out of range");
+    *out = (int32_t)m->m.nh();
+  });
+}
+
+gbdt_status gbdt_model_export(const gbdt_model* m, int32_t tree, gbdt_node* nodes) {
+  return guarded([&] {
+    if (!m || !nodes) fail(GBDT_E_INVAL, "NULL argument");
+    if (tree < 0 || tree >= m->m.n_trees) fail(GBDT_E_RANGE, "tree index out of range");
+    const int64_t NH = m->m.nh();
+    std::memcpy(nodes, m->m.nodes.data() + (size_t)tree * NH, sizeof(gbdt_node) * (size_t)NH);
+  });
+}
+
+gbdt_status gbdt_get_timings(const gbdt_model* m, double* ms, int32_t n) {
+  return guarded([&] {
+    if (!m || !ms) fail(GBDT_E_INVAL, "NULL argument");
+    for (int i = 0; i < n && i < GBDT_N_PHASES; ++i) ms[i] = m->m.timings[i];
+  });
+}
+
+gbdt_status gbdt_dataset_info(const gbdt_dataset* d, int32_t shard, int64_t info[7]) {
+  return guarded([&] {
+    if (!d || !info) fail(GBDT_E_INVAL, "NULL argument");
+    const Dataset& ds = d->ds;
+    if (shard < 0 || shard >= (int)ds.shards.size()) fail(GBDT_E_RANGE, "shard out of range");
+    const Shard& s = *ds.shards[shard];
+    info[0] = ds.n; info[1] = ds.m; info[2] = s.nnz; info[3] = (int64_t)ds.shards.size();
+    info[4] = s.a_begin; info[5] = s.a_end; info[6] = s.rle ? s.runs : -1;
+  });
+}
+
+gbdt_status gbdt_dataset_export_layout(const gbdt_dataset* d, int32_t shard, int64_t* col_ptr, float* val,
+                                       int32_t* ins) {
+  return guarded([&] {
+    if (!d) fail(GBDT_E_INVAL, "NULL argument");
+    const Dataset& ds = d->ds;
+    if (shard < 0 || shard >= (int)ds.shards.size()) fail(GBDT_E_RANGE, "shard out of range");
+    const Shard& s = *ds.shards[shard];
+    GBDT_CUDA(cudaSetDevice(ds.device));
+    int64_t off = 0;
+    if (col_ptr) col_ptr[0] = 0;
+    for (int a = 0; a < s.m; ++a) {
+      const int64_t L = s.h_col_len[a];
+      if (val && L) GBDT_CUDA(cudaMemcpy(val + off, s.val0.as<float>() + s.h_col_start[a], L * 4, cudaMemcpyDeviceToHost));
+      if (ins && L) GBDT_CUDA(cudaMemcpy(ins + off, s.ins0.as<int32_t>() + s.h_col_start[a], L * 4, cudaMemcpyDeviceToHost));
+      off += L;
+      if (col_ptr) col_ptr[a + 1] = off;
+    }
+  });
+}
+
+gbdt_status gbdt_dataset_export_rle(const gbdt_dataset* d, int32_t shard, int64_t* run_ptr, float* run_val,
+                                    int32_t* run_len) {
+  return guarded([&] {
+    if (!d) fail(GBDT_E_INVAL, "NULL argument");
+    const Dataset& ds = d->ds;
+    if (shard < 0 || shard >= (int)ds.shards.size()) fail(GBDT_E_RANGE, "shard out of range");
+    const Shard& s = *ds.shards[shard];
+    if (!s.rle) fail(GBDT_E_STATE, "shard is not RLE-compressed");
+    GBDT_CUDA(cudaSetDevice(ds.device));
+    if (run_ptr) GBDT_CUDA(cudaMemcpy(run_ptr, s.run_ptr.p, (size_t)(s.m + 1) * 8, cudaMemcpyDeviceToHost));
+    if (run_val && s.runs) GBDT_CUDA(cudaMemcpy(run_val, s.run_val.p, (size_t)s.runs * 4, cudaMemcpyDeviceToHost));
+    if (run_len && s.runs) GBDT_CUDA(cudaMemcpy(run_len, s.run_len.p, (size_t)s.runs * 4, cudaMemcpyDeviceToHost));
+  });
+}
+
+gbdt_status gbdt_comm_unique_id(uint8_t id[128]) {
+  return guarded([&] {
+    if (!id) fail(GBDT_E_INVAL, "NULL argument");
+    comm_unique_id(id);
+  });
+}
+
+gbdt_status gbdt_comm_init(int32_t rank, int32_t world, const uint8_t id[128], int32_t device, gbdt_comm** out) {
+  if (out) *out = nullptr;
+  return guarded([&] {
+    if (!id || !out) fail(GBDT_E_INVAL, "NULL argument");
+    if (world < 1 || world > 8 || (world & (world - 1))) fail(GBDT_E_RANGE, "world must be 1, 2, 4 or 8");
+    if (rank < 0 || rank >= world) fail(GBDT_E_RANGE, "rank out of range");
+    auto* c = new gbdt_comm();
+    c->c = comm_init(rank, world, id, device);
+    *out = c;
+  });
+}
+
+void gbdt_comm_free(gbdt_comm* c) {
+  if (!c) return;
+  comm_free(c->c);
+  delete c;
+}
+
+void gbdt_dataset_free(gbdt_dataset* d) {
+  if (!d) return;
+  cudaSetDevice(d->ds.device);
+  cudaStream_t st = d->ds.stream;
+  delete d;
+  cudaStreamSynchronize(st);
+}
+
+void gbdt_model_free(gbdt_model* m) { delete m; }
+
+}  // extern "C"

@@ -1,0 +1,148 @@
+// internal.h -- host-side structures of libgbdt.so (not part of the C ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "../../include/gbdt.h"
+
+namespace gbdt {
+
+struct Error {
+  gbdt_status st;
+  std::string msg;
+};
+
+[[noreturn]] void fail(gbdt_status st, const std::string& msg);
+
+#define GBDT_CUDA(x)                                                                        \
+  do {                                                                                      \
+    cudaError_t e_ = (x);                                                                   \
+    if (e_ != cudaSuccess)                                                                  \
+      ::gbdt::fail(e_ == cudaErrorMemoryAllocation ? GBDT_E_NOMEM : GBDT_E_CUDA,            \
+                   std::string(#x) + ": " + cudaGetErrorString(e_) + " (" __FILE__ ":" +    \
+                       std::to_string(__LINE__) + ")");                                     \
+  } while (0)
+
+#define GBDT_LAUNCH_CHECK() GBDT_CUDA(cudaGetLastError())
+
+// Counts kernel launches of the current gbdt_train (bench "gpu_launches" evidence).
+void count_launch(int k = 1);
+
+// Stream-ordered device buffer (cudaMallocAsync / cudaFreeAsync).
+struct DBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+  cudaStream_t st = nullptr;
+  DBuf() = default;
+  DBuf(size_t b, cudaStream_t s) { alloc(b, s); }
+  void alloc(size_t b, cudaStream_t s);
+  void release();
+  ~DBuf() { release(); }
+  DBuf(const DBuf&) = delete;
+  DBuf& operator=(const DBuf&) = delete;
+  DBuf(DBuf&& o) noexcept { *this = std::move(o); }
+  DBuf& operator=(DBuf&& o) noexcept {
+    if (this != &o) {
+      release();
+      p = o.p; bytes = o.bytes; st = o.st;
+      o.p = nullptr; o.bytes = 0;
+    }
+    return *this;
+  }
+  template <class T> T* as() const { return static_cast<T*>(p); }
+};
+
+// Per-level attribute/segment tables of one shard (device pointers).
+// Segment s = a*K + j is node j's part of attribute a's list; it occupies
+// [seg_start[s], seg_start[s] + seg_cnt[s]) of the level buffer.
+struct Tables {
+  int64_t* col_start = nullptr;   // [m+1] padded start of each attribute list
+  int64_t* col_len = nullptr;     // [m]   entries of each attribute list at this level
+  int32_t* tile_start = nullptr;  // [m+1] first tile of each attribute (tiles never straddle)
+  int64_t* seg_start = nullptr;   // [m*Kcap]
+  int64_t* seg_cnt = nullptr;     // [m*Kcap]
+  int32_t* T = nullptr;           // [1] tiles at this level
+};
+
+// Best split of one node found in one shard ("piece" records are reduced to this).
+struct Rec {
+  double gain;
+  double GL, HL;      // high/left child totals (include the missing part when dir == 1)
+  long long cntL;     // high/left child instance count
+  long long pos;      // level-buffer position of the last present high entry (owner shard)
+  float value;        // split value (smallest value on the high side)
+  int attr;           // global attribute id
+  int dir;            // 1: missing -> high/left
+  int node;           // node index at this level
+  int epoch;          // level epoch that produced it
+  int shard;          // owner shard (global index)
+};
+
+struct Comm;  // comm.cpp
+
+struct Shard {
+  int32_t index = 0;             // global shard index
+  int32_t a_begin = 0, a_end = 0, m = 0;
+  int64_t nnz = 0;               // stored entries of this shard
+  int64_t cap = 0;               // padded level-buffer length (+ slack)
+  int32_t T0 = 0;                // tiles at the root
+  DBuf val0, ins0;               // pristine root layout (padded)
+  DBuf valw[2], insw[2];         // ping-pong level buffers
+  DBuf root_tab;                 // root tables storage
+  Tables root;
+  std::vector<int64_t> h_col_len;  // host copy, unpadded lengths
+  std::vector<int64_t> h_col_start;
+  // RLE
+  bool rle = false;
+  int64_t runs = 0;
+  DBuf run_ptr, run_val, run_len;
+};
+
+struct Dataset {
+  int64_t n = 0, m = 0, nnz = 0;
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  bool has_missing = false;      // some instance lacks some attribute
+  DBuf y;                        // labels (device, fp32)
+  std::vector<float> h_labels_minmax;  // [min, max]
+  std::vector<std::unique_ptr<Shard>> shards;  // local shards
+  int32_t n_total_shards = 1;    // across all ranks
+  Comm* comm = nullptr;
+  int rle = 0;
+};
+
+struct Model {
+  int32_t n_trees = 0, max_depth = 0, loss = 0;
+  int64_t n_cols = 0;
+  double eta = 0, base_margin = 0, lambda = 0;
+  std::vector<gbdt_node> nodes;  // n_trees * NH
+  double timings[GBDT_N_PHASES] = {0};
+  int device = 0;
+  int64_t nh() const { return (int64_t(1) << (max_depth + 1)) - 1; }
+};
+
+struct Comm {
+  int rank = 0, world = 1, device = 0;
+  void* nccl = nullptr;  // ncclComm_t
+  void allgather(const void* send, void* recv, size_t bytes, cudaStream_t st);
+  void allreduce_sum_u8(void* buf, size_t n, cudaStream_t st);
+};
+
+// layout.cu
+void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices,
+                  const float* d_values, const std::vector<int64_t>& col_counts,
+                  double rle_min_ratio);
+// train.cu
+void train(Dataset& ds, const gbdt_params& p, Model& model, double* margin_out);
+// predict.cu
+void predict(const Model& m, int64_t n_rows, int64_t n_cols, const int64_t* indptr,
+             const int32_t* indices, const float* values, int output_margin, double* out);
+
+inline int64_t pad4(int64_t x) { return (x + 3) & ~int64_t(3); }
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+}  // namespace gbdt

@@ -1,0 +1,267 @@
+"""Thin ctypes binding of libgbdt.so (include/gbdt.h).  Argument marshalling only: every step of
+training and prediction runs in the library's CUDA kernels.  There is no CPU fallback -- if the
+shared library is missing or no CUDA device is usable, calls raise.
+
+Function names follow the C ABI: load_csr, train, predict, comm_unique_id, comm_init.
+PyTorch is used only to obtain the current CUDA stream and, for multi-process sharding, to
+broadcast the NCCL unique id over torch.distributed.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libgbdt.so")
+
+GBDT_OK = 0
+STATUS = {0: "OK", 1: "E_INVAL", 2: "E_NOMEM", 3: "E_CUDA", 4: "E_NCCL", 5: "E_STATE", 6: "E_RANGE"}
+LOSS = {"squared": 0, "logistic": 1}
+RLE = {"off": 0, "on": 1, "auto": 2, False: 0, True: 1, None: 0}
+PHASES = ["grad", "split_find", "decide", "nodemap", "partition", "comm", "total"]
+
+NODE_DTYPE = np.dtype([
+    ("heap_id", np.int32), ("is_leaf", np.int32), ("attr", np.int32), ("default_left", np.int32),
+    ("split_value", np.float32), ("reserved", np.int32),
+    ("gain", np.float64), ("G", np.float64), ("H", np.float64), ("weight", np.float64),
+    ("count", np.int64),
+])
+assert NODE_DTYPE.itemsize == 64
+
+
+class GbdtError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class _LoadOpts(C.Structure):
+    _fields_ = [("rle", C.c_int32), ("rle_min_ratio", C.c_double), ("n_shards", C.c_int32),
+                ("device", C.c_int32), ("stream", C.c_void_p), ("comm", C.c_void_p)]
+
+
+class _Params(C.Structure):
+    _fields_ = [("max_depth", C.c_int32), ("n_trees", C.c_int32), ("lam", C.c_double),
+                ("gamma", C.c_double), ("eta", C.c_double), ("base_margin", C.c_double),
+                ("loss", C.c_int32), ("profile", C.c_int32)]
+
+
+_lib = None
+
+
+def lib():
+    """Loads the in-tree libgbdt.so; raises if it has not been built."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is not built: run `python -c 'import __graft_entry__ as g; g.build()'`")
+    L = C.CDLL(LIB_PATH)
+    p, i32, i64 = C.c_void_p, C.c_int32, C.c_int64
+    L.gbdt_last_error.restype = C.c_char_p
+    L.gbdt_last_launch_count.restype = C.c_int64
+    L.gbdt_load_csr.argtypes = [i64, i64, p, p, p, p, C.POINTER(_LoadOpts), C.POINTER(p)]
+    L.gbdt_train.argtypes = [p, C.POINTER(_Params), C.POINTER(p), p]
+    L.gbdt_predict.argtypes = [p, i64, i64, p, p, p, i32, p]
+    L.gbdt_model_num_trees.argtypes = [p, C.POINTER(i32)]
+    L.gbdt_model_num_nodes.argtypes = [p, i32, C.POINTER(i32)]
+    L.gbdt_model_export.argtypes = [p, i32, p]
+    L.gbdt_get_timings.argtypes = [p, p, i32]
+    L.gbdt_dataset_info.argtypes = [p, i32, p]
+    L.gbdt_dataset_export_layout.argtypes = [p, i32, p, p, p]
+    L.gbdt_dataset_export_rle.argtypes = [p, i32, p, p, p]
+    L.gbdt_comm_unique_id.argtypes = [p]
+    L.gbdt_comm_init.argtypes = [i32, i32, p, i32, C.POINTER(p)]
+    L.gbdt_comm_free.argtypes = [p]
+    L.gbdt_dataset_free.argtypes = [p]
+    L.gbdt_model_free.argtypes = [p]
+    for f in ("gbdt_load_csr", "gbdt_train", "gbdt_predict", "gbdt_model_num_trees", "gbdt_model_num_nodes",
+              "gbdt_model_export", "gbdt_get_timings", "gbdt_dataset_info", "gbdt_dataset_export_layout",
+              "gbdt_dataset_export_rle", "gbdt_comm_unique_id", "gbdt_comm_init"):
+        getattr(L, f).restype = C.c_int
+    _lib = L
+    return L
+
+
+def _check(st):
+    if st != GBDT_OK:
+        raise GbdtError(st, lib().gbdt_last_error().decode())
+
+
+def _p(a):
+    return None if a is None else a.ctypes.data_as(C.c_void_p)
+
+
+def _current_stream():
+    try:
+        import torch
+        if torch.cuda.is_available():
+            return torch.cuda.current_stream().cuda_stream
+    except Exception:
+        pass
+    return None
+
+
+def last_launch_count() -> int:
+    return int(lib().gbdt_last_launch_count())
+
+
+class Comm:
+    """NCCL communicator (one process per GPU).  Use :func:`comm_from_torch` under torchrun."""
+
+    def __init__(self, handle):
+        self._h = handle
+
+    def __del__(self):
+        if getattr(self, "_h", None) and _lib is not None:
+            _lib.gbdt_comm_free(self._h)
+            self._h = None
+
+
+def comm_unique_id() -> bytes:
+    buf = (C.c_uint8 * 128)()
+    _check(lib().gbdt_comm_unique_id(C.cast(buf, C.c_void_p)))
+    return bytes(buf)
+
+
+def comm_init(rank: int, world: int, uid: bytes, device: int = -1) -> Comm:
+    buf = (C.c_uint8 * 128).from_buffer_copy(uid)
+    h = C.c_void_p()
+    _check(lib().gbdt_comm_init(rank, world, C.cast(buf, C.c_void_p), device, C.byref(h)))
+    return Comm(h)
+
+
+def comm_from_torch(device: int = -1) -> Comm:
+    """Bootstraps the NCCL id through the default torch.distributed process group."""
+    import torch
+    import torch.distributed as dist
+    rank, world = dist.get_rank(), dist.get_world_size()
+    uid = comm_unique_id() if rank == 0 else bytes(128)
+    t = torch.tensor(list(uid), dtype=torch.uint8)
+    if dist.get_backend() == "nccl":
+        t = t.cuda()
+    dist.broadcast(t, 0)
+    return comm_init(rank, world, bytes(t.cpu().tolist()), device)
+
+
+class Dataset:
+    def __init__(self, handle, n, m, keep):
+        self._h = handle
+        self.n, self.m = n, m
+        self._keep = keep
+
+    def __del__(self):
+        if getattr(self, "_h", None) and _lib is not None:
+            _lib.gbdt_dataset_free(self._h)
+            self._h = None
+
+    def info(self, shard=0):
+        a = np.zeros(7, np.int64)
+        _check(lib().gbdt_dataset_info(self._h, shard, _p(a)))
+        return dict(n=int(a[0]), m=int(a[1]), nnz=int(a[2]), n_shards=int(a[3]), attr_begin=int(a[4]),
+                    attr_end=int(a[5]), runs=int(a[6]))
+
+    def export_layout(self, shard=0):
+        inf = self.info(shard)
+        ms = inf["attr_end"] - inf["attr_begin"]
+        col_ptr = np.zeros(ms + 1, np.int64)
+        val = np.zeros(max(inf["nnz"], 1), np.float32)
+        ins = np.zeros(max(inf["nnz"], 1), np.int32)
+        _check(lib().gbdt_dataset_export_layout(self._h, shard, _p(col_ptr), _p(val), _p(ins)))
+        return col_ptr, val[:inf["nnz"]], ins[:inf["nnz"]]
+
+    def export_rle(self, shard=0):
+        inf = self.info(shard)
+        ms = inf["attr_end"] - inf["attr_begin"]
+        run_ptr = np.zeros(ms + 1, np.int64)
+        R = max(inf["runs"], 1)
+        rv = np.zeros(R, np.float32)
+        rl = np.zeros(R, np.int32)
+        _check(lib().gbdt_dataset_export_rle(self._h, shard, _p(run_ptr), _p(rv), _p(rl)))
+        return run_ptr, rv[:inf["runs"]], rl[:inf["runs"]]
+
+
+class Model:
+    def __init__(self, handle):
+        self._h = handle
+
+    def __del__(self):
+        if getattr(self, "_h", None) and _lib is not None:
+            _lib.gbdt_model_free(self._h)
+            self._h = None
+
+    @property
+    def n_trees(self):
+        v = C.c_int32()
+        _check(lib().gbdt_model_num_trees(self._h, C.byref(v)))
+        return v.value
+
+    def nodes(self) -> np.ndarray:
+        """All trees, heap order: array of shape (n_trees, 2^(d+1)-1) with NODE_DTYPE."""
+        T = self.n_trees
+        v = C.c_int32()
+        _check(lib().gbdt_model_num_nodes(self._h, 0, C.byref(v)))
+        out = np.zeros((T, v.value), NODE_DTYPE)
+        for t in range(T):
+            row = np.zeros(v.value, NODE_DTYPE)
+            _check(lib().gbdt_model_export(self._h, t, _p(row)))
+            out[t] = row
+        return out
+
+    def timings(self) -> dict:
+        a = np.zeros(len(PHASES), np.float64)
+        _check(lib().gbdt_get_timings(self._h, _p(a), len(PHASES)))
+        return dict(zip(PHASES, a.tolist()))
+
+    def predict(self, indptr, indices, values, n_cols, output_margin=True) -> np.ndarray:
+        return predict(self, indptr, indices, values, n_cols, output_margin)
+
+
+def load_csr(indptr, indices, values, labels, n_cols, rle="off", rle_min_ratio=0.0, n_shards=1,
+             device=-1, stream="current", comm: Comm | None = None) -> Dataset:
+    indptr = np.ascontiguousarray(indptr, np.int64)
+    indices = np.ascontiguousarray(indices, np.int32)
+    values = np.ascontiguousarray(values, np.float32)
+    labels = np.ascontiguousarray(labels, np.float32)
+    n = indptr.size - 1
+    if stream == "current":
+        stream = _current_stream()
+    o = _LoadOpts(RLE[rle], float(rle_min_ratio), int(n_shards), int(device), stream,
+                  comm._h if comm is not None else None)
+    h = C.c_void_p()
+    _check(lib().gbdt_load_csr(n, int(n_cols), _p(indptr), _p(indices), _p(values), _p(labels), C.byref(o),
+                               C.byref(h)))
+    return Dataset(h, n, int(n_cols), None)
+
+
+def train(ds: Dataset, max_depth=6, n_trees=40, lam=1.0, gamma=0.0, eta=0.3, base_margin=0.0,
+          loss="squared", profile=False, want_margin=True):
+    prm = _Params(int(max_depth), int(n_trees), float(lam), float(gamma), float(eta), float(base_margin),
+                  LOSS[loss], int(bool(profile)))
+    h = C.c_void_p()
+    margin = np.zeros(ds.n, np.float64) if want_margin else None
+    _check(lib().gbdt_train(ds._h, C.byref(prm), C.byref(h), _p(margin)))
+    return Model(h), margin
+
+
+def predict(model: Model, indptr, indices, values, n_cols, output_margin=True) -> np.ndarray:
+    indptr = np.ascontiguousarray(indptr, np.int64)
+    indices = np.ascontiguousarray(indices, np.int32)
+    values = np.ascontiguousarray(values, np.float32)
+    n = indptr.size - 1
+    out = np.zeros(n, np.float64)
+    _check(lib().gbdt_predict(model._h, n, int(n_cols), _p(indptr), _p(indices), _p(values),
+                              int(bool(output_margin)), _p(out)))
+    return out
+
+
+def train_problem(prob, **overrides):
+    """Convenience: load + train a datagen.synth.Problem with its own parameters."""
+    P = dict(prob.params)
+    P.update(overrides)
+    rle = P.pop("rle", "off")
+    n_shards = P.pop("n_shards", 1)
+    ds = load_csr(prob.indptr, prob.indices, prob.values, prob.labels, prob.m, rle=rle, n_shards=n_shards)
+    return train(ds, **P)

@@ -1,0 +1,198 @@
+"""CUDA path vs the CPU oracle, element by element on the same seeded inputs (-m gpu).
+
+Every call goes through the C ABI (libgbdt.so) via the ctypes binding.
+"""
+import numpy as np
+import pytest
+
+from datagen import synth
+from oracle import oracle
+from paper_conf_ipps_wenhkls18_b200 import gbdt
+
+from parity import compare, structural_invariants
+
+pytestmark = pytest.mark.gpu
+
+
+def _train(prob, **kw):
+    return gbdt.train_problem(prob, **kw)
+
+
+# ------------------------------------------------------------------ a1 layout (bit-exact)
+@pytest.mark.parametrize("maker", [
+    lambda: synth.table1(),
+    lambda: synth.c1(n=3000),
+    lambda: synth.random_small(11, n=5000, m=7, nan_frac=0.3, n_distinct=40),
+    lambda: synth.c4(seed=5, n=800, m=3000, density=0.01),
+])
+def test_layout_bit_exact(maker):
+    p = maker()
+    ds = gbdt.load_csr(p.indptr, p.indices, p.values, p.labels, p.m)
+    col_ptr, val, ins = ds.export_layout()
+    ocp, oval, oins = oracle.presort(p.indptr, p.indices, p.values, p.n, p.m)
+    assert np.array_equal(col_ptr, ocp)
+    assert np.array_equal(val.view(np.uint32), oval.view(np.uint32))
+    assert np.array_equal(ins, oins)
+
+
+def test_layout_sharded_equals_unsharded():
+    p = synth.c1(n=2000)
+    base = gbdt.load_csr(p.indptr, p.indices, p.values, p.labels, p.m).export_layout()
+    for k in (2, 4, 8):
+        ds = gbdt.load_csr(p.indptr, p.indices, p.values, p.labels, p.m, n_shards=k)
+        cols = []
+        vals = []
+        inss = []
+        for s in range(k):
+            cp, v, i = ds.export_layout(s)
+            cols.append(np.diff(cp))
+            vals.append(v)
+            inss.append(i)
+        assert np.array_equal(np.concatenate(cols), np.diff(base[0]))
+        assert np.array_equal(np.concatenate(vals), base[1])
+        assert np.array_equal(np.concatenate(inss), base[2])
+
+
+# ------------------------------------------------------------------ worked example
+def test_table1_appendix_a_on_gpu():
+    p = synth.table1(loss="squared", d=2, T=2, lam=1.0, eta=1.0)
+    model, margin = _train(p)
+    nodes = model.nodes()
+    compare(p, nodes, margin, allow_near_ties=False)
+    assert nodes[0, 0]["attr"] == 0 and nodes[0, 0]["split_value"] == np.float32(1.2)
+    np.testing.assert_allclose(margin, [0.96, 0.0, 0.96, 0.0], rtol=1e-12, atol=1e-15)
+
+
+# ------------------------------------------------------------------ C1 (full config) and friends
+def test_c1_full_config_exact():
+    p = synth.c1()
+    model, margin = _train(p)
+    nodes = model.nodes()
+    st = compare(p, nodes, margin, allow_near_ties=False)
+    assert st["exact"] > 0
+    assert not np.any(nodes["attr"] == 7)  # a7 duplicates a0: exact ties resolve to a0
+
+
+@pytest.mark.parametrize("seed", range(8))
+@pytest.mark.parametrize("loss", ["squared", "logistic"])
+def test_random_missing_values(seed, loss):
+    p = synth.random_small(seed + 100, n=200 + 37 * seed, m=3 + seed % 5, nan_frac=0.3,
+                           n_distinct=3 + 2 * seed, loss=loss, d=4, T=3, lam=1.0,
+                           gamma=0.02 if seed % 3 == 2 else 0.0, eta=0.4)
+    model, margin = _train(p)
+    compare(p, model.nodes(), margin)
+
+
+@pytest.mark.parametrize("maker,T", [
+    (lambda: synth.c2(n=20000, T=4), 4),
+    (lambda: synth.c3(n=40000, T=3), 3),
+    (lambda: synth.c5(n=30000, T=3), 3),
+])
+def test_shaped_subsamples(maker, T):
+    p = maker()
+    model, margin = _train(p)
+    nodes = model.nodes()
+    compare(p, nodes, margin)
+    structural_invariants(nodes, p.n, p.params["max_depth"], p.params["lam"], p.params["gamma"])
+
+
+def test_sparse_many_segments():
+    p = synth.c4(seed=9, n=1500, m=4000, density=0.01, T=3)
+    model, margin = _train(p)
+    compare(p, model.nodes(), margin)
+
+
+def test_multi_tile_ragged():
+    # columns of 2048*k + ragged tails; exercises the Fenwick look-back across many tiles
+    p = synth.random_small(77, n=2048 * 9 + 123, m=3, nan_frac=0.0, n_distinct=5000, loss="logistic",
+                           d=5, T=2)
+    model, margin = _train(p)
+    compare(p, model.nodes(), margin)
+
+
+# ------------------------------------------------------------------ edge cases
+def test_constant_labels_no_split():
+    p = synth.c1(n=500)
+    p.labels[:] = 0.25
+    model, margin = _train(p, eta=1.0, lam=1.0)
+    nodes = model.nodes()
+    # g == 0 everywhere -> every gain is exactly 0 -> no split (strict >)
+    assert nodes[0, 0]["is_leaf"] == 1
+    compare(p, nodes, margin, params=dict(eta=1.0), allow_near_ties=False)
+
+
+def test_constant_and_missing_columns():
+    X = np.random.default_rng(1).normal(size=(300, 4))
+    X[:, 1] = 3.0
+    X[:, 2] = np.nan
+    X[::7, 3] = np.nan
+    y = X[:, 0] + (np.nan_to_num(X[:, 3]) > 0)
+    p = synth.from_dense("edge", X, y, dict(loss="squared", max_depth=3, n_trees=2, lam=1.0, gamma=0.0,
+                                             eta=0.5, base_margin=0.0))
+    model, margin = _train(p)
+    compare(p, model.nodes(), margin)
+
+
+def test_single_row_and_depth_one():
+    p = synth.c1(n=1)
+    model, margin = _train(p)
+    compare(p, model.nodes(), margin)
+    q = synth.c1(n=700)
+    model, margin = _train(q, max_depth=1, n_trees=3)
+    compare(q, model.nodes(), margin, params=dict(max_depth=1, n_trees=3))
+
+
+def test_gamma_blocks_splits():
+    p = synth.c1(n=700)
+    model, margin = _train(p, gamma=1e9)
+    nodes = model.nodes()
+    assert np.all(nodes[:, 0]["is_leaf"] == 1)
+    compare(p, nodes, margin, params=dict(gamma=1e9))
+
+
+# ------------------------------------------------------------------ prediction
+def test_predict_reproduces_training_margin_and_oracle():
+    p = synth.random_small(5, n=3000, m=6, nan_frac=0.2, n_distinct=50, loss="logistic", d=5, T=4)
+    model, margin = _train(p)
+    pred = model.predict(p.indptr, p.indices, p.values, p.m)
+    assert np.array_equal(pred, margin)
+    opred = oracle.predict(_as_oracle(model.nodes()), p.indptr, p.indices, p.values, eta=p.params["eta"])
+    assert np.array_equal(pred, opred)  # same trees, same op order -> bit-identical
+    prob = gbdt.predict(model, p.indptr, p.indices, p.values, p.m, output_margin=False)
+    np.testing.assert_allclose(prob, 1 / (1 + np.exp(-margin)), rtol=1e-15)
+
+
+def _as_oracle(nodes):
+    out = np.zeros(nodes.shape, oracle.NODE_DTYPE)
+    for f in oracle.NODE_DTYPE.names:
+        if f in nodes.dtype.names:
+            out[f] = nodes[f]
+    return out
+
+
+# ------------------------------------------------------------------ sharding (loopback, 1 GPU)
+@pytest.mark.parametrize("k", [2, 4, 8])
+def test_loopback_shards_bit_identical(k):
+    p = synth.c2(n=12000, T=3)
+    ref_model, ref_margin = _train(p)
+    ref = ref_model.nodes()
+    model, margin = _train(p, n_shards=k)
+    nodes = model.nodes()
+    assert np.array_equal(nodes.view(np.uint8), ref.view(np.uint8))
+    assert np.array_equal(margin, ref_margin)
+
+
+def test_loopback_shards_sparse_missing():
+    p = synth.c4(seed=3, n=1200, m=2500, density=0.01, T=2)
+    ref_model, ref_margin = _train(p)
+    model, margin = _train(p, n_shards=4)
+    assert np.array_equal(model.nodes().view(np.uint8), ref_model.nodes().view(np.uint8))
+    assert np.array_equal(margin, ref_margin)
+
+
+def test_deterministic_across_runs():
+    p = synth.c3(n=30000, T=2)
+    a, ma = _train(p)
+    b, mb = _train(p)
+    assert np.array_equal(a.nodes().view(np.uint8), b.nodes().view(np.uint8))
+    assert np.array_equal(ma, mb)
