@@ -1,0 +1,293 @@
+#!/usr/bin/env python
+"""Benchmark of the GPU-GBDT hot path on B200 (BASELINE.json metric: seconds per tree at depth 6;
+split-find HBM GB/s vs peak).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C3] [--impl ours|reference]
+
+A step is one tree: one pass of the whole per-tree hot path (SmartGD gradients, then for every
+level split finding, decision, node map and partition) over the resident synthetic dataset.
+`value` = device seconds per tree of a K-tree gbdt_train (CUDA events on the library's stream,
+max over ranks), after a W-tree warm-up training.  The dataset (2.5 GB of sorted lists for C3)
+is larger than L2, so no flush is needed between steps.  `e2e` = the same metric through the C
+ABI from pinned host buffers: gbdt_load_csr (H2D + layout build) + gbdt_train + margin D2H.
+For N > 1 (torchrun) the attributes are sharded over the ranks (NCCL allgather of node bests +
+bitmap allreduce per level) and the total work is fixed ("strong" scaling).
+
+--impl reference times the CPU oracle (oracle/, single thread) on a bounded row sample of the
+same workload and scales it to the full workload's entries (the paper's cost model is linear in
+the number of entries per level).
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "seconds per tree (depth 6) at 1/2/4/8 B200; split-find HBM GB/s vs peak"
+UNIT = "s/tree"
+BYTES_PER_ENTRY_SPLIT_FIND = 24  # val 4 + ins 4 + (g,h) fp64 gather 16
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=40)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C3")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--rle", default="off")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle CPU time for cpu_baseline")
+    return ap.parse_args()
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+def clock_sampler_start():
+    try:
+        return subprocess.Popen(
+            ["nvidia-smi", "--query-gpu=index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+             "--format=csv,noheader,nounits", "-lms", "100"],
+            stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+    except Exception:
+        return None
+
+
+def clock_sampler_stop(proc, dev=0):
+    if proc is None:
+        return None
+    time.sleep(0.15)
+    proc.terminate()
+    try:
+        out, _ = proc.communicate(timeout=5)
+    except Exception:
+        proc.kill()
+        out = ""
+    sm, smax, reasons = [], 0.0, set()
+    names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+    for line in out.strip().splitlines():
+        f = [x.strip() for x in line.split(",")]
+        if len(f) < 9 or f[0] != str(dev):
+            continue
+        try:
+            sm.append(float(f[1]))
+            smax = max(smax, float(f[2]))
+        except ValueError:
+            continue
+        for nm, v in zip(names, f[5:9]):
+            if v.lower().startswith("active"):
+                reasons.add(nm)
+    if not sm:
+        return None
+    return {"sm_mhz": statistics.median(sm), "sm_max_mhz": smax, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def entries_per_level(nodes, m_local, d):
+    """Entries the split-find kernel reads per level, from the trees: a node at depth l is active at
+    level l and, for dense data, owns count x m_local entries of the shard's lists."""
+    out = np.zeros(d, np.int64)
+    present = nodes["heap_id"] >= 0
+    heap = np.arange(nodes.shape[1])
+    depth = np.floor(np.log2(heap + 1)).astype(int)
+    for lvl in range(d):
+        sel = present & (depth[None, :] == lvl)
+        out[lvl] = int(nodes["count"][sel].sum()) * m_local
+    return out
+
+
+def oracle_sample_rate(prob, target_s, trees=2):
+    """Oracle seconds per tree on the full workload, estimated from a bounded row sample."""
+    from datagen import synth
+    from oracle import oracle
+    n_s = min(prob.n, 20000)
+    while True:
+        sub = _rows(prob, n_s)
+        t0 = time.perf_counter()
+        oracle.presort(sub.indptr, sub.indices, sub.values, sub.n, sub.m)
+        t1 = time.perf_counter()
+        oracle.train(sub, params=dict(n_trees=trees))
+        t2 = time.perf_counter()
+        per_tree = max((t2 - t1) - (t1 - t0), 1e-9) / trees
+        if t2 - t0 > target_s / 4 or n_s >= prob.n:
+            break
+        n_s = min(prob.n, int(n_s * min(8.0, max(2.0, (target_s / 4) / max(t2 - t0, 1e-3)))))
+    scale = prob.nnz / sub.nnz
+    return per_tree * scale, dict(n_rows=n_s, entries=sub.nnz, trees=trees, per_tree_s=per_tree,
+                                  scale=scale, presort_s=t1 - t0), synth
+
+
+def _rows(prob, n_s):
+    from datagen import synth
+    if n_s >= prob.n:
+        return prob
+    e = int(prob.indptr[n_s])
+    return synth.Problem(prob.name + f"[:{n_s}]", n_s, prob.m, prob.indptr[:n_s + 1].copy(),
+                         prob.indices[:e], prob.values[:e], prob.labels[:n_s], prob.params)
+
+
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    from datagen import synth
+
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        prob = synth.make(args.config)
+        P = prob.params
+        from oracle import oracle
+        # warm-up: W trees on a small sample (untimed), then the bounded timed sample
+        sub = _rows(prob, min(prob.n, 2000))
+        oracle.train(sub, params=dict(n_trees=max(1, min(args.warmup, 3))))
+        rate, info, _ = oracle_sample_rate(prob, args.cpu_seconds * 2, trees=min(args.steps, 3))
+        line = {
+            "impl": "reference", "metric": METRIC, "value": rate, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": rate * 1e3, "higher_is_better": False,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": args.config, "n": prob.n, "m": prob.m, "nnz": prob.nnz, "loss": P["loss"],
+                       "max_depth": P["max_depth"], "n_trees": P["n_trees"]},
+            "cpu_baseline": {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"first {info['n_rows']} rows ({info['entries']} entries), "
+                                       f"{info['trees']} trees, presort excluded, scaled x{info['scale']:.1f} by entries"},
+            "e2e": {"value": rate, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        }
+        print(json.dumps(line))
+        return
+
+    import torch
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    from paper_conf_ipps_wenhkls18_b200 import gbdt
+
+    prob = synth.make(args.config)
+    P = dict(prob.params)
+    d = P["max_depth"]
+    comm = gbdt.comm_from_torch(local) if world > 1 else None
+    stream = torch.cuda.current_stream()
+    ds = gbdt.load_csr(prob.indptr, prob.indices, prob.values, prob.labels, prob.m, rle=args.rle,
+                       stream=stream.cuda_stream, comm=comm)
+    info = ds.info(0)
+    m_local = info["attr_end"] - info["attr_begin"]
+    tp = dict(max_depth=d, lam=P["lam"], gamma=P["gamma"], eta=P["eta"], base_margin=P["base_margin"],
+              loss=P["loss"])
+
+    # warm-up (untimed)
+    gbdt.train(ds, n_trees=max(args.warmup, 1), want_margin=False, **tp)
+    torch.cuda.synchronize()
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clk = clock_sampler_start()
+    time.sleep(0.3)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record(stream)
+    model, _ = gbdt.train(ds, n_trees=args.steps, want_margin=False, profile=True, **tp)
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    clocks = clock_sampler_stop(clk, local)
+    launches = gbdt.last_launch_count()
+    ms = ev0.elapsed_time(ev1)
+    if dist:
+        t = torch.tensor([ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+        dist.barrier()
+    torch.cuda.synchronize()
+    tim = model.timings()
+    nodes = model.nodes()
+    ent = entries_per_level(nodes, m_local, d)       # summed over the K trees
+    sf_launches = args.steps * d
+    sf_bytes = float(ent.sum()) * BYTES_PER_ENTRY_SPLIT_FIND
+    sf_ms = tim["split_find"]
+    peak, peak_kind = peaks()
+    achieved = (sf_bytes / 1e9) / (sf_ms / 1e3) if sf_ms > 0 else None
+    traffic = None
+    tp_path = os.path.join(ROOT, "profiles", f"ncu_split_find_{args.config}.json")
+    if os.path.exists(tp_path):
+        with open(tp_path) as f:
+            traffic = json.load(f).get("dram_bytes_per_launch")
+
+    # e2e through the C ABI from pinned host buffers
+    e2e = None
+    if not args.no_e2e:
+        pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory().numpy()
+        hp, hi, hv, hl = pin(prob.indptr), pin(prob.indices), pin(prob.values), pin(prob.labels)
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        ds2 = gbdt.load_csr(hp, hi, hv, hl, prob.m, rle=args.rle, stream=stream.cuda_stream, comm=comm)
+        model2, margin2 = gbdt.train(ds2, n_trees=args.steps, want_margin=True, **tp)
+        torch.cuda.synchronize()
+        te = time.perf_counter() - t0
+        if dist:
+            t = torch.tensor([te], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            te = float(t.item())
+        h2d = hp.nbytes + hi.nbytes + hv.nbytes + hl.nbytes
+        d2h = margin2.nbytes + nodes.nbytes
+        e2e = {"value": te / args.steps, "unit": UNIT, "h2d_bytes_per_step": int(h2d / args.steps),
+               "d2h_bytes_per_step": int(d2h / args.steps),
+               "note": "one gbdt_load_csr (H2D + layout sort) + K-tree gbdt_train + margin D2H, amortised per tree"}
+        del ds2, model2
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        rate, cinfo, _ = oracle_sample_rate(prob, args.cpu_seconds)
+        cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"first {cinfo['n_rows']} rows ({cinfo['entries']} entries), {cinfo['trees']} trees, "
+                         f"presort excluded, scaled x{cinfo['scale']:.1f} by entries"}
+
+    if rank == 0:
+        value = ms / 1e3 / args.steps
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": False,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": args.config, "n": prob.n, "m": prob.m, "nnz": prob.nnz, "loss": P["loss"],
+                       "max_depth": d, "trees_timed": args.steps, "lambda": P["lam"], "eta": P["eta"],
+                       "rle": args.rle, "parallelism": f"attr-shard{world}",
+                       "l2": "inputs larger than L2 (sorted lists %.2f GB)" % (prob.nnz * 8 / 1e9)},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": (achieved / peak) if achieved else None, "traffic": traffic,
+                         "kernel": "k_split_find", "peak_kind": peak_kind,
+                         "bytes_per_entry": BYTES_PER_ENTRY_SPLIT_FIND, "launches": sf_launches,
+                         "avg_launch_ms": sf_ms / sf_launches},
+            "phases_ms_per_tree": {k: v / args.steps for k, v in tim.items()},
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "clocks": clocks,
+            "context": {"paper_gpu_gbdt_titanx_higgs10M_mse_s_per_tree": 5.50,
+                        "paper_xgbst40_higgs10M_mse_s_per_tree": 9.66, "source": "PAPER.md P:478-487 /40"},
+        }
+        print(json.dumps(line))
+    if dist:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

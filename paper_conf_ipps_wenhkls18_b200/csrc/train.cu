@@ -346,20 +346,13 @@ __global__ void __launch_bounds__(kThreads, 2) k_split_find(SplitArgs A) {
       const int u = sm.u;
       const int tb = t - u;
       const int jpub = __ffs(u + 1) - 1;  // top block of tile u covers (u - 2^jpub, u]
+      // (1) publish this tile's Fenwick block first: it depends only on other tiles' blocks,
+      //     never on any exclusive prefix, so the dependency depth stays <= log2(tiles)
       SVf got = svf_zero();
       if (lane < jpub) {
         const int tt = tb + u - (1 << lane);
         wait_flag(A.fw.E + tt, epoch);
         got = SVf{__ldcg(A.fw.G + tt), __ldcg(A.fw.H + tt), __ldcg(A.fw.C + tt), __ldcg(A.fw.F + tt)};
-      }
-      const int pc = __popc(u);
-      SVf q = svf_zero();
-      if (lane >= 16 && lane < 16 + pc) {
-        int i = u;
-        for (int r = 0; r < lane - 16; ++r) i &= i - 1;
-        const int tt = tb + i - 1;
-        wait_flag(A.fw.E + tt, epoch);
-        q = SVf{__ldcg(A.fw.G + tt), __ldcg(A.fw.H + tt), __ldcg(A.fw.C + tt), __ldcg(A.fw.F + tt)};
       }
       SVf B = agg;
       for (int i = 0; i < jpub; ++i) B = comb(shfl_idx(got, i), B);
@@ -367,8 +360,18 @@ __global__ void __launch_bounds__(kThreads, 2) k_split_find(SplitArgs A) {
         A.fw.G[t] = B.g; A.fw.H[t] = B.h; A.fw.C[t] = B.c; A.fw.F[t] = B.f;
         st_release(A.fw.E + t, epoch);
       }
+      // (2) exclusive prefix of the tile = fold of the Fenwick blocks covering [0, u)
+      const int pc = __popc(u);
+      SVf q = svf_zero();
+      if (lane < pc) {
+        int i = u;
+        for (int r = 0; r < lane; ++r) i &= i - 1;
+        const int tt = tb + i - 1;
+        wait_flag(A.fw.E + tt, epoch);
+        q = SVf{__ldcg(A.fw.G + tt), __ldcg(A.fw.H + tt), __ldcg(A.fw.C + tt), __ldcg(A.fw.F + tt)};
+      }
       SVf E = svf_zero();
-      for (int b = pc - 1; b >= 0; --b) E = comb(E, shfl_idx(q, 16 + b));
+      for (int b = pc - 1; b >= 0; --b) E = comb(E, shfl_idx(q, b));
       __syncwarp();
       if (lane < kWarps) s_wcar[lane] = comb(E, s_wcar[lane]);
     }
@@ -1126,14 +1129,16 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       NodeTab& nxt = nt[(lvl + 1) & 1];
       const bool last = (lvl == d - 1);
       const int Kl = 1 << lvl;  // upper bound of active nodes at this level
-      tm.begin(GBDT_PHASE_SPLIT_FIND);
+      tm.begin(GBDT_PHASE_DECIDE);
       k_level_begin<<<1, 1024, 0, st>>>(epoch, sw[0].counters, 0, nrec, nloc, cur.K, gkey, tkey, Kcap);
       GBDT_LAUNCH_CHECK();
       count_launch();
+      for (int li = 0; li < nloc; ++li) GBDT_CUDA(cudaMemsetAsync(sw[li].counters, 0, 4 * sizeof(int), st));
+      tm.end();
+      tm.begin(GBDT_PHASE_SPLIT_FIND);
       for (int li = 0; li < nloc; ++li) {
         Shard& sh = *ds.shards[li];
         ShardWork& w = sw[li];
-        GBDT_CUDA(cudaMemsetAsync(w.counters, 0, 4 * sizeof(int), st));
         if (sh.m == 0) continue;
         const Tables tb = lvl == 0 ? sh.root : w.tab[lvl & 1];
         const float* val = lvl == 0 ? sh.val0.as<float>() : sh.valw[lvl & 1].as<float>();
