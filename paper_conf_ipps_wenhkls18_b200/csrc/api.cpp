@@ -109,7 +109,9 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
     validate_csr(n_rows, n_cols, indptr, indices, values, true);
     if (!labels) fail(GBDT_E_INVAL, "labels is NULL");
     float lmin = std::numeric_limits<float>::infinity(), lmax = -lmin;
+    bool binary = true;
     for (int64_t i = 0; i < n_rows; ++i) {
+      binary &= (labels[i] == 0.0f || labels[i] == 1.0f);
       if (!std::isfinite(labels[i])) fail(GBDT_E_INVAL, "labels must be finite (row " + std::to_string(i) + ")");
       lmin = std::min(lmin, labels[i]);
       lmax = std::max(lmax, labels[i]);
@@ -146,6 +148,7 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
       ds.device = dev;
       ds.stream = (cudaStream_t)o.stream;
       ds.has_missing = missing;
+      ds.binary_labels = binary;
       ds.comm = comm;
       ds.rle = o.rle;
       ds.h_labels_minmax = {lmin, lmax};

@@ -107,6 +107,7 @@ struct Dataset {
   int device = 0;
   cudaStream_t stream = nullptr;
   bool has_missing = false;      // some instance lacks some attribute
+  bool binary_labels = false;    // every label is 0 or 1
   DBuf y;                        // labels (device, fp32)
   std::vector<float> h_labels_minmax;  // [min, max]
   std::vector<std::unique_ptr<Shard>> shards;  // local shards

@@ -1,4 +1,4 @@
-// kernels.cuh -- argument blocks of the per-level sm_100a kernels (train.cu).
+// kernels.cuh -- argument blocks of the per-level sm_100a kernels (train.cu, levels.cu).
 #pragma once
 #include "common.cuh"
 
@@ -15,15 +15,6 @@ struct NodeTab {
   double* pterm;    // [Kcap] G^2/(H+lambda), the parent term of Eq. 2
 };
 
-// Fenwick-tree look-back storage: top block of every tile (see split_find in train.cu).
-struct Fenwick {
-  double* G;
-  double* H;
-  int32_t* C;
-  int32_t* F;   // 1: the block contains a segment head
-  int32_t* E;   // publication flag = level epoch
-};
-
 struct TileArgs {
   const float* val;
   const int32_t* ins;
@@ -34,36 +25,77 @@ struct TileArgs {
   int* counter;        // dynamic tile claim counter (reset per level)
 };
 
+// Gradient storage mode of the split-find kernels:
+//   0: squared loss, h == 2 (only g is gathered)
+//   1: logistic loss with 0/1 labels, h = max(q(1-q), 1e-16), q = g + [g < 0] (reading R5b)
+//   2: general: h gathered too
+enum { kHConst2 = 0, kHFromG = 1, kHGather = 2 };
+
 struct SplitArgs {
   TileArgs t;
-  const double2* gh;
+  const double* g;       // per instance
+  const double* h;       // per instance (mode 2)
+  double* glist;         // per list entry: g of the entry's instance (written by k_tile_agg)
+  double* hlist;         // per list entry: h (mode 2)
+  unsigned long long* tagg;   // [T][5] tile aggregate: fixed-point g, h (lo,hi each), count | head << 32
+  unsigned long long* carry;  // [T][5] exclusive segmented prefix of the tile (same layout)
   NodeTab nodes;
   const double* segPG;   // [m*K] present totals per segment (only with missing values)
   const double* segPH;
   double lam;
   const int32_t* epochp;
-  Fenwick fw;
-  Rec* rec;              // per-piece records (appended)
+  const int32_t* fx;     // [2] fixed-point scales F_g, F_h of this tree (value * 2^F fits in 2^125)
+  Rec* rec;              // node-best records (appended)
   int* nrec;
   unsigned long long* gkey;  // [Kcap] per node max gain key
   int shard;
-  int totals_only;       // 1: write segPG/segPH instead of evaluating gains
-  double* segPG_out;
+  double* segPG_out;     // totals pass output
   double* segPH_out;
 };
 
 struct PartArgs {
   TileArgs t;
   const uint8_t* side;    // per instance: 0 drop, 1 high, 2 low
-  uint32_t* tile_cnt;     // [T] packed hi | lo<<16
-  int32_t* segH;          // [m*K]
+  int32_t* segH;          // [m*K] counted (missing values) or derived from node counts (dense)
   int32_t* segL;
-  const unsigned long long* tile_pre;  // [T] packed hi | lo<<32 exclusive
-  const unsigned long long* seg_pre;   // [m*K]
+  uint32_t* tcnt;         // [T] tile (high | low << 16) counts
+  unsigned long long* tpre;  // [T] exclusive (high | low << 32) count of the attribute before the tile
+  const unsigned long long* seg_pre;   // [m*K] exclusive count of the attribute before the segment
   const int64_t* out_hi;  // [m*K]
   const int64_t* out_lo;
   float* val_out;
   int32_t* ins_out;
+};
+
+struct PlanArgs {
+  int m;
+  int counted;            // 1: segH/segL were counted (missing values); 0: derive from node counts
+  const int32_t* Kp;      // current K
+  const int32_t* Knp;     // next K
+  const int32_t* cidx;
+  const int32_t* ncnt;    // next-level node counts
+  int32_t* segH;
+  int32_t* segL;
+  unsigned long long* seg_pre;
+  int64_t* out_hi;
+  int64_t* out_lo;
+  int64_t* len_tmp;       // [m]
+  Tables nxt;
+};
+
+// levels.cu launchers
+struct LevelKernels {
+  int sms = 148;
+  unsigned grid_sf[3][2] = {{0}};  // [hmode][missing]
+  unsigned grid_tot[3] = {0};
+  unsigned grid_agg[3] = {0};
+  unsigned grid_scatter = 0, grid_count = 0;
+  void init(int device);
+  // a3/a4: tile aggregates (+ g/h lists) and the exact segmented carry scan
+  void tile_prefix(const SplitArgs& A, int hmode, cudaStream_t st);
+  void split_find(const SplitArgs& A, int hmode, bool missing, cudaStream_t st);
+  void seg_totals(const SplitArgs& A, int hmode, cudaStream_t st);
+  void partition(const PartArgs& A, const PlanArgs& P, bool counted, cudaStream_t st);
 };
 
 }  // namespace gbdt
