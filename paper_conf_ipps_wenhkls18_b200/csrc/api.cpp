@@ -131,6 +131,13 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
     if (dev >= ndev) fail(GBDT_E_RANGE, "device ordinal out of range");
     if (comm) dev = comm->device;
     GBDT_CUDA(cudaSetDevice(dev));
+    {
+      // keep freed stream-ordered allocations cached in the pool across gbdt_train calls
+      cudaMemPool_t pool;
+      GBDT_CUDA(cudaDeviceGetDefaultMemPool(&pool, dev));
+      uint64_t thr = UINT64_MAX;
+      GBDT_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+    }
 
     const int64_t nnz = indptr[n_rows];
     std::vector<int64_t> col_counts(n_cols, 0);

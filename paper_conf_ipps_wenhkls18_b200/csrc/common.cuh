@@ -13,6 +13,7 @@ constexpr int kThreads = 256;          // threads per tile CTA (8 warps)
 constexpr int kItems = 8;              // entries per thread, blocked arrangement
 constexpr int kTile = kThreads * kItems;  // 2048 entries per tile (attribute-aligned)
 constexpr int kWarps = kThreads / 32;
+constexpr int kChunk = 32 * kItems;    // 256 entries: the unit of one warp (8 per tile)
 
 // ----------------------------------------------------------------------------- memory order
 __device__ __forceinline__ int ld_acquire(const int* p) {
@@ -80,6 +81,12 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
           smem_u32(dst)),
       "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
       : "memory");
+}
+// read-only load that L2 should keep (gathered per-instance gradients)
+__device__ __forceinline__ double ld_keep(const double* p, unsigned long long pol) {
+  double v;
+  asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(pol));
+  return v;
 }
 // per-thread async gathers (LDGSTS)
 __device__ __forceinline__ void cp_async8(void* dst, const void* src, unsigned long long pol) {

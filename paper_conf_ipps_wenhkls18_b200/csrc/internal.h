@@ -63,9 +63,11 @@ struct Tables {
   int64_t* col_start = nullptr;   // [m+1] padded start of each attribute list
   int64_t* col_len = nullptr;     // [m]   entries of each attribute list at this level
   int32_t* tile_start = nullptr;  // [m+1] first tile of each attribute (tiles never straddle)
+  int32_t* chunk_start = nullptr; // [m+1] first 256-entry chunk of each attribute (8 per tile)
   int64_t* seg_start = nullptr;   // [m*Kcap]
   int64_t* seg_cnt = nullptr;     // [m*Kcap]
   int32_t* T = nullptr;           // [1] tiles at this level
+  int32_t* C = nullptr;           // [1] chunks at this level
 };
 
 // Best split of one node found in one shard ("piece" records are reduced to this).
@@ -90,6 +92,7 @@ struct Shard {
   int64_t nnz = 0;               // stored entries of this shard
   int64_t cap = 0;               // padded level-buffer length (+ slack)
   int32_t T0 = 0;                // tiles at the root
+  int32_t C0 = 0;                // 256-entry chunks at the root
   DBuf val0, ins0;               // pristine root layout (padded)
   DBuf valw[2], insw[2];         // ping-pong level buffers
   DBuf root_tab;                 // root tables storage

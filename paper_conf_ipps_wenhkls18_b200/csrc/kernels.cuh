@@ -37,8 +37,9 @@ struct SplitArgs {
   const double* h;       // per instance (mode 2)
   double* glist;         // per list entry: g of the entry's instance (written by k_tile_agg)
   double* hlist;         // per list entry: h (mode 2)
-  unsigned long long* tagg;   // [T][5] tile aggregate: fixed-point g, h (lo,hi each), count | head << 32
-  unsigned long long* carry;  // [T][5] exclusive segmented prefix of the tile (same layout)
+  unsigned long long* cagg;   // [C][5] chunk aggregate: fixed-point g, h (lo,hi each), count | flags
+  unsigned long long* carry;  // [C][5] exclusive segmented prefix of the chunk (same layout)
+  unsigned long long* sgrp;   // scan scratch (group aggregates / carries)
   NodeTab nodes;
   const double* segPG;   // [m*K] present totals per segment (only with missing values)
   const double* segPH;
@@ -53,13 +54,28 @@ struct SplitArgs {
   double* segPH_out;
 };
 
+// Decoupled look-back storage of the partition's (high, low) counts: integers, exact in any order.
+struct LookBack {
+  int32_t* flag;                 // 2*epoch+1: aggregate published, 2*epoch+2: inclusive prefix published
+  unsigned long long* agg;       // packed hi | lo << 32
+  unsigned long long* incl;
+};
+
 struct PartArgs {
   TileArgs t;
+  const double* g_in;     // g-list (h-list) of this level, moved with the entries
+  const double* h_in;
+  double* g_out;
+  double* h_out;
+  const int32_t* epochp;
+  LookBack lb;
   const uint8_t* side;    // per instance: 0 drop, 1 high, 2 low
+  uint8_t* slist;         // per list entry: side of its instance (k_part_count -> k_part_scatter)
   int32_t* segH;          // [m*K] counted (missing values) or derived from node counts (dense)
   int32_t* segL;
-  uint32_t* tcnt;         // [T] tile (high | low << 16) counts
-  unsigned long long* tpre;  // [T] exclusive (high | low << 32) count of the attribute before the tile
+  unsigned long long* ccnt;  // [C][2] chunk (high | low << 32) counts, reset flag
+  unsigned long long* cpre;  // [C][2] exclusive count of the attribute before the chunk
+  unsigned long long* sgrp;  // scan scratch
   const unsigned long long* seg_pre;   // [m*K] exclusive count of the attribute before the segment
   const int64_t* out_hi;  // [m*K]
   const int64_t* out_lo;
@@ -89,13 +105,15 @@ struct LevelKernels {
   unsigned grid_sf[3][2] = {{0}};  // [hmode][missing]
   unsigned grid_tot[3] = {0};
   unsigned grid_agg[3] = {0};
-  unsigned grid_scatter = 0, grid_count = 0;
+  unsigned grid_scatter[2] = {0}, grid_count = 0, grid_agg_list[3] = {0};
   void init(int device);
   // a3/a4: tile aggregates (+ g/h lists) and the exact segmented carry scan
-  void tile_prefix(const SplitArgs& A, int hmode, cudaStream_t st);
+  static unsigned scan_groups(int64_t max_chunks);
+  void tile_prefix(const SplitArgs& A, int hmode, bool gather, unsigned groups, cudaStream_t st);
   void split_find(const SplitArgs& A, int hmode, bool missing, cudaStream_t st);
   void seg_totals(const SplitArgs& A, int hmode, cudaStream_t st);
-  void partition(const PartArgs& A, const PlanArgs& P, bool counted, cudaStream_t st);
+  void partition(const PartArgs& A, const PlanArgs& P, bool counted, bool with_h, unsigned groups,
+                 cudaStream_t st);
 };
 
 }  // namespace gbdt

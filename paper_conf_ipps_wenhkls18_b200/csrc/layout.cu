@@ -254,12 +254,14 @@ void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices
     sh.nnz = 0;
     for (int a = 0; a < m; ++a) { sh.h_col_len[a] = col_counts[sh.a_begin + a]; sh.nnz += sh.h_col_len[a]; }
     sh.h_col_start.assign(m + 1, 0);
-    std::vector<int32_t> tstart(m + 1, 0);
+    std::vector<int32_t> tstart(m + 1, 0), cstart(m + 1, 0);
     for (int a = 0; a < m; ++a) {
       sh.h_col_start[a + 1] = sh.h_col_start[a] + pad4(sh.h_col_len[a]);
       tstart[a + 1] = tstart[a] + (int32_t)ceil_div(sh.h_col_len[a], kTile);
+      cstart[a + 1] = cstart[a] + (int32_t)ceil_div(sh.h_col_len[a], kChunk);
     }
     sh.T0 = tstart[m];
+    sh.C0 = cstart[m];
     sh.cap = sh.h_col_start[m] + 16;
     sh.val0.alloc(sh.cap * 4, st);
     sh.ins0.alloc(sh.cap * 4, st);
@@ -272,7 +274,7 @@ void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices
       GBDT_CUDA(cudaMemsetAsync(sh.insw[b].p, 0, sh.cap * 4, st));
     }
     // root tables: col_start[m+1], col_len[m], tile_start[m+1], seg_start[m], seg_cnt[m], T
-    const size_t rb = (size_t)(m + 1) * 8 + (size_t)m * 8 + (size_t)(m + 1) * 4 + (size_t)m * 16 + 16;
+    const size_t rb = (size_t)(m + 1) * 8 + (size_t)m * 8 + (size_t)(m + 1) * 8 + (size_t)m * 16 + 64;
     sh.root_tab.alloc(rb + 64, st);
     char* q = sh.root_tab.as<char>();
     sh.root.col_start = (int64_t*)q; q += (size_t)(m + 1) * 8;
@@ -280,7 +282,9 @@ void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices
     sh.root.seg_start = (int64_t*)q; q += (size_t)m * 8;
     sh.root.seg_cnt = (int64_t*)q; q += (size_t)m * 8;
     sh.root.T = (int32_t*)q; q += 16;
-    sh.root.tile_start = (int32_t*)q;
+    sh.root.C = (int32_t*)q; q += 16;
+    sh.root.tile_start = (int32_t*)q; q += (size_t)(m + 1) * 4;
+    sh.root.chunk_start = (int32_t*)q;
     GBDT_CUDA(cudaMemcpyAsync(sh.root.col_start, sh.h_col_start.data(), (m + 1) * 8, cudaMemcpyHostToDevice, st));
     if (m) {
       GBDT_CUDA(cudaMemcpyAsync(sh.root.col_len, sh.h_col_len.data(), m * 8, cudaMemcpyHostToDevice, st));
@@ -289,6 +293,8 @@ void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices
     }
     GBDT_CUDA(cudaMemcpyAsync(sh.root.tile_start, tstart.data(), (m + 1) * 4, cudaMemcpyHostToDevice, st));
     GBDT_CUDA(cudaMemcpyAsync(sh.root.T, &sh.T0, 4, cudaMemcpyHostToDevice, st));
+    GBDT_CUDA(cudaMemcpyAsync(sh.root.chunk_start, cstart.data(), (m + 1) * 4, cudaMemcpyHostToDevice, st));
+    GBDT_CUDA(cudaMemcpyAsync(sh.root.C, &sh.C0, 4, cudaMemcpyHostToDevice, st));
     GBDT_CUDA(cudaStreamSynchronize(st));  // host vectors above must outlive the copies
     if (m == 0 || sh.nnz == 0) continue;
 

@@ -1,33 +1,32 @@
 // levels.cu -- the per-level streaming kernels of the hot path on sm_100a:
 //
-//   k_sf          a3-a6: segmented prefix sum of (g, h, count) over every (node, attribute)
-//                 segment of the level's attribute-sorted lists (Fig. 1), Eq. 2 gain at
-//                 the end of every run of equal values, both missing directions
-//                 (P:116), best split per node
-//   k_part_*      a8: order-preserving stable partition of every segment into its two children,
-//                 entries of new leaves dropped
+//   a3-a6 split find: segmented prefix sum of (g, h, count) over every (node,
+//         attribute) segment of the level's attribute-sorted lists (Fig. 1), Eq. 2 gain at the end
+//         of every run of equal values, both missing directions,
+//         best split per node
+//   a8    partition: order-preserving stable partition of every segment into its two
+//         children; entries of new leaves are dropped
 //
-// The work unit is a tile: 2048 consecutive entries of one attribute list (tiles never straddle
-// attributes).  The segmented scan is done reduce-then-scan, so no CTA ever waits on another:
-//   k_tile_agg   per tile: gathers g (h) of the tile's instances -- the only random access of the
-//                level, into an L2-resident array (n x 8 B: 88 MB for the 11M-row config, loaded
-//                evict-last) -- writes them as a contiguous g-list next to the attribute list, and
-//                publishes the tile's segmented aggregate
-//   k_tile_scan  one warp per attribute: exact segmented carry of every tile
-//   k_sf         persistent, 3-stage shared-memory ring fed by TMA 1-D bulk copies
-//                (cp.async.bulk / UBLKCP, mbarrier completion, evict-first) of the tile's value
-//                list and g-list; computes in-tile prefixes + carry, the Eq. 2 gains and the
-//                per-node argmax while the next two tiles stream in
-//   k_part_count / k_part_tscan / k_part_plan / k_part_scatter   same count -> scan -> scatter
-//                shape for the partition
+// Work decomposition.  An attribute list is cut into 256-entry CHUNKS (one warp: 32 lanes x 8
+// consecutive entries) and 2048-entry TILES (8 chunks); neither straddles attributes.  Every
+// streaming kernel is warp-granular -- a warp owns a chunk end to end and never waits for
+// another warp -- so latency is hidden by warp parallelism alone:
+//   k_chunk_agg   per chunk: g (h) of its entries -- gathered from the L2-resident per-instance
+//                 array at the root (the only random access of the level), read from the g-list
+//                 the partition carried along below it -- and the chunk's segmented aggregate
+//   k_scan1/2/3   exact segmented exclusive scan of the chunk aggregates (three parallel phases)
+//   k_sf          persistent tile loop over a 3-stage shared-memory ring fed by TMA 1-D bulk
+//                 copies (cp.async.bulk / UBLKCP, mbarrier completion, L2 evict-first) of the
+//                 tile's value list and g-list; each warp scans its chunk from its carry, ranks
+//                 its run ends (Eq. 2), and posts its best candidates to a per-CTA node table
+//   k_part_count / k_scan1/2/3 / k_part_plan / k_part_scatter   count -> scan -> stable scatter,
+//                 the entry's g (h) moving with it
 //
-// Determinism: inside a tile every sum has a fixed association.  Across tiles, each tile's fp64
-// aggregate is converted ONCE to an exact 128-bit fixed-point integer (trunc(x * 2^F), F per tree),
-// and the carry into a tile is the integer sum of its predecessors' published values, assembled by
-// a CTA-wide decoupled look-back.  Integer addition is exact and associative, so the carry -- and
-// every prefix, gain and tree built from it -- is bit-identical whatever the timing, the tile
-// schedule, or the attribute sharding (tiles are attribute-aligned).  The partition's carry is an
-// integer count and equally exact.
+// Determinism.  Inside a chunk every sum has a fixed association.  Across chunks, each chunk's
+// fp64 aggregate is converted ONCE to an exact 128-bit fixed-point integer (trunc(x * 2^F), F per
+// tree so that every sum stays below 2^125) and carries are integer sums: exact and associative,
+// so every prefix, gain and tree is bit-identical whatever the schedule, the scan decomposition or
+// the attribute sharding (chunks are attribute-aligned).  Partition offsets are integer counts.
 #include <algorithm>
 #include <climits>
 
@@ -40,8 +39,10 @@ constexpr int kStages = 3;
 constexpr int kSegCache = 32;     // segment starts/counts of a tile's attribute cached per stage
 constexpr int kCtaK = 64;         // per-CTA node-best table when K <= kCtaK
 constexpr int kTabCache = 64;     // attribute tables cached in smem when m <= kTabCache
-constexpr int kPieceList = 32;
-constexpr int kLiteBlocks = 4;    // target CTAs/SM of the light streaming kernels
+constexpr int kPieceList = 64;
+constexpr int kChunksPerTile = kTile / kChunk;  // 8 == kWarps
+constexpr int kScanGroup = 1024;  // elements per CTA in the 3-phase scans
+static_assert(kChunksPerTile == kWarps, "one warp per chunk of a tile");
 
 // ============================================================================ scan algebra
 struct SVf {
@@ -58,42 +59,90 @@ __device__ __forceinline__ SVf shfl_up(const SVf& x, int o) {
   return SVf{__shfl_up_sync(0xffffffffu, x.g, o), __shfl_up_sync(0xffffffffu, x.h, o),
              __shfl_up_sync(0xffffffffu, x.c, o), __shfl_up_sync(0xffffffffu, x.f, o)};
 }
-__device__ __forceinline__ SVf shfl_idx(const SVf& x, int l) {
-  return SVf{__shfl_sync(0xffffffffu, x.g, l), __shfl_sync(0xffffffffu, x.h, l),
-             __shfl_sync(0xffffffffu, x.c, l), __shfl_sync(0xffffffffu, x.f, l)};
+
+// ============================================================================ exact fixed point
+// x -> trunc(x * 2^F) as a 128-bit integer.  A pure function of x, and integer addition is
+// associative, so sums of converted values are bit-identical in any order.
+__device__ __forceinline__ __int128 to_fx(double x, int F) {
+  if (x == 0.0) return 0;
+  const long long b = __double_as_longlong(x);
+  const int e = (int)((b >> 52) & 0x7ff);
+  const unsigned long long mant = (unsigned long long)(b & 0xfffffffffffffll) | (e ? (1ull << 52) : 0ull);
+  const int sh = (e ? e : 1) - 1075 + F;
+  unsigned __int128 v;
+  if (sh >= 0) v = (unsigned __int128)mant << (sh > 74 ? 74 : sh);
+  else v = (sh > -64) ? (unsigned __int128)(mant >> (-sh)) : (unsigned __int128)0;
+  return b < 0 ? -(__int128)v : (__int128)v;
+}
+__device__ __forceinline__ double from_fx(__int128 v, int F) {
+  const bool neg = v < 0;
+  const unsigned __int128 u = neg ? (unsigned __int128)(-v) : (unsigned __int128)v;
+  const double hi = (double)(unsigned long long)(u >> 64), lo = (double)(unsigned long long)u;
+  double r = __dadd_rn(__dmul_rn(hi, 18446744073709551616.0), lo);
+  r = __dmul_rn(r, __longlong_as_double((long long)(1023 - F) << 52));  // exact power of two
+  return neg ? -r : r;
+}
+__device__ __forceinline__ __int128 shfl_up128(__int128 v, int o) {
+  const unsigned long long lo = __shfl_up_sync(0xffffffffu, (unsigned long long)v, o);
+  const unsigned long long hi = __shfl_up_sync(0xffffffffu, (unsigned long long)((unsigned __int128)v >> 64), o);
+  return (__int128)(((unsigned __int128)hi << 64) | lo);
+}
+__device__ __forceinline__ __int128 shfl_idx128(__int128 v, int l) {
+  const unsigned long long lo = __shfl_sync(0xffffffffu, (unsigned long long)v, l);
+  const unsigned long long hi = __shfl_sync(0xffffffffu, (unsigned long long)((unsigned __int128)v >> 64), l);
+  return (__int128)(((unsigned __int128)hi << 64) | lo);
 }
 
-// argmax element within a piece (attr fixed): gain desc, value desc, dir low first (R12)
-struct AM {
-  double gain;
-  float value;
-  int meta;  // bits 0-11 item index in tile, bit 12 dir, bit 13 valid
-  int f;     // piece start inside
+// Element of the exact scans: fixed-point (g, h), count, head-inside flag.  In global memory:
+// 5 words  g.lo g.hi h.lo h.hi  count | f << 32 | reset-before << 33.
+struct FXV {
+  __int128 g, h;
+  int c, f;
 };
-__device__ __forceinline__ AM am_none() { return AM{0.0, 0.f, 0, 0}; }
-__device__ __forceinline__ bool am_valid(const AM& a) { return (a.meta >> 13) & 1; }
-__device__ __forceinline__ AM am_best(const AM& a, const AM& b) {
-  if (!am_valid(a)) return b;
-  if (!am_valid(b)) return a;
-  if (a.gain != b.gain) return a.gain > b.gain ? a : b;
-  if (a.value != b.value) return a.value > b.value ? a : b;
-  return ((a.meta >> 12) & 1) <= ((b.meta >> 12) & 1) ? a : b;
-}
-__device__ __forceinline__ AM am_comb(const AM& l, const AM& r) {
+__device__ __forceinline__ FXV fxv_comb(const FXV& l, const FXV& r) {
   if (r.f) return r;
-  AM x = am_best(l, r);
-  x.f = l.f;
-  return x;
+  return FXV{l.g + r.g, l.h + r.h, l.c + r.c, l.f};
 }
-__device__ __forceinline__ AM shfl_up(const AM& x, int o) {
-  return AM{__shfl_up_sync(0xffffffffu, x.gain, o), __shfl_up_sync(0xffffffffu, x.value, o),
-            __shfl_up_sync(0xffffffffu, x.meta, o), __shfl_up_sync(0xffffffffu, x.f, o)};
+__device__ __forceinline__ void fxv_store(unsigned long long* dst, const FXV& x, int reset) {
+  dst[0] = (unsigned long long)x.g;
+  dst[1] = (unsigned long long)((unsigned __int128)x.g >> 64);
+  dst[2] = (unsigned long long)x.h;
+  dst[3] = (unsigned long long)((unsigned __int128)x.h >> 64);
+  dst[4] = (unsigned long long)(unsigned)x.c | ((unsigned long long)(x.f & 1) << 32) |
+           ((unsigned long long)(reset & 1) << 33);
+}
+__device__ __forceinline__ FXV fxv_load(const unsigned long long* src, int* reset = nullptr) {
+  const unsigned long long w = src[4];
+  if (reset) *reset = (int)((w >> 33) & 1);
+  return FXV{(__int128)(((unsigned __int128)src[1] << 64) | src[0]),
+             (__int128)(((unsigned __int128)src[3] << 64) | src[2]), (int)(unsigned)w, (int)((w >> 32) & 1)};
 }
 
-// ============================================================================ tile plumbing
+template <int HMODE>
+__device__ __forceinline__ double hess_of(double g) {
+  if (HMODE == kHConst2) return 2.0;
+  // logistic, 0/1 labels: y = [g < 0] (g = p - y with p in [0,1]); q = g + y; reading R5b
+  const double q = g < 0.0 ? __dadd_rn(g, 1.0) : g;
+  const double hh = __dmul_rn(q, __dsub_rn(1.0, q));
+  return hh > 1e-16 ? hh : 1e-16;
+}
+
+// 1/x for x > 0 (normal): hardware seed + two Newton steps (~1 ulp).  Used only to RANK the
+// candidates of a chunk; the winner's Eq. 2 gain is then recomputed with IEEE divisions.
+__device__ __forceinline__ double rcp_nr(double x) {
+  double r;
+  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
+  double e = __fma_rn(-x, r, 1.0);
+  r = __fma_rn(r, e, r);
+  e = __fma_rn(-x, r, 1.0);
+  return __fma_rn(r, e, r);
+}
+
+// ============================================================================ plumbing
 struct TabCache {
   int use;
   int tile_start[kTabCache + 1];
+  int chunk_start[kTabCache + 1];
   long long col_start[kTabCache + 1];
   long long col_len[kTabCache];
 };
@@ -104,44 +153,50 @@ __device__ __forceinline__ void tab_load(TabCache& tc, const TileArgs& A) {
   if (use) {
     for (int i = threadIdx.x; i <= A.m; i += blockDim.x) {
       tc.tile_start[i] = A.tb.tile_start[i];
+      tc.chunk_start[i] = A.tb.chunk_start[i];
       tc.col_start[i] = A.tb.col_start[i];
       if (i < A.m) tc.col_len[i] = A.tb.col_len[i];
     }
   }
 }
 
-
-// Tile metadata computed by one thread.
-struct TileMeta {
-  long long p0, p1, colend, sb;
-  int t, a, u, pad;
-};
-
-__device__ __forceinline__ void tile_meta(const TabCache& tc, const TileArgs& A, int K, int t, TileMeta& M) {
-  const bool c = tc.use;
-  const int* ts = c ? tc.tile_start : A.tb.tile_start;
-  int lo = 0, hi = A.m - 1;  // largest a with tile_start[a] <= t
+// largest a with start[a] <= x
+__device__ __forceinline__ int find_attr(const int* start, int m, int x) {
+  int lo = 0, hi = m - 1;
   while (lo < hi) {
     const int mid = (lo + hi + 1) >> 1;
-    if (ts[mid] <= t) lo = mid; else hi = mid - 1;
+    if (start[mid] <= x) lo = mid; else hi = mid - 1;
   }
-  const int a = lo;
-  const long long cs = c ? tc.col_start[a] : A.tb.col_start[a];
-  const long long cl = c ? tc.col_len[a] : A.tb.col_len[a];
-  M.t = t;
-  M.a = a;
-  M.u = t - ts[a];
-  M.colend = cs + cl;
-  M.p0 = cs + (long long)M.u * kTile;
-  M.p1 = min(M.p0 + (long long)kTile, M.colend);
-  M.sb = (long long)a * K;
+  return lo;
 }
 
-// Segment (node) of each of the thread's items; head / piece-end / run-end masks.
+// Range of one chunk (all lanes compute it; the tables are in smem when m is small).
+struct ChunkMeta {
+  long long p0, p1, sb;
+  int a, reset;
+};
+__device__ __forceinline__ ChunkMeta chunk_meta(const TabCache& tc, const TileArgs& A, int K, int c) {
+  const bool u = tc.use;
+  const int* cs = u ? tc.chunk_start : A.tb.chunk_start;
+  const int a = find_attr(cs, A.m, c);
+  const long long c0 = u ? tc.col_start[a] : A.tb.col_start[a];
+  const long long cl = u ? tc.col_len[a] : A.tb.col_len[a];
+  const int k = c - cs[a];
+  ChunkMeta M;
+  M.a = a;
+  M.reset = (k == 0);
+  M.p0 = c0 + (long long)k * kChunk;
+  M.p1 = min(M.p0 + (long long)kChunk, c0 + cl);
+  M.sb = (long long)a * K;
+  return M;
+}
+
+// Segment (node) of each of the thread's items; head / piece-end / run-end masks.  ss/sc are the
+// attribute's segment starts/counts; p1 bounds the piece (chunk end).
 template <bool kNeedVal>
-__device__ __forceinline__ void assign_segments(const long long* ss, const long long* sc, long long p1, int K, long long base,
-                                                unsigned vm, const float* v, float vnext, int* sj,
-                                                unsigned& hm, unsigned& pem, unsigned& rem) {
+__device__ __forceinline__ void assign_segments(const long long* ss, const long long* sc, long long p1, int K,
+                                                long long base, unsigned vm, const float* v, float vnext,
+                                                int* sj, unsigned& hm, unsigned& pem, unsigned& rem) {
   hm = pem = rem = 0;
   if (!vm) return;
   int lo = 0, hi = K - 1;
@@ -169,148 +224,85 @@ __device__ __forceinline__ void assign_segments(const long long* ss, const long 
   }
 }
 
-// ---- exact 128-bit fixed point: x -> trunc(x * 2^F).  F is chosen per tree so that every sum of
-// |g| (|h|) over the level fits below 2^125; conversion of a given double is a pure function, and
-// integer addition is associative, so cross-tile carries are bit-identical in any order.
-__device__ __forceinline__ __int128 to_fx(double x, int F) {
-  if (x == 0.0) return 0;
-  const long long b = __double_as_longlong(x);
-  const int e = (int)((b >> 52) & 0x7ff);
-  const unsigned long long mant = (unsigned long long)(b & 0xfffffffffffffll) | (e ? (1ull << 52) : 0ull);
-  const int sh = (e ? e : 1) - 1075 + F;
-  unsigned __int128 v;
-  if (sh >= 0) v = (unsigned __int128)mant << (sh > 74 ? 74 : sh);
-  else v = (sh > -64) ? (unsigned __int128)(mant >> (-sh)) : (unsigned __int128)0;
-  return b < 0 ? -(__int128)v : (__int128)v;
-}
-__device__ __forceinline__ double from_fx(__int128 v, int F) {
-  const bool neg = v < 0;
-  const unsigned __int128 u = neg ? (unsigned __int128)(-v) : (unsigned __int128)v;
-  const double hi = (double)(unsigned long long)(u >> 64), lo = (double)(unsigned long long)u;
-  double r = __dadd_rn(__dmul_rn(hi, 18446744073709551616.0), lo);
-  r = __dmul_rn(r, __longlong_as_double((long long)(1023 - F) << 52));  // exact power of two
-  return neg ? -r : r;
-}
-__device__ __forceinline__ __int128 shfl_xor128(__int128 v, int o) {
-  const unsigned long long lo = __shfl_xor_sync(0xffffffffu, (unsigned long long)v, o);
-  const unsigned long long hi = __shfl_xor_sync(0xffffffffu, (unsigned long long)((unsigned __int128)v >> 64), o);
-  return (__int128)(((unsigned __int128)hi << 64) | lo);
-}
-__device__ __forceinline__ __int128 ld128(const unsigned long long* p) {
-  return (__int128)(((unsigned __int128)__ldcg(p + 1) << 64) | __ldcg(p));
-}
-__device__ __forceinline__ void st128(unsigned long long* p, __int128 v) {
-  p[0] = (unsigned long long)v;
-  p[1] = (unsigned long long)((unsigned __int128)v >> 64);
-}
-
-struct FX {
-  __int128 g, h;
-  int c, f;
-};
-
-__device__ __forceinline__ void fx_publish(unsigned long long* dst, const FX& x) {
-  st128(dst, x.g);
-  st128(dst + 2, x.h);
-  dst[4] = (unsigned long long)(unsigned)x.c | ((unsigned long long)(unsigned)x.f << 32);
-}
-
-
-struct FXV {
-  __int128 g, h;
-  int c, f;
-};
-__device__ __forceinline__ FXV fxv_comb(const FXV& l, const FXV& r) {  // segmented, exact
-  if (r.f) return r;
-  return FXV{l.g + r.g, l.h + r.h, l.c + r.c, l.f};
-}
-__device__ __forceinline__ __int128 shfl_up128(__int128 v, int o) {
-  const unsigned long long lo = __shfl_up_sync(0xffffffffu, (unsigned long long)v, o);
-  const unsigned long long hi = __shfl_up_sync(0xffffffffu, (unsigned long long)((unsigned __int128)v >> 64), o);
-  return (__int128)(((unsigned __int128)hi << 64) | lo);
-}
-__device__ __forceinline__ void fxv_store(unsigned long long* dst, const FXV& x) {
-  st128(dst, x.g);
-  st128(dst + 2, x.h);
-  dst[4] = (unsigned long long)(unsigned)x.c | ((unsigned long long)(unsigned)x.f << 32);
-}
-__device__ __forceinline__ FXV fxv_load(const unsigned long long* src) {
-  const unsigned long long cf = src[4];
-  return FXV{(__int128)(((unsigned __int128)src[1] << 64) | src[0]),
-             (__int128)(((unsigned __int128)src[3] << 64) | src[2]), (int)(unsigned)cf, (int)(cf >> 32)};
-}
-
-template <int HMODE>
-__device__ __forceinline__ double hess_of(double g) {
-  if (HMODE == kHConst2) return 2.0;
-  // logistic, 0/1 labels: y = [g < 0] (g = p - y with p in [0,1]); q = g + y; reading R5b
-  const double q = g < 0.0 ? __dadd_rn(g, 1.0) : g;
-  const double hh = __dmul_rn(q, __dsub_rn(1.0, q));
-  return hh > 1e-16 ? hh : 1e-16;
-}
-
-// ============================================================================ a4: tile aggregates
-// Per tile: gather g (h) of its instances (L2-resident, evict-last), write them as the tile's
-// g-list (h-list), and publish the tile's segmented aggregate (sum since its last segment head,
-// fixed in-tile association) as an exact fixed-point value.
-template <int HMODE>
-__global__ void __launch_bounds__(kThreads, kLiteBlocks) k_tile_agg(SplitArgs A) {
+// ============================================================================ a4: chunk aggregates
+// One warp per chunk: g (h) of its entries -- gathered at the root (L2 evict-last) and laid out as
+// the chunk's g-list, read from the partition-carried g-list below -- and the chunk's segmented
+// aggregate (sum since its last segment head, fixed association) as an exact fixed-point value.
+template <int HMODE, bool kGather>
+__global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
   __shared__ TabCache tc;
-  __shared__ TileMeta sm;
-  __shared__ SVf wtot[kWarps];
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int lane = threadIdx.x & 31;
   const int K = *A.t.Kp;
-  const int T = *A.t.tb.T;
-  if (K == 0 || T == 0) return;
+  const int C = *A.t.tb.C;
+  if (K == 0 || C == 0) return;
   const int Fg = A.fx[0], Fh = A.fx[1];
+  const unsigned long long pol_keep = policy_evict_last();
   tab_load(tc, A.t);
   __syncthreads();
-  for (int t = blockIdx.x; t < T; t += gridDim.x) {
-    if (tid == 0) tile_meta(tc, A.t, K, t, sm);
-    __syncthreads();
-    const long long p1 = sm.p1;
-    const long long base = sm.p0 + (long long)tid * kItems;
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nw) {
+    const ChunkMeta M = chunk_meta(tc, A.t, K, c);
+    const long long p1 = M.p1;
+    const long long base = M.p0 + (long long)lane * kItems;
     unsigned vm = 0;
     double g[kItems], h[kItems];
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) { g[k] = 0.0; h[k] = 0.0; }
     if (base < p1) {
-      const int4 i0 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base));
-      const int4 i1 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base + 4));
-      const int id[kItems] = {i0.x, i0.y, i0.z, i0.w, i1.x, i1.y, i1.z, i1.w};
-#pragma unroll
-      for (int k = 0; k < kItems; ++k) {
-        if (base + k < p1) {
-          vm |= 1u << k;
-          g[k] = __ldg(A.g + id[k]);
-          h[k] = HMODE == kHGather ? __ldg(A.h + id[k]) : hess_of<HMODE>(g[k]);
-        } else {
-          g[k] = 0.0; h[k] = 0.0;
-        }
-      }
-      // lists are padded to 4 entries only: never write past the tile's own entries
-      if (base + kItems <= p1) {
-        double2* go = reinterpret_cast<double2*>(A.glist + base);
-#pragma unroll
-        for (int k = 0; k < kItems / 2; ++k) go[k] = make_double2(g[2 * k], g[2 * k + 1]);
-        if (HMODE == kHGather) {
-          double2* ho = reinterpret_cast<double2*>(A.hlist + base);
-#pragma unroll
-          for (int k = 0; k < kItems / 2; ++k) ho[k] = make_double2(h[2 * k], h[2 * k + 1]);
-        }
-      } else {
+      if (kGather) {
+        const int4 i0 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base));
+        const int4 i1 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base + 4));
+        const int id[kItems] = {i0.x, i0.y, i0.z, i0.w, i1.x, i1.y, i1.z, i1.w};
 #pragma unroll
         for (int k = 0; k < kItems; ++k) {
           if (base + k < p1) {
-            A.glist[base + k] = g[k];
-            if (HMODE == kHGather) A.hlist[base + k] = h[k];
+            vm |= 1u << k;
+            g[k] = ld_keep(A.g + id[k], pol_keep);
+            h[k] = HMODE == kHGather ? ld_keep(A.h + id[k], pol_keep) : hess_of<HMODE>(g[k]);
+          }
+        }
+        if (base + kItems <= p1) {  // lists are padded to 4 entries only: never write past the chunk
+          double2* go = reinterpret_cast<double2*>(A.glist + base);
+#pragma unroll
+          for (int q = 0; q < kItems / 2; ++q) __stcs(go + q, make_double2(g[2 * q], g[2 * q + 1]));
+          if (HMODE == kHGather) {
+            double2* ho = reinterpret_cast<double2*>(A.hlist + base);
+#pragma unroll
+            for (int q = 0; q < kItems / 2; ++q) __stcs(ho + q, make_double2(h[2 * q], h[2 * q + 1]));
+          }
+        } else {
+#pragma unroll
+          for (int k = 0; k < kItems; ++k)
+            if (base + k < p1) {
+              A.glist[base + k] = g[k];
+              if (HMODE == kHGather) A.hlist[base + k] = h[k];
+            }
+        }
+      } else {
+        const double2* gi = reinterpret_cast<const double2*>(A.glist + base);
+        const double2* hi2 = reinterpret_cast<const double2*>(A.hlist + base);
+#pragma unroll
+        for (int q = 0; q < kItems / 2; ++q) {
+          const double2 x = __ldcs(gi + q);
+          g[2 * q] = x.x; g[2 * q + 1] = x.y;
+          if (HMODE == kHGather) { const double2 y = __ldcs(hi2 + q); h[2 * q] = y.x; h[2 * q + 1] = y.y; }
+        }
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+          if (base + k < p1) {
+            vm |= 1u << k;
+            if (HMODE != kHGather) h[k] = hess_of<HMODE>(g[k]);
+          } else {
+            g[k] = 0.0; h[k] = 0.0;
           }
         }
       }
     }
     int sj[kItems];
     unsigned hm, pem, rem;
-    float vdummy[kItems];
-    assign_segments<false>((const long long*)(A.t.tb.seg_start + sm.sb), (const long long*)(A.t.tb.seg_cnt + sm.sb),
-                           p1, K, base, vm, vdummy, 0.f, sj, hm, pem, rem);
+    float vd[kItems];
+    assign_segments<false>((const long long*)(A.t.tb.seg_start + M.sb), (const long long*)(A.t.tb.seg_cnt + M.sb),
+                           p1, K, base, vm, vd, 0.f, sj, hm, pem, rem);
     SVf run = svf_zero();
 #pragma unroll
     for (int k = 0; k < kItems; ++k) {
@@ -318,67 +310,174 @@ __global__ void __launch_bounds__(kThreads, kLiteBlocks) k_tile_agg(SplitArgs A)
       if ((hm >> k) & 1) { run.g = g[k]; run.h = h[k]; run.c = 1; run.f = 1; }
       else { run.g = run.g + g[k]; run.h = run.h + h[k]; run.c += 1; }
     }
-    SVf inc = run;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-      const SVf y = shfl_up(inc, o);
-      if (lane >= o) inc = comb(y, inc);
+      const SVf y = shfl_up(run, o);
+      if (lane >= o) run = comb(y, run);
     }
-    if (lane == 31) wtot[wid] = inc;
-    __syncthreads();
-    if (tid == 0) {
-      SVf agg = svf_zero();
-      for (int w = 0; w < kWarps; ++w) agg = comb(agg, wtot[w]);
-      fxv_store(A.tagg + 5ll * t, FXV{to_fx(agg.g, Fg), to_fx(agg.h, Fh), agg.c, agg.f});
-    }
-    __syncthreads();
+    if (lane == 31)
+      fxv_store(A.cagg + 5ll * c, FXV{to_fx(run.g, Fg), to_fx(run.h, Fh), run.c, run.f}, M.reset);
   }
 }
 
-// One warp per attribute: exact segmented exclusive scan of the tile aggregates -> carry per tile.
-__global__ void __launch_bounds__(256) k_tile_scan(SplitArgs A) {
-  const int K = *A.t.Kp;
-  if (K == 0) return;
+// ============================================================================ exact scans
+// Segmented exclusive scan over chunk elements x_c with head-inside flags f_c and reset-before
+// flags r_c (first chunk of an attribute):
+//   I_c = (f_c | r_c) ? x_c : I_{c-1} + x_c,    E_c = r_c ? 0 : I_{c-1}.
+// Integer arithmetic, so the result does not depend on how the scan is decomposed:
+//   k_scan1: per group of kScanGroup elements, the group's segmented aggregate
+//   k_scan2: one warp, exclusive segmented scan over the group aggregates (in place)
+//   k_scan3: per group, every element's exclusive value from the group's carry
+struct PK {  // packed count element (partition): hi | lo << 32
+  unsigned long long v;
+  int f;
+};
+
+template <bool kFx>
+struct ScanOps;
+template <>
+struct ScanOps<true> {
+  using T = FXV;
+  static constexpr int W = 5;
+  static __device__ T zero() { return FXV{0, 0, 0, 0}; }
+  static __device__ T load(const unsigned long long* a, long long i, int& r) {
+    T x = fxv_load(a + W * i, &r);
+    x.f |= r;
+    return x;
+  }
+  static __device__ T load_plain(const unsigned long long* a, long long i) { return fxv_load(a + W * i); }
+  static __device__ void store(unsigned long long* a, long long i, const T& x) { fxv_store(a + W * i, x, 0); }
+  static __device__ T comb(const T& l, const T& r) { return fxv_comb(l, r); }
+  static __device__ T up(const T& x, int o) {
+    return FXV{shfl_up128(x.g, o), shfl_up128(x.h, o), __shfl_up_sync(0xffffffffu, x.c, o),
+               __shfl_up_sync(0xffffffffu, x.f, o)};
+  }
+  static __device__ T idx(const T& x, int l) {
+    return FXV{shfl_idx128(x.g, l), shfl_idx128(x.h, l), __shfl_sync(0xffffffffu, x.c, l),
+               __shfl_sync(0xffffffffu, x.f, l)};
+  }
+};
+template <>
+struct ScanOps<false> {
+  using T = PK;
+  static constexpr int W = 2;
+  static __device__ T zero() { return PK{0ull, 0}; }
+  static __device__ T load(const unsigned long long* a, long long i, int& r) {
+    r = (int)(a[W * i + 1] & 1);
+    return PK{a[W * i], r};
+  }
+  static __device__ T load_plain(const unsigned long long* a, long long i) {
+    return PK{a[W * i], (int)(a[W * i + 1] & 1)};
+  }
+  static __device__ void store(unsigned long long* a, long long i, const T& x) {
+    a[W * i] = x.v;
+    a[W * i + 1] = (unsigned long long)x.f;
+  }
+  static __device__ T comb(const T& l, const T& r) { return r.f ? r : PK{l.v + r.v, l.f}; }
+  static __device__ T up(const T& x, int o) {
+    return PK{__shfl_up_sync(0xffffffffu, x.v, o), __shfl_up_sync(0xffffffffu, x.f, o)};
+  }
+  static __device__ T idx(const T& x, int l) {
+    return PK{__shfl_sync(0xffffffffu, x.v, l), __shfl_sync(0xffffffffu, x.f, l)};
+  }
+};
+
+template <bool kFx>
+__global__ void __launch_bounds__(kThreads) k_scan1(const int32_t* __restrict__ Cp, const unsigned long long* __restrict__ in,
+                                                   unsigned long long* __restrict__ gagg) {
+  using O = ScanOps<kFx>;
+  using T = typename O::T;
+  constexpr int kPer = kScanGroup / kThreads;
+  __shared__ T wt[kWarps];
+  const int C = *Cp, lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const long long g0 = (long long)blockIdx.x * kScanGroup;
+  if (g0 >= C) return;
+  T run = O::zero();
+  for (int k = 0; k < kPer; ++k) {
+    const long long i = g0 + (long long)threadIdx.x * kPer + k;
+    if (i < C) { int r; run = O::comb(run, O::load(in, i, r)); }
+  }
+  for (int o = 1; o < 32; o <<= 1) {
+    const T y = O::up(run, o);
+    if (lane >= o) run = O::comb(y, run);
+  }
+  if (lane == 31) wt[wid] = run;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    T acc = O::zero();
+    for (int w = 0; w < kWarps; ++w) acc = O::comb(acc, wt[w]);
+    O::store(gagg, blockIdx.x, acc);
+  }
+}
+
+template <bool kFx>
+__global__ void k_scan2(const int32_t* __restrict__ Cp, unsigned long long* __restrict__ gagg) {
+  using O = ScanOps<kFx>;
+  using T = typename O::T;
+  const int C = *Cp;
+  const int G = (C + kScanGroup - 1) / kScanGroup;
   const int lane = threadIdx.x & 31;
-  const int warps = gridDim.x * (blockDim.x >> 5);
-  for (int a = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); a < A.t.m; a += warps) {
-    const int t0 = A.t.tb.tile_start[a], t1 = A.t.tb.tile_start[a + 1];
-    FXV carry{0, 0, 0, 0};
-    for (int base = t0; base < t1; base += 32) {
-      const int t = base + lane;
-      FXV x{0, 0, 0, 0};
-      if (t < t1) x = fxv_load(A.tagg + 5ll * t);
-      FXV inc = x;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        FXV y;
-        y.g = shfl_up128(inc.g, o);
-        y.h = shfl_up128(inc.h, o);
-        y.c = __shfl_up_sync(0xffffffffu, inc.c, o);
-        y.f = __shfl_up_sync(0xffffffffu, inc.f, o);
-        if (lane >= o) inc = fxv_comb(y, inc);
-      }
-      FXV exc;
-      exc.g = shfl_up128(inc.g, 1);
-      exc.h = shfl_up128(inc.h, 1);
-      exc.c = __shfl_up_sync(0xffffffffu, inc.c, 1);
-      exc.f = __shfl_up_sync(0xffffffffu, inc.f, 1);
-      if (lane == 0) exc = FXV{0, 0, 0, 0};
-      const FXV ex = fxv_comb(carry, exc);
-      if (t < t1) fxv_store(A.carry + 5ll * t, ex);
-      FXV last;
-      {
-        const unsigned long long lo = __shfl_sync(0xffffffffu, (unsigned long long)inc.g, 31);
-        const unsigned long long hi = __shfl_sync(0xffffffffu, (unsigned long long)((unsigned __int128)inc.g >> 64), 31);
-        last.g = (__int128)(((unsigned __int128)hi << 64) | lo);
-        const unsigned long long lo2 = __shfl_sync(0xffffffffu, (unsigned long long)inc.h, 31);
-        const unsigned long long hi2 = __shfl_sync(0xffffffffu, (unsigned long long)((unsigned __int128)inc.h >> 64), 31);
-        last.h = (__int128)(((unsigned __int128)hi2 << 64) | lo2);
-        last.c = __shfl_sync(0xffffffffu, inc.c, 31);
-        last.f = __shfl_sync(0xffffffffu, inc.f, 31);
-      }
-      carry = fxv_comb(carry, last);
+  T carry = O::zero();
+  for (int base = 0; base < G; base += 32) {
+    const int i = base + lane;
+    T x = O::zero();
+    if (i < G) x = O::load_plain(gagg, i);
+    T inc = x;
+    for (int o = 1; o < 32; o <<= 1) {
+      const T y = O::up(inc, o);
+      if (lane >= o) inc = O::comb(y, inc);
     }
+    T ex = O::up(inc, 1);
+    if (lane == 0) ex = O::zero();
+    const T e = O::comb(carry, ex);
+    if (i < G) O::store(gagg, i, e);
+    carry = O::comb(carry, O::idx(inc, 31));
+  }
+}
+
+template <bool kFx>
+__global__ void __launch_bounds__(kThreads) k_scan3(const int32_t* __restrict__ Cp, const unsigned long long* __restrict__ in,
+                                                   const unsigned long long* __restrict__ gcar,
+                                                   unsigned long long* __restrict__ out) {
+  using O = ScanOps<kFx>;
+  using T = typename O::T;
+  constexpr int kPer = kScanGroup / kThreads;
+  __shared__ T wt[kWarps];
+  __shared__ T wc[kWarps];
+  const int C = *Cp, lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const long long g0 = (long long)blockIdx.x * kScanGroup;
+  if (g0 >= C) return;
+  T x[kPer];
+  int r[kPer];
+  T run = O::zero();
+#pragma unroll
+  for (int k = 0; k < kPer; ++k) {
+    const long long i = g0 + (long long)threadIdx.x * kPer + k;
+    r[k] = 0;
+    x[k] = O::zero();
+    if (i < C) x[k] = O::load(in, i, r[k]);
+    run = O::comb(run, x[k]);
+  }
+  T inc = run;
+  for (int o = 1; o < 32; o <<= 1) {
+    const T y = O::up(inc, o);
+    if (lane >= o) inc = O::comb(y, inc);
+  }
+  T ex = O::up(inc, 1);
+  if (lane == 0) ex = O::zero();
+  if (lane == 31) wt[wid] = inc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    T acc = O::load_plain(gcar, blockIdx.x);
+    for (int w = 0; w < kWarps; ++w) { wc[w] = acc; acc = O::comb(acc, wt[w]); }
+  }
+  __syncthreads();
+  T prev = O::comb(wc[wid], ex);  // inclusive value before this thread's first element
+#pragma unroll
+  for (int k = 0; k < kPer; ++k) {
+    const long long i = g0 + (long long)threadIdx.x * kPer + k;
+    if (i < C) O::store(out, i, r[k] ? O::zero() : prev);
+    prev = O::comb(prev, x[k]);
   }
 }
 
@@ -386,39 +485,46 @@ __global__ void __launch_bounds__(256) k_tile_scan(SplitArgs A) {
 struct StageMeta {
   long long p0, p1, colend, sb;
   int t, a, u, seg_cached;
-  unsigned long long carry[5];
+  unsigned long long carry[kChunksPerTile * 5];
   long long seg_s[kSegCache];
   long long seg_c[kSegCache];
 };
 
-// lane 0 of warp 0: metadata of tile t and the TMA bulk loads of its lists into a stage; lanes
-// fetch the tile's carry and the attribute's segment table with cp.async.
+// lane 0 of warp 0: metadata of tile t and the TMA bulk loads of its lists into a stage; the
+// lanes fetch the tile's chunk carries and the attribute's segment table with cp.async.
 template <bool kVal, bool kH>
 __device__ __forceinline__ void issue_stage(int lane, int t, int T, int K, const TabCache& tc,
                                             const SplitArgs& A, StageMeta& M, float* sval, double* sg,
                                             double* sh, unsigned long long* bar, unsigned long long pol) {
   if (lane == 0) {
-    TileMeta tm;
-    tm.t = t;
     M.t = t;
     if (t < T) {
-      tile_meta(tc, A.t, K, t, tm);
-      M.a = tm.a; M.u = tm.u; M.p0 = tm.p0; M.p1 = tm.p1; M.colend = tm.colend; M.sb = tm.sb;
+      const bool u = tc.use;
+      const int* ts = u ? tc.tile_start : A.t.tb.tile_start;
+      const int a = find_attr(ts, A.t.m, t);
+      const long long cs = u ? tc.col_start[a] : A.t.tb.col_start[a];
+      const long long cl = u ? tc.col_len[a] : A.t.tb.col_len[a];
+      M.a = a;
+      M.u = t - ts[a];
+      M.colend = cs + cl;
+      M.p0 = cs + (long long)M.u * kTile;
+      M.p1 = min(M.p0 + (long long)kTile, M.colend);
+      M.sb = (long long)a * K;
       M.seg_cached = K <= kSegCache;
-      const long long cs = tc.use ? tc.col_start[tm.a] : A.t.tb.col_start[tm.a];
-      const long long cl = tc.use ? tc.col_len[tm.a] : A.t.tb.col_len[tm.a];
-      const long long r1 = min((tm.p1 + 3) & ~3ll, cs + ((cl + 3) & ~3ll));  // 16-byte granules
-      const uint32_t n = (uint32_t)(r1 - tm.p0);
+      const long long r1 = min((M.p1 + 3) & ~3ll, cs + ((cl + 3) & ~3ll));  // 16-byte granules
+      const uint32_t n = (uint32_t)(r1 - M.p0);
       fence_proxy_async();
       mbar_arrive_expect_tx(bar, (kVal ? 4u * n : 0u) + 8u * n + (kH ? 8u * n : 0u));
-      if (kVal) tma_load_1d(sval, A.t.val + tm.p0, 4u * n, bar, pol);
-      tma_load_1d(sg, A.glist + tm.p0, 8u * n, bar, pol);
-      if (kH) tma_load_1d(sh, A.hlist + tm.p0, 8u * n, bar, pol);
+      if (kVal) tma_load_1d(sval, A.t.val + M.p0, 4u * n, bar, pol);
+      tma_load_1d(sg, A.glist + M.p0, 8u * n, bar, pol);
+      if (kH) tma_load_1d(sh, A.hlist + M.p0, 8u * n, bar, pol);
     }
   }
   __syncwarp();
   if (t < T) {
-    if (lane < 5) cp_async8(&M.carry[lane], A.carry + 5ll * t + lane, pol);
+    const int nch = (int)((M.p1 - M.p0 + kChunk - 1) / kChunk);
+    const int c0 = (tc.use ? tc.chunk_start[M.a] : A.t.tb.chunk_start[M.a]) + M.u * kChunksPerTile;
+    for (int q = lane; q < nch * 5; q += 32) cp_async8(&M.carry[q], A.carry + 5ll * c0 + q, pol);
     if (K <= kSegCache) {
       const long long sb = M.sb;
       for (int j = lane; j < K; j += 32) {
@@ -435,9 +541,7 @@ struct SFSmem {
   StageMeta meta[kStages];
   unsigned long long bar[kStages];
   int npw;
-  SVf wtot[kWarps], wcar[kWarps];
-  AM mtot[kWarps], mcar[kWarps];
-  unsigned char win[kTile];
+  unsigned char flg[kTile];  // general path: per-item candidate flags of the current tile
   unsigned long long cg[kCtaK], ct[kCtaK];
   Rec cb[kCtaK];
   Rec pw[kPieceList];
@@ -455,6 +559,18 @@ __device__ __forceinline__ void cta_merge(SFSmem& S) {
   S.npw = 0;
 }
 
+__device__ __forceinline__ void push_record(SFSmem& S, const SplitArgs& A, const Rec& r, bool cta_table) {
+  int slot = kPieceList;
+  if (cta_table) slot = atomicAdd(&S.npw, 1);
+  if (slot < kPieceList) {
+    S.pw[slot] = r;
+  } else {
+    const int gs = atomicAdd(A.nrec, 1);
+    A.rec[gs] = r;
+    atomicMax(A.gkey + r.node, gain_key(r.gain));
+  }
+}
+
 template <int HMODE, bool kMissing, bool kTotals>
 __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -469,8 +585,9 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
   const int epoch = *A.epochp;
   const int Fg = A.fx[0], Fh = A.fx[1];
   const bool cta_table = !kTotals && K <= kCtaK;
+  const double lam = A.lam;
   const unsigned long long pol_stream = policy_evict_first();
-  // static round-robin tiles (no inter-CTA dependencies: carries come from k_tile_scan)
+  // static round-robin tiles: there are no inter-CTA dependencies (carries come from the scans)
   auto tile_of = [&](int i) { return (int)blockIdx.x + i * (int)gridDim.x; };
   if (tid == 0) {
     for (int s = 0; s < kStages; ++s) mbar_init(&S.bar[s], 1);
@@ -478,7 +595,6 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
     S.npw = 0;
   }
   tab_load(S.tc, A.t);
-  for (int i = tid; i < kTile; i += kThreads) S.win[i] = 0;
   for (int j = tid; j < kCtaK; j += kThreads) { S.cg[j] = 0ull; S.ct[j] = ~0ull; }
   __syncthreads();
   auto issue = [&](int i) {
@@ -494,7 +610,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
   for (int it = 0;; ++it) {
     const int s0 = it % kStages;
     issue(it + 2);
-    cp_async_wait<2>();                   // this tile's carry / segment table (cp.async)
+    cp_async_wait<2>();  // this tile's carries / segment table (cp.async)
     __syncthreads();
     if (tid == 0 && S.npw) cta_merge(S);
     const StageMeta& M = S.meta[s0];
@@ -502,199 +618,258 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
     if (t >= T) break;
     mbar_wait(&S.bar[s0], (uint32_t)((it / kStages) & 1));  // this tile's lists (TMA)
 
-    const long long p0 = M.p0, p1 = M.p1;
-    const int ibase = tid * kItems;
-    const long long base = p0 + ibase;
-    // ---------------------------------------------------------------- items from shared memory
-    float v[kItems];
-    double g[kItems], h[kItems];
-    int c[kItems];
-    unsigned vm = 0;
-    float vnext = 0.f;
+    // ---------------------------------------------------------------- this warp's chunk
+    const int ibase = tid * kItems;  // position in the tile
+    const long long base = M.p0 + ibase;
+    const long long cp0 = M.p0 + (long long)wid * kChunk;
+    const long long cp1 = min(cp0 + (long long)kChunk, M.p1);
+    if (cp0 < M.p1) {
+      float v[kItems];
+      double g[kItems], h[kItems];
+      int c[kItems];
+      unsigned vm = 0;
+      float vnext = 0.f;
 #pragma unroll
-    for (int k = 0; k < kItems; ++k)
-      if (base + k < p1) vm |= 1u << k;
-    if (!kTotals) {
-      const float4 v0 = *reinterpret_cast<const float4*>(&S.val[s0][ibase]);
-      const float4 v1 = *reinterpret_cast<const float4*>(&S.val[s0][ibase + 4]);
-      v[0] = v0.x; v[1] = v0.y; v[2] = v0.z; v[3] = v0.w;
-      v[4] = v1.x; v[5] = v1.y; v[6] = v1.z; v[7] = v1.w;
-      if (base + kItems < p1) vnext = S.val[s0][ibase + kItems];
-      else if (base + kItems < M.colend && base + kItems == p1) vnext = __ldg(A.t.val + p1);
-    } else {
-#pragma unroll
-      for (int k = 0; k < kItems; ++k) v[k] = 0.f;
-    }
-#pragma unroll
-    for (int k = 0; k < kItems; ++k) {
-      if ((vm >> k) & 1) {
-        g[k] = S.g[s0][ibase + k];
-        h[k] = kH ? sH[(size_t)s0 * kTile + ibase + k] : hess_of<HMODE>(g[k]);
+      for (int k = 0; k < kItems; ++k)
+        if (base + k < cp1) vm |= 1u << k;
+      if (!kTotals) {
+        const float4 v0 = *reinterpret_cast<const float4*>(&S.val[s0][ibase]);
+        const float4 v1 = *reinterpret_cast<const float4*>(&S.val[s0][ibase + 4]);
+        v[0] = v0.x; v[1] = v0.y; v[2] = v0.z; v[3] = v0.w;
+        v[4] = v1.x; v[5] = v1.y; v[6] = v1.z; v[7] = v1.w;
+        if (base + kItems < M.p1) vnext = S.val[s0][ibase + kItems];
+        else if (base + kItems < M.colend && base + kItems == M.p1) vnext = __ldg(A.t.val + M.p1);
       } else {
-        g[k] = 0.0; h[k] = 0.0;
-      }
-    }
-    int sj[kItems];
-    unsigned hm, pem, rem;
-    {
-      const long long* ss = M.seg_cached ? M.seg_s : (const long long*)(A.t.tb.seg_start + M.sb);
-      const long long* sc = M.seg_cached ? M.seg_c : (const long long*)(A.t.tb.seg_cnt + M.sb);
-      assign_segments<!kTotals>(ss, sc, p1, K, base, vm, v, vnext, sj, hm, pem, rem);
-    }
-
-    // ---------------------------------------------------------------- segmented scan
-    SVf run = svf_zero();
 #pragma unroll
-    for (int k = 0; k < kItems; ++k) {
-      if ((vm >> k) & 1) {
-        if ((hm >> k) & 1) { run.g = g[k]; run.h = h[k]; run.c = 1; run.f = 1; }
-        else { run.g = run.g + g[k]; run.h = run.h + h[k]; run.c += 1; }
+        for (int k = 0; k < kItems; ++k) v[k] = 0.f;
       }
-      g[k] = run.g; h[k] = run.h; c[k] = run.c;
-    }
-    SVf inc = run;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const SVf y = shfl_up(inc, o);
-      if (lane >= o) inc = comb(y, inc);
-    }
-    SVf exc = shfl_up(inc, 1);
-    if (lane == 0) exc = svf_zero();
-    if (lane == 31) S.wtot[wid] = inc;
-    __syncthreads();
-    if (tid == 0) {
-      // carry into the tile (exact fixed point from k_tile_scan), then the fixed-order fold of
-      // the warp totals
-      const FXV cx = fxv_load(M.carry);
-      SVf acc = SVf{from_fx(cx.g, Fg), from_fx(cx.h, Fh), cx.c, 0};
-      for (int w = 0; w < kWarps; ++w) { S.wcar[w] = acc; acc = comb(acc, S.wtot[w]); }
-    }
-    __syncthreads();
-    {
-      const SVf car = comb(S.wcar[wid], exc);
 #pragma unroll
       for (int k = 0; k < kItems; ++k) {
-        const bool head_before = (hm & ((2u << k) - 1u)) != 0u;
-        if (!head_before) { g[k] = car.g + g[k]; h[k] = car.h + h[k]; c[k] = car.c + c[k]; }
-      }
-    }
-
-    if (kTotals) {
-#pragma unroll
-      for (int k = 0; k < kItems; ++k) {
-        if (((vm & rem) >> k) & 1) {
-          const long long s = M.sb + sj[k];
-          A.segPG_out[s] = g[k];
-          A.segPH_out[s] = h[k];
+        if ((vm >> k) & 1) {
+          g[k] = S.g[s0][ibase + k];
+          h[k] = kH ? sH[(size_t)s0 * kTile + ibase + k] : hess_of<HMODE>(g[k]);
+        } else {
+          g[k] = 0.0; h[k] = 0.0;
         }
       }
-      __syncthreads();
-      continue;
-    }
+      const FXV cx = fxv_load(M.carry + 5 * wid);
+      const SVf carry = SVf{from_fx(cx.g, Fg), from_fx(cx.h, Fh), cx.c, 0};
+      const long long* ss = M.seg_cached ? M.seg_s : (const long long*)(A.t.tb.seg_start + M.sb);
+      const long long* sc = M.seg_cached ? M.seg_c : (const long long*)(A.t.tb.seg_cnt + M.sb);
 
-    // ---------------------------------------------------------------- Eq. 2 at run ends
-    double gn[kItems];
-    unsigned dm = 0, okm = 0;
+      // ============================================================ fast path: the chunk lies
+      // inside ONE segment and no value is missing -> plain scans, candidates ranked with one
+      // Newton reciprocal, warp argmax, exact Eq. 2 only for the chunk's winner.
+      bool done = false;
+      if (!kTotals && !kMissing && M.seg_cached) {
+        int j0, j1;
+        {
+          int lo = 0, hi = K - 1;
+          while (lo < hi) { const int mid = (lo + hi + 1) >> 1; if (ss[mid] <= cp0) lo = mid; else hi = mid - 1; }
+          j0 = lo;
+          hi = K - 1;
+          while (lo < hi) { const int mid = (lo + hi + 1) >> 1; if (ss[mid] <= cp1 - 1) lo = mid; else hi = mid - 1; }
+          j1 = lo;
+        }
+        if (j0 == j1) {  // warp-uniform
+          done = true;
+          const int j = j0;
+          const long long se = ss[j] + sc[j];
+          const bool head0 = (cp0 == ss[j]);
+          double lg = 0.0, lh = 0.0;
+          int lc = 0;
 #pragma unroll
-    for (int k = 0; k < kItems; ++k) {
-      gn[k] = 0.0;
-      if (!(((vm & rem) >> k) & 1)) continue;
-      const int j = sj[k];
-      const double Gt = A.nodes.G[j], Ht = A.nodes.H[j], pt = A.nodes.pterm[j];
-      const int Ct = A.nodes.cnt[j];
-      const int cL = c[k];
-      bool ok = false;
-      double best = 0.0;
-      int bd = 0;
-      if (cL >= 1 && Ct - cL >= 1) { best = eq2_gain(g[k], h[k], Gt, Ht, A.lam, pt); ok = true; }
-      if (kMissing) {
-        const long long s = M.sb + j;
-        const int cM = Ct - (int)A.t.tb.seg_cnt[s];
-        if (cM > 0) {
-          const double GM = Gt - A.segPG[s], HM = Ht - A.segPH[s];
-          const int cL1 = cL + cM;
-          if (cL1 >= 1 && Ct - cL1 >= 1) {
-            const double g1 = eq2_gain(g[k] + GM, h[k] + HM, Gt, Ht, A.lam, pt);
-            if (!ok || g1 > best) { best = g1; bd = 1; ok = true; }
+          for (int k = 0; k < kItems; ++k) {
+            lg = lg + g[k]; lh = lh + h[k]; lc += (vm >> k) & 1;  // invalid items are 0
+            g[k] = lg; h[k] = lh; c[k] = lc;
+          }
+          double wg = lg, wh = lh;
+          int wcn = lc;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const double yg = __shfl_up_sync(0xffffffffu, wg, o), yh = __shfl_up_sync(0xffffffffu, wh, o);
+            const int yc = __shfl_up_sync(0xffffffffu, wcn, o);
+            if (lane >= o) { wg = yg + wg; wh = yh + wh; wcn += yc; }
+          }
+          double eg = __shfl_up_sync(0xffffffffu, wg, 1), eh = __shfl_up_sync(0xffffffffu, wh, 1);
+          int ec = __shfl_up_sync(0xffffffffu, wcn, 1);
+          if (lane == 0) { eg = 0.0; eh = 0.0; ec = 0; }
+          const double bg = (head0 ? 0.0 : carry.g) + eg, bh = (head0 ? 0.0 : carry.h) + eh;
+          const int bc = (head0 ? 0 : carry.c) + ec;
+          const double Gt = A.nodes.G[j], Ht = A.nodes.H[j];
+          const int Ct = A.nodes.cnt[j];
+          double best = -INFINITY;
+          int bk = -1;
+#pragma unroll
+          for (int k = 0; k < kItems; ++k) {
+            const long long p = base + k;
+            const float nv = (k < kItems - 1) ? v[k + 1] : vnext;
+            const bool cand = ((vm >> k) & 1) && (p + 1 == se || nv != v[k]);
+            const int cL = bc + c[k];
+            if (cand && cL >= 1 && Ct - cL >= 1) {
+              const double GL = bg + g[k], HL = bh + h[k];
+              const double dl = HL + lam, dr = (Ht - HL) + lam, GR = Gt - GL;
+              const double sc2 = __dmul_rn(__fma_rn(GL * GL, dr, __dmul_rn(GR * GR, dl)), rcp_nr(__dmul_rn(dl, dr)));
+              if (sc2 > best) { best = sc2; bk = k; }
+            }
+          }
+          int bpos = bk >= 0 ? ibase + bk : INT_MAX;
+#pragma unroll
+          for (int o = 16; o; o >>= 1) {
+            const double ob = __shfl_xor_sync(0xffffffffu, best, o);
+            const int op = __shfl_xor_sync(0xffffffffu, bpos, o);
+            if (ob > best || (ob == best && op < bpos)) { best = ob; bpos = op; }
+          }
+          if (bpos != INT_MAX && bpos / kItems == tid) {
+            const int k = bpos % kItems;
+            Rec r;
+            r.GL = bg + g[k];
+            r.HL = bh + h[k];
+            r.cntL = bc + c[k];
+            r.gain = eq2_gain(r.GL, r.HL, Gt, Ht, lam, A.nodes.pterm[j]);
+            r.value = v[k];
+            r.attr = A.t.a_base + M.a;
+            r.dir = 0;
+            r.node = j;
+            r.epoch = epoch;
+            r.shard = A.shard;
+            r.pos = base + k;
+            push_record(S, A, r, cta_table);
           }
         }
       }
-      gn[k] = best;
-      dm |= (unsigned)bd << k;
-      okm |= (unsigned)ok << k;
-    }
 
-    // ---------------------------------------------------------------- per-piece argmax scan
-    AM mrun = am_none();
+      if (!done) {
+        // ============================================================ general path (per warp)
+        int sj[kItems];
+        unsigned hm, pem, rem;
+        assign_segments<!kTotals>(ss, sc, cp1, K, base, vm, v, vnext, sj, hm, pem, rem);
+        SVf run = svf_zero();
 #pragma unroll
-    for (int k = 0; k < kItems; ++k) {
-      if (!((vm >> k) & 1)) continue;
-      AM x;
-      x.gain = gn[k]; x.value = v[k];
-      x.meta = (ibase + k) | (int)(((dm >> k) & 1) << 12) | (int)(((okm >> k) & 1) << 13);
-      x.f = ((hm >> k) & 1) || (tid == 0 && k == 0);
-      mrun = am_comb(mrun, x);
-    }
-    AM minc = mrun;
+        for (int k = 0; k < kItems; ++k) {
+          if ((vm >> k) & 1) {
+            if ((hm >> k) & 1) { run.g = g[k]; run.h = h[k]; run.c = 1; run.f = 1; }
+            else { run.g = run.g + g[k]; run.h = run.h + h[k]; run.c += 1; }
+          }
+          g[k] = run.g; h[k] = run.h; c[k] = run.c;
+        }
+        SVf inc = run;
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const AM y = shfl_up(minc, o);
-      if (lane >= o) minc = am_comb(y, minc);
-    }
-    AM mexc = shfl_up(minc, 1);
-    if (lane == 0) mexc = am_none();
-    if (lane == 31) S.mtot[wid] = minc;
-    __syncthreads();
-    if (tid == 0) {
-      AM acc = am_none();
-      for (int w = 0; w < kWarps; ++w) { S.mcar[w] = acc; acc = am_comb(acc, S.mtot[w]); }
-    }
-    __syncthreads();
-    {
-      AM r = am_comb(S.mcar[wid], mexc);
+        for (int o = 1; o < 32; o <<= 1) {
+          const SVf y = shfl_up(inc, o);
+          if (lane >= o) inc = comb(y, inc);
+        }
+        SVf exc = shfl_up(inc, 1);
+        if (lane == 0) exc = svf_zero();
+        {
+          const SVf car = comb(carry, exc);
 #pragma unroll
-      for (int k = 0; k < kItems; ++k) {
-        if (!((vm >> k) & 1)) continue;
-        AM x;
-        x.gain = gn[k]; x.value = v[k];
-        x.meta = (ibase + k) | (int)(((dm >> k) & 1) << 12) | (int)(((okm >> k) & 1) << 13);
-        x.f = ((hm >> k) & 1) || (tid == 0 && k == 0);
-        r = am_comb(r, x);
-        if (((pem >> k) & 1) && am_valid(r)) S.win[r.meta & 0xfff] = 1;
-      }
-    }
-    __syncthreads();
+          for (int k = 0; k < kItems; ++k) {
+            const bool head_before = (hm & ((2u << k) - 1u)) != 0u;
+            if (!head_before) { g[k] = car.g + g[k]; h[k] = car.h + h[k]; c[k] = car.c + c[k]; }
+          }
+        }
+        if (kTotals) {
 #pragma unroll
-    for (int k = 0; k < kItems; ++k) {
-      if (!((vm >> k) & 1) || !S.win[ibase + k]) continue;
-      S.win[ibase + k] = 0;
-      const int j = sj[k];
-      const long long s = M.sb + j;
-      Rec r;
-      r.gain = gn[k];
-      r.value = v[k];
-      r.attr = A.t.a_base + M.a;
-      r.dir = (dm >> k) & 1;
-      r.node = j;
-      r.epoch = epoch;
-      r.shard = A.shard;
-      r.pos = base + k;
-      if (r.dir) {
-        const int cM = A.nodes.cnt[j] - (int)A.t.tb.seg_cnt[s];
-        r.GL = g[k] + (A.nodes.G[j] - A.segPG[s]);
-        r.HL = h[k] + (A.nodes.H[j] - A.segPH[s]);
-        r.cntL = c[k] + cM;
-      } else {
-        r.GL = g[k]; r.HL = h[k]; r.cntL = c[k];
-      }
-      int slot = kPieceList;
-      if (cta_table) slot = atomicAdd(&S.npw, 1);
-      if (slot < kPieceList) {
-        S.pw[slot] = r;
-      } else {
-        const int gs = atomicAdd(A.nrec, 1);
-        A.rec[gs] = r;
-        atomicMax(A.gkey + j, gain_key(r.gain));
+          for (int k = 0; k < kItems; ++k) {
+            if (((vm & rem) >> k) & 1) {
+              const long long s = M.sb + sj[k];
+              A.segPG_out[s] = g[k];
+              A.segPH_out[s] = h[k];
+            }
+          }
+        } else {
+          // Eq. 2 at run ends (both missing directions when the segment has missing values)
+          double gn[kItems];
+          unsigned dm = 0, okm = 0;
+#pragma unroll
+          for (int k = 0; k < kItems; ++k) {
+            gn[k] = 0.0;
+            if (!(((vm & rem) >> k) & 1)) continue;
+            const int j = sj[k];
+            const double Gt = A.nodes.G[j], Ht = A.nodes.H[j], pt = A.nodes.pterm[j];
+            const int Ct = A.nodes.cnt[j];
+            const int cL = c[k];
+            bool ok = false;
+            double best = 0.0;
+            int bd = 0;
+            if (cL >= 1 && Ct - cL >= 1) { best = eq2_gain(g[k], h[k], Gt, Ht, lam, pt); ok = true; }
+            if (kMissing) {
+              const long long s = M.sb + j;
+              const int cM = Ct - (int)A.t.tb.seg_cnt[s];
+              if (cM > 0) {
+                const double GM = Gt - A.segPG[s], HM = Ht - A.segPH[s];
+                const int cL1 = cL + cM;
+                if (cL1 >= 1 && Ct - cL1 >= 1) {
+                  const double g1 = eq2_gain(g[k] + GM, h[k] + HM, Gt, Ht, lam, pt);
+                  if (!ok || g1 > best) { best = g1; bd = 1; ok = true; }
+                }
+              }
+            }
+            gn[k] = best;
+            dm |= (unsigned)bd << k;
+            okm |= (unsigned)ok << k;
+          }
+          // per-piece argmax inside the chunk (pieces = segments of the chunk): the item that ends
+          // a piece walks back to the piece start; R12 order gain desc, value desc, dir low first.
+          // The chunk's g slots of the stage are free now and hold the gains.
+          double* sgn = &S.g[s0][wid * kChunk];
+          const float* svv = &S.val[s0][wid * kChunk];
+          unsigned char* sfl = &S.flg[wid * kChunk];
+          __syncwarp();
+#pragma unroll
+          for (int k = 0; k < kItems; ++k) {
+            sgn[lane * kItems + k] = gn[k];
+            sfl[lane * kItems + k] = (unsigned char)(((okm >> k) & 1) | (((dm >> k) & 1) << 1) |
+                                                     (((hm >> k) & 1) << 2));
+          }
+          __syncwarp();
+#pragma unroll
+          for (int k = 0; k < kItems; ++k) {
+            if (!(((vm & pem) >> k) & 1)) continue;
+            int q = lane * kItems + k, bq = -1;
+            for (;;) {
+              const int fl = sfl[q];
+              if (fl & 1) {
+                if (bq < 0) {
+                  bq = q;
+                } else {
+                  const double a = sgn[q], b = sgn[bq];
+                  const float va = svv[q], vb = svv[bq];
+                  if (a > b || (a == b && (va > vb || (va == vb && ((fl >> 1) & 1) < ((sfl[bq] >> 1) & 1))))) bq = q;
+                }
+              }
+              if ((fl & 4) || q == 0) break;
+              --q;
+            }
+            if (bq >= 0) sfl[bq] |= 8;  // each piece marks exactly one item
+          }
+          __syncwarp();
+#pragma unroll
+          for (int k = 0; k < kItems; ++k) {
+            if (!(sfl[lane * kItems + k] & 8)) continue;
+            const int j = sj[k];
+            const long long s = M.sb + j;
+            Rec r;
+            r.gain = gn[k];
+            r.value = v[k];
+            r.attr = A.t.a_base + M.a;
+            r.dir = (dm >> k) & 1;
+            r.node = j;
+            r.epoch = epoch;
+            r.shard = A.shard;
+            r.pos = base + k;
+            if (r.dir) {
+              const int cM = A.nodes.cnt[j] - (int)A.t.tb.seg_cnt[s];
+              r.GL = g[k] + (A.nodes.G[j] - A.segPG[s]);
+              r.HL = h[k] + (A.nodes.H[j] - A.segPH[s]);
+              r.cntL = c[k] + cM;
+            } else {
+              r.GL = g[k]; r.HL = h[k]; r.cntL = c[k];
+            }
+            push_record(S, A, r, cta_table);
+          }
+        }
       }
     }
     __syncthreads();
@@ -715,52 +890,55 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
 }
 
 // ============================================================================ a8: partition
-// Per tile: (high, low) counts; with missing values also the per-segment counts.
-__global__ void __launch_bounds__(kThreads, kLiteBlocks) k_part_count(PartArgs A, int counted) {
+// One warp per chunk: (high, low) entry counts (packed hi | lo << 32) + reset flag; with missing
+// values also the per-segment counts (the plan needs them).
+__global__ void __launch_bounds__(kThreads) k_part_count(PartArgs A, int counted) {
   __shared__ TabCache tc;
-  __shared__ TileMeta sm;
-  __shared__ unsigned ws[kWarps];
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int lane = threadIdx.x & 31;
   const int K = *A.t.Kp;
-  const int T = *A.t.tb.T;
-  if (K == 0 || T == 0) return;
+  const int C = *A.t.tb.C;
+  if (K == 0 || C == 0) return;
   tab_load(tc, A.t);
   __syncthreads();
-  for (int t = blockIdx.x; t < T; t += gridDim.x) {
-    if (tid == 0) tile_meta(tc, A.t, K, t, sm);
-    __syncthreads();
-    const long long p1 = sm.p1;
-    const long long base = sm.p0 + (long long)tid * kItems;
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nw) {
+    const ChunkMeta M = chunk_meta(tc, A.t, K, c);
+    const long long base = M.p0 + (long long)lane * kItems;
     unsigned vm = 0, loc = 0;
     uint8_t sd[kItems];
-    if (base < p1) {
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) sd[k] = 0;
+    if (base < M.p1) {
       const int4 i0 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base));
       const int4 i1 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base + 4));
       const int id[kItems] = {i0.x, i0.y, i0.z, i0.w, i1.x, i1.y, i1.z, i1.w};
 #pragma unroll
-      for (int k = 0; k < kItems; ++k) {
-        sd[k] = 0;
-        if (base + k < p1) { vm |= 1u << k; sd[k] = __ldg(A.side + id[k]); }
-        loc += sd[k] == 1 ? 1u : (sd[k] == 2 ? (1u << 16) : 0u);
-      }
-    } else {
+      for (int k = 0; k < kItems; ++k)
+        if (base + k < M.p1) { vm |= 1u << k; sd[k] = __ldg(A.side + id[k]); }
 #pragma unroll
-      for (int k = 0; k < kItems; ++k) sd[k] = 0;
+      for (int k = 0; k < kItems; ++k) loc += sd[k] == 1 ? 1u : (sd[k] == 2 ? (1u << 16) : 0u);
+      // the entry-aligned side-list lets the scatter stream sides instead of gathering again
+      // (4-entry granules: lists are padded to 4 entries, so never write past this list)
+      unsigned w0 = 0, w1 = 0;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) { w0 |= (unsigned)sd[k] << (8 * k); w1 |= (unsigned)sd[k + 4] << (8 * k); }
+      reinterpret_cast<unsigned*>(A.slist + base)[0] = w0;
+      if (base + 4 < M.p1) reinterpret_cast<unsigned*>(A.slist + base)[1] = w1;
     }
     if (counted && vm) {
       int sj[kItems];
       unsigned hm, pem, rem;
       float vd[kItems];
-      assign_segments<false>((const long long*)(A.t.tb.seg_start + sm.sb), (const long long*)(A.t.tb.seg_cnt + sm.sb),
-                             p1, K, base, vm, vd, 0.f, sj, hm, pem, rem);
+      assign_segments<false>((const long long*)(A.t.tb.seg_start + M.sb), (const long long*)(A.t.tb.seg_cnt + M.sb),
+                             M.p1, K, base, vm, vd, 0.f, sj, hm, pem, rem);
       int cur = -1, ch = 0, cl = 0;
 #pragma unroll
       for (int k = 0; k < kItems; ++k) {
         if (!((vm >> k) & 1)) continue;
         if (sj[k] != cur) {
           if (cur >= 0) {
-            if (ch) atomicAdd(A.segH + sm.sb + cur, ch);
-            if (cl) atomicAdd(A.segL + sm.sb + cur, cl);
+            if (ch) atomicAdd(A.segH + M.sb + cur, ch);
+            if (cl) atomicAdd(A.segL + M.sb + cur, cl);
           }
           cur = sj[k]; ch = cl = 0;
         }
@@ -768,44 +946,15 @@ __global__ void __launch_bounds__(kThreads, kLiteBlocks) k_part_count(PartArgs A
         cl += sd[k] == 2;
       }
       if (cur >= 0) {
-        if (ch) atomicAdd(A.segH + sm.sb + cur, ch);
-        if (cl) atomicAdd(A.segL + sm.sb + cur, cl);
+        if (ch) atomicAdd(A.segH + M.sb + cur, ch);
+        if (cl) atomicAdd(A.segL + M.sb + cur, cl);
       }
     }
 #pragma unroll
     for (int o = 16; o; o >>= 1) loc += __shfl_xor_sync(0xffffffffu, loc, o);
-    if (lane == 0) ws[wid] = loc;
-    __syncthreads();
-    if (tid == 0) {
-      unsigned x = 0;
-      for (int w = 0; w < kWarps; ++w) x += ws[w];
-      A.tcnt[t] = x;
-    }
-    __syncthreads();
-  }
-}
-
-// One warp per attribute: exclusive scan of the tile counts within the attribute list.
-__global__ void __launch_bounds__(256) k_part_tscan(PartArgs A) {
-  const int K = *A.t.Kp;
-  if (K == 0) return;
-  const int lane = threadIdx.x & 31;
-  const int warps = gridDim.x * (blockDim.x >> 5);
-  for (int a = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); a < A.t.m; a += warps) {
-    const int t0 = A.t.tb.tile_start[a], t1 = A.t.tb.tile_start[a + 1];
-    unsigned long long carry = 0;
-    for (int base = t0; base < t1; base += 32) {
-      const int t = base + lane;
-      unsigned long long x = 0;
-      if (t < t1) { const unsigned c = A.tcnt[t]; x = (unsigned long long)(c & 0xffffu) | ((unsigned long long)(c >> 16) << 32); }
-      unsigned long long inc = x;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const unsigned long long y = __shfl_up_sync(0xffffffffu, inc, o);
-        if (lane >= o) inc += y;
-      }
-      if (t < t1) A.tpre[t] = carry + inc - x;
-      carry += __shfl_sync(0xffffffffu, inc, 31);
+    if (lane == 0) {
+      A.ccnt[2ll * c] = (unsigned long long)(loc & 0xffffu) | ((unsigned long long)(loc >> 16) << 32);
+      A.ccnt[2ll * c + 1] = (unsigned long long)M.reset;
     }
   }
 }
@@ -839,7 +988,7 @@ __device__ unsigned long long block_exscan_u64(unsigned long long x, unsigned lo
 }
 
 // Single thread block: places every child segment (stable, attribute-major, children in heap
-// order) and builds the next level's attribute/tile/segment tables.
+// order) and builds the next level's attribute / tile / chunk / segment tables.
 __global__ void __launch_bounds__(1024) k_part_plan(PlanArgs A) {
   const int K = *A.Kp, Kn = *A.Knp, m = A.m;
   if (!A.counted) {
@@ -866,20 +1015,28 @@ __global__ void __launch_bounds__(1024) k_part_plan(PlanArgs A) {
     A.nxt.col_len[a] = L;
   }
   __syncthreads();
-  unsigned long long cpos = 0, ctile = 0, t1, t2;
+  unsigned long long cpos = 0, ctile = 0, cchunk = 0, t1, t2, t3;
   for (int base = 0; base < m; base += blockDim.x) {
     const int a = base + threadIdx.x;
     const unsigned long long L = a < m ? (unsigned long long)A.len_tmp[a] : 0ull;
     const unsigned long long ep = block_exscan_u64((L + 3) & ~3ull, t1);
     const unsigned long long et = block_exscan_u64((L + kTile - 1) / kTile, t2);
-    if (a < m) { A.nxt.col_start[a] = (int64_t)(cpos + ep); A.nxt.tile_start[a] = (int32_t)(ctile + et); }
+    const unsigned long long ec = block_exscan_u64((L + kChunk - 1) / kChunk, t3);
+    if (a < m) {
+      A.nxt.col_start[a] = (int64_t)(cpos + ep);
+      A.nxt.tile_start[a] = (int32_t)(ctile + et);
+      A.nxt.chunk_start[a] = (int32_t)(cchunk + ec);
+    }
     cpos += t1;
     ctile += t2;
+    cchunk += t3;
   }
   if (threadIdx.x == 0) {
     A.nxt.col_start[m] = (int64_t)cpos;
     A.nxt.tile_start[m] = (int32_t)ctile;
+    A.nxt.chunk_start[m] = (int32_t)cchunk;
     *A.nxt.T = (int32_t)ctile;
+    *A.nxt.C = (int32_t)cchunk;
   }
   __syncthreads();
   for (int a = threadIdx.x; a < m; a += blockDim.x) {
@@ -901,47 +1058,70 @@ __global__ void __launch_bounds__(1024) k_part_plan(PlanArgs A) {
   }
 }
 
-// Stable scatter ("Scatter"): out(e) = out_base(seg, side) + rank of e among the
-// segment's same-side entries = C_side(e) - C_side(seg start), C counted within the attribute.
-__global__ void __launch_bounds__(kThreads, kLiteBlocks) k_part_scatter(PartArgs A) {
+// Stable scatter ("Scatter"), one warp per chunk: out(e) = out_base(seg, side) + rank of
+// e among the segment's same-side entries = C_side(e) - C_side(seg start), C counted within the
+// attribute (chunk prefix from the count scan + in-warp exclusive count).  The kept entries are
+// staged in shared memory in destination order (the chunk's high entries, then its low ones) so
+// that the stores go out as coalesced runs; g (h) move along.
+struct ScatterStage {
+  long long dst[kChunk];
+  double g[kChunk];
+  float v[kChunk];
+  int id[kChunk];
+};
+
+template <bool kH>
+__global__ void __launch_bounds__(kThreads) k_part_scatter(PartArgs A) {
   __shared__ TabCache tc;
-  __shared__ TileMeta sm;
-  __shared__ unsigned ws[kWarps];
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  extern __shared__ __align__(16) unsigned char sc_raw[];
+  ScatterStage* stg = reinterpret_cast<ScatterStage*>(sc_raw);
+  double* stgh = reinterpret_cast<double*>(sc_raw + sizeof(ScatterStage) * kWarps);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int K = *A.t.Kp;
-  const int T = *A.t.tb.T;
-  if (K == 0 || T == 0) return;
+  const int C = *A.t.tb.C;
+  if (K == 0 || C == 0) return;
   tab_load(tc, A.t);
   __syncthreads();
-  for (int t = blockIdx.x; t < T; t += gridDim.x) {
-    if (tid == 0) tile_meta(tc, A.t, K, t, sm);
-    __syncthreads();
-    const long long p1 = sm.p1;
-    const long long base = sm.p0 + (long long)tid * kItems;
+  ScatterStage& W = stg[wid];
+  double* Wh = stgh + (size_t)wid * kChunk;
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nw) {
+    const ChunkMeta M = chunk_meta(tc, A.t, K, c);
+    const long long p1 = M.p1;
+    const long long base = M.p0 + (long long)lane * kItems;
     unsigned vm = 0, loc = 0;
     float v[kItems];
     int id[kItems];
+    double g[kItems], h[kItems];
     uint8_t sd[kItems];
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) { sd[k] = 0; v[k] = 0.f; id[k] = 0; g[k] = 0.0; h[k] = 0.0; }
     if (base < p1) {
       const int4 i0 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base));
       const int4 i1 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base + 4));
       const float4 v0 = __ldcs(reinterpret_cast<const float4*>(A.t.val + base));
       const float4 v1 = __ldcs(reinterpret_cast<const float4*>(A.t.val + base + 4));
+      const unsigned long long pk = (unsigned long long)__ldcs(reinterpret_cast<const unsigned*>(A.slist + base)) |
+                                    ((unsigned long long)__ldcs(reinterpret_cast<const unsigned*>(A.slist + base) + 1) << 32);
       id[0] = i0.x; id[1] = i0.y; id[2] = i0.z; id[3] = i0.w; id[4] = i1.x; id[5] = i1.y; id[6] = i1.z; id[7] = i1.w;
       v[0] = v0.x; v[1] = v0.y; v[2] = v0.z; v[3] = v0.w; v[4] = v1.x; v[5] = v1.y; v[6] = v1.z; v[7] = v1.w;
+      const double2* gi = reinterpret_cast<const double2*>(A.g_in + base);
+      const double2* hi2 = reinterpret_cast<const double2*>(A.h_in + base);
+#pragma unroll
+      for (int q = 0; q < kItems / 2; ++q) {
+        const double2 x = __ldcs(gi + q);
+        g[2 * q] = x.x; g[2 * q + 1] = x.y;
+        if (kH) { const double2 y = __ldcs(hi2 + q); h[2 * q] = y.x; h[2 * q + 1] = y.y; }
+      }
 #pragma unroll
       for (int k = 0; k < kItems; ++k) {
-        sd[k] = 0;
-        if (base + k < p1) { vm |= 1u << k; sd[k] = __ldg(A.side + id[k]); }
+        if (base + k < p1) { vm |= 1u << k; sd[k] = (uint8_t)((pk >> (8 * k)) & 0xff); }
         loc += sd[k] == 1 ? 1u : (sd[k] == 2 ? (1u << 16) : 0u);
       }
-    } else {
-#pragma unroll
-      for (int k = 0; k < kItems; ++k) { sd[k] = 0; v[k] = 0.f; id[k] = 0; }
     }
     int sj[kItems];
     unsigned hm, pem, rem;
-    assign_segments<false>((const long long*)(A.t.tb.seg_start + sm.sb), (const long long*)(A.t.tb.seg_cnt + sm.sb),
+    assign_segments<false>((const long long*)(A.t.tb.seg_start + M.sb), (const long long*)(A.t.tb.seg_cnt + M.sb),
                            p1, K, base, vm, v, 0.f, sj, hm, pem, rem);
     unsigned inc = loc;
 #pragma unroll
@@ -949,27 +1129,39 @@ __global__ void __launch_bounds__(kThreads, kLiteBlocks) k_part_scatter(PartArgs
       const unsigned y = __shfl_up_sync(0xffffffffu, inc, o);
       if (lane >= o) inc += y;
     }
-    if (lane == 31) ws[wid] = inc;
-    __syncthreads();
-    unsigned wex = 0;
-    for (int w = 0; w < wid; ++w) wex += ws[w];
-    unsigned ex = wex + inc - loc;
-    const unsigned long long tp = A.tpre[t];
-    const long long chi0 = (long long)(tp & 0xffffffffull), clo0 = (long long)(tp >> 32);
+    const unsigned tot = __shfl_sync(0xffffffffu, inc, 31);
+    const unsigned nhi = tot & 0xffffu, nkeep = nhi + (tot >> 16);
+    unsigned ex = inc - loc;
+    const unsigned long long cpv = A.cpre[2ll * c];
+    const long long chi0 = (long long)(cpv & 0xffffffffull), clo0 = (long long)(cpv >> 32);
+    __syncwarp();
 #pragma unroll
     for (int k = 0; k < kItems; ++k) {
       if (sd[k]) {
-        const long long s = sm.sb + sj[k];
+        const long long s = M.sb + sj[k];
         const unsigned long long sp = A.seg_pre[s];
+        const unsigned rh = ex & 0xffffu, rl = ex >> 16;
         long long dst;
-        if (sd[k] == 1) dst = A.out_hi[s] + (chi0 + (long long)(ex & 0xffffu) - (long long)(sp & 0xffffffffull));
-        else dst = A.out_lo[s] + (clo0 + (long long)(ex >> 16) - (long long)(sp >> 32));
-        A.val_out[dst] = v[k];
-        A.ins_out[dst] = id[k];
+        int slot;
+        if (sd[k] == 1) { dst = A.out_hi[s] + (chi0 + (long long)rh - (long long)(sp & 0xffffffffull)); slot = (int)rh; }
+        else { dst = A.out_lo[s] + (clo0 + (long long)rl - (long long)(sp >> 32)); slot = (int)(nhi + rl); }
+        W.dst[slot] = dst;
+        W.v[slot] = v[k];
+        W.id[slot] = id[k];
+        W.g[slot] = g[k];
+        if (kH) Wh[slot] = h[k];
         ex += sd[k] == 1 ? 1u : (1u << 16);
       }
     }
-    __syncthreads();
+    __syncwarp();
+    for (int i = lane; i < (int)nkeep; i += 32) {
+      const long long d = W.dst[i];
+      A.val_out[d] = W.v[i];
+      A.ins_out[d] = W.id[i];
+      A.g_out[d] = W.g[i];
+      if (kH) A.h_out[d] = Wh[i];
+    }
+    __syncwarp();
   }
 }
 
@@ -982,6 +1174,8 @@ unsigned grid_for(KernelT kern, size_t smem, int sms) {
   return (unsigned)(occ * sms);
 }
 
+size_t scatter_smem(bool h) { return sizeof(ScatterStage) * kWarps + (h ? sizeof(double) * kChunk * kWarps : 0); }
+
 size_t sf_smem(int hmode) {
   size_t b = (sizeof(SFSmem) + 127) & ~size_t(127);
   if (hmode == kHGather) b += sizeof(double) * kStages * kTile;
@@ -992,6 +1186,16 @@ template <int HM>
 void launch_sf(const SplitArgs& A, bool missing, unsigned grid, cudaStream_t st) {
   if (missing) k_sf<HM, true, false><<<grid, kThreads, sf_smem(HM), st>>>(A);
   else k_sf<HM, false, false><<<grid, kThreads, sf_smem(HM), st>>>(A);
+}
+
+template <bool kFx>
+void launch_scan(const int32_t* Cp, unsigned long long* in, unsigned long long* gbuf, unsigned long long* out,
+                 unsigned groups, cudaStream_t st) {
+  k_scan1<kFx><<<groups, kThreads, 0, st>>>(Cp, in, gbuf);
+  k_scan2<kFx><<<1, 32, 0, st>>>(Cp, gbuf);
+  k_scan3<kFx><<<groups, kThreads, 0, st>>>(Cp, in, gbuf, out);
+  GBDT_LAUNCH_CHECK();
+  count_launch(3);
 }
 
 }  // namespace
@@ -1007,22 +1211,34 @@ void LevelKernels::init(int device) {
   grid_tot[0] = grid_for(k_sf<0, true, true>, sf_smem(0), sms);
   grid_tot[1] = grid_for(k_sf<1, true, true>, sf_smem(1), sms);
   grid_tot[2] = grid_for(k_sf<2, true, true>, sf_smem(2), sms);
-  grid_agg[0] = grid_for(k_tile_agg<0>, 0, sms);
-  grid_agg[1] = grid_for(k_tile_agg<1>, 0, sms);
-  grid_agg[2] = grid_for(k_tile_agg<2>, 0, sms);
-  grid_scatter = grid_for(k_part_scatter, 0, sms);
+  grid_agg[0] = grid_for(k_chunk_agg<0, true>, 0, sms);
+  grid_agg[1] = grid_for(k_chunk_agg<1, true>, 0, sms);
+  grid_agg[2] = grid_for(k_chunk_agg<2, true>, 0, sms);
+  grid_agg_list[0] = grid_for(k_chunk_agg<0, false>, 0, sms);
+  grid_agg_list[1] = grid_for(k_chunk_agg<1, false>, 0, sms);
+  grid_agg_list[2] = grid_for(k_chunk_agg<2, false>, 0, sms);
+  grid_scatter[0] = grid_for(k_part_scatter<false>, scatter_smem(false), sms);
+  grid_scatter[1] = grid_for(k_part_scatter<true>, scatter_smem(true), sms);
   grid_count = grid_for(k_part_count, 0, sms);
 }
 
-void LevelKernels::tile_prefix(const SplitArgs& A, int hmode, cudaStream_t st) {
-  if (hmode == 0) k_tile_agg<0><<<grid_agg[0], kThreads, 0, st>>>(A);
-  else if (hmode == 1) k_tile_agg<1><<<grid_agg[1], kThreads, 0, st>>>(A);
-  else k_tile_agg<2><<<grid_agg[2], kThreads, 0, st>>>(A);
+unsigned LevelKernels::scan_groups(int64_t max_chunks) {
+  return (unsigned)std::max<int64_t>(1, (max_chunks + kScanGroup - 1) / kScanGroup);
+}
+
+void LevelKernels::tile_prefix(const SplitArgs& A, int hmode, bool gather, unsigned groups, cudaStream_t st) {
+  if (gather) {
+    if (hmode == 0) k_chunk_agg<0, true><<<grid_agg[0], kThreads, 0, st>>>(A);
+    else if (hmode == 1) k_chunk_agg<1, true><<<grid_agg[1], kThreads, 0, st>>>(A);
+    else k_chunk_agg<2, true><<<grid_agg[2], kThreads, 0, st>>>(A);
+  } else {
+    if (hmode == 0) k_chunk_agg<0, false><<<grid_agg_list[0], kThreads, 0, st>>>(A);
+    else if (hmode == 1) k_chunk_agg<1, false><<<grid_agg_list[1], kThreads, 0, st>>>(A);
+    else k_chunk_agg<2, false><<<grid_agg_list[2], kThreads, 0, st>>>(A);
+  }
   GBDT_LAUNCH_CHECK();
-  const unsigned g = (unsigned)std::max(1, std::min(A.t.m, sms * 64) / 8 + 1);
-  k_tile_scan<<<g, 256, 0, st>>>(A);
-  GBDT_LAUNCH_CHECK();
-  count_launch(2);
+  count_launch();
+  launch_scan<true>(A.t.tb.C, A.cagg, A.sgrp, A.carry, groups, st);
 }
 
 void LevelKernels::split_find(const SplitArgs& A, int hmode, bool missing, cudaStream_t st) {
@@ -1041,17 +1257,18 @@ void LevelKernels::seg_totals(const SplitArgs& A, int hmode, cudaStream_t st) {
   count_launch();
 }
 
-void LevelKernels::partition(const PartArgs& A, const PlanArgs& P, bool counted, cudaStream_t st) {
+void LevelKernels::partition(const PartArgs& A, const PlanArgs& P, bool counted, bool with_h, unsigned groups,
+                             cudaStream_t st) {
   k_part_count<<<grid_count, kThreads, 0, st>>>(A, counted ? 1 : 0);
   GBDT_LAUNCH_CHECK();
-  const unsigned g = (unsigned)std::max(1, std::min(A.t.m, sms * 64) / 8 + 1);
-  k_part_tscan<<<g, 256, 0, st>>>(A);
-  GBDT_LAUNCH_CHECK();
+  count_launch();
+  launch_scan<false>(A.t.tb.C, A.ccnt, A.sgrp, A.cpre, groups, st);
   k_part_plan<<<1, 1024, 0, st>>>(P);
   GBDT_LAUNCH_CHECK();
-  k_part_scatter<<<grid_scatter, kThreads, 0, st>>>(A);
+  if (with_h) k_part_scatter<true><<<grid_scatter[1], kThreads, scatter_smem(true), st>>>(A);
+  else k_part_scatter<false><<<grid_scatter[0], kThreads, scatter_smem(false), st>>>(A);
   GBDT_LAUNCH_CHECK();
-  count_launch(4);
+  count_launch(2);
 }
 
 }  // namespace gbdt

@@ -342,11 +342,14 @@ struct Carve {
 struct ShardWork {
   DBuf mem;
   Tables tab[2];
-  DBuf lists;                 // g-list (+ h-list) of the level, entry-aligned with val/ins
-  double *glist, *hlist;
-  unsigned long long *tagg, *carry;   // [T0][5]
-  uint32_t* tcnt;
-  unsigned long long* tpre;
+  DBuf lists;                 // g-lists (+ h-lists) of two levels, entry-aligned with val/ins
+  double *glist[2], *hlist[2];
+  uint8_t* slist;
+  unsigned long long *cagg, *carry;   // [C0][5]
+  unsigned long long *ccnt, *cpre;    // [C0][2]
+  unsigned long long* sgrp;           // scan scratch
+  unsigned groups;
+  LookBack lb;                        // partition look-back
   Rec* rec;
   int* nrec;
   unsigned long long *gkey, *tkey;
@@ -470,13 +473,17 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     const int m = sh.m;
     const int64_t S = (int64_t)m * Kcap;
     const int64_t T0 = std::max(sh.T0, 1);
+    const int64_t C0 = std::max(sh.C0, 1);
     const int64_t R = (int64_t)LK.grid_sf[2][1] * 64 + T0 + S;  // node-best records per level
     auto sz = [&](Carve& q) {
       for (int b = 0; b < 2; ++b) {
-        q.take<int64_t>(m + 1); q.take<int64_t>(m); q.take<int32_t>(m + 1); q.take<int64_t>(S); q.take<int64_t>(S); q.take<int32_t>(1);
+        q.take<int64_t>(m + 1); q.take<int64_t>(m); q.take<int32_t>(m + 1); q.take<int32_t>(m + 1);
+        q.take<int64_t>(S); q.take<int64_t>(S); q.take<int32_t>(1); q.take<int32_t>(1);
       }
-      q.take<unsigned long long>(5 * T0); q.take<unsigned long long>(5 * T0);
-      q.take<uint32_t>(T0); q.take<unsigned long long>(T0);
+      q.take<unsigned long long>(5 * C0); q.take<unsigned long long>(5 * C0);
+      q.take<unsigned long long>(2 * C0); q.take<unsigned long long>(2 * C0);
+      q.take<unsigned long long>(5 * (size_t)LevelKernels::scan_groups(C0) + 8);
+      q.take<int32_t>(T0); q.take<unsigned long long>(T0); q.take<unsigned long long>(T0);
       q.take<Rec>(R);
       q.take<int32_t>(S); q.take<int32_t>(S); q.take<unsigned long long>(S); q.take<int64_t>(S); q.take<int64_t>(S);
       q.take<int64_t>(m); q.take<double>(S); q.take<double>(S); q.take<int>(4);
@@ -488,14 +495,22 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     Carve q{w.mem.as<char>()};
     for (int b = 0; b < 2; ++b) {
       w.tab[b].col_start = q.take<int64_t>(m + 1); w.tab[b].col_len = q.take<int64_t>(m);
-      w.tab[b].tile_start = q.take<int32_t>(m + 1); w.tab[b].seg_start = q.take<int64_t>(S);
-      w.tab[b].seg_cnt = q.take<int64_t>(S); w.tab[b].T = q.take<int32_t>(1);
+      w.tab[b].tile_start = q.take<int32_t>(m + 1); w.tab[b].chunk_start = q.take<int32_t>(m + 1);
+      w.tab[b].seg_start = q.take<int64_t>(S); w.tab[b].seg_cnt = q.take<int64_t>(S);
+      w.tab[b].T = q.take<int32_t>(1); w.tab[b].C = q.take<int32_t>(1);
     }
-    w.tagg = q.take<unsigned long long>(5 * T0); w.carry = q.take<unsigned long long>(5 * T0);
-    w.tcnt = q.take<uint32_t>(T0); w.tpre = q.take<unsigned long long>(T0);
-    w.lists.alloc((size_t)sh.cap * 8 * (hmode == kHGather ? 2 : 1), st);
-    w.glist = w.lists.as<double>();
-    w.hlist = hmode == kHGather ? w.glist + sh.cap : nullptr;
+    w.cagg = q.take<unsigned long long>(5 * C0); w.carry = q.take<unsigned long long>(5 * C0);
+    w.ccnt = q.take<unsigned long long>(2 * C0); w.cpre = q.take<unsigned long long>(2 * C0);
+    w.groups = LevelKernels::scan_groups(C0);
+    w.sgrp = q.take<unsigned long long>(5 * (size_t)w.groups + 8);
+    w.lb.flag = q.take<int32_t>(T0); w.lb.agg = q.take<unsigned long long>(T0); w.lb.incl = q.take<unsigned long long>(T0);
+    const int nl = hmode == kHGather ? 4 : 2;
+    w.lists.alloc((size_t)sh.cap * 8 * nl + (size_t)sh.cap + 64, st);
+    w.slist = reinterpret_cast<uint8_t*>(w.lists.as<double>() + (size_t)sh.cap * nl);
+    for (int b = 0; b < 2; ++b) {
+      w.glist[b] = w.lists.as<double>() + (size_t)b * sh.cap;
+      w.hlist[b] = hmode == kHGather ? w.lists.as<double>() + (size_t)(2 + b) * sh.cap : nullptr;
+    }
     w.rec = q.take<Rec>(R);
     w.segH = q.take<int32_t>(S); w.segL = q.take<int32_t>(S);
     w.seg_pre = q.take<unsigned long long>(S);
@@ -555,9 +570,10 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         A.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters};
         A.g = gv; A.h = hv; A.nodes = cur; A.segPG = w.segPG; A.segPH = w.segPH; A.lam = P.lambda;
         A.epochp = epoch; A.fx = fxs; A.rec = w.rec;
-        A.glist = w.glist; A.hlist = w.hlist; A.tagg = w.tagg; A.carry = w.carry; A.nrec = w.nrec; A.gkey = w.gkey; A.shard = sh.index;
+        A.glist = w.glist[lvl & 1]; A.hlist = w.hlist[lvl & 1]; A.cagg = w.cagg; A.carry = w.carry;
+        A.sgrp = w.sgrp; A.nrec = w.nrec; A.gkey = w.gkey; A.shard = sh.index;
         A.segPG_out = w.segPG; A.segPH_out = w.segPH;
-        LK.tile_prefix(A, hmode, st);
+        LK.tile_prefix(A, hmode, /*gather=*/lvl == 0, w.groups, st);
         // present totals per segment first (needed for the missing direction)
         if (ds.has_missing) LK.seg_totals(A, hmode, st);
         LK.split_find(A, hmode, ds.has_missing, st);
@@ -630,16 +646,19 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         }
         PartArgs PA;
         PA.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters + 1};
-        PA.side = side; PA.segH = w.segH; PA.segL = w.segL;
+        PA.side = side; PA.slist = w.slist; PA.segH = w.segH; PA.segL = w.segL;
         PA.seg_pre = w.seg_pre; PA.out_hi = w.out_hi; PA.out_lo = w.out_lo;
         PA.val_out = sh.valw[(lvl + 1) & 1].as<float>();
         PA.ins_out = sh.insw[(lvl + 1) & 1].as<int32_t>();
-        PA.tcnt = w.tcnt; PA.tpre = w.tpre;
+        PA.ccnt = w.ccnt; PA.cpre = w.cpre; PA.sgrp = w.sgrp;
+        PA.g_in = w.glist[lvl & 1]; PA.h_in = w.hlist[lvl & 1];
+        PA.g_out = w.glist[(lvl + 1) & 1]; PA.h_out = w.hlist[(lvl + 1) & 1];
+        PA.epochp = epoch; PA.lb = w.lb;
         PlanArgs PL;
         PL.m = sh.m; PL.counted = ds.has_missing; PL.Kp = cur.K; PL.Knp = nxt.K; PL.cidx = cidx; PL.ncnt = nxt.cnt;
         PL.segH = w.segH; PL.segL = w.segL; PL.seg_pre = w.seg_pre;
         PL.out_hi = w.out_hi; PL.out_lo = w.out_lo; PL.len_tmp = w.len_tmp; PL.nxt = tn;
-        LK.partition(PA, PL, ds.has_missing, st);
+        LK.partition(PA, PL, ds.has_missing, hmode == kHGather, w.groups, st);
       }
       tm.end();
     }
