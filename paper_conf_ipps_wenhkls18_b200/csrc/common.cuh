@@ -137,6 +137,17 @@ __device__ __forceinline__ double parent_term(double G, double H, double lam) {
   return __ddiv_rn(__dmul_rn(G, G), __dadd_rn(H, lam));
 }
 
+// ----------------------------------------------------------------------------- RLE chunk index
+// Run o covers list positions [P, P+L) of attribute a: record it as the run of every chunk whose
+// first entry it holds (chunk starts are col_start[a] + 256 k).
+__device__ __forceinline__ void fill_run_chunks(int32_t* run_chunk, const Tables& tb, int a, long long P,
+                                                long long L, int o) {
+  const long long cs = tb.col_start[a];
+  const long long k0 = (P - cs + kChunk - 1) / kChunk;
+  const long long c0 = tb.chunk_start[a];
+  for (long long q = cs + k0 * kChunk; q < P + L; q += kChunk) run_chunk[c0 + (q - cs) / kChunk] = o;
+}
+
 // ----------------------------------------------------------------------------- scan value
 struct SV {
   double g, h;

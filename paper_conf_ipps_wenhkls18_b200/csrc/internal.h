@@ -68,6 +68,14 @@ struct Tables {
   int64_t* seg_cnt = nullptr;     // [m*Kcap]
   int32_t* T = nullptr;           // [1] tiles at this level
   int32_t* C = nullptr;           // [1] chunks at this level
+  // RLE: the runs of segment s are [seg_run[s], seg_run[s+1]); run r covers list
+  // positions [run_pos[r], run_pos[r] + run_len[r]) with value run_val[r]
+  int32_t* seg_run = nullptr;     // [m*Kcap + 1]
+  float* run_val = nullptr;
+  int32_t* run_len = nullptr;
+  int64_t* run_pos = nullptr;
+  int32_t* R = nullptr;           // [1] runs at this level
+  int32_t* run_chunk = nullptr;   // [C] the run holding each chunk's first entry
 };
 
 // Best split of one node found in one shard ("piece" records are reduced to this).
@@ -102,7 +110,7 @@ struct Shard {
   // RLE
   bool rle = false;
   int64_t runs = 0;
-  DBuf run_ptr, run_val, run_len;
+  DBuf run_ptr, run_val, run_len, run_pos, run_seg, run_chunk;
 };
 
 struct Dataset {

@@ -99,6 +99,23 @@ struct PlanArgs {
   Tables nxt;
 };
 
+struct RunArgs {
+  int m;
+  const int32_t* Kp;
+  const int32_t* Knp;
+  const int32_t* cidx;
+  Tables cur, nxt;                 // run tables of this level / the next (nxt.seg_start from the plan)
+  const uint8_t* slist;
+  const unsigned long long* cpre;  // [C][2] the partition's chunk prefix counts (attribute-relative)
+  int32_t* run_seg;                // [Rcap] parent segment of each run
+  unsigned long long* run_hl;      // [Rcap] h_r | l_r << 32
+  unsigned long long* cnt;         // [Rcap][2] scan elements (h_r | l_r << 32, segment head)
+  unsigned long long* fl;          // [Rcap+1][2] scan elements ([h_r>0] | [l_r>0] << 32, 0)
+  int32_t* Rp1;                    // R + 1 (length of the flag scan)
+  unsigned long long* sgrp;        // scan scratch
+  unsigned groups;
+};
+
 // levels.cu launchers
 struct LevelKernels {
   int sms = 148;
@@ -110,10 +127,10 @@ struct LevelKernels {
   // a3/a4: tile aggregates (+ g/h lists) and the exact segmented carry scan
   static unsigned scan_groups(int64_t max_chunks);
   void tile_prefix(const SplitArgs& A, int hmode, bool gather, unsigned groups, cudaStream_t st);
-  void split_find(const SplitArgs& A, int hmode, bool missing, cudaStream_t st);
+  void split_find(const SplitArgs& A, int hmode, bool missing, bool rle, cudaStream_t st);
   void seg_totals(const SplitArgs& A, int hmode, cudaStream_t st);
   void partition(const PartArgs& A, const PlanArgs& P, bool counted, bool with_h, unsigned groups,
-                 cudaStream_t st);
+                 const RunArgs* rle, cudaStream_t st);
 };
 
 }  // namespace gbdt

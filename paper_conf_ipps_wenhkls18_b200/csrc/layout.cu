@@ -215,6 +215,27 @@ __global__ void k_run_fill(int m, const int64_t* __restrict__ col_start, const i
   }
 }
 
+// run positions in the padded list: prefix of the run lengths inside each attribute
+__global__ void k_run_pos(int m, const int64_t* __restrict__ col_start, const int64_t* __restrict__ run_ptr,
+                          const int32_t* __restrict__ run_len, int64_t* __restrict__ run_pos,
+                          int32_t* __restrict__ seg_run, int32_t* __restrict__ R) {
+  for (int a = blockIdx.x * blockDim.x + threadIdx.x; a <= m; a += gridDim.x * blockDim.x) {
+    seg_run[a] = (int32_t)run_ptr[a];
+    if (a == m) { *R = (int32_t)run_ptr[m]; continue; }
+    int64_t p = col_start[a];
+    for (int64_t r = run_ptr[a]; r < run_ptr[a + 1]; ++r) { run_pos[r] = p; p += run_len[r]; }
+  }
+}
+
+__global__ void k_run_chunk_root(int m, Tables tb) {
+  const int R = *tb.R;
+  for (int r = blockIdx.x * blockDim.x + threadIdx.x; r < R; r += gridDim.x * blockDim.x) {
+    int lo = 0, hi = m - 1;  // attribute of run r
+    while (lo < hi) { const int mid = (lo + hi + 1) >> 1; if (tb.seg_run[mid] <= r) lo = mid; else hi = mid - 1; }
+    fill_run_chunks(tb.run_chunk, tb, lo, tb.run_pos[r], tb.run_len[r], r);
+  }
+}
+
 }  // namespace
 
 static void radix_sort(unsigned long long*& keys, uint32_t*& ids, unsigned long long*& kalt,
@@ -343,6 +364,23 @@ void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices
         k_run_fill<<<(unsigned)std::min<int64_t>(ceil_div(m, 8), (int64_t)sms * 8), 256, 0, st>>>(
             m, sh.root.col_start, sh.root.col_len, sh.val0.as<float>(), sh.run_ptr.as<int64_t>(),
             sh.run_val.as<float>(), sh.run_len.as<int32_t>());
+        GBDT_LAUNCH_CHECK();
+        sh.run_pos.alloc((size_t)std::max<int64_t>(R, 1) * 8 + 64, st);
+        sh.run_seg.alloc((size_t)(m + 1) * 4 + 64, st);
+        int32_t* Rdev = reinterpret_cast<int32_t*>(sh.run_seg.as<char>() + (size_t)(m + 1) * 4 + 16);
+        k_run_pos<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(m + 1, 256), (int64_t)sms * 4)), 256, 0, st>>>(
+            m, sh.root.col_start, sh.run_ptr.as<int64_t>(), sh.run_len.as<int32_t>(), sh.run_pos.as<int64_t>(),
+            sh.run_seg.as<int32_t>(), Rdev);
+        GBDT_LAUNCH_CHECK();
+        sh.root.seg_run = sh.run_seg.as<int32_t>();
+        sh.root.run_val = sh.run_val.as<float>();
+        sh.root.run_len = sh.run_len.as<int32_t>();
+        sh.root.run_pos = sh.run_pos.as<int64_t>();
+        sh.root.R = Rdev;
+        sh.run_chunk.alloc((size_t)std::max(sh.C0, 1) * 4 + 64, st);
+        sh.root.run_chunk = sh.run_chunk.as<int32_t>();
+        k_run_chunk_root<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, 256), (int64_t)sms * 8)), 256, 0, st>>>(
+            m, sh.root);
         GBDT_LAUNCH_CHECK();
         GBDT_CUDA(cudaStreamSynchronize(st));
       }

@@ -571,7 +571,7 @@ __device__ __forceinline__ void push_record(SFSmem& S, const SplitArgs& A, const
   }
 }
 
-template <int HMODE, bool kMissing, bool kTotals>
+template <int HMODE, bool kMissing, bool kTotals, bool kRLE>
 __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
   SFSmem& S = *reinterpret_cast<SFSmem*>(smem_raw);
@@ -600,7 +600,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
   auto issue = [&](int i) {
     const int s = i % kStages;
     if (wid == 0)
-      issue_stage<!kTotals, kH>(lane, tile_of(i), T, K, S.tc, A, S.meta[s], S.val[s], S.g[s],
+      issue_stage<!kTotals && !kRLE, kH>(lane, tile_of(i), T, K, S.tc, A, S.meta[s], S.val[s], S.g[s],
                                 kH ? sH + (size_t)s * kTile : nullptr, &S.bar[s], pol_stream);
     cp_async_commit();
   };
@@ -632,7 +632,28 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
 #pragma unroll
       for (int k = 0; k < kItems; ++k)
         if (base + k < cp1) vm |= 1u << k;
-      if (!kTotals) {
+      if (kRLE && !kTotals) {
+        // direct RLE: the values come from the runs covering this thread's entries; the
+        // chunk index gives the runs holding the first entries of this chunk and the next one
+        const Tables& tb = A.t.tb;
+        const int cg = (S.tc.use ? S.tc.chunk_start[M.a] : tb.chunk_start[M.a]) + M.u * kChunksPerTile + wid;
+        int lo = tb.run_chunk[cg];
+        int hi = cp1 < M.colend ? tb.run_chunk[cg + 1] : tb.seg_run[M.sb + K] - 1;
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (tb.run_pos[mid] <= base) lo = mid; else hi = mid - 1;
+        }
+        int r = lo;
+        long long rend = tb.run_pos[r] + tb.run_len[r];
+        float rv = tb.run_val[r];
+#pragma unroll
+        for (int k = 0; k <= kItems; ++k) {
+          const long long p = base + k;
+          if (p >= M.colend || p > cp1) { if (k < kItems) v[k] = 0.f; continue; }
+          while (p >= rend) { ++r; rend = tb.run_pos[r] + tb.run_len[r]; rv = tb.run_val[r]; }
+          if (k < kItems) v[k] = rv; else vnext = rv;
+        }
+      } else if (!kTotals) {
         const float4 v0 = *reinterpret_cast<const float4*>(&S.val[s0][ibase]);
         const float4 v1 = *reinterpret_cast<const float4*>(&S.val[s0][ibase + 4]);
         v[0] = v0.x; v[1] = v0.y; v[2] = v0.z; v[3] = v0.w;
@@ -1070,7 +1091,7 @@ struct ScatterStage {
   int id[kChunk];
 };
 
-template <bool kH>
+template <bool kH, bool kRLE>
 __global__ void __launch_bounds__(kThreads) k_part_scatter(PartArgs A) {
   __shared__ TabCache tc;
   extern __shared__ __align__(16) unsigned char sc_raw[];
@@ -1099,8 +1120,11 @@ __global__ void __launch_bounds__(kThreads) k_part_scatter(PartArgs A) {
     if (base < p1) {
       const int4 i0 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base));
       const int4 i1 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base + 4));
-      const float4 v0 = __ldcs(reinterpret_cast<const float4*>(A.t.val + base));
-      const float4 v1 = __ldcs(reinterpret_cast<const float4*>(A.t.val + base + 4));
+      float4 v0 = make_float4(0.f, 0.f, 0.f, 0.f), v1 = v0;
+      if (!kRLE) {  // with RLE the values live in the runs, which are split separately
+        v0 = __ldcs(reinterpret_cast<const float4*>(A.t.val + base));
+        v1 = __ldcs(reinterpret_cast<const float4*>(A.t.val + base + 4));
+      }
       const unsigned long long pk = (unsigned long long)__ldcs(reinterpret_cast<const unsigned*>(A.slist + base)) |
                                     ((unsigned long long)__ldcs(reinterpret_cast<const unsigned*>(A.slist + base) + 1) << 32);
       id[0] = i0.x; id[1] = i0.y; id[2] = i0.z; id[3] = i0.w; id[4] = i1.x; id[5] = i1.y; id[6] = i1.z; id[7] = i1.w;
@@ -1156,12 +1180,150 @@ __global__ void __launch_bounds__(kThreads) k_part_scatter(PartArgs A) {
     __syncwarp();
     for (int i = lane; i < (int)nkeep; i += 32) {
       const long long d = W.dst[i];
-      A.val_out[d] = W.v[i];
+      if (!kRLE) A.val_out[d] = W.v[i];
       A.ins_out[d] = W.id[i];
       A.g_out[d] = W.g[i];
       if (kH) A.h_out[d] = Wh[i];
     }
     __syncwarp();
+  }
+}
+
+// ============================================================================ a8 RLE: direct split
+// "each RLE element is potentially split into two ... we compute the length of each new RLE element
+// using the instance to node mapping ... prefix sum to remove the RLE element with length of 0"
+// (P:250).  k_run_count: one warp per run counts its entries going high (h_r) / low (l_r) from the
+// side-list.  Two exact integer scans follow: (h_r, l_r) segmented by parent segment (the child
+// run's offset inside its child segment) and the non-empty flags ([h_r>0], [l_r>0]) over all runs
+// (the compaction).  k_run_scatter writes the child runs -- high child of every parent segment,
+// then its low child, in segment order -- and the next level's segment -> run table.
+// (high | low << 32) side counts of the attribute before list position p (p inside the attribute
+// list, or its end): the chunk prefix from the count scan + the warp's count inside the chunk.
+__device__ __forceinline__ unsigned long long side_prefix(const RunArgs& A, int a, long long p, int lane) {
+  const long long cs = A.cur.col_start[a];
+  const long long k = (p - cs - 1) / kChunk;  // chunk of entry p-1 (p > cs)
+  const long long q0 = cs + k * kChunk;
+  const unsigned long long pre = A.cpre[2 * ((long long)A.cur.chunk_start[a] + k)];
+  const long long b = q0 + lane * kItems;
+  unsigned h = 0, l = 0;
+  if (b < p) {
+    const unsigned w0 = reinterpret_cast<const unsigned*>(A.slist + b)[0];
+    const unsigned w1 = b + 4 < p ? reinterpret_cast<const unsigned*>(A.slist + b)[1] : 0u;
+#pragma unroll
+    for (int i = 0; i < kItems; ++i) {
+      const unsigned sd = ((i < 4 ? w0 : w1) >> (8 * (i & 3))) & 0xffu;
+      const bool in = b + i < p;
+      h += in && sd == 1;
+      l += in && sd == 2;
+    }
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    h += __shfl_xor_sync(0xffffffffu, h, o);
+    l += __shfl_xor_sync(0xffffffffu, l, o);
+  }
+  return pre + ((unsigned long long)h | ((unsigned long long)l << 32));
+}
+
+__global__ void __launch_bounds__(kThreads) k_run_count(RunArgs A) {
+  const int R = *A.cur.R;
+  const int K = *A.Kp;
+  const long long S = (long long)A.m * K;
+  const int lane = threadIdx.x & 31;
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    A.fl[2ll * R] = 0ull;
+    A.fl[2ll * R + 1] = 0ull;
+    *A.Rp1 = R + 1;
+  }
+  for (int r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; r < R; r += nw) {
+    long long lo = 0, hi = S - 1;  // last segment whose first run is <= r (it contains r)
+    while (lo < hi) {
+      const long long mid = (lo + hi + 1) >> 1;
+      if (A.cur.seg_run[mid] <= r) lo = mid; else hi = mid - 1;
+    }
+    const long long p0 = A.cur.run_pos[r];
+    const int len = A.cur.run_len[r];
+    unsigned long long hl;
+    if (len <= 2 * kChunk) {  // short run: count its own sides
+      unsigned h = 0, l = 0;
+      for (int q = lane; q < len; q += 32) {
+        const uint8_t sd = A.slist[p0 + q];
+        h += sd == 1;
+        l += sd == 2;
+      }
+#pragma unroll
+      for (int o = 16; o; o >>= 1) {
+        h += __shfl_xor_sync(0xffffffffu, h, o);
+        l += __shfl_xor_sync(0xffffffffu, l, o);
+      }
+      hl = (unsigned long long)h | ((unsigned long long)l << 32);
+    } else {  // long run: difference of two attribute prefixes (work independent of the length)
+      const int a = (int)(lo / K);
+      hl = side_prefix(A, a, p0 + len, lane) - side_prefix(A, a, p0 + 1, lane);
+      const uint8_t sd0 = A.slist[p0];  // side_prefix(p0 + 1) counted entry p0 too
+      hl += (unsigned long long)(sd0 == 1) | ((unsigned long long)(sd0 == 2) << 32);
+    }
+    if (lane == 0) {
+      const unsigned h = (unsigned)(hl & 0xffffffffull), l = (unsigned)(hl >> 32);
+      A.run_seg[r] = (int32_t)lo;
+      A.run_hl[r] = hl;
+      A.cnt[2ll * r] = hl;
+      A.cnt[2ll * r + 1] = A.cur.seg_run[lo] == r ? 1ull : 0ull;
+      A.fl[2ll * r] = (unsigned long long)(h > 0) | ((unsigned long long)(l > 0) << 32);
+      A.fl[2ll * r + 1] = 0ull;
+    }
+  }
+}
+
+__global__ void __launch_bounds__(kThreads) k_run_scatter(RunArgs A) {
+  const int R = *A.cur.R;
+  const int K = *A.Kp, Kn = *A.Knp;
+  const long long S = (long long)A.m * K;
+  auto eh = [&](long long r) { return (long long)(A.fl[2 * r] & 0xffffffffull); };
+  auto el = [&](long long r) { return (long long)(A.fl[2 * r] >> 32); };
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  const long long i0 = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i0 == 0) {
+    const int tot = (int)(eh(R) + el(R));
+    *A.nxt.R = tot;
+    A.nxt.seg_run[(long long)A.m * Kn] = tot;
+  }
+  for (long long s = i0; s < S; s += stride) {  // next level's segment -> first run
+    const int c = A.cidx[s % K];
+    if (c < 0) continue;
+    const long long chi = (s / K) * Kn + c;
+    const long long r0 = A.cur.seg_run[s], r1 = A.cur.seg_run[s + 1];
+    A.nxt.seg_run[chi] = (int32_t)(eh(r0) + el(r0));
+    A.nxt.seg_run[chi + 1] = (int32_t)(eh(r1) + el(r0));
+  }
+  for (long long r = i0; r < R; r += stride) {
+    const unsigned long long hl = A.run_hl[r];
+    if (hl == 0ull) continue;
+    const long long s = A.run_seg[r];
+    const int c = A.cidx[s % K];
+    const long long chi = (s / K) * Kn + c;
+    const long long r0 = A.cur.seg_run[s], r1 = A.cur.seg_run[s + 1];
+    const unsigned long long off = A.cnt[2 * r];  // exclusive (h, l) inside the parent segment
+    const float v = A.cur.run_val[r];
+    const unsigned h = (unsigned)(hl & 0xffffffffull), l = (unsigned)(hl >> 32);
+    const int a = (int)(s / K);
+    if (h) {
+      const long long o = eh(r) + el(r0);
+      const long long P = A.nxt.seg_start[chi] + (long long)(off & 0xffffffffull);
+      A.nxt.run_val[o] = v;
+      A.nxt.run_len[o] = (int32_t)h;
+      A.nxt.run_pos[o] = P;
+      fill_run_chunks(A.nxt.run_chunk, A.nxt, a, P, h, (int)o);
+    }
+    if (l) {
+      const long long o = eh(r1) + el(r);
+      const long long P = A.nxt.seg_start[chi + 1] + (long long)(off >> 32);
+      A.nxt.run_val[o] = v;
+      A.nxt.run_len[o] = (int32_t)l;
+      A.nxt.run_pos[o] = P;
+      fill_run_chunks(A.nxt.run_chunk, A.nxt, a, P, l, (int)o);
+    }
   }
 }
 
@@ -1183,9 +1345,14 @@ size_t sf_smem(int hmode) {
 }
 
 template <int HM>
-void launch_sf(const SplitArgs& A, bool missing, unsigned grid, cudaStream_t st) {
-  if (missing) k_sf<HM, true, false><<<grid, kThreads, sf_smem(HM), st>>>(A);
-  else k_sf<HM, false, false><<<grid, kThreads, sf_smem(HM), st>>>(A);
+void launch_sf(const SplitArgs& A, bool missing, bool rle, unsigned grid, cudaStream_t st) {
+  if (rle) {
+    if (missing) k_sf<HM, true, false, true><<<grid, kThreads, sf_smem(HM), st>>>(A);
+    else k_sf<HM, false, false, true><<<grid, kThreads, sf_smem(HM), st>>>(A);
+  } else {
+    if (missing) k_sf<HM, true, false, false><<<grid, kThreads, sf_smem(HM), st>>>(A);
+    else k_sf<HM, false, false, false><<<grid, kThreads, sf_smem(HM), st>>>(A);
+  }
 }
 
 template <bool kFx>
@@ -1202,23 +1369,31 @@ void launch_scan(const int32_t* Cp, unsigned long long* in, unsigned long long* 
 
 void LevelKernels::init(int device) {
   GBDT_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device));
-  grid_sf[0][0] = grid_for(k_sf<0, false, false>, sf_smem(0), sms);
-  grid_sf[0][1] = grid_for(k_sf<0, true, false>, sf_smem(0), sms);
-  grid_sf[1][0] = grid_for(k_sf<1, false, false>, sf_smem(1), sms);
-  grid_sf[1][1] = grid_for(k_sf<1, true, false>, sf_smem(1), sms);
-  grid_sf[2][0] = grid_for(k_sf<2, false, false>, sf_smem(2), sms);
-  grid_sf[2][1] = grid_for(k_sf<2, true, false>, sf_smem(2), sms);
-  grid_tot[0] = grid_for(k_sf<0, true, true>, sf_smem(0), sms);
-  grid_tot[1] = grid_for(k_sf<1, true, true>, sf_smem(1), sms);
-  grid_tot[2] = grid_for(k_sf<2, true, true>, sf_smem(2), sms);
+  grid_sf[0][0] = grid_for(k_sf<0, false, false, false>, sf_smem(0), sms);
+  grid_sf[0][1] = grid_for(k_sf<0, true, false, false>, sf_smem(0), sms);
+  grid_sf[1][0] = grid_for(k_sf<1, false, false, false>, sf_smem(1), sms);
+  grid_sf[1][1] = grid_for(k_sf<1, true, false, false>, sf_smem(1), sms);
+  grid_sf[2][0] = grid_for(k_sf<2, false, false, false>, sf_smem(2), sms);
+  grid_sf[2][1] = grid_for(k_sf<2, true, false, false>, sf_smem(2), sms);
+  grid_for(k_sf<0, false, false, true>, sf_smem(0), sms);
+  grid_for(k_sf<0, true, false, true>, sf_smem(0), sms);
+  grid_for(k_sf<1, false, false, true>, sf_smem(1), sms);
+  grid_for(k_sf<1, true, false, true>, sf_smem(1), sms);
+  grid_for(k_sf<2, false, false, true>, sf_smem(2), sms);
+  grid_for(k_sf<2, true, false, true>, sf_smem(2), sms);
+  grid_tot[0] = grid_for(k_sf<0, true, true, false>, sf_smem(0), sms);
+  grid_tot[1] = grid_for(k_sf<1, true, true, false>, sf_smem(1), sms);
+  grid_tot[2] = grid_for(k_sf<2, true, true, false>, sf_smem(2), sms);
   grid_agg[0] = grid_for(k_chunk_agg<0, true>, 0, sms);
   grid_agg[1] = grid_for(k_chunk_agg<1, true>, 0, sms);
   grid_agg[2] = grid_for(k_chunk_agg<2, true>, 0, sms);
   grid_agg_list[0] = grid_for(k_chunk_agg<0, false>, 0, sms);
   grid_agg_list[1] = grid_for(k_chunk_agg<1, false>, 0, sms);
   grid_agg_list[2] = grid_for(k_chunk_agg<2, false>, 0, sms);
-  grid_scatter[0] = grid_for(k_part_scatter<false>, scatter_smem(false), sms);
-  grid_scatter[1] = grid_for(k_part_scatter<true>, scatter_smem(true), sms);
+  grid_scatter[0] = grid_for(k_part_scatter<false, false>, scatter_smem(false), sms);
+  grid_scatter[1] = grid_for(k_part_scatter<true, false>, scatter_smem(true), sms);
+  grid_for(k_part_scatter<false, true>, scatter_smem(false), sms);
+  grid_for(k_part_scatter<true, true>, scatter_smem(true), sms);
   grid_count = grid_for(k_part_count, 0, sms);
 }
 
@@ -1241,32 +1416,45 @@ void LevelKernels::tile_prefix(const SplitArgs& A, int hmode, bool gather, unsig
   launch_scan<true>(A.t.tb.C, A.cagg, A.sgrp, A.carry, groups, st);
 }
 
-void LevelKernels::split_find(const SplitArgs& A, int hmode, bool missing, cudaStream_t st) {
-  if (hmode == 0) launch_sf<0>(A, missing, grid_sf[0][missing], st);
-  else if (hmode == 1) launch_sf<1>(A, missing, grid_sf[1][missing], st);
-  else launch_sf<2>(A, missing, grid_sf[2][missing], st);
+void LevelKernels::split_find(const SplitArgs& A, int hmode, bool missing, bool rle, cudaStream_t st) {
+  if (hmode == 0) launch_sf<0>(A, missing, rle, grid_sf[0][missing], st);
+  else if (hmode == 1) launch_sf<1>(A, missing, rle, grid_sf[1][missing], st);
+  else launch_sf<2>(A, missing, rle, grid_sf[2][missing], st);
   GBDT_LAUNCH_CHECK();
   count_launch();
 }
 
 void LevelKernels::seg_totals(const SplitArgs& A, int hmode, cudaStream_t st) {
-  if (hmode == 0) k_sf<0, true, true><<<grid_tot[0], kThreads, sf_smem(0), st>>>(A);
-  else if (hmode == 1) k_sf<1, true, true><<<grid_tot[1], kThreads, sf_smem(1), st>>>(A);
-  else k_sf<2, true, true><<<grid_tot[2], kThreads, sf_smem(2), st>>>(A);
+  if (hmode == 0) k_sf<0, true, true, false><<<grid_tot[0], kThreads, sf_smem(0), st>>>(A);
+  else if (hmode == 1) k_sf<1, true, true, false><<<grid_tot[1], kThreads, sf_smem(1), st>>>(A);
+  else k_sf<2, true, true, false><<<grid_tot[2], kThreads, sf_smem(2), st>>>(A);
   GBDT_LAUNCH_CHECK();
   count_launch();
 }
 
 void LevelKernels::partition(const PartArgs& A, const PlanArgs& P, bool counted, bool with_h, unsigned groups,
-                             cudaStream_t st) {
+                             const RunArgs* rle, cudaStream_t st) {
   k_part_count<<<grid_count, kThreads, 0, st>>>(A, counted ? 1 : 0);
   GBDT_LAUNCH_CHECK();
   count_launch();
   launch_scan<false>(A.t.tb.C, A.ccnt, A.sgrp, A.cpre, groups, st);
   k_part_plan<<<1, 1024, 0, st>>>(P);
   GBDT_LAUNCH_CHECK();
-  if (with_h) k_part_scatter<true><<<grid_scatter[1], kThreads, scatter_smem(true), st>>>(A);
-  else k_part_scatter<false><<<grid_scatter[0], kThreads, scatter_smem(false), st>>>(A);
+  if (rle) {
+    if (with_h) k_part_scatter<true, true><<<grid_scatter[1], kThreads, scatter_smem(true), st>>>(A);
+    else k_part_scatter<false, true><<<grid_scatter[0], kThreads, scatter_smem(false), st>>>(A);
+    GBDT_LAUNCH_CHECK();
+    k_run_count<<<(unsigned)(sms * 8), kThreads, 0, st>>>(*rle);
+    GBDT_LAUNCH_CHECK();
+    count_launch();
+    launch_scan<false>(rle->cur.R, rle->cnt, rle->sgrp, rle->cnt, rle->groups, st);
+    launch_scan<false>(rle->Rp1, rle->fl, rle->sgrp, rle->fl, rle->groups, st);
+    k_run_scatter<<<(unsigned)(sms * 8), kThreads, 0, st>>>(*rle);
+    count_launch();
+  } else {
+    if (with_h) k_part_scatter<true, false><<<grid_scatter[1], kThreads, scatter_smem(true), st>>>(A);
+    else k_part_scatter<false, false><<<grid_scatter[0], kThreads, scatter_smem(false), st>>>(A);
+  }
   GBDT_LAUNCH_CHECK();
   count_launch(2);
 }

@@ -358,6 +358,12 @@ struct ShardWork {
   int64_t *out_hi, *out_lo, *len_tmp;
   double *segPG, *segPH;
   int* counters;  // [4]
+  // RLE (a8): run tables of two levels live in tab[b]; scratch of the direct run split
+  DBuf runs;
+  int32_t* run_seg = nullptr;
+  unsigned long long *run_hl = nullptr, *rcnt = nullptr, *rfl = nullptr, *rsgrp = nullptr;
+  int32_t* Rp1 = nullptr;
+  unsigned rgroups = 1;
 };
 
 struct PhaseTimer {
@@ -518,6 +524,34 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     w.len_tmp = q.take<int64_t>(m);
     w.segPG = q.take<double>(S); w.segPH = q.take<double>(S);
     w.counters = q.take<int>(4);
+    if (sh.rle) {
+      // child runs: every run splits in at most two, and there are never more runs than entries
+      const int64_t Rcap = std::max<int64_t>(1, std::min<int64_t>(sh.runs * Kcap, sh.cap));
+      w.rgroups = LevelKernels::scan_groups(Rcap + 1);
+      auto rz = [&](Carve& q) {
+        for (int b = 0; b < 2; ++b) {
+          q.take<float>(Rcap); q.take<int32_t>(Rcap); q.take<int64_t>(Rcap); q.take<int32_t>(S + 1); q.take<int32_t>(1);
+          q.take<int32_t>(C0 + 1);
+        }
+        q.take<int32_t>(Rcap); q.take<unsigned long long>(Rcap); q.take<unsigned long long>(2 * Rcap);
+        q.take<unsigned long long>(2 * (Rcap + 1)); q.take<int32_t>(1);
+        q.take<unsigned long long>(2 * (size_t)w.rgroups + 8);
+      };
+      Carve rp{nullptr};
+      rz(rp);
+      w.runs.alloc(rp.off + 1024, st);
+      GBDT_CUDA(cudaMemsetAsync(w.runs.p, 0, w.runs.bytes, st));
+      Carve r{w.runs.as<char>()};
+      for (int b = 0; b < 2; ++b) {
+        w.tab[b].run_val = r.take<float>(Rcap); w.tab[b].run_len = r.take<int32_t>(Rcap);
+        w.tab[b].run_pos = r.take<int64_t>(Rcap); w.tab[b].seg_run = r.take<int32_t>(S + 1);
+        w.tab[b].R = r.take<int32_t>(1);
+        w.tab[b].run_chunk = r.take<int32_t>(C0 + 1);
+      }
+      w.run_seg = r.take<int32_t>(Rcap); w.run_hl = r.take<unsigned long long>(Rcap);
+      w.rcnt = r.take<unsigned long long>(2 * Rcap); w.rfl = r.take<unsigned long long>(2 * (Rcap + 1));
+      w.Rp1 = r.take<int32_t>(1); w.rsgrp = r.take<unsigned long long>(2 * (size_t)w.rgroups + 8);
+    }
     w.nrec = nrec + li;
     w.gkey = gkey + (size_t)li * Kcap;
     w.tkey = tkey + (size_t)li * Kcap;
@@ -576,7 +610,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         LK.tile_prefix(A, hmode, /*gather=*/lvl == 0, w.groups, st);
         // present totals per segment first (needed for the missing direction)
         if (ds.has_missing) LK.seg_totals(A, hmode, st);
-        LK.split_find(A, hmode, ds.has_missing, st);
+        LK.split_find(A, hmode, ds.has_missing, sh.rle, st);
       }
       tm.end();
       tm.begin(GBDT_PHASE_DECIDE);
@@ -658,7 +692,13 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         PL.m = sh.m; PL.counted = ds.has_missing; PL.Kp = cur.K; PL.Knp = nxt.K; PL.cidx = cidx; PL.ncnt = nxt.cnt;
         PL.segH = w.segH; PL.segL = w.segL; PL.seg_pre = w.seg_pre;
         PL.out_hi = w.out_hi; PL.out_lo = w.out_lo; PL.len_tmp = w.len_tmp; PL.nxt = tn;
-        LK.partition(PA, PL, ds.has_missing, hmode == kHGather, w.groups, st);
+        RunArgs RA;
+        if (sh.rle) {
+          RA.m = sh.m; RA.Kp = cur.K; RA.Knp = nxt.K; RA.cidx = cidx; RA.cur = tb; RA.nxt = tn;
+          RA.slist = w.slist; RA.cpre = w.cpre; RA.run_seg = w.run_seg; RA.run_hl = w.run_hl; RA.cnt = w.rcnt; RA.fl = w.rfl;
+          RA.Rp1 = w.Rp1; RA.sgrp = w.rsgrp; RA.groups = w.rgroups;
+        }
+        LK.partition(PA, PL, ds.has_missing, hmode == kHGather, w.groups, sh.rle ? &RA : nullptr, st);
       }
       tm.end();
     }

@@ -196,3 +196,50 @@ def test_deterministic_across_runs():
     b, mb = _train(p)
     assert np.array_equal(a.nodes().view(np.uint8), b.nodes().view(np.uint8))
     assert np.array_equal(ma, mb)
+
+
+# ------------------------------------------------------------------ a8 RLE: direct split
+# The RLE path reads values from the runs and splits the runs themselves (no decompression in HBM);
+# it sees the same entry streams, so its trees and margins must be bit-identical to the plain path,
+# and both match the oracle.
+@pytest.mark.parametrize("maker", [
+    lambda: synth.c5(n=40000, T=3),
+    lambda: synth.table1(),
+    lambda: synth.random_small(7, n=6000, m=6, nan_frac=0.25, n_distinct=12),
+    lambda: synth.random_small(8, n=9000, m=5, nan_frac=0.0, n_distinct=3000),
+    lambda: synth.c4(seed=9, n=1500, m=2000, density=0.01, T=2),
+    lambda: synth.c1(n=5000),
+])
+def test_rle_direct_split_bit_identical(maker):
+    p = maker()
+    ref_model, ref_margin = _train(p)
+    model, margin = _train(p, rle="on")
+    assert np.array_equal(model.nodes().view(np.uint8), ref_model.nodes().view(np.uint8))
+    assert np.array_equal(margin, ref_margin)
+
+
+def test_rle_c5_against_oracle():
+    p = synth.c5(n=20000, T=2)
+    model, margin = _train(p, rle="on")
+    compare(p, model.nodes(), margin)
+
+
+@pytest.mark.parametrize("k", [2, 4])
+def test_rle_with_shards(k):
+    p = synth.c5(n=30000, T=2)
+    ref_model, ref_margin = _train(p)
+    model, margin = _train(p, rle="on", n_shards=k)
+    assert np.array_equal(model.nodes().view(np.uint8), ref_model.nodes().view(np.uint8))
+    assert np.array_equal(margin, ref_margin)
+
+
+def test_rle_export_matches_oracle_encoding():
+    p = synth.c5(n=20000, T=1)
+    ds = gbdt.load_csr(p.indptr, p.indices, p.values, p.labels, p.m, rle="on")
+    run_ptr, rv, rl = ds.export_rle()
+    ocp, oval, _ = oracle.presort(p.indptr, p.indices, p.values, p.n, p.m)
+    for a in range(p.m):
+        orv, orl = oracle.rle_encode(oval[ocp[a]:ocp[a + 1]])
+        assert np.array_equal(rv[run_ptr[a]:run_ptr[a + 1]].view(np.uint32), orv.view(np.uint32))
+        assert np.array_equal(rl[run_ptr[a]:run_ptr[a + 1]], orl)
+    assert run_ptr[-1] == rv.size
