@@ -96,6 +96,10 @@ struct PlanArgs {
   int64_t* out_hi;
   int64_t* out_lo;
   int64_t* len_tmp;       // [m]
+  unsigned long long* el; // [m+1][2] scan elements: padded list length | chunks << 32
+  unsigned long long* egrp;
+  unsigned egroups;
+  const int32_t* mp1;     // m + 1 (device)
   Tables nxt;
 };
 

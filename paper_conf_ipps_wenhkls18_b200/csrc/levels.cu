@@ -141,7 +141,6 @@ __device__ __forceinline__ double rcp_nr(double x) {
 // ============================================================================ plumbing
 struct TabCache {
   int use;
-  int tile_start[kTabCache + 1];
   int chunk_start[kTabCache + 1];
   long long col_start[kTabCache + 1];
   long long col_len[kTabCache];
@@ -152,7 +151,6 @@ __device__ __forceinline__ void tab_load(TabCache& tc, const TileArgs& A) {
   if (threadIdx.x == 0) tc.use = use;
   if (use) {
     for (int i = threadIdx.x; i <= A.m; i += blockDim.x) {
-      tc.tile_start[i] = A.tb.tile_start[i];
       tc.chunk_start[i] = A.tb.chunk_start[i];
       tc.col_start[i] = A.tb.col_start[i];
       if (i < A.m) tc.col_len[i] = A.tb.col_len[i];
@@ -482,54 +480,69 @@ __global__ void __launch_bounds__(kThreads) k_scan3(const int32_t* __restrict__ 
 }
 
 // ============================================================================ a3-a6: split find
-struct StageMeta {
+// A tile is 8 CONSECUTIVE chunks of the level (chunks 8t .. 8t+7), which may belong to different
+// attributes: chunks are attribute-aligned, tiles are not, so thousands of short attribute lists
+// (C4: ~20 entries each) share one tile instead of each occupying a mostly empty one (a3,
+// many-segment load balance).  The chunks of a tile are contiguous in the list buffer up to the
+// <= 3-entry padding between attributes, so one bulk copy per list stages the whole tile.
+constexpr int kTileSpan = kTile + 4 * kChunksPerTile;  // entries a stage can hold
+struct WarpMeta {
   long long p0, p1, colend, sb;
-  int t, a, u, seg_cached;
+  int a, off;  // attribute; chunk offset in the stage
+};
+struct StageMeta {
+  long long P0, P1;
+  int t, nch;
+  WarpMeta w[kChunksPerTile];
   unsigned long long carry[kChunksPerTile * 5];
-  long long seg_s[kSegCache];
-  long long seg_c[kSegCache];
+  long long seg_s[kChunksPerTile][kSegCache];
+  long long seg_c[kChunksPerTile][kSegCache];
 };
 
-// lane 0 of warp 0: metadata of tile t and the TMA bulk loads of its lists into a stage; the
-// lanes fetch the tile's chunk carries and the attribute's segment table with cp.async.
+// warp 0: lanes 0..7 locate the tile's chunks; lane 0 issues the TMA bulk loads of the tile's lists
+// into a stage; the lanes fetch the chunk carries and the segment tables with cp.async.
 template <bool kVal, bool kH>
-__device__ __forceinline__ void issue_stage(int lane, int t, int T, int K, const TabCache& tc,
+__device__ __forceinline__ void issue_stage(int lane, int t, int T, int C, int K, const TabCache& tc,
                                             const SplitArgs& A, StageMeta& M, float* sval, double* sg,
                                             double* sh, unsigned long long* bar, unsigned long long pol) {
-  if (lane == 0) {
-    M.t = t;
-    if (t < T) {
-      const bool u = tc.use;
-      const int* ts = u ? tc.tile_start : A.t.tb.tile_start;
-      const int a = find_attr(ts, A.t.m, t);
-      const long long cs = u ? tc.col_start[a] : A.t.tb.col_start[a];
-      const long long cl = u ? tc.col_len[a] : A.t.tb.col_len[a];
-      M.a = a;
-      M.u = t - ts[a];
-      M.colend = cs + cl;
-      M.p0 = cs + (long long)M.u * kTile;
-      M.p1 = min(M.p0 + (long long)kTile, M.colend);
-      M.sb = (long long)a * K;
-      M.seg_cached = K <= kSegCache;
-      const long long r1 = min((M.p1 + 3) & ~3ll, cs + ((cl + 3) & ~3ll));  // 16-byte granules
-      const uint32_t n = (uint32_t)(r1 - M.p0);
-      fence_proxy_async();
-      mbar_arrive_expect_tx(bar, (kVal ? 4u * n : 0u) + 8u * n + (kH ? 8u * n : 0u));
-      if (kVal) tma_load_1d(sval, A.t.val + M.p0, 4u * n, bar, pol);
-      tma_load_1d(sg, A.glist + M.p0, 8u * n, bar, pol);
-      if (kH) tma_load_1d(sh, A.hlist + M.p0, 8u * n, bar, pol);
-    }
+  if (lane == 0) M.t = t;
+  if (t >= T) return;
+  const int c0 = t * kChunksPerTile;
+  const int nch = min(kChunksPerTile, C - c0);
+  long long p0 = 0, p1 = 0;
+  if (lane < nch) {
+    const ChunkMeta cm = chunk_meta(tc, A.t, K, c0 + lane);
+    p0 = cm.p0;
+    p1 = cm.p1;
+    WarpMeta& W = M.w[lane];
+    W.p0 = cm.p0;
+    W.p1 = cm.p1;
+    W.colend = (tc.use ? tc.col_start[cm.a] + tc.col_len[cm.a] : A.t.tb.col_start[cm.a] + A.t.tb.col_len[cm.a]);
+    W.sb = cm.sb;
+    W.a = cm.a;
   }
-  __syncwarp();
-  if (t < T) {
-    const int nch = (int)((M.p1 - M.p0 + kChunk - 1) / kChunk);
-    const int c0 = (tc.use ? tc.chunk_start[M.a] : A.t.tb.chunk_start[M.a]) + M.u * kChunksPerTile;
-    for (int q = lane; q < nch * 5; q += 32) cp_async8(&M.carry[q], A.carry + 5ll * c0 + q, pol);
-    if (K <= kSegCache) {
-      const long long sb = M.sb;
-      for (int j = lane; j < K; j += 32) {
-        cp_async8(&M.seg_s[j], A.t.tb.seg_start + sb + j, pol);
-        cp_async8(&M.seg_c[j], A.t.tb.seg_cnt + sb + j, pol);
+  const long long P0 = __shfl_sync(0xffffffffu, p0, 0);
+  const long long P1 = __shfl_sync(0xffffffffu, p1, nch - 1);
+  if (lane < nch) M.w[lane].off = (int)(p0 - P0);
+  if (lane == 0) {
+    M.P0 = P0;
+    M.P1 = P1;
+    M.nch = nch;
+    const uint32_t n = (uint32_t)(((P1 + 3) & ~3ll) - P0);  // 16-byte granules inside the padding
+    fence_proxy_async();
+    mbar_arrive_expect_tx(bar, (kVal ? 4u * n : 0u) + 8u * n + (kH ? 8u * n : 0u));
+    if (kVal) tma_load_1d(sval, A.t.val + P0, 4u * n, bar, pol);
+    tma_load_1d(sg, A.glist + P0, 8u * n, bar, pol);
+    if (kH) tma_load_1d(sh, A.hlist + P0, 8u * n, bar, pol);
+  }
+  for (int q = lane; q < nch * 5; q += 32) cp_async8(&M.carry[q], A.carry + 5ll * c0 + q, pol);
+  if (K <= kSegCache) {
+    const long long sbl = lane < nch ? M.w[lane].sb : 0ll;
+    for (int w = 0; w < nch; ++w) {
+      const long long sb = __shfl_sync(0xffffffffu, sbl, w);
+      if (lane < K) {
+        cp_async8(&M.seg_s[w][lane], A.t.tb.seg_start + sb + lane, pol);
+        cp_async8(&M.seg_c[w][lane], A.t.tb.seg_cnt + sb + lane, pol);
       }
     }
   }
@@ -580,7 +593,8 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
 
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int K = *A.t.Kp;
-  const int T = *A.t.tb.T;
+  const int C = *A.t.tb.C;
+  const int T = (C + kChunksPerTile - 1) / kChunksPerTile;
   if (K == 0 || T == 0) return;
   const int epoch = *A.epochp;
   const int Fg = A.fx[0], Fh = A.fx[1];
@@ -600,8 +614,8 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
   auto issue = [&](int i) {
     const int s = i % kStages;
     if (wid == 0)
-      issue_stage<!kTotals && !kRLE, kH>(lane, tile_of(i), T, K, S.tc, A, S.meta[s], S.val[s], S.g[s],
-                                kH ? sH + (size_t)s * kTile : nullptr, &S.bar[s], pol_stream);
+      issue_stage<!kTotals && !kRLE, kH>(lane, tile_of(i), T, C, K, S.tc, A, S.meta[s], S.val[s], S.g[s],
+                                         kH ? sH + (size_t)s * kTileSpan : nullptr, &S.bar[s], pol_stream);
     cp_async_commit();
   };
   issue(0);
@@ -619,11 +633,11 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
     mbar_wait(&S.bar[s0], (uint32_t)((it / kStages) & 1));  // this tile's lists (TMA)
 
     // ---------------------------------------------------------------- this warp's chunk
-    const int ibase = tid * kItems;  // position in the tile
-    const long long base = M.p0 + ibase;
-    const long long cp0 = M.p0 + (long long)wid * kChunk;
-    const long long cp1 = min(cp0 + (long long)kChunk, M.p1);
-    if (cp0 < M.p1) {
+    if (wid < M.nch) {
+      const WarpMeta& W = M.w[wid];
+      const int ibase = W.off + lane * kItems;  // position in the stage
+      const long long cp0 = W.p0, cp1 = W.p1;
+      const long long base = cp0 + lane * kItems;
       float v[kItems];
       double g[kItems], h[kItems];
       int c[kItems];
@@ -636,9 +650,9 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
         // direct RLE: the values come from the runs covering this thread's entries; the
         // chunk index gives the runs holding the first entries of this chunk and the next one
         const Tables& tb = A.t.tb;
-        const int cg = (S.tc.use ? S.tc.chunk_start[M.a] : tb.chunk_start[M.a]) + M.u * kChunksPerTile + wid;
+        const int cg = t * kChunksPerTile + wid;
         int lo = tb.run_chunk[cg];
-        int hi = cp1 < M.colend ? tb.run_chunk[cg + 1] : tb.seg_run[M.sb + K] - 1;
+        int hi = cp1 < W.colend ? tb.run_chunk[cg + 1] : tb.seg_run[W.sb + K] - 1;
         while (lo < hi) {
           const int mid = (lo + hi + 1) >> 1;
           if (tb.run_pos[mid] <= base) lo = mid; else hi = mid - 1;
@@ -649,7 +663,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
 #pragma unroll
         for (int k = 0; k <= kItems; ++k) {
           const long long p = base + k;
-          if (p >= M.colend || p > cp1) { if (k < kItems) v[k] = 0.f; continue; }
+          if (p >= W.colend || p > cp1) { if (k < kItems) v[k] = 0.f; continue; }
           while (p >= rend) { ++r; rend = tb.run_pos[r] + tb.run_len[r]; rv = tb.run_val[r]; }
           if (k < kItems) v[k] = rv; else vnext = rv;
         }
@@ -658,8 +672,8 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
         const float4 v1 = *reinterpret_cast<const float4*>(&S.val[s0][ibase + 4]);
         v[0] = v0.x; v[1] = v0.y; v[2] = v0.z; v[3] = v0.w;
         v[4] = v1.x; v[5] = v1.y; v[6] = v1.z; v[7] = v1.w;
-        if (base + kItems < M.p1) vnext = S.val[s0][ibase + kItems];
-        else if (base + kItems < M.colend && base + kItems == M.p1) vnext = __ldg(A.t.val + M.p1);
+        const long long pn = base + kItems;  // the entry after this thread's items
+        if (pn < W.colend) vnext = pn < M.P1 ? S.val[s0][ibase + kItems] : __ldg(A.t.val + pn);
       } else {
 #pragma unroll
         for (int k = 0; k < kItems; ++k) v[k] = 0.f;
@@ -668,21 +682,22 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
       for (int k = 0; k < kItems; ++k) {
         if ((vm >> k) & 1) {
           g[k] = S.g[s0][ibase + k];
-          h[k] = kH ? sH[(size_t)s0 * kTile + ibase + k] : hess_of<HMODE>(g[k]);
+          h[k] = kH ? sH[(size_t)s0 * kTileSpan + ibase + k] : hess_of<HMODE>(g[k]);
         } else {
           g[k] = 0.0; h[k] = 0.0;
         }
       }
       const FXV cx = fxv_load(M.carry + 5 * wid);
       const SVf carry = SVf{from_fx(cx.g, Fg), from_fx(cx.h, Fh), cx.c, 0};
-      const long long* ss = M.seg_cached ? M.seg_s : (const long long*)(A.t.tb.seg_start + M.sb);
-      const long long* sc = M.seg_cached ? M.seg_c : (const long long*)(A.t.tb.seg_cnt + M.sb);
+      const bool seg_cached = K <= kSegCache;
+      const long long* ss = seg_cached ? M.seg_s[wid] : (const long long*)(A.t.tb.seg_start + W.sb);
+      const long long* sc = seg_cached ? M.seg_c[wid] : (const long long*)(A.t.tb.seg_cnt + W.sb);
 
       // ============================================================ fast path: the chunk lies
       // inside ONE segment and no value is missing -> plain scans, candidates ranked with one
       // Newton reciprocal, warp argmax, exact Eq. 2 only for the chunk's winner.
       bool done = false;
-      if (!kTotals && !kMissing && M.seg_cached) {
+      if (!kTotals && !kMissing && seg_cached) {
         int j0, j1;
         {
           int lo = 0, hi = K - 1;
@@ -734,14 +749,14 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
               if (sc2 > best) { best = sc2; bk = k; }
             }
           }
-          int bpos = bk >= 0 ? ibase + bk : INT_MAX;
+          int bpos = bk >= 0 ? lane * kItems + bk : INT_MAX;
 #pragma unroll
           for (int o = 16; o; o >>= 1) {
             const double ob = __shfl_xor_sync(0xffffffffu, best, o);
             const int op = __shfl_xor_sync(0xffffffffu, bpos, o);
             if (ob > best || (ob == best && op < bpos)) { best = ob; bpos = op; }
           }
-          if (bpos != INT_MAX && bpos / kItems == tid) {
+          if (bpos != INT_MAX && bpos / kItems == lane) {
             const int k = bpos % kItems;
             Rec r;
             r.GL = bg + g[k];
@@ -749,7 +764,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
             r.cntL = bc + c[k];
             r.gain = eq2_gain(r.GL, r.HL, Gt, Ht, lam, A.nodes.pterm[j]);
             r.value = v[k];
-            r.attr = A.t.a_base + M.a;
+            r.attr = A.t.a_base + W.a;
             r.dir = 0;
             r.node = j;
             r.epoch = epoch;
@@ -794,7 +809,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
 #pragma unroll
           for (int k = 0; k < kItems; ++k) {
             if (((vm & rem) >> k) & 1) {
-              const long long s = M.sb + sj[k];
+              const long long s = W.sb + sj[k];
               A.segPG_out[s] = g[k];
               A.segPH_out[s] = h[k];
             }
@@ -816,7 +831,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
             int bd = 0;
             if (cL >= 1 && Ct - cL >= 1) { best = eq2_gain(g[k], h[k], Gt, Ht, lam, pt); ok = true; }
             if (kMissing) {
-              const long long s = M.sb + j;
+              const long long s = W.sb + j;
               const int cM = Ct - (int)A.t.tb.seg_cnt[s];
               if (cM > 0) {
                 const double GM = Gt - A.segPG[s], HM = Ht - A.segPH[s];
@@ -834,13 +849,17 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
           // per-piece argmax inside the chunk (pieces = segments of the chunk): the item that ends
           // a piece walks back to the piece start; R12 order gain desc, value desc, dir low first.
           // The chunk's g slots of the stage are free now and hold the gains.
-          double* sgn = &S.g[s0][wid * kChunk];
-          const float* svv = &S.val[s0][wid * kChunk];
-          unsigned char* sfl = &S.flg[wid * kChunk];
+          double* sgn = &S.g[s0][W.off];
+          float* svv = &S.val[s0][W.off];
+          unsigned char* sfl = &S.flg[W.off];
           __syncwarp();
+          // (only the chunk's own entries: the chunks of a tile are packed, so slots past the
+          // chunk's end belong to the next chunk)
 #pragma unroll
           for (int k = 0; k < kItems; ++k) {
+            if (!((vm >> k) & 1)) continue;
             sgn[lane * kItems + k] = gn[k];
+            if (kRLE) svv[lane * kItems + k] = v[k];  // the stage holds no values with RLE
             sfl[lane * kItems + k] = (unsigned char)(((okm >> k) & 1) | (((dm >> k) & 1) << 1) |
                                                      (((hm >> k) & 1) << 2));
           }
@@ -868,13 +887,13 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
           __syncwarp();
 #pragma unroll
           for (int k = 0; k < kItems; ++k) {
-            if (!(sfl[lane * kItems + k] & 8)) continue;
+            if (!((vm >> k) & 1) || !(sfl[lane * kItems + k] & 8)) continue;
             const int j = sj[k];
-            const long long s = M.sb + j;
+            const long long s = W.sb + j;
             Rec r;
             r.gain = gn[k];
             r.value = v[k];
-            r.attr = A.t.a_base + M.a;
+            r.attr = A.t.a_base + W.a;
             r.dir = (dm >> k) & 1;
             r.node = j;
             r.epoch = epoch;
@@ -1008,60 +1027,51 @@ __device__ unsigned long long block_exscan_u64(unsigned long long x, unsigned lo
   return ex;
 }
 
-// Single thread block: places every child segment (stable, attribute-major, children in heap
-// order) and builds the next level's attribute / tile / chunk / segment tables.
-__global__ void __launch_bounds__(1024) k_part_plan(PlanArgs A) {
-  const int K = *A.Kp, Kn = *A.Knp, m = A.m;
-  if (!A.counted) {
-    // no missing values: every instance of a node is present in every attribute list
-    for (long long s = threadIdx.x; s < (long long)m * K; s += blockDim.x) {
-      const int c = A.cidx[s % K];
-      A.segH[s] = c >= 0 ? A.ncnt[c] : 0;
-      A.segL[s] = c >= 0 ? A.ncnt[c + 1] : 0;
-    }
-    __syncthreads();
-  }
-  // per attribute: exclusive (high, low) counts before each segment, and the child list length
-  for (int a = threadIdx.x; a < m; a += blockDim.x) {
+// Child placement (stable, attribute-major, children in heap order) and the next level's
+// attribute / chunk / segment tables, attribute-parallel:
+//   k_plan_attr  per attribute: (high, low) counts before each segment and the child list length
+//   (exact integer scan over the attributes of (padded length | chunks << 32))
+//   k_plan_seg   per attribute: list start, chunk start, every child segment's start and count
+__global__ void __launch_bounds__(kThreads) k_plan_attr(PlanArgs A) {
+  const int K = *A.Kp, m = A.m;
+  const int stride = gridDim.x * blockDim.x;
+  for (int a = blockIdx.x * blockDim.x + threadIdx.x; a <= m; a += stride) {
+    if (a == m) { A.el[2ll * m] = 0ull; A.el[2ll * m + 1] = 0ull; continue; }
     unsigned long long pre = 0;
     long long L = 0;
     for (int j = 0; j < K; ++j) {
       const long long s = (long long)a * K + j;
+      const int c = A.cidx[j];
+      if (!A.counted) {  // no missing values: every instance of a node is in every attribute list
+        A.segH[s] = c >= 0 ? A.ncnt[c] : 0;
+        A.segL[s] = c >= 0 ? A.ncnt[c + 1] : 0;
+      }
       const unsigned hi = (unsigned)A.segH[s], lo = (unsigned)A.segL[s];
       A.seg_pre[s] = pre;
       pre += (unsigned long long)hi | ((unsigned long long)lo << 32);
-      if (A.cidx[j] >= 0) L += (long long)hi + lo;
+      if (c >= 0) L += (long long)hi + lo;
     }
-    A.len_tmp[a] = L;
     A.nxt.col_len[a] = L;
+    A.el[2ll * a] = (unsigned long long)((L + 3) & ~3ll) | ((unsigned long long)((L + kChunk - 1) / kChunk) << 32);
+    A.el[2ll * a + 1] = 0ull;
   }
-  __syncthreads();
-  unsigned long long cpos = 0, ctile = 0, cchunk = 0, t1, t2, t3;
-  for (int base = 0; base < m; base += blockDim.x) {
-    const int a = base + threadIdx.x;
-    const unsigned long long L = a < m ? (unsigned long long)A.len_tmp[a] : 0ull;
-    const unsigned long long ep = block_exscan_u64((L + 3) & ~3ull, t1);
-    const unsigned long long et = block_exscan_u64((L + kTile - 1) / kTile, t2);
-    const unsigned long long ec = block_exscan_u64((L + kChunk - 1) / kChunk, t3);
-    if (a < m) {
-      A.nxt.col_start[a] = (int64_t)(cpos + ep);
-      A.nxt.tile_start[a] = (int32_t)(ctile + et);
-      A.nxt.chunk_start[a] = (int32_t)(cchunk + ec);
+}
+
+__global__ void __launch_bounds__(kThreads) k_plan_seg(PlanArgs A) {
+  const int K = *A.Kp, Kn = *A.Knp, m = A.m;
+  const int stride = gridDim.x * blockDim.x;
+  for (int a = blockIdx.x * blockDim.x + threadIdx.x; a <= m; a += stride) {
+    const unsigned long long ex = A.el[2ll * a];
+    const long long cs = (long long)(ex & 0xffffffffull);
+    const int ch = (int)(ex >> 32);
+    A.nxt.col_start[a] = cs;
+    A.nxt.chunk_start[a] = ch;
+    if (a == m) {
+      *A.nxt.C = ch;
+      *A.nxt.T = (ch + kChunksPerTile - 1) / kChunksPerTile;
+      continue;
     }
-    cpos += t1;
-    ctile += t2;
-    cchunk += t3;
-  }
-  if (threadIdx.x == 0) {
-    A.nxt.col_start[m] = (int64_t)cpos;
-    A.nxt.tile_start[m] = (int32_t)ctile;
-    A.nxt.chunk_start[m] = (int32_t)cchunk;
-    *A.nxt.T = (int32_t)ctile;
-    *A.nxt.C = (int32_t)cchunk;
-  }
-  __syncthreads();
-  for (int a = threadIdx.x; a < m; a += blockDim.x) {
-    long long r = A.nxt.col_start[a];
+    long long r = cs;
     for (int j = 0; j < K; ++j) {
       const int c = A.cidx[j];
       if (c < 0) continue;
@@ -1340,7 +1350,7 @@ size_t scatter_smem(bool h) { return sizeof(ScatterStage) * kWarps + (h ? sizeof
 
 size_t sf_smem(int hmode) {
   size_t b = (sizeof(SFSmem) + 127) & ~size_t(127);
-  if (hmode == kHGather) b += sizeof(double) * kStages * kTile;
+  if (hmode == kHGather) b += sizeof(double) * kStages * kTileSpan;
   return b;
 }
 
@@ -1438,8 +1448,12 @@ void LevelKernels::partition(const PartArgs& A, const PlanArgs& P, bool counted,
   GBDT_LAUNCH_CHECK();
   count_launch();
   launch_scan<false>(A.t.tb.C, A.ccnt, A.sgrp, A.cpre, groups, st);
-  k_part_plan<<<1, 1024, 0, st>>>(P);
+  const unsigned pg = (unsigned)std::max(1, std::min((P.m + kThreads) / kThreads, sms * 8));
+  k_plan_attr<<<pg, kThreads, 0, st>>>(P);
+  launch_scan<false>(P.mp1, P.el, P.egrp, P.el, P.egroups, st);
+  k_plan_seg<<<pg, kThreads, 0, st>>>(P);
   GBDT_LAUNCH_CHECK();
+  count_launch(2);
   if (rle) {
     if (with_h) k_part_scatter<true, true><<<grid_scatter[1], kThreads, scatter_smem(true), st>>>(A);
     else k_part_scatter<false, true><<<grid_scatter[0], kThreads, scatter_smem(false), st>>>(A);

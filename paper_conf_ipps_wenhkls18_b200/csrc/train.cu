@@ -364,6 +364,10 @@ struct ShardWork {
   unsigned long long *run_hl = nullptr, *rcnt = nullptr, *rfl = nullptr, *rsgrp = nullptr;
   int32_t* Rp1 = nullptr;
   unsigned rgroups = 1;
+  // attribute-parallel partition plan
+  unsigned long long *pel = nullptr, *pgrp = nullptr;
+  int32_t* mp1 = nullptr;
+  unsigned pgroups = 1;
 };
 
 struct PhaseTimer {
@@ -493,6 +497,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       q.take<Rec>(R);
       q.take<int32_t>(S); q.take<int32_t>(S); q.take<unsigned long long>(S); q.take<int64_t>(S); q.take<int64_t>(S);
       q.take<int64_t>(m); q.take<double>(S); q.take<double>(S); q.take<int>(4);
+      q.take<unsigned long long>(2 * (size_t)(m + 1)); q.take<unsigned long long>(2 * (size_t)LevelKernels::scan_groups(m + 1) + 8);
+      q.take<int32_t>(1);
     };
     Carve pq{nullptr};
     sz(pq);
@@ -524,6 +530,15 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     w.len_tmp = q.take<int64_t>(m);
     w.segPG = q.take<double>(S); w.segPH = q.take<double>(S);
     w.counters = q.take<int>(4);
+    w.pgroups = LevelKernels::scan_groups(m + 1);
+    w.pel = q.take<unsigned long long>(2 * (size_t)(m + 1));
+    w.pgrp = q.take<unsigned long long>(2 * (size_t)w.pgroups + 8);
+    w.mp1 = q.take<int32_t>(1);
+    {
+      const int32_t mp1 = m + 1;
+      GBDT_CUDA(cudaMemcpyAsync(w.mp1, &mp1, 4, cudaMemcpyHostToDevice, st));
+      GBDT_CUDA(cudaStreamSynchronize(st));
+    }
     if (sh.rle) {
       // child runs: every run splits in at most two, and there are never more runs than entries
       const int64_t Rcap = std::max<int64_t>(1, std::min<int64_t>(sh.runs * Kcap, sh.cap));
@@ -692,6 +707,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         PL.m = sh.m; PL.counted = ds.has_missing; PL.Kp = cur.K; PL.Knp = nxt.K; PL.cidx = cidx; PL.ncnt = nxt.cnt;
         PL.segH = w.segH; PL.segL = w.segL; PL.seg_pre = w.seg_pre;
         PL.out_hi = w.out_hi; PL.out_lo = w.out_lo; PL.len_tmp = w.len_tmp; PL.nxt = tn;
+        PL.el = w.pel; PL.egrp = w.pgrp; PL.egroups = w.pgroups; PL.mp1 = w.mp1;
         RunArgs RA;
         if (sh.rle) {
           RA.m = sh.m; RA.Kp = cur.K; RA.Knp = nxt.K; RA.cidx = cidx; RA.cur = tb; RA.nxt = tn;
