@@ -68,6 +68,7 @@ struct Tables {
   int64_t* seg_cnt = nullptr;     // [m*Kcap]
   int32_t* T = nullptr;           // [1] tiles at this level
   int32_t* C = nullptr;           // [1] chunks at this level
+  int32_t* chunk_attr = nullptr;  // [C] attribute of each chunk
   // RLE: the runs of segment s are [seg_run[s], seg_run[s+1]); run r covers list
   // positions [run_pos[r], run_pos[r] + run_len[r]) with value run_val[r]
   int32_t* seg_run = nullptr;     // [m*Kcap + 1]
@@ -104,6 +105,7 @@ struct Shard {
   DBuf val0, ins0;               // pristine root layout (padded)
   DBuf valw[2], insw[2];         // ping-pong level buffers
   DBuf root_tab;                 // root tables storage
+  DBuf root_chunk_attr;
   Tables root;
   std::vector<int64_t> h_col_len;  // host copy, unpadded lengths
   std::vector<int64_t> h_col_start;

@@ -316,6 +316,12 @@ void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices
     GBDT_CUDA(cudaMemcpyAsync(sh.root.T, &sh.T0, 4, cudaMemcpyHostToDevice, st));
     GBDT_CUDA(cudaMemcpyAsync(sh.root.chunk_start, cstart.data(), (m + 1) * 4, cudaMemcpyHostToDevice, st));
     GBDT_CUDA(cudaMemcpyAsync(sh.root.C, &sh.C0, 4, cudaMemcpyHostToDevice, st));
+    std::vector<int32_t> cattr((size_t)std::max(sh.C0, 1), 0);
+    for (int a = 0; a < m; ++a)
+      for (int c = cstart[a]; c < cstart[a + 1]; ++c) cattr[c] = a;
+    sh.root_chunk_attr.alloc(cattr.size() * 4, st);
+    sh.root.chunk_attr = sh.root_chunk_attr.as<int32_t>();
+    GBDT_CUDA(cudaMemcpyAsync(sh.root.chunk_attr, cattr.data(), cattr.size() * 4, cudaMemcpyHostToDevice, st));
     GBDT_CUDA(cudaStreamSynchronize(st));  // host vectors above must outlive the copies
     if (m == 0 || sh.nnz == 0) continue;
 

@@ -37,9 +37,7 @@ namespace {
 
 constexpr int kStages = 3;
 constexpr int kSegCache = 32;     // segment starts/counts of a tile's attribute cached per stage
-constexpr int kCtaK = 64;         // per-CTA node-best table when K <= kCtaK
 constexpr int kTabCache = 64;     // attribute tables cached in smem when m <= kTabCache
-constexpr int kPieceList = 64;
 constexpr int kChunksPerTile = kTile / kChunk;  // 8 == kWarps
 constexpr int kScanGroup = 1024;  // elements per CTA in the 3-phase scans
 static_assert(kChunksPerTile == kWarps, "one warp per chunk of a tile");
@@ -176,7 +174,7 @@ struct ChunkMeta {
 __device__ __forceinline__ ChunkMeta chunk_meta(const TabCache& tc, const TileArgs& A, int K, int c) {
   const bool u = tc.use;
   const int* cs = u ? tc.chunk_start : A.tb.chunk_start;
-  const int a = find_attr(cs, A.m, c);
+  const int a = A.tb.chunk_attr[c];
   const long long c0 = u ? tc.col_start[a] : A.tb.col_start[a];
   const long long cl = u ? tc.col_len[a] : A.tb.col_len[a];
   const int k = c - cs[a];
@@ -548,39 +546,35 @@ __device__ __forceinline__ void issue_stage(int lane, int t, int T, int C, int K
   }
 }
 
+constexpr int kWarpK = 32;  // per-warp node-best tables when K <= kWarpK
 struct SFSmem {
-  float val[kStages][kTile];
-  double g[kStages][kTile];
+  float val[kStages][kTileSpan];
+  double g[kStages][kTileSpan];
   StageMeta meta[kStages];
   unsigned long long bar[kStages];
-  int npw;
-  unsigned char flg[kTile];  // general path: per-item candidate flags of the current tile
-  unsigned long long cg[kCtaK], ct[kCtaK];
-  Rec cb[kCtaK];
-  Rec pw[kPieceList];
+  unsigned char flg[kTileSpan];  // general path: winner marks of the current tile
+  // Per-warp best record per node.  A chunk lies in one attribute, whose segments belong to
+  // distinct nodes, so a warp never has two candidates for one node at once: no atomics.
+  unsigned long long wg[kWarps][kWarpK];
+  Rec wb[kWarps][kWarpK];
   TabCache tc;
 };
 
-__device__ __forceinline__ void cta_merge(SFSmem& S) {
-  const int n = min(S.npw, kPieceList);
-  for (int q = 0; q < n; ++q) {
-    const Rec& r = S.pw[q];
-    const unsigned long long gk = gain_key(r.gain), tk = tie_key(r.attr, r.value, r.dir);
-    const int j = r.node;
-    if (gk > S.cg[j] || (gk == S.cg[j] && tk < S.ct[j])) { S.cg[j] = gk; S.ct[j] = tk; S.cb[j] = r; }
-  }
-  S.npw = 0;
+__device__ __forceinline__ bool rec_better(unsigned long long gk, const Rec& r, unsigned long long gk0, const Rec& r0) {
+  return gk > gk0 || (gk == gk0 && tie_key(r.attr, r.value, r.dir) < tie_key(r0.attr, r0.value, r0.dir));
 }
 
-__device__ __forceinline__ void push_record(SFSmem& S, const SplitArgs& A, const Rec& r, bool cta_table) {
-  int slot = kPieceList;
-  if (cta_table) slot = atomicAdd(&S.npw, 1);
-  if (slot < kPieceList) {
-    S.pw[slot] = r;
+__device__ __forceinline__ void push_record(SFSmem& S, const SplitArgs& A, const Rec& r, bool warp_table, int wid) {
+  const unsigned long long gk = gain_key(r.gain);
+  if (warp_table) {
+    if (rec_better(gk, r, S.wg[wid][r.node], S.wb[wid][r.node])) {
+      S.wg[wid][r.node] = gk;
+      S.wb[wid][r.node] = r;
+    }
   } else {
     const int gs = atomicAdd(A.nrec, 1);
     A.rec[gs] = r;
-    atomicMax(A.gkey + r.node, gain_key(r.gain));
+    atomicMax(A.gkey + r.node, gk);
   }
 }
 
@@ -598,7 +592,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
   if (K == 0 || T == 0) return;
   const int epoch = *A.epochp;
   const int Fg = A.fx[0], Fh = A.fx[1];
-  const bool cta_table = !kTotals && K <= kCtaK;
+  const bool warp_table = !kTotals && K <= kWarpK;
   const double lam = A.lam;
   const unsigned long long pol_stream = policy_evict_first();
   // static round-robin tiles: there are no inter-CTA dependencies (carries come from the scans)
@@ -606,10 +600,9 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
   if (tid == 0) {
     for (int s = 0; s < kStages; ++s) mbar_init(&S.bar[s], 1);
     fence_mbar_init();
-    S.npw = 0;
   }
   tab_load(S.tc, A.t);
-  for (int j = tid; j < kCtaK; j += kThreads) { S.cg[j] = 0ull; S.ct[j] = ~0ull; }
+  for (int j = tid; j < kWarps * kWarpK; j += kThreads) S.wg[j / kWarpK][j % kWarpK] = 0ull;
   __syncthreads();
   auto issue = [&](int i) {
     const int s = i % kStages;
@@ -626,7 +619,6 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
     issue(it + 2);
     cp_async_wait<2>();  // this tile's carries / segment table (cp.async)
     __syncthreads();
-    if (tid == 0 && S.npw) cta_merge(S);
     const StageMeta& M = S.meta[s0];
     const int t = M.t;
     if (t >= T) break;
@@ -770,7 +762,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
             r.epoch = epoch;
             r.shard = A.shard;
             r.pos = base + k;
-            push_record(S, A, r, cta_table);
+            push_record(S, A, r, warp_table, wid);
           }
         }
       }
@@ -846,48 +838,44 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
             dm |= (unsigned)bd << k;
             okm |= (unsigned)ok << k;
           }
-          // per-piece argmax inside the chunk (pieces = segments of the chunk): the item that ends
-          // a piece walks back to the piece start; R12 order gain desc, value desc, dir low first.
-          // The chunk's g slots of the stage are free now and hold the gains.
-          double* sgn = &S.g[s0][W.off];
-          float* svv = &S.val[s0][W.off];
+          // per-piece argmax inside the chunk (pieces = the chunk's segments): segmented max-scan
+          // over the warp of (gain, position).  Inside a segment the candidates are distinct values
+          // in descending order, so "earlier position" is R12's "larger value" (the direction tie
+          // was settled per item, low first).  The end item of every piece marks its winner.
           unsigned char* sfl = &S.flg[W.off];
-          __syncwarp();
-          // (only the chunk's own entries: the chunks of a tile are packed, so slots past the
-          // chunk's end belong to the next chunk)
+          double lg = -INFINITY;
+          int lq = INT_MAX, lf = 0;
 #pragma unroll
           for (int k = 0; k < kItems; ++k) {
             if (!((vm >> k) & 1)) continue;
-            sgn[lane * kItems + k] = gn[k];
-            if (kRLE) svv[lane * kItems + k] = v[k];  // the stage holds no values with RLE
-            sfl[lane * kItems + k] = (unsigned char)(((okm >> k) & 1) | (((dm >> k) & 1) << 1) |
-                                                     (((hm >> k) & 1) << 2));
+            sfl[lane * kItems + k] = 0;
+            if ((hm >> k) & 1) { lg = -INFINITY; lq = INT_MAX; lf = 1; }
+            if (((okm >> k) & 1) && gn[k] > lg) { lg = gn[k]; lq = lane * kItems + k; }
           }
-          __syncwarp();
 #pragma unroll
-          for (int k = 0; k < kItems; ++k) {
-            if (!(((vm & pem) >> k) & 1)) continue;
-            int q = lane * kItems + k, bq = -1;
-            for (;;) {
-              const int fl = sfl[q];
-              if (fl & 1) {
-                if (bq < 0) {
-                  bq = q;
-                } else {
-                  const double a = sgn[q], b = sgn[bq];
-                  const float va = svv[q], vb = svv[bq];
-                  if (a > b || (a == b && (va > vb || (va == vb && ((fl >> 1) & 1) < ((sfl[bq] >> 1) & 1))))) bq = q;
-                }
-              }
-              if ((fl & 4) || q == 0) break;
-              --q;
+          for (int o = 1; o < 32; o <<= 1) {
+            const double yg = __shfl_up_sync(0xffffffffu, lg, o);
+            const int yq = __shfl_up_sync(0xffffffffu, lq, o), yf = __shfl_up_sync(0xffffffffu, lf, o);
+            if (lane >= o) {
+              if (!lf && (yg > lg || (yg == lg && yq < lq))) { lg = yg; lq = yq; }
+              lf |= yf;
             }
-            if (bq >= 0) sfl[bq] |= 8;  // each piece marks exactly one item
+          }
+          double cg_ = __shfl_up_sync(0xffffffffu, lg, 1);
+          int cq = __shfl_up_sync(0xffffffffu, lq, 1);
+          if (lane == 0) { cg_ = -INFINITY; cq = INT_MAX; }
+          __syncwarp();
+#pragma unroll
+          for (int k = 0; k < kItems; ++k) {
+            if (!((vm >> k) & 1)) continue;
+            if ((hm >> k) & 1) { cg_ = -INFINITY; cq = INT_MAX; }
+            if (((okm >> k) & 1) && gn[k] > cg_) { cg_ = gn[k]; cq = lane * kItems + k; }
+            if (((pem >> k) & 1) && cq != INT_MAX) sfl[cq] = 1;  // each piece marks one item
           }
           __syncwarp();
 #pragma unroll
           for (int k = 0; k < kItems; ++k) {
-            if (!((vm >> k) & 1) || !(sfl[lane * kItems + k] & 8)) continue;
+            if (!((vm >> k) & 1) || !sfl[lane * kItems + k]) continue;
             const int j = sj[k];
             const long long s = W.sb + j;
             Rec r;
@@ -907,23 +895,24 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
             } else {
               r.GL = g[k]; r.HL = h[k]; r.cntL = c[k];
             }
-            push_record(S, A, r, cta_table);
+            push_record(S, A, r, warp_table, wid);
           }
         }
       }
     }
     __syncthreads();
   }
-  // flush the CTA's node bests
-  if (cta_table) {
+  // flush the CTA's node bests (merge of the warp tables)
+  if (warp_table) {
     __syncthreads();
-    if (tid == 0 && S.npw) cta_merge(S);
-    __syncthreads();
-    for (int j = tid; j < K; j += kThreads) {
-      if (S.cg[j]) {
+    if (tid < K) {
+      int bw = -1;
+      for (int w = 0; w < kWarps; ++w)
+        if (S.wg[w][tid] && (bw < 0 || rec_better(S.wg[w][tid], S.wb[w][tid], S.wg[bw][tid], S.wb[bw][tid]))) bw = w;
+      if (bw >= 0) {
         const int gs = atomicAdd(A.nrec, 1);
-        A.rec[gs] = S.cb[j];
-        atomicMax(A.gkey + j, S.cg[j]);
+        A.rec[gs] = S.wb[bw][tid];
+        atomicMax(A.gkey + tid, S.wg[bw][tid]);
       }
     }
   }
@@ -1087,6 +1076,13 @@ __global__ void __launch_bounds__(kThreads) k_plan_seg(PlanArgs A) {
       r += lo;
     }
   }
+}
+
+// attribute of every chunk of the next level (the largest a with chunk_start[a] <= c)
+__global__ void __launch_bounds__(kThreads) k_chunk_attr(PlanArgs A) {
+  const int C = *A.nxt.C, m = A.m;
+  for (int c = blockIdx.x * blockDim.x + threadIdx.x; c < C; c += gridDim.x * blockDim.x)
+    A.nxt.chunk_attr[c] = find_attr(A.nxt.chunk_start, m, c);
 }
 
 // Stable scatter ("Scatter"), one warp per chunk: out(e) = out_base(seg, side) + rank of
@@ -1452,8 +1448,9 @@ void LevelKernels::partition(const PartArgs& A, const PlanArgs& P, bool counted,
   k_plan_attr<<<pg, kThreads, 0, st>>>(P);
   launch_scan<false>(P.mp1, P.el, P.egrp, P.el, P.egroups, st);
   k_plan_seg<<<pg, kThreads, 0, st>>>(P);
+  k_chunk_attr<<<(unsigned)(sms * 8), kThreads, 0, st>>>(P);
   GBDT_LAUNCH_CHECK();
-  count_launch(2);
+  count_launch(3);
   if (rle) {
     if (with_h) k_part_scatter<true, true><<<grid_scatter[1], kThreads, scatter_smem(true), st>>>(A);
     else k_part_scatter<false, true><<<grid_scatter[0], kThreads, scatter_smem(false), st>>>(A);

@@ -488,7 +488,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     auto sz = [&](Carve& q) {
       for (int b = 0; b < 2; ++b) {
         q.take<int64_t>(m + 1); q.take<int64_t>(m); q.take<int32_t>(m + 1); q.take<int32_t>(m + 1);
-        q.take<int64_t>(S); q.take<int64_t>(S); q.take<int32_t>(1); q.take<int32_t>(1);
+        q.take<int64_t>(S); q.take<int64_t>(S); q.take<int32_t>(1); q.take<int32_t>(1); q.take<int32_t>(C0);
       }
       q.take<unsigned long long>(5 * C0); q.take<unsigned long long>(5 * C0);
       q.take<unsigned long long>(2 * C0); q.take<unsigned long long>(2 * C0);
@@ -510,6 +510,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       w.tab[b].tile_start = q.take<int32_t>(m + 1); w.tab[b].chunk_start = q.take<int32_t>(m + 1);
       w.tab[b].seg_start = q.take<int64_t>(S); w.tab[b].seg_cnt = q.take<int64_t>(S);
       w.tab[b].T = q.take<int32_t>(1); w.tab[b].C = q.take<int32_t>(1);
+      w.tab[b].chunk_attr = q.take<int32_t>(C0);
     }
     w.cagg = q.take<unsigned long long>(5 * C0); w.carry = q.take<unsigned long long>(5 * C0);
     w.ccnt = q.take<unsigned long long>(2 * C0); w.cpre = q.take<unsigned long long>(2 * C0);
