@@ -31,8 +31,22 @@ struct TileArgs {
 //   2: general: h gathered too
 enum { kHConst2 = 0, kHFromG = 1, kHGather = 2 };
 
+// Per-chunk descriptor written by k_chunk_agg for the split-find kernels (32 bytes).
+struct ChunkDesc {
+  long long p0;   // first entry
+  long long se;   // end of the segment holding the chunk's first entry
+  int len;        // entries
+  int a;          // attribute (shard-local)
+  int jf;         // bits 0-15: segment (node) j of the first entry; 16: the chunk starts at that
+                  // segment's start; 17: the chunk lies in that one segment; 18: vnext valid
+  float vnext;    // value of the entry after the chunk when it is in the same attribute (plain)
+};
+constexpr int kDescHead0 = 1 << 16, kDescSingle = 1 << 17, kDescNext = 1 << 18;
+
 struct SplitArgs {
   TileArgs t;
+  ChunkDesc* desc;       // [C]
+  int rle;               // the level's values live in runs (t.val is not maintained)
   const double* g;       // per instance
   const double* h;       // per instance (mode 2)
   double* glist;         // per list entry: g of the entry's instance (written by k_tile_agg)
@@ -123,8 +137,8 @@ struct RunArgs {
 // levels.cu launchers
 struct LevelKernels {
   int sms = 148;
-  unsigned grid_sf[3][2] = {{0}};  // [hmode][missing]
-  unsigned grid_tot[3] = {0};
+  unsigned grid_fast[3][2] = {{0}};  // [hmode][rle]
+  unsigned grid_gen = 0;
   unsigned grid_agg[3] = {0};
   unsigned grid_scatter[2] = {0}, grid_count = 0, grid_agg_list[3] = {0};
   void init(int device);

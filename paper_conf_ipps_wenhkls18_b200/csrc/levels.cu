@@ -299,6 +299,28 @@ __global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
     float vd[kItems];
     assign_segments<false>((const long long*)(A.t.tb.seg_start + M.sb), (const long long*)(A.t.tb.seg_cnt + M.sb),
                            p1, K, base, vm, vd, 0.f, sj, hm, pem, rem);
+    {  // the chunk's descriptor: its first entry's segment, and whether the chunk stays in it
+      const int len = (int)(p1 - M.p0);
+      const int ll = (len - 1) / kItems, lk = (len - 1) % kItems;
+      int jl = 0;
+#pragma unroll
+      for (int k = 0; k < kItems; ++k)
+        if (k == lk) jl = sj[k];
+      jl = __shfl_sync(0xffffffffu, jl, ll);
+      if (lane == 0) {
+        const int j0 = sj[0];
+        const long long ss0 = A.t.tb.seg_start[M.sb + j0];
+        const long long colend = A.t.tb.col_start[M.a] + A.t.tb.col_len[M.a];
+        ChunkDesc d;
+        d.p0 = M.p0;
+        d.se = ss0 + A.t.tb.seg_cnt[M.sb + j0];
+        d.len = len;
+        d.a = M.a;
+        d.jf = j0 | (ss0 == M.p0 ? kDescHead0 : 0) | (jl == j0 ? kDescSingle : 0) | (p1 < colend ? kDescNext : 0);
+        d.vnext = (p1 < colend && !A.rle) ? A.t.val[p1] : 0.f;
+        A.desc[c] = d;
+      }
+    }
     SVf run = svf_zero();
 #pragma unroll
     for (int k = 0; k < kItems; ++k) {
@@ -478,444 +500,502 @@ __global__ void __launch_bounds__(kThreads) k_scan3(const int32_t* __restrict__ 
 }
 
 // ============================================================================ a3-a6: split find
-// A tile is 8 CONSECUTIVE chunks of the level (chunks 8t .. 8t+7), which may belong to different
-// attributes: chunks are attribute-aligned, tiles are not, so thousands of short attribute lists
-// (C4: ~20 entries each) share one tile instead of each occupying a mostly empty one (a3,
-// many-segment load balance).  The chunks of a tile are contiguous in the list buffer up to the
-// <= 3-entry padding between attributes, so one bulk copy per list stages the whole tile.
-constexpr int kTileSpan = kTile + 4 * kChunksPerTile;  // entries a stage can hold
-struct WarpMeta {
-  long long p0, p1, colend, sb;
-  int a, off;  // attribute; chunk offset in the stage
-};
-struct StageMeta {
-  long long P0, P1;
-  int t, nch;
-  WarpMeta w[kChunksPerTile];
-  unsigned long long carry[kChunksPerTile * 5];
-  long long seg_s[kChunksPerTile][kSegCache];
-  long long seg_c[kChunksPerTile][kSegCache];
+// Two kernels per level (both warp-granular: a warp owns one 256-entry chunk at a time and never
+// waits for another warp):
+//   k_sf_fast  every chunk that lies inside ONE segment (nearly all chunks of dense data): the
+//              chunk's value list and g-list stream through a per-warp 2-stage shared-memory ring
+//              fed by TMA 1-D bulk copies (UBLKCP + mbarrier, L2 evict-first); plain warp scans,
+//              candidates ranked by a Newton-reciprocal score, exact Eq. 2 for the chunk's winner
+//   k_sf_gen   every other chunk (chunks that cross segment boundaries; all chunks when values are
+//              missing, where both default directions need the segments' present totals):
+//              segmented scans and a log-time per-segment argmax, direct vector loads
+// Node bests are merged per CTA in shared memory (a per-node lock; posts are rare: one per chunk
+// and segment) and flushed once per CTA.
+constexpr int kWarpK = 32;  // CTA node tables when K <= kWarpK (d <= 6); else global records
+
+struct NodeBest {
+  unsigned long long gk[kWarpK];
+  Rec rec[kWarpK];
+  double G[kWarpK], H[kWarpK], P[kWarpK];
+  int C[kWarpK];
+  int lock[kWarpK];
 };
 
-// warp 0: lanes 0..7 locate the tile's chunks; lane 0 issues the TMA bulk loads of the tile's lists
-// into a stage; the lanes fetch the chunk carries and the segment tables with cp.async.
-template <bool kVal, bool kH>
-__device__ __forceinline__ void issue_stage(int lane, int t, int T, int C, int K, const TabCache& tc,
-                                            const SplitArgs& A, StageMeta& M, float* sval, double* sg,
-                                            double* sh, unsigned long long* bar, unsigned long long pol) {
-  if (lane == 0) M.t = t;
-  if (t >= T) return;
-  const int c0 = t * kChunksPerTile;
-  const int nch = min(kChunksPerTile, C - c0);
-  long long p0 = 0, p1 = 0;
-  if (lane < nch) {
-    const ChunkMeta cm = chunk_meta(tc, A.t, K, c0 + lane);
-    p0 = cm.p0;
-    p1 = cm.p1;
-    WarpMeta& W = M.w[lane];
-    W.p0 = cm.p0;
-    W.p1 = cm.p1;
-    W.colend = (tc.use ? tc.col_start[cm.a] + tc.col_len[cm.a] : A.t.tb.col_start[cm.a] + A.t.tb.col_len[cm.a]);
-    W.sb = cm.sb;
-    W.a = cm.a;
-  }
-  const long long P0 = __shfl_sync(0xffffffffu, p0, 0);
-  const long long P1 = __shfl_sync(0xffffffffu, p1, nch - 1);
-  if (lane < nch) M.w[lane].off = (int)(p0 - P0);
-  if (lane == 0) {
-    M.P0 = P0;
-    M.P1 = P1;
-    M.nch = nch;
-    const uint32_t n = (uint32_t)(((P1 + 3) & ~3ll) - P0);  // 16-byte granules inside the padding
-    fence_proxy_async();
-    mbar_arrive_expect_tx(bar, (kVal ? 4u * n : 0u) + 8u * n + (kH ? 8u * n : 0u));
-    if (kVal) tma_load_1d(sval, A.t.val + P0, 4u * n, bar, pol);
-    tma_load_1d(sg, A.glist + P0, 8u * n, bar, pol);
-    if (kH) tma_load_1d(sh, A.hlist + P0, 8u * n, bar, pol);
-  }
-  for (int q = lane; q < nch * 5; q += 32) cp_async8(&M.carry[q], A.carry + 5ll * c0 + q, pol);
-  if (K <= kSegCache) {
-    const long long sbl = lane < nch ? M.w[lane].sb : 0ll;
-    for (int w = 0; w < nch; ++w) {
-      const long long sb = __shfl_sync(0xffffffffu, sbl, w);
-      if (lane < K) {
-        cp_async8(&M.seg_s[w][lane], A.t.tb.seg_start + sb + lane, pol);
-        cp_async8(&M.seg_c[w][lane], A.t.tb.seg_cnt + sb + lane, pol);
-      }
-    }
-  }
+struct NodeV {
+  double G, H, P;
+  int C;
+};
+__device__ __forceinline__ NodeV node_v(const NodeBest& B, const SplitArgs& A, int K, int j) {
+  if (K <= kWarpK) return NodeV{B.G[j], B.H[j], B.P[j], B.C[j]};
+  return NodeV{A.nodes.G[j], A.nodes.H[j], A.nodes.pterm[j], A.nodes.cnt[j]};
 }
 
-constexpr int kWarpK = 32;  // per-warp node-best tables when K <= kWarpK
-struct SFSmem {
-  float val[kStages][kTileSpan];
-  double g[kStages][kTileSpan];
-  StageMeta meta[kStages];
-  unsigned long long bar[kStages];
-  unsigned char flg[kTileSpan];  // general path: winner marks of the current tile
-  // Per-warp best record per node.  A chunk lies in one attribute, whose segments belong to
-  // distinct nodes, so a warp never has two candidates for one node at once: no atomics.
-  unsigned long long wg[kWarps][kWarpK];
-  Rec wb[kWarps][kWarpK];
-  TabCache tc;
-};
+__device__ __forceinline__ void nb_init(NodeBest& B, const SplitArgs& A, int K) {
+  for (int j = threadIdx.x; j < kWarpK; j += blockDim.x) {
+    B.gk[j] = 0ull;
+    B.lock[j] = 0;
+    if (j < K) { B.G[j] = A.nodes.G[j]; B.H[j] = A.nodes.H[j]; B.P[j] = A.nodes.pterm[j]; B.C[j] = A.nodes.cnt[j]; }
+  }
+}
 
 __device__ __forceinline__ bool rec_better(unsigned long long gk, const Rec& r, unsigned long long gk0, const Rec& r0) {
   return gk > gk0 || (gk == gk0 && tie_key(r.attr, r.value, r.dir) < tie_key(r0.attr, r0.value, r0.dir));
 }
 
-__device__ __forceinline__ void push_record(SFSmem& S, const SplitArgs& A, const Rec& r, bool warp_table, int wid) {
+// R12 order merge of one candidate record into the CTA table (or the global record list)
+__device__ __forceinline__ void post_record(NodeBest& B, const SplitArgs& A, int K, const Rec& r) {
   const unsigned long long gk = gain_key(r.gain);
-  if (warp_table) {
-    if (rec_better(gk, r, S.wg[wid][r.node], S.wb[wid][r.node])) {
-      S.wg[wid][r.node] = gk;
-      S.wb[wid][r.node] = r;
-    }
-  } else {
+  if (K > kWarpK) {
     const int gs = atomicAdd(A.nrec, 1);
     A.rec[gs] = r;
     atomicMax(A.gkey + r.node, gk);
+    return;
+  }
+  const int j = r.node;
+  if (gk < *reinterpret_cast<volatile unsigned long long*>(&B.gk[j])) return;  // keys only grow
+  while (atomicCAS(&B.lock[j], 0, 1) != 0) {
+  }
+  __threadfence_block();
+  if (rec_better(gk, r, B.gk[j], B.rec[j])) {
+    B.rec[j] = r;
+    B.gk[j] = gk;
+  }
+  __threadfence_block();
+  atomicExch(&B.lock[j], 0);
+}
+
+__device__ __forceinline__ void nb_flush(NodeBest& B, const SplitArgs& A, int K) {
+  if (K > kWarpK) return;
+  __syncthreads();
+  for (int j = threadIdx.x; j < K; j += blockDim.x) {
+    if (B.gk[j]) {
+      const int gs = atomicAdd(A.nrec, 1);
+      A.rec[gs] = B.rec[j];
+      atomicMax(A.gkey + j, B.gk[j]);
+    }
   }
 }
 
-template <int HMODE, bool kMissing, bool kTotals, bool kRLE>
-__global__ void __launch_bounds__(kThreads, 2) k_sf(SplitArgs A) {
-  extern __shared__ __align__(128) unsigned char smem_raw[];
-  SFSmem& S = *reinterpret_cast<SFSmem*>(smem_raw);
-  double* sH = reinterpret_cast<double*>(smem_raw + ((sizeof(SFSmem) + 127) & ~size_t(127)));  // mode 2
-  constexpr bool kH = HMODE == kHGather;
+// rank score of a split: GL^2/(HL+l) + GR^2/(HR+l) = 2 Eq. 2 + G^2/(H+l); one Newton reciprocal
+__device__ __forceinline__ double split_score(double GL, double HL, double G, double H, double lam) {
+  const double dl = HL + lam, dr = (H - HL) + lam, GR = G - GL;
+  return __dmul_rn(__fma_rn(GL * GL, dr, __dmul_rn(GR * GR, dl)), rcp_nr(__dmul_rn(dl, dr)));
+}
 
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+// value of list position p from the level's runs (RLE): the run holding it, searched between
+// the runs holding the first entries of chunk cg and of the next chunk
+__device__ __forceinline__ void rle_values(const Tables& tb, int cg, long long p0, long long len, bool has_next,
+                                           long long base, int K, int sb_end_seg, float* v, float& vnext) {
+  int lo = tb.run_chunk[cg];
+  int hi = has_next ? tb.run_chunk[cg + 1] : tb.seg_run[sb_end_seg] - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (tb.run_pos[mid] <= base) lo = mid; else hi = mid - 1;
+  }
+  int r = lo;
+  long long rend = tb.run_pos[r] + tb.run_len[r];
+  float rv = tb.run_val[r];
+  const long long pend = p0 + len + (has_next ? 1 : 0);
+#pragma unroll
+  for (int k = 0; k <= kItems; ++k) {
+    const long long p = base + k;
+    if (p >= pend) { if (k < kItems) v[k] = 0.f; continue; }
+    while (p >= rend) { ++r; rend = tb.run_pos[r] + tb.run_len[r]; rv = tb.run_val[r]; }
+    if (k < kItems) v[k] = rv; else vnext = rv;
+  }
+}
+
+// ---------------------------------------------------------------------------- k_sf_fast
+constexpr int kFS = 2;  // stages per warp
+template <bool kH>
+struct __align__(16) FastWarp {
+  float val[kFS][kChunk + 4];  // + the value after the chunk
+  double g[kFS][kChunk];
+  double h[kH ? kFS : 1][kH ? kChunk : 2];
+  unsigned long long carry[kFS][6];
+  ChunkDesc d[4];
+  unsigned long long bar[kFS];
+};
+template <bool kH>
+struct FastSmem {
+  FastWarp<kH> w[kWarps];
+  NodeBest B;
+};
+
+template <int HMODE, bool kRLE>
+__global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
+  constexpr bool kH = HMODE == kHGather;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  FastSmem<kH>& S = *reinterpret_cast<FastSmem<kH>*>(smem_raw);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int K = *A.t.Kp;
   const int C = *A.t.tb.C;
-  const int T = (C + kChunksPerTile - 1) / kChunksPerTile;
-  if (K == 0 || T == 0) return;
+  if (K == 0 || C == 0) return;
   const int epoch = *A.epochp;
   const int Fg = A.fx[0], Fh = A.fx[1];
-  const bool warp_table = !kTotals && K <= kWarpK;
   const double lam = A.lam;
-  const unsigned long long pol_stream = policy_evict_first();
-  // static round-robin tiles: there are no inter-CTA dependencies (carries come from the scans)
-  auto tile_of = [&](int i) { return (int)blockIdx.x + i * (int)gridDim.x; };
-  if (tid == 0) {
-    for (int s = 0; s < kStages; ++s) mbar_init(&S.bar[s], 1);
+  FastWarp<kH>& W = S.w[wid];
+  nb_init(S.B, A, K);
+  if (lane == 0) {
+    for (int s = 0; s < kFS; ++s) mbar_init(&W.bar[s], 1);
     fence_mbar_init();
   }
-  tab_load(S.tc, A.t);
-  for (int j = tid; j < kWarps * kWarpK; j += kThreads) S.wg[j / kWarpK][j % kWarpK] = 0ull;
   __syncthreads();
-  auto issue = [&](int i) {
-    const int s = i % kStages;
-    if (wid == 0)
-      issue_stage<!kTotals && !kRLE, kH>(lane, tile_of(i), T, C, K, S.tc, A, S.meta[s], S.val[s], S.g[s],
-                                         kH ? sH + (size_t)s * kTileSpan : nullptr, &S.bar[s], pol_stream);
-    cp_async_commit();
+  const int NW = gridDim.x * kWarps;
+  const int gw = blockIdx.x * kWarps + wid;
+  const unsigned long long pol = policy_evict_first();
+  auto chunk = [&](int i) { return gw + i * NW; };
+  // descriptor (and carry) prefetch into the warp's rings
+  auto fetch = [&](int i, bool with_desc, bool with_carry) {
+    const int c = chunk(i);
+    if (c < C) {
+      if (with_desc && lane < 4) cp_async8(reinterpret_cast<unsigned long long*>(&W.d[i & 3]) + lane,
+                                          reinterpret_cast<const unsigned long long*>(A.desc + c) + lane, pol);
+      if (with_carry && lane < 5) cp_async8(&W.carry[i & 1][lane], A.carry + 5ll * c + lane, pol);
+    }
   };
+  // TMA of chunk i's lists into stage i & 1 (single-segment chunks only)
+  auto issue = [&](int i) {
+    const int c = chunk(i);
+    if (lane == 0 && c < C) {
+      const ChunkDesc& d = W.d[i & 3];
+      if (d.jf & kDescSingle) {
+        const int st = i & 1;
+        const uint32_t n = (uint32_t)((d.len + 3) & ~3);
+        fence_proxy_async();
+        mbar_arrive_expect_tx(&W.bar[st], (kRLE ? 0u : 4u * n) + 8u * n + (kH ? 8u * n : 0u));
+        if (!kRLE) tma_load_1d(W.val[st], A.t.val + d.p0, 4u * n, &W.bar[st], pol);
+        tma_load_1d(W.g[st], A.glist + d.p0, 8u * n, &W.bar[st], pol);
+        if (kH) tma_load_1d(W.h[st], A.hlist + d.p0, 8u * n, &W.bar[st], pol);
+      }
+    }
+  };
+  fetch(0, true, true);
+  fetch(1, true, true);
+  fetch(2, true, false);
+  cp_async_commit();
+  cp_async_wait<0>();
+  __syncwarp();
   issue(0);
   issue(1);
-
-  for (int it = 0;; ++it) {
-    const int s0 = it % kStages;
-    issue(it + 2);
-    cp_async_wait<2>();  // this tile's carries / segment table (cp.async)
-    __syncthreads();
-    const StageMeta& M = S.meta[s0];
-    const int t = M.t;
-    if (t >= T) break;
-    mbar_wait(&S.bar[s0], (uint32_t)((it / kStages) & 1));  // this tile's lists (TMA)
-
-    // ---------------------------------------------------------------- this warp's chunk
-    if (wid < M.nch) {
-      const WarpMeta& W = M.w[wid];
-      const int ibase = W.off + lane * kItems;  // position in the stage
-      const long long cp0 = W.p0, cp1 = W.p1;
-      const long long base = cp0 + lane * kItems;
-      float v[kItems];
-      double g[kItems], h[kItems];
-      int c[kItems];
-      unsigned vm = 0;
-      float vnext = 0.f;
+  uint32_t ph = 0;
+  for (int i = 0; chunk(i) < C; ++i) {
+    const int st = i & 1;
+    const ChunkDesc& d = W.d[i & 3];
+    const int jf = d.jf;
+    if (jf & kDescSingle) {
+      mbar_wait(&W.bar[st], (ph >> st) & 1);
+      ph ^= 1u << st;
+      const long long p0 = d.p0, se = d.se;
+      const int len = d.len;
+      const int j = jf & 0xffff;
+      float* sv = W.val[st];
+      const double* sg = W.g[st];
+      const int q0 = lane * kItems;
+      if (kRLE) {
+        float v[kItems], vn = 0.f;
+        if (q0 < len)
+          rle_values(A.t.tb, chunk(i), p0, len, (jf & kDescNext) != 0, p0 + q0, K, d.a * K + K, v, vn);
 #pragma unroll
-      for (int k = 0; k < kItems; ++k)
-        if (base + k < cp1) vm |= 1u << k;
-      if (kRLE && !kTotals) {
-        // direct RLE: the values come from the runs covering this thread's entries; the
-        // chunk index gives the runs holding the first entries of this chunk and the next one
-        const Tables& tb = A.t.tb;
-        const int cg = t * kChunksPerTile + wid;
-        int lo = tb.run_chunk[cg];
-        int hi = cp1 < W.colend ? tb.run_chunk[cg + 1] : tb.seg_run[W.sb + K] - 1;
-        while (lo < hi) {
-          const int mid = (lo + hi + 1) >> 1;
-          if (tb.run_pos[mid] <= base) lo = mid; else hi = mid - 1;
+        for (int k = 0; k < kItems; ++k)
+          if (q0 + k <= len) sv[q0 + k] = v[k];  // slot len: the value after the chunk
+        if (q0 + kItems == len) sv[len] = vn;
+      } else if (lane == 0) {
+        sv[len] = d.vnext;
+      }
+      __syncwarp();
+      // pass 1: the lane's sums
+      double lg = 0.0, lh = 0.0;
+      int lc = 0;
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) {
+        if (q0 + k < len) {
+          const double gk = sg[q0 + k];
+          const double hk = kH ? W.h[st][q0 + k] : hess_of<HMODE>(gk);
+          lg = lg + gk; lh = lh + hk; ++lc;
         }
-        int r = lo;
-        long long rend = tb.run_pos[r] + tb.run_len[r];
-        float rv = tb.run_val[r];
+      }
+      double wg = lg, wh = lh;
+      int wc = lc;
 #pragma unroll
-        for (int k = 0; k <= kItems; ++k) {
-          const long long p = base + k;
-          if (p >= W.colend || p > cp1) { if (k < kItems) v[k] = 0.f; continue; }
-          while (p >= rend) { ++r; rend = tb.run_pos[r] + tb.run_len[r]; rv = tb.run_val[r]; }
-          if (k < kItems) v[k] = rv; else vnext = rv;
+      for (int o = 1; o < 32; o <<= 1) {
+        const double yg = __shfl_up_sync(0xffffffffu, wg, o), yh = __shfl_up_sync(0xffffffffu, wh, o);
+        const int yc = __shfl_up_sync(0xffffffffu, wc, o);
+        if (lane >= o) { wg = yg + wg; wh = yh + wh; wc += yc; }
+      }
+      double eg = __shfl_up_sync(0xffffffffu, wg, 1), eh = __shfl_up_sync(0xffffffffu, wh, 1);
+      int ec = __shfl_up_sync(0xffffffffu, wc, 1);
+      if (lane == 0) { eg = 0.0; eh = 0.0; ec = 0; }
+      const bool head0 = (jf & kDescHead0) != 0;
+      double bg, bh;
+      int bc;
+      {
+        const FXV cx = fxv_load(W.carry[st]);
+        bg = (head0 ? 0.0 : from_fx(cx.g, Fg)) + eg;
+        bh = (head0 ? 0.0 : from_fx(cx.h, Fh)) + eh;
+        bc = (head0 ? 0 : cx.c) + ec;
+      }
+      const NodeV nv = node_v(S.B, A, K, j);
+      // pass 2: prefix at every run end, ranked by the score
+      double best = -INFINITY, xg = 0.0, xh = 0.0;
+      int bq = INT_MAX, xc = 0;
+      double pg = 0.0, phh = 0.0;
+      int pc = 0;
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) {
+        const int q = q0 + k;
+        if (q < len) {
+          const double gk = sg[q];
+          const double hk = kH ? W.h[st][q] : hess_of<HMODE>(gk);
+          pg = pg + gk; phh = phh + hk; ++pc;
+          const bool cand = (p0 + q + 1 == se) || (sv[q + 1] != sv[q]);
+          const int cL = bc + pc;
+          if (cand && cL >= 1 && nv.C - cL >= 1) {
+            const double GL = bg + pg, HL = bh + phh;
+            const double sc = split_score(GL, HL, nv.G, nv.H, lam);
+            if (sc > best) { best = sc; bq = q; xg = GL; xh = HL; xc = cL; }
+          }
         }
-      } else if (!kTotals) {
-        const float4 v0 = *reinterpret_cast<const float4*>(&S.val[s0][ibase]);
-        const float4 v1 = *reinterpret_cast<const float4*>(&S.val[s0][ibase + 4]);
-        v[0] = v0.x; v[1] = v0.y; v[2] = v0.z; v[3] = v0.w;
-        v[4] = v1.x; v[5] = v1.y; v[6] = v1.z; v[7] = v1.w;
-        const long long pn = base + kItems;  // the entry after this thread's items
-        if (pn < W.colend) vnext = pn < M.P1 ? S.val[s0][ibase + kItems] : __ldg(A.t.val + pn);
-      } else {
+      }
+      double wb = best;
+      int wq = bq;
 #pragma unroll
-        for (int k = 0; k < kItems; ++k) v[k] = 0.f;
+      for (int o = 16; o; o >>= 1) {
+        const double ob = __shfl_xor_sync(0xffffffffu, wb, o);
+        const int oq = __shfl_xor_sync(0xffffffffu, wq, o);
+        if (ob > wb || (ob == wb && oq < wq)) { wb = ob; wq = oq; }
+      }
+      if (wq != INT_MAX && wq == bq) {
+        Rec r;
+        r.GL = xg;
+        r.HL = xh;
+        r.cntL = xc;
+        r.gain = eq2_gain(xg, xh, nv.G, nv.H, lam, nv.P);
+        r.value = sv[bq];
+        r.attr = A.t.a_base + d.a;
+        r.dir = 0;
+        r.node = j;
+        r.epoch = epoch;
+        r.shard = A.shard;
+        r.pos = p0 + bq;
+        post_record(S.B, A, K, r);
+      }
+    }
+    __syncwarp();  // stage st and descriptor slot i & 3 are free
+    cp_async_wait<0>();  // descriptor of chunk i + 2 (and carry of chunk i + 1)
+    __syncwarp();
+    issue(i + 2);
+    fetch(i + 3, true, false);
+    fetch(i + 2, false, true);
+    cp_async_commit();
+  }
+  cp_async_wait<0>();
+  nb_flush(S.B, A, K);
+}
+
+// ---------------------------------------------------------------------------- k_sf_gen
+template <int HMODE, bool kMissing, bool kTotals, bool kRLE>
+__global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
+  constexpr bool kH = HMODE == kHGather;
+  __shared__ NodeBest B;
+  __shared__ unsigned char flg[kWarps][kChunk];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int K = *A.t.Kp;
+  const int C = *A.t.tb.C;
+  if (K == 0 || C == 0) return;
+  const int epoch = *A.epochp;
+  const int Fg = A.fx[0], Fh = A.fx[1];
+  const double lam = A.lam;
+  nb_init(B, A, K);
+  __syncthreads();
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nw) {
+    const ChunkDesc d = A.desc[c];
+    if (!kMissing && !kTotals && (d.jf & kDescSingle)) continue;  // k_sf_fast's
+    const long long p0 = d.p0;
+    const long long cp1 = p0 + d.len;
+    const long long sb = (long long)d.a * K;
+    const long long base = p0 + lane * kItems;
+    const long long* ss = (const long long*)(A.t.tb.seg_start + sb);
+    const long long* sc = (const long long*)(A.t.tb.seg_cnt + sb);
+    float v[kItems];
+    double g[kItems], h[kItems];
+    int cnt[kItems];
+    unsigned vm = 0;
+    float vnext = 0.f;
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) {
+      v[k] = 0.f; g[k] = 0.0; h[k] = 0.0;
+      if (base + k < cp1) vm |= 1u << k;
+    }
+    if (vm) {
+      if (!kTotals) {
+        if (kRLE) {
+          rle_values(A.t.tb, c, p0, d.len, (d.jf & kDescNext) != 0, base, K, (int)(sb + K), v, vnext);
+        } else {
+          const float4 v0 = __ldcs(reinterpret_cast<const float4*>(A.t.val + base));
+          const float4 v1 = __ldcs(reinterpret_cast<const float4*>(A.t.val + base + 4));
+          v[0] = v0.x; v[1] = v0.y; v[2] = v0.z; v[3] = v0.w; v[4] = v1.x; v[5] = v1.y; v[6] = v1.z; v[7] = v1.w;
+          if (base + kItems < cp1) vnext = __ldg(A.t.val + base + kItems);
+          else if (d.jf & kDescNext) vnext = d.vnext;
+        }
+      }
+      const double2* gi = reinterpret_cast<const double2*>(A.glist + base);
+      const double2* hi2 = reinterpret_cast<const double2*>(A.hlist + base);
+#pragma unroll
+      for (int q = 0; q < kItems / 2; ++q) {
+        const double2 x = __ldcs(gi + q);
+        g[2 * q] = x.x; g[2 * q + 1] = x.y;
+        if (kH) { const double2 y = __ldcs(hi2 + q); h[2 * q] = y.x; h[2 * q + 1] = y.y; }
       }
 #pragma unroll
       for (int k = 0; k < kItems; ++k) {
-        if ((vm >> k) & 1) {
-          g[k] = S.g[s0][ibase + k];
-          h[k] = kH ? sH[(size_t)s0 * kTileSpan + ibase + k] : hess_of<HMODE>(g[k]);
-        } else {
-          g[k] = 0.0; h[k] = 0.0;
-        }
-      }
-      const FXV cx = fxv_load(M.carry + 5 * wid);
-      const SVf carry = SVf{from_fx(cx.g, Fg), from_fx(cx.h, Fh), cx.c, 0};
-      const bool seg_cached = K <= kSegCache;
-      const long long* ss = seg_cached ? M.seg_s[wid] : (const long long*)(A.t.tb.seg_start + W.sb);
-      const long long* sc = seg_cached ? M.seg_c[wid] : (const long long*)(A.t.tb.seg_cnt + W.sb);
-
-      // ============================================================ fast path: the chunk lies
-      // inside ONE segment and no value is missing -> plain scans, candidates ranked with one
-      // Newton reciprocal, warp argmax, exact Eq. 2 only for the chunk's winner.
-      bool done = false;
-      if (!kTotals && !kMissing && seg_cached) {
-        int j0, j1;
-        {
-          int lo = 0, hi = K - 1;
-          while (lo < hi) { const int mid = (lo + hi + 1) >> 1; if (ss[mid] <= cp0) lo = mid; else hi = mid - 1; }
-          j0 = lo;
-          hi = K - 1;
-          while (lo < hi) { const int mid = (lo + hi + 1) >> 1; if (ss[mid] <= cp1 - 1) lo = mid; else hi = mid - 1; }
-          j1 = lo;
-        }
-        if (j0 == j1) {  // warp-uniform
-          done = true;
-          const int j = j0;
-          const long long se = ss[j] + sc[j];
-          const bool head0 = (cp0 == ss[j]);
-          double lg = 0.0, lh = 0.0;
-          int lc = 0;
-#pragma unroll
-          for (int k = 0; k < kItems; ++k) {
-            lg = lg + g[k]; lh = lh + h[k]; lc += (vm >> k) & 1;  // invalid items are 0
-            g[k] = lg; h[k] = lh; c[k] = lc;
-          }
-          double wg = lg, wh = lh;
-          int wcn = lc;
-#pragma unroll
-          for (int o = 1; o < 32; o <<= 1) {
-            const double yg = __shfl_up_sync(0xffffffffu, wg, o), yh = __shfl_up_sync(0xffffffffu, wh, o);
-            const int yc = __shfl_up_sync(0xffffffffu, wcn, o);
-            if (lane >= o) { wg = yg + wg; wh = yh + wh; wcn += yc; }
-          }
-          double eg = __shfl_up_sync(0xffffffffu, wg, 1), eh = __shfl_up_sync(0xffffffffu, wh, 1);
-          int ec = __shfl_up_sync(0xffffffffu, wcn, 1);
-          if (lane == 0) { eg = 0.0; eh = 0.0; ec = 0; }
-          const double bg = (head0 ? 0.0 : carry.g) + eg, bh = (head0 ? 0.0 : carry.h) + eh;
-          const int bc = (head0 ? 0 : carry.c) + ec;
-          const double Gt = A.nodes.G[j], Ht = A.nodes.H[j];
-          const int Ct = A.nodes.cnt[j];
-          double best = -INFINITY;
-          int bk = -1;
-#pragma unroll
-          for (int k = 0; k < kItems; ++k) {
-            const long long p = base + k;
-            const float nv = (k < kItems - 1) ? v[k + 1] : vnext;
-            const bool cand = ((vm >> k) & 1) && (p + 1 == se || nv != v[k]);
-            const int cL = bc + c[k];
-            if (cand && cL >= 1 && Ct - cL >= 1) {
-              const double GL = bg + g[k], HL = bh + h[k];
-              const double dl = HL + lam, dr = (Ht - HL) + lam, GR = Gt - GL;
-              const double sc2 = __dmul_rn(__fma_rn(GL * GL, dr, __dmul_rn(GR * GR, dl)), rcp_nr(__dmul_rn(dl, dr)));
-              if (sc2 > best) { best = sc2; bk = k; }
-            }
-          }
-          int bpos = bk >= 0 ? lane * kItems + bk : INT_MAX;
-#pragma unroll
-          for (int o = 16; o; o >>= 1) {
-            const double ob = __shfl_xor_sync(0xffffffffu, best, o);
-            const int op = __shfl_xor_sync(0xffffffffu, bpos, o);
-            if (ob > best || (ob == best && op < bpos)) { best = ob; bpos = op; }
-          }
-          if (bpos != INT_MAX && bpos / kItems == lane) {
-            const int k = bpos % kItems;
-            Rec r;
-            r.GL = bg + g[k];
-            r.HL = bh + h[k];
-            r.cntL = bc + c[k];
-            r.gain = eq2_gain(r.GL, r.HL, Gt, Ht, lam, A.nodes.pterm[j]);
-            r.value = v[k];
-            r.attr = A.t.a_base + W.a;
-            r.dir = 0;
-            r.node = j;
-            r.epoch = epoch;
-            r.shard = A.shard;
-            r.pos = base + k;
-            push_record(S, A, r, warp_table, wid);
-          }
-        }
-      }
-
-      if (!done) {
-        // ============================================================ general path (per warp)
-        int sj[kItems];
-        unsigned hm, pem, rem;
-        assign_segments<!kTotals>(ss, sc, cp1, K, base, vm, v, vnext, sj, hm, pem, rem);
-        SVf run = svf_zero();
-#pragma unroll
-        for (int k = 0; k < kItems; ++k) {
-          if ((vm >> k) & 1) {
-            if ((hm >> k) & 1) { run.g = g[k]; run.h = h[k]; run.c = 1; run.f = 1; }
-            else { run.g = run.g + g[k]; run.h = run.h + h[k]; run.c += 1; }
-          }
-          g[k] = run.g; h[k] = run.h; c[k] = run.c;
-        }
-        SVf inc = run;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const SVf y = shfl_up(inc, o);
-          if (lane >= o) inc = comb(y, inc);
-        }
-        SVf exc = shfl_up(inc, 1);
-        if (lane == 0) exc = svf_zero();
-        {
-          const SVf car = comb(carry, exc);
-#pragma unroll
-          for (int k = 0; k < kItems; ++k) {
-            const bool head_before = (hm & ((2u << k) - 1u)) != 0u;
-            if (!head_before) { g[k] = car.g + g[k]; h[k] = car.h + h[k]; c[k] = car.c + c[k]; }
-          }
-        }
-        if (kTotals) {
-#pragma unroll
-          for (int k = 0; k < kItems; ++k) {
-            if (((vm & rem) >> k) & 1) {
-              const long long s = W.sb + sj[k];
-              A.segPG_out[s] = g[k];
-              A.segPH_out[s] = h[k];
-            }
-          }
-        } else {
-          // Eq. 2 at run ends (both missing directions when the segment has missing values)
-          double gn[kItems];
-          unsigned dm = 0, okm = 0;
-#pragma unroll
-          for (int k = 0; k < kItems; ++k) {
-            gn[k] = 0.0;
-            if (!(((vm & rem) >> k) & 1)) continue;
-            const int j = sj[k];
-            const double Gt = A.nodes.G[j], Ht = A.nodes.H[j], pt = A.nodes.pterm[j];
-            const int Ct = A.nodes.cnt[j];
-            const int cL = c[k];
-            bool ok = false;
-            double best = 0.0;
-            int bd = 0;
-            if (cL >= 1 && Ct - cL >= 1) { best = eq2_gain(g[k], h[k], Gt, Ht, lam, pt); ok = true; }
-            if (kMissing) {
-              const long long s = W.sb + j;
-              const int cM = Ct - (int)A.t.tb.seg_cnt[s];
-              if (cM > 0) {
-                const double GM = Gt - A.segPG[s], HM = Ht - A.segPH[s];
-                const int cL1 = cL + cM;
-                if (cL1 >= 1 && Ct - cL1 >= 1) {
-                  const double g1 = eq2_gain(g[k] + GM, h[k] + HM, Gt, Ht, lam, pt);
-                  if (!ok || g1 > best) { best = g1; bd = 1; ok = true; }
-                }
-              }
-            }
-            gn[k] = best;
-            dm |= (unsigned)bd << k;
-            okm |= (unsigned)ok << k;
-          }
-          // per-piece argmax inside the chunk (pieces = the chunk's segments): segmented max-scan
-          // over the warp of (gain, position).  Inside a segment the candidates are distinct values
-          // in descending order, so "earlier position" is R12's "larger value" (the direction tie
-          // was settled per item, low first).  The end item of every piece marks its winner.
-          unsigned char* sfl = &S.flg[W.off];
-          double lg = -INFINITY;
-          int lq = INT_MAX, lf = 0;
-#pragma unroll
-          for (int k = 0; k < kItems; ++k) {
-            if (!((vm >> k) & 1)) continue;
-            sfl[lane * kItems + k] = 0;
-            if ((hm >> k) & 1) { lg = -INFINITY; lq = INT_MAX; lf = 1; }
-            if (((okm >> k) & 1) && gn[k] > lg) { lg = gn[k]; lq = lane * kItems + k; }
-          }
-#pragma unroll
-          for (int o = 1; o < 32; o <<= 1) {
-            const double yg = __shfl_up_sync(0xffffffffu, lg, o);
-            const int yq = __shfl_up_sync(0xffffffffu, lq, o), yf = __shfl_up_sync(0xffffffffu, lf, o);
-            if (lane >= o) {
-              if (!lf && (yg > lg || (yg == lg && yq < lq))) { lg = yg; lq = yq; }
-              lf |= yf;
-            }
-          }
-          double cg_ = __shfl_up_sync(0xffffffffu, lg, 1);
-          int cq = __shfl_up_sync(0xffffffffu, lq, 1);
-          if (lane == 0) { cg_ = -INFINITY; cq = INT_MAX; }
-          __syncwarp();
-#pragma unroll
-          for (int k = 0; k < kItems; ++k) {
-            if (!((vm >> k) & 1)) continue;
-            if ((hm >> k) & 1) { cg_ = -INFINITY; cq = INT_MAX; }
-            if (((okm >> k) & 1) && gn[k] > cg_) { cg_ = gn[k]; cq = lane * kItems + k; }
-            if (((pem >> k) & 1) && cq != INT_MAX) sfl[cq] = 1;  // each piece marks one item
-          }
-          __syncwarp();
-#pragma unroll
-          for (int k = 0; k < kItems; ++k) {
-            if (!((vm >> k) & 1) || !sfl[lane * kItems + k]) continue;
-            const int j = sj[k];
-            const long long s = W.sb + j;
-            Rec r;
-            r.gain = gn[k];
-            r.value = v[k];
-            r.attr = A.t.a_base + W.a;
-            r.dir = (dm >> k) & 1;
-            r.node = j;
-            r.epoch = epoch;
-            r.shard = A.shard;
-            r.pos = base + k;
-            if (r.dir) {
-              const int cM = A.nodes.cnt[j] - (int)A.t.tb.seg_cnt[s];
-              r.GL = g[k] + (A.nodes.G[j] - A.segPG[s]);
-              r.HL = h[k] + (A.nodes.H[j] - A.segPH[s]);
-              r.cntL = c[k] + cM;
-            } else {
-              r.GL = g[k]; r.HL = h[k]; r.cntL = c[k];
-            }
-            push_record(S, A, r, warp_table, wid);
-          }
-        }
+        if ((vm >> k) & 1) { if (!kH) h[k] = hess_of<HMODE>(g[k]); }
+        else { g[k] = 0.0; h[k] = 0.0; }
       }
     }
-    __syncthreads();
-  }
-  // flush the CTA's node bests (merge of the warp tables)
-  if (warp_table) {
-    __syncthreads();
-    if (tid < K) {
-      int bw = -1;
-      for (int w = 0; w < kWarps; ++w)
-        if (S.wg[w][tid] && (bw < 0 || rec_better(S.wg[w][tid], S.wb[w][tid], S.wg[bw][tid], S.wb[bw][tid]))) bw = w;
-      if (bw >= 0) {
-        const int gs = atomicAdd(A.nrec, 1);
-        A.rec[gs] = S.wb[bw][tid];
-        atomicMax(A.gkey + tid, S.wg[bw][tid]);
+    const FXV cx = fxv_load(A.carry + 5ll * c);
+    const SVf carry = SVf{from_fx(cx.g, Fg), from_fx(cx.h, Fh), cx.c, 0};
+    int sj[kItems];
+    unsigned hm, pem, rem;
+    assign_segments<!kTotals>(ss, sc, cp1, K, base, vm, v, vnext, sj, hm, pem, rem);
+    SVf run = svf_zero();
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) {
+      if ((vm >> k) & 1) {
+        if ((hm >> k) & 1) { run.g = g[k]; run.h = h[k]; run.c = 1; run.f = 1; }
+        else { run.g = run.g + g[k]; run.h = run.h + h[k]; run.c += 1; }
+      }
+      g[k] = run.g; h[k] = run.h; cnt[k] = run.c;
+    }
+    SVf inc = run;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const SVf y = shfl_up(inc, o);
+      if (lane >= o) inc = comb(y, inc);
+    }
+    SVf exc = shfl_up(inc, 1);
+    if (lane == 0) exc = svf_zero();
+    {
+      const SVf car = comb(carry, exc);
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) {
+        const bool head_before = (hm & ((2u << k) - 1u)) != 0u;
+        if (!head_before) { g[k] = car.g + g[k]; h[k] = car.h + h[k]; cnt[k] = car.c + cnt[k]; }
       }
     }
+    if (kTotals) {
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) {
+        if (((vm & rem) >> k) & 1) {
+          const long long s = sb + sj[k];
+          A.segPG_out[s] = g[k];
+          A.segPH_out[s] = h[k];
+        }
+      }
+      continue;
+    }
+    // Eq. 2 at run ends, both default directions when the segment has missing values; ranked by
+    // the score, exact Eq. 2 for each segment's winner.  Segment j's present totals sit in lane j.
+    double lPG = 0.0, lPH = 0.0;
+    if (kMissing && K <= kWarpK && lane < K) {
+      lPG = A.segPG[sb + lane];
+      lPH = A.segPH[sb + lane];
+    }
+    double gn[kItems];
+    unsigned dm = 0, okm = 0;
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) {
+      gn[k] = 0.0;
+      const int j = sj[k];
+      double PG = 0.0, PH = 0.0;
+      if (kMissing && K <= kWarpK) {  // every lane takes part in the shuffles
+        PG = __shfl_sync(0xffffffffu, lPG, j & 31);
+        PH = __shfl_sync(0xffffffffu, lPH, j & 31);
+      }
+      if (!(((vm & rem) >> k) & 1)) continue;
+      const NodeV nv = node_v(B, A, K, j);
+      const int cL = cnt[k];
+      bool ok = false;
+      double best = 0.0;
+      int bd = 0;
+      if (cL >= 1 && nv.C - cL >= 1) { best = split_score(g[k], h[k], nv.G, nv.H, lam); ok = true; }
+      if (kMissing) {
+        const int cM = nv.C - (int)sc[j];
+        if (cM > 0) {
+          if (K > kWarpK) { PG = A.segPG[sb + j]; PH = A.segPH[sb + j]; }
+          const int cL1 = cL + cM;
+          if (cL1 >= 1 && nv.C - cL1 >= 1) {
+            const double g1 = split_score(g[k] + (nv.G - PG), h[k] + (nv.H - PH), nv.G, nv.H, lam);
+            if (!ok || g1 > best) { best = g1; bd = 1; ok = true; }
+          }
+        }
+      }
+      gn[k] = best;
+      dm |= (unsigned)bd << k;
+      okm |= (unsigned)ok << k;
+    }
+    // per-segment argmax inside the chunk: segmented max-scan over the warp of (score, position).
+    // Inside a segment the candidates are distinct values in descending order, so "earlier
+    // position" is R12's "larger value"; the direction tie was settled per item (low first).
+    unsigned char* sfl = flg[wid];
+    double lg = -INFINITY;
+    int lq = INT_MAX, lf = 0;
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) {
+      if (!((vm >> k) & 1)) continue;
+      sfl[lane * kItems + k] = 0;
+      if ((hm >> k) & 1) { lg = -INFINITY; lq = INT_MAX; lf = 1; }
+      if (((okm >> k) & 1) && gn[k] > lg) { lg = gn[k]; lq = lane * kItems + k; }
+    }
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const double yg = __shfl_up_sync(0xffffffffu, lg, o);
+      const int yq = __shfl_up_sync(0xffffffffu, lq, o), yf = __shfl_up_sync(0xffffffffu, lf, o);
+      if (lane >= o) {
+        if (!lf && (yg > lg || (yg == lg && yq < lq))) { lg = yg; lq = yq; }
+        lf |= yf;
+      }
+    }
+    double cg_ = __shfl_up_sync(0xffffffffu, lg, 1);
+    int cq = __shfl_up_sync(0xffffffffu, lq, 1);
+    if (lane == 0) { cg_ = -INFINITY; cq = INT_MAX; }
+    __syncwarp();
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) {
+      if (!((vm >> k) & 1)) continue;
+      if ((hm >> k) & 1) { cg_ = -INFINITY; cq = INT_MAX; }
+      if (((okm >> k) & 1) && gn[k] > cg_) { cg_ = gn[k]; cq = lane * kItems + k; }
+      if (((pem >> k) & 1) && cq != INT_MAX) sfl[cq] = 1;  // each segment marks one item
+    }
+    __syncwarp();
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) {
+      if (!((vm >> k) & 1) || !sfl[lane * kItems + k]) continue;
+      const int j = sj[k];
+      const long long s = sb + j;
+      const NodeV nv = node_v(B, A, K, j);
+      Rec r;
+      r.value = v[k];
+      r.attr = A.t.a_base + d.a;
+      r.dir = (dm >> k) & 1;
+      r.node = j;
+      r.epoch = epoch;
+      r.shard = A.shard;
+      r.pos = base + k;
+      if (r.dir) {
+        r.GL = g[k] + (nv.G - A.segPG[s]);
+        r.HL = h[k] + (nv.H - A.segPH[s]);
+        r.cntL = cnt[k] + (nv.C - (int)sc[j]);
+      } else {
+        r.GL = g[k]; r.HL = h[k]; r.cntL = cnt[k];
+      }
+      r.gain = eq2_gain(r.GL, r.HL, nv.G, nv.H, lam, nv.P);
+      post_record(B, A, K, r);
+    }
+    __syncwarp();
   }
+  if (!kTotals) nb_flush(B, A, K);
 }
 
 // ============================================================================ a8: partition
@@ -1344,21 +1424,15 @@ unsigned grid_for(KernelT kern, size_t smem, int sms) {
 
 size_t scatter_smem(bool h) { return sizeof(ScatterStage) * kWarps + (h ? sizeof(double) * kChunk * kWarps : 0); }
 
-size_t sf_smem(int hmode) {
-  size_t b = (sizeof(SFSmem) + 127) & ~size_t(127);
-  if (hmode == kHGather) b += sizeof(double) * kStages * kTileSpan;
-  return b;
-}
+size_t fast_smem(int hmode) { return hmode == kHGather ? sizeof(FastSmem<true>) : sizeof(FastSmem<false>); }
 
-template <int HM>
-void launch_sf(const SplitArgs& A, bool missing, bool rle, unsigned grid, cudaStream_t st) {
-  if (rle) {
-    if (missing) k_sf<HM, true, false, true><<<grid, kThreads, sf_smem(HM), st>>>(A);
-    else k_sf<HM, false, false, true><<<grid, kThreads, sf_smem(HM), st>>>(A);
-  } else {
-    if (missing) k_sf<HM, true, false, false><<<grid, kThreads, sf_smem(HM), st>>>(A);
-    else k_sf<HM, false, false, false><<<grid, kThreads, sf_smem(HM), st>>>(A);
-  }
+template <int HM, bool kR>
+void launch_fast(const SplitArgs& A, unsigned grid, cudaStream_t st) {
+  k_sf_fast<HM, kR><<<grid, kThreads, fast_smem(HM), st>>>(A);
+}
+template <int HM, bool kM, bool kT, bool kR>
+void launch_gen(const SplitArgs& A, unsigned grid, cudaStream_t st) {
+  k_sf_gen<HM, kM, kT, kR><<<grid, kThreads, 0, st>>>(A);
 }
 
 template <bool kFx>
@@ -1375,21 +1449,13 @@ void launch_scan(const int32_t* Cp, unsigned long long* in, unsigned long long* 
 
 void LevelKernels::init(int device) {
   GBDT_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device));
-  grid_sf[0][0] = grid_for(k_sf<0, false, false, false>, sf_smem(0), sms);
-  grid_sf[0][1] = grid_for(k_sf<0, true, false, false>, sf_smem(0), sms);
-  grid_sf[1][0] = grid_for(k_sf<1, false, false, false>, sf_smem(1), sms);
-  grid_sf[1][1] = grid_for(k_sf<1, true, false, false>, sf_smem(1), sms);
-  grid_sf[2][0] = grid_for(k_sf<2, false, false, false>, sf_smem(2), sms);
-  grid_sf[2][1] = grid_for(k_sf<2, true, false, false>, sf_smem(2), sms);
-  grid_for(k_sf<0, false, false, true>, sf_smem(0), sms);
-  grid_for(k_sf<0, true, false, true>, sf_smem(0), sms);
-  grid_for(k_sf<1, false, false, true>, sf_smem(1), sms);
-  grid_for(k_sf<1, true, false, true>, sf_smem(1), sms);
-  grid_for(k_sf<2, false, false, true>, sf_smem(2), sms);
-  grid_for(k_sf<2, true, false, true>, sf_smem(2), sms);
-  grid_tot[0] = grid_for(k_sf<0, true, true, false>, sf_smem(0), sms);
-  grid_tot[1] = grid_for(k_sf<1, true, true, false>, sf_smem(1), sms);
-  grid_tot[2] = grid_for(k_sf<2, true, true, false>, sf_smem(2), sms);
+  grid_fast[0][0] = grid_for(k_sf_fast<0, false>, fast_smem(0), sms);
+  grid_fast[0][1] = grid_for(k_sf_fast<0, true>, fast_smem(0), sms);
+  grid_fast[1][0] = grid_for(k_sf_fast<1, false>, fast_smem(1), sms);
+  grid_fast[1][1] = grid_for(k_sf_fast<1, true>, fast_smem(1), sms);
+  grid_fast[2][0] = grid_for(k_sf_fast<2, false>, fast_smem(2), sms);
+  grid_fast[2][1] = grid_for(k_sf_fast<2, true>, fast_smem(2), sms);
+  grid_gen = grid_for(k_sf_gen<2, true, false, true>, 0, sms);  // the largest variant
   grid_agg[0] = grid_for(k_chunk_agg<0, true>, 0, sms);
   grid_agg[1] = grid_for(k_chunk_agg<1, true>, 0, sms);
   grid_agg[2] = grid_for(k_chunk_agg<2, true>, 0, sms);
@@ -1423,17 +1489,29 @@ void LevelKernels::tile_prefix(const SplitArgs& A, int hmode, bool gather, unsig
 }
 
 void LevelKernels::split_find(const SplitArgs& A, int hmode, bool missing, bool rle, cudaStream_t st) {
-  if (hmode == 0) launch_sf<0>(A, missing, rle, grid_sf[0][missing], st);
-  else if (hmode == 1) launch_sf<1>(A, missing, rle, grid_sf[1][missing], st);
-  else launch_sf<2>(A, missing, rle, grid_sf[2][missing], st);
+  const unsigned gg = grid_gen;
+  if (!missing) {  // single-segment chunks stream through k_sf_fast; the rest go through k_sf_gen
+    const unsigned gf = grid_fast[hmode][rle];
+    if (hmode == 0) { if (rle) launch_fast<0, true>(A, gf, st); else launch_fast<0, false>(A, gf, st); }
+    else if (hmode == 1) { if (rle) launch_fast<1, true>(A, gf, st); else launch_fast<1, false>(A, gf, st); }
+    else { if (rle) launch_fast<2, true>(A, gf, st); else launch_fast<2, false>(A, gf, st); }
+    if (hmode == 0) { if (rle) launch_gen<0, false, false, true>(A, gg, st); else launch_gen<0, false, false, false>(A, gg, st); }
+    else if (hmode == 1) { if (rle) launch_gen<1, false, false, true>(A, gg, st); else launch_gen<1, false, false, false>(A, gg, st); }
+    else { if (rle) launch_gen<2, false, false, true>(A, gg, st); else launch_gen<2, false, false, false>(A, gg, st); }
+    count_launch(2);
+  } else {
+    if (hmode == 0) { if (rle) launch_gen<0, true, false, true>(A, gg, st); else launch_gen<0, true, false, false>(A, gg, st); }
+    else if (hmode == 1) { if (rle) launch_gen<1, true, false, true>(A, gg, st); else launch_gen<1, true, false, false>(A, gg, st); }
+    else { if (rle) launch_gen<2, true, false, true>(A, gg, st); else launch_gen<2, true, false, false>(A, gg, st); }
+    count_launch();
+  }
   GBDT_LAUNCH_CHECK();
-  count_launch();
 }
 
 void LevelKernels::seg_totals(const SplitArgs& A, int hmode, cudaStream_t st) {
-  if (hmode == 0) k_sf<0, true, true, false><<<grid_tot[0], kThreads, sf_smem(0), st>>>(A);
-  else if (hmode == 1) k_sf<1, true, true, false><<<grid_tot[1], kThreads, sf_smem(1), st>>>(A);
-  else k_sf<2, true, true, false><<<grid_tot[2], kThreads, sf_smem(2), st>>>(A);
+  if (hmode == 0) launch_gen<0, true, true, false>(A, grid_gen, st);
+  else if (hmode == 1) launch_gen<1, true, true, false>(A, grid_gen, st);
+  else launch_gen<2, true, true, false>(A, grid_gen, st);
   GBDT_LAUNCH_CHECK();
   count_launch();
 }
