@@ -46,6 +46,8 @@ constexpr int kDescHead0 = 1 << 16, kDescSingle = 1 << 17, kDescNext = 1 << 18;
 struct SplitArgs {
   TileArgs t;
   ChunkDesc* desc;       // [C]
+  int32_t* genlist;      // [C] chunks that cross a segment boundary (k_sf_gen), appended
+  int32_t* ngen;
   int rle;               // the level's values live in runs (t.val is not maintained)
   const double* g;       // per instance
   const double* h;       // per instance (mode 2)

@@ -169,7 +169,7 @@ __device__ __forceinline__ int find_attr(const int* start, int m, int x) {
 // Range of one chunk (all lanes compute it; the tables are in smem when m is small).
 struct ChunkMeta {
   long long p0, p1, sb;
-  int a, reset;
+  int a, reset, more;  // more: the attribute continues after the chunk
 };
 __device__ __forceinline__ ChunkMeta chunk_meta(const TabCache& tc, const TileArgs& A, int K, int c) {
   const bool u = tc.use;
@@ -183,6 +183,7 @@ __device__ __forceinline__ ChunkMeta chunk_meta(const TabCache& tc, const TileAr
   M.reset = (k == 0);
   M.p0 = c0 + (long long)k * kChunk;
   M.p1 = min(M.p0 + (long long)kChunk, c0 + cl);
+  M.more = M.p1 < c0 + cl;
   M.sb = (long long)a * K;
   return M;
 }
@@ -192,7 +193,8 @@ __device__ __forceinline__ ChunkMeta chunk_meta(const TabCache& tc, const TileAr
 template <bool kNeedVal>
 __device__ __forceinline__ void assign_segments(const long long* ss, const long long* sc, long long p1, int K,
                                                 long long base, unsigned vm, const float* v, float vnext,
-                                                int* sj, unsigned& hm, unsigned& pem, unsigned& rem) {
+                                                int* sj, unsigned& hm, unsigned& pem, unsigned& rem,
+                                                long long* first = nullptr) {
   hm = pem = rem = 0;
   if (!vm) return;
   int lo = 0, hi = K - 1;
@@ -202,6 +204,7 @@ __device__ __forceinline__ void assign_segments(const long long* ss, const long 
   }
   int j = lo;
   long long s0 = ss[j], se = s0 + sc[j];
+  if (first) { first[0] = s0; first[1] = se; }  // segment of the thread's first entry
 #pragma unroll
   for (int k = 0; k < kItems; ++k) {
     const long long p = base + k;
@@ -240,6 +243,8 @@ __global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
     const ChunkMeta M = chunk_meta(tc, A.t, K, c);
     const long long p1 = M.p1;
     const long long base = M.p0 + (long long)lane * kItems;
+    // value after the chunk (same attribute), for the descriptor; loaded early
+    const float vnx = (lane == 0 && M.more && !A.rle) ? __ldg(A.t.val + p1) : 0.f;
     unsigned vm = 0;
     double g[kItems], h[kItems];
 #pragma unroll
@@ -297,8 +302,9 @@ __global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
     int sj[kItems];
     unsigned hm, pem, rem;
     float vd[kItems];
+    long long fs[2] = {0, 0};
     assign_segments<false>((const long long*)(A.t.tb.seg_start + M.sb), (const long long*)(A.t.tb.seg_cnt + M.sb),
-                           p1, K, base, vm, vd, 0.f, sj, hm, pem, rem);
+                           p1, K, base, vm, vd, 0.f, sj, hm, pem, rem, fs);
     {  // the chunk's descriptor: its first entry's segment, and whether the chunk stays in it
       const int len = (int)(p1 - M.p0);
       const int ll = (len - 1) / kItems, lk = (len - 1) % kItems;
@@ -309,16 +315,15 @@ __global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
       jl = __shfl_sync(0xffffffffu, jl, ll);
       if (lane == 0) {
         const int j0 = sj[0];
-        const long long ss0 = A.t.tb.seg_start[M.sb + j0];
-        const long long colend = A.t.tb.col_start[M.a] + A.t.tb.col_len[M.a];
         ChunkDesc d;
         d.p0 = M.p0;
-        d.se = ss0 + A.t.tb.seg_cnt[M.sb + j0];
+        d.se = fs[1];
         d.len = len;
         d.a = M.a;
-        d.jf = j0 | (ss0 == M.p0 ? kDescHead0 : 0) | (jl == j0 ? kDescSingle : 0) | (p1 < colend ? kDescNext : 0);
-        d.vnext = (p1 < colend && !A.rle) ? A.t.val[p1] : 0.f;
+        d.jf = j0 | (fs[0] == M.p0 ? kDescHead0 : 0) | (jl == j0 ? kDescSingle : 0) | (M.more ? kDescNext : 0);
+        d.vnext = vnx;
         A.desc[c] = d;
+        if (jl != j0) A.genlist[atomicAdd(A.ngen, 1)] = c;  // chunks for k_sf_gen
       }
     }
     SVf run = svf_zero();
@@ -605,6 +610,34 @@ __device__ __forceinline__ void rle_values(const Tables& tb, int cg, long long p
   }
 }
 
+// A lane's 8 consecutive entries [8 lane, 8 lane + 8) of a chunk staged in shared memory, read
+// as 16-byte pieces in a lane-rotated order so that every quarter-warp touches 8 distinct 16-byte
+// bank groups (the natural order would be a 16-way bank conflict), then rotated back.
+__device__ __forceinline__ void lds_blocked8(const double* chunk, int lane, double* out) {
+  const double2* p = reinterpret_cast<const double2*>(chunk) + lane * 4;
+  const int s = (lane >> 1) & 3;
+  double2 x[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) x[j] = p[(j + s) & 3];  // x[j] = piece (j + s) & 3
+#pragma unroll
+  for (int r = 0; r < 4; ++r) {
+    double2 y = x[0];
+#pragma unroll
+    for (int j = 1; j < 4; ++j)
+      if (((j + s) & 3) == r) y = x[j];
+    out[2 * r] = y.x;
+    out[2 * r + 1] = y.y;
+  }
+}
+__device__ __forceinline__ void lds_blocked8f(const float* chunk, int lane, float* out) {
+  const float4* p = reinterpret_cast<const float4*>(chunk) + lane * 2;
+  const int s = (lane >> 2) & 1;
+  const float4 a = p[s], b = p[s ^ 1];
+  const float4 x0 = s ? b : a, x1 = s ? a : b;
+  out[0] = x0.x; out[1] = x0.y; out[2] = x0.z; out[3] = x0.w;
+  out[4] = x1.x; out[5] = x1.y; out[6] = x1.z; out[7] = x1.w;
+}
+
 // ---------------------------------------------------------------------------- k_sf_fast
 constexpr int kFS = 2;  // stages per warp
 template <bool kH>
@@ -690,29 +723,36 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
       const int len = d.len;
       const int j = jf & 0xffff;
       float* sv = W.val[st];
-      const double* sg = W.g[st];
       const int q0 = lane * kItems;
+      // the lane's 8 consecutive entries into registers with bank-rotated 16-byte loads
+      double g[kItems], hh[kH ? kItems : 1];
+      float v[kItems], vn = 0.f;
+      lds_blocked8(W.g[st], lane, g);
+      if (kH) lds_blocked8(W.h[st], lane, hh);
       if (kRLE) {
-        float v[kItems], vn = 0.f;
-        if (q0 < len)
-          rle_values(A.t.tb, chunk(i), p0, len, (jf & kDescNext) != 0, p0 + q0, K, d.a * K + K, v, vn);
+        if (q0 < len) rle_values(A.t.tb, chunk(i), p0, len, (jf & kDescNext) != 0, p0 + q0, K, d.a * K + K, v, vn);
+      } else {
+        lds_blocked8f(sv, lane, v);
+        vn = __shfl_down_sync(0xffffffffu, v[0], 1);
+        if (q0 + kItems >= len) vn = d.vnext;  // the entry after the chunk
+      }
+      // value after item k (the chunk's last item: the value after the chunk, when there is one)
+      auto next_v = [&](int k) { return (k < kItems - 1 && q0 + k + 1 < len) ? v[k + 1] : vn; };
+      if (kRLE && q0 + kItems > len) {
+        // rle_values filled the value after the chunk into v[len - q0]
+        const int kl = len - q0;
 #pragma unroll
         for (int k = 0; k < kItems; ++k)
-          if (q0 + k <= len) sv[q0 + k] = v[k];  // slot len: the value after the chunk
-        if (q0 + kItems == len) sv[len] = vn;
-      } else if (lane == 0) {
-        sv[len] = d.vnext;
+          if (k == kl) vn = v[k];
       }
-      __syncwarp();
       // pass 1: the lane's sums
       double lg = 0.0, lh = 0.0;
       int lc = 0;
 #pragma unroll
       for (int k = 0; k < kItems; ++k) {
         if (q0 + k < len) {
-          const double gk = sg[q0 + k];
-          const double hk = kH ? W.h[st][q0 + k] : hess_of<HMODE>(gk);
-          lg = lg + gk; lh = lh + hk; ++lc;
+          const double hk = kH ? hh[k] : hess_of<HMODE>(g[k]);
+          lg = lg + g[k]; lh = lh + hk; ++lc;
         }
       }
       double wg = lg, wh = lh;
@@ -739,21 +779,21 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
       // pass 2: prefix at every run end, ranked by the score
       double best = -INFINITY, xg = 0.0, xh = 0.0;
       int bq = INT_MAX, xc = 0;
+      float xv = 0.f;
       double pg = 0.0, phh = 0.0;
       int pc = 0;
 #pragma unroll
       for (int k = 0; k < kItems; ++k) {
         const int q = q0 + k;
         if (q < len) {
-          const double gk = sg[q];
-          const double hk = kH ? W.h[st][q] : hess_of<HMODE>(gk);
-          pg = pg + gk; phh = phh + hk; ++pc;
-          const bool cand = (p0 + q + 1 == se) || (sv[q + 1] != sv[q]);
+          const double hk = kH ? hh[k] : hess_of<HMODE>(g[k]);
+          pg = pg + g[k]; phh = phh + hk; ++pc;
+          const bool cand = (p0 + q + 1 == se) || (next_v(k) != v[k]);
           const int cL = bc + pc;
           if (cand && cL >= 1 && nv.C - cL >= 1) {
             const double GL = bg + pg, HL = bh + phh;
             const double sc = split_score(GL, HL, nv.G, nv.H, lam);
-            if (sc > best) { best = sc; bq = q; xg = GL; xh = HL; xc = cL; }
+            if (sc > best) { best = sc; bq = q; xg = GL; xh = HL; xc = cL; xv = v[k]; }
           }
         }
       }
@@ -771,7 +811,7 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
         r.HL = xh;
         r.cntL = xc;
         r.gain = eq2_gain(xg, xh, nv.G, nv.H, lam, nv.P);
-        r.value = sv[bq];
+        r.value = xv;
         r.attr = A.t.a_base + d.a;
         r.dir = 0;
         r.node = j;
@@ -809,9 +849,12 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
   nb_init(B, A, K);
   __syncthreads();
   const int nw = (gridDim.x * blockDim.x) >> 5;
-  for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nw) {
+  // with missing values every chunk; else the chunks k_chunk_agg listed (they cross segments)
+  constexpr bool kAll = kMissing || kTotals;
+  const int n = kAll ? C : *A.ngen;
+  for (int i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < n; i += nw) {
+    const int c = kAll ? i : A.genlist[i];
     const ChunkDesc d = A.desc[c];
-    if (!kMissing && !kTotals && (d.jf & kDescSingle)) continue;  // k_sf_fast's
     const long long p0 = d.p0;
     const long long cp1 = p0 + d.len;
     const long long sb = (long long)d.a * K;

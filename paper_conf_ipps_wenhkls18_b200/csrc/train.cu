@@ -352,6 +352,7 @@ struct ShardWork {
   LookBack lb;                        // partition look-back
   Rec* rec;
   ChunkDesc* desc;
+  int32_t* genlist;
   int* nrec;
   unsigned long long *gkey, *tkey;
   int32_t *segH, *segL;
@@ -497,7 +498,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       q.take<unsigned long long>(2 * C0); q.take<unsigned long long>(2 * C0);
       q.take<unsigned long long>(5 * (size_t)LevelKernels::scan_groups(C0) + 8);
       q.take<int32_t>(T0); q.take<unsigned long long>(T0); q.take<unsigned long long>(T0);
-      q.take<Rec>(R); q.take<ChunkDesc>(C0);
+      q.take<Rec>(R); q.take<ChunkDesc>(C0); q.take<int32_t>(C0);
       q.take<int32_t>(S); q.take<int32_t>(S); q.take<unsigned long long>(S); q.take<int64_t>(S); q.take<int64_t>(S);
       q.take<int64_t>(m); q.take<double>(S); q.take<double>(S); q.take<int>(4);
       q.take<unsigned long long>(2 * (size_t)(m + 1)); q.take<unsigned long long>(2 * (size_t)LevelKernels::scan_groups(m + 1) + 8);
@@ -529,6 +530,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     }
     w.rec = q.take<Rec>(R);
     w.desc = q.take<ChunkDesc>(C0);
+    w.genlist = q.take<int32_t>(C0);
     w.segH = q.take<int32_t>(S); w.segL = q.take<int32_t>(S);
     w.seg_pre = q.take<unsigned long long>(S);
     w.out_hi = q.take<int64_t>(S); w.out_lo = q.take<int64_t>(S);
@@ -622,7 +624,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         const int32_t* ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
         SplitArgs A;
         A.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters};
-        A.desc = w.desc; A.rle = sh.rle ? 1 : 0;
+        A.desc = w.desc; A.rle = sh.rle ? 1 : 0; A.genlist = w.genlist; A.ngen = w.counters + 2;
         A.g = gv; A.h = hv; A.nodes = cur; A.segPG = w.segPG; A.segPH = w.segPH; A.lam = P.lambda;
         A.epochp = epoch; A.fx = fxs; A.rec = w.rec;
         A.glist = w.glist[lvl & 1]; A.hlist = w.hlist[lvl & 1]; A.cagg = w.cagg; A.carry = w.carry;
