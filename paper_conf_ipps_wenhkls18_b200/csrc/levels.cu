@@ -188,6 +188,12 @@ __device__ __forceinline__ ChunkMeta chunk_meta(const TabCache& tc, const TileAr
   return M;
 }
 
+// L2 prefetch of a chunk's list bytes [p0, p0 + 256) * elem (lanes take one 128-byte line each)
+__device__ __forceinline__ void prefetch_chunk(const void* list, long long p0, int elem, int lane) {
+  const char* b = reinterpret_cast<const char*>(list) + p0 * elem;
+  if (lane * 128 < kChunk * elem) asm volatile("prefetch.global.L2 [%0];" ::"l"(b + lane * 128));
+}
+
 // Segment (node) of each of the thread's items; head / piece-end / run-end masks.  ss/sc are the
 // attribute's segment starts/counts; p1 bounds the piece (chunk end).
 template <bool kNeedVal>
@@ -243,6 +249,11 @@ __global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
     const ChunkMeta M = chunk_meta(tc, A.t, K, c);
     const long long p1 = M.p1;
     const long long base = M.p0 + (long long)lane * kItems;
+    if (!kGather && c + nw < C) {  // the warp's next chunk streams into L2 meanwhile
+      const ChunkMeta Mn = chunk_meta(tc, A.t, K, c + nw);
+      prefetch_chunk(A.glist, Mn.p0, 8, lane);
+      if (HMODE == kHGather) prefetch_chunk(A.hlist, Mn.p0, 8, lane);
+    }
     // value after the chunk (same attribute), for the descriptor; loaded early
     const float vnx = (lane == 0 && M.more && !A.rle) ? __ldg(A.t.val + p1) : 0.f;
     unsigned vm = 0;
@@ -299,32 +310,57 @@ __global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
         }
       }
     }
+    // segment of the chunk's first entry (warp-uniform search; the attribute's table is in L1)
+    const long long* ss = (const long long*)(A.t.tb.seg_start + M.sb);
+    const long long* sc = (const long long*)(A.t.tb.seg_cnt + M.sb);
+    int j0;
+    {
+      int lo = 0, hi = K - 1;
+      while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (ss[mid] <= M.p0) lo = mid; else hi = mid - 1;
+      }
+      j0 = lo;
+    }
+    const long long s0 = ss[j0], se = s0 + sc[j0];
+    const int len = (int)(p1 - M.p0);
+    if (p1 <= se) {
+      // one segment: the aggregate is the whole chunk (a head can only be its first entry)
+      double lg = 0.0, lh = 0.0;
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) { lg = lg + g[k]; lh = lh + h[k]; }  // invalid items are 0
+#pragma unroll
+      for (int o = 16; o; o >>= 1) {
+        lg = lg + __shfl_xor_sync(0xffffffffu, lg, o);
+        lh = lh + __shfl_xor_sync(0xffffffffu, lh, o);
+      }
+      if (lane == 0) {
+        ChunkDesc d;
+        d.p0 = M.p0;
+        d.se = se;
+        d.len = len;
+        d.a = M.a;
+        d.jf = j0 | (s0 == M.p0 ? kDescHead0 : 0) | kDescSingle | (M.more ? kDescNext : 0);
+        d.vnext = vnx;
+        A.desc[c] = d;
+        fxv_store(A.cagg + 5ll * c, FXV{to_fx(lg, Fg), to_fx(lh, Fh), len, s0 == M.p0 ? 1 : 0}, M.reset);
+      }
+      continue;
+    }
     int sj[kItems];
     unsigned hm, pem, rem;
     float vd[kItems];
-    long long fs[2] = {0, 0};
-    assign_segments<false>((const long long*)(A.t.tb.seg_start + M.sb), (const long long*)(A.t.tb.seg_cnt + M.sb),
-                           p1, K, base, vm, vd, 0.f, sj, hm, pem, rem, fs);
-    {  // the chunk's descriptor: its first entry's segment, and whether the chunk stays in it
-      const int len = (int)(p1 - M.p0);
-      const int ll = (len - 1) / kItems, lk = (len - 1) % kItems;
-      int jl = 0;
-#pragma unroll
-      for (int k = 0; k < kItems; ++k)
-        if (k == lk) jl = sj[k];
-      jl = __shfl_sync(0xffffffffu, jl, ll);
-      if (lane == 0) {
-        const int j0 = sj[0];
-        ChunkDesc d;
-        d.p0 = M.p0;
-        d.se = fs[1];
-        d.len = len;
-        d.a = M.a;
-        d.jf = j0 | (fs[0] == M.p0 ? kDescHead0 : 0) | (jl == j0 ? kDescSingle : 0) | (M.more ? kDescNext : 0);
-        d.vnext = vnx;
-        A.desc[c] = d;
-        if (jl != j0) A.genlist[atomicAdd(A.ngen, 1)] = c;  // chunks for k_sf_gen
-      }
+    assign_segments<false>(ss, sc, p1, K, base, vm, vd, 0.f, sj, hm, pem, rem);
+    if (lane == 0) {  // the chunk crosses a segment boundary: k_sf_gen's
+      ChunkDesc d;
+      d.p0 = M.p0;
+      d.se = se;
+      d.len = len;
+      d.a = M.a;
+      d.jf = j0 | (s0 == M.p0 ? kDescHead0 : 0) | (M.more ? kDescNext : 0);
+      d.vnext = vnx;
+      A.desc[c] = d;
+      A.genlist[atomicAdd(A.ngen, 1)] = c;
     }
     SVf run = svf_zero();
 #pragma unroll
@@ -776,28 +812,33 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
         bc = (head0 ? 0 : cx.c) + ec;
       }
       const NodeV nv = node_v(S.B, A, K, j);
-      // pass 2: prefix at every run end, ranked by the score
-      double best = -INFINITY, xg = 0.0, xh = 0.0;
+      // pass 2: prefix at every run end, ranked inside the lane by the score num/den compared by
+      // cross-multiplication (no division), num = GL^2 (HR+l) + GR^2 (HL+l), den = (HL+l)(HR+l)
+      double bnum = 0.0, bden = 1.0, xg = 0.0, xh = 0.0;
       int bq = INT_MAX, xc = 0;
       float xv = 0.f;
       double pg = 0.0, phh = 0.0;
       int pc = 0;
+      const int se_q = (int)min(se - p0, (long long)kChunk + 1);  // segment end, chunk-relative
 #pragma unroll
       for (int k = 0; k < kItems; ++k) {
         const int q = q0 + k;
         if (q < len) {
           const double hk = kH ? hh[k] : hess_of<HMODE>(g[k]);
           pg = pg + g[k]; phh = phh + hk; ++pc;
-          const bool cand = (p0 + q + 1 == se) || (next_v(k) != v[k]);
+          const bool cand = (q + 1 == se_q) || (next_v(k) != v[k]);
           const int cL = bc + pc;
           if (cand && cL >= 1 && nv.C - cL >= 1) {
             const double GL = bg + pg, HL = bh + phh;
-            const double sc = split_score(GL, HL, nv.G, nv.H, lam);
-            if (sc > best) { best = sc; bq = q; xg = GL; xh = HL; xc = cL; xv = v[k]; }
+            const double dl = HL + lam, dr = (nv.H - HL) + lam, GR = nv.G - GL;
+            const double num = __fma_rn(GL * GL, dr, __dmul_rn(GR * GR, dl)), den = __dmul_rn(dl, dr);
+            if (bq == INT_MAX || __dmul_rn(num, bden) > __dmul_rn(bnum, den)) {
+              bnum = num; bden = den; bq = q; xg = GL; xh = HL; xc = cL; xv = v[k];
+            }
           }
         }
       }
-      double wb = best;
+      double wb = bq == INT_MAX ? -INFINITY : __dmul_rn(bnum, rcp_nr(bden));
       int wq = bq;
 #pragma unroll
       for (int o = 16; o; o >>= 1) {
@@ -1056,6 +1097,7 @@ __global__ void __launch_bounds__(kThreads) k_part_count(PartArgs A, int counted
   for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nw) {
     const ChunkMeta M = chunk_meta(tc, A.t, K, c);
     const long long base = M.p0 + (long long)lane * kItems;
+    if (c + nw < C) prefetch_chunk(A.t.ins, chunk_meta(tc, A.t, K, c + nw).p0, 4, lane);
     unsigned vm = 0, loc = 0;
     uint8_t sd[kItems];
 #pragma unroll
@@ -1239,6 +1281,13 @@ __global__ void __launch_bounds__(kThreads) k_part_scatter(PartArgs A) {
     const ChunkMeta M = chunk_meta(tc, A.t, K, c);
     const long long p1 = M.p1;
     const long long base = M.p0 + (long long)lane * kItems;
+    if (c + nw < C) {  // the warp's next chunk streams into L2 meanwhile
+      const long long pn = chunk_meta(tc, A.t, K, c + nw).p0;
+      prefetch_chunk(A.t.ins, pn, 4, lane);
+      prefetch_chunk(A.g_in, pn, 8, lane);
+      if (!kRLE) prefetch_chunk(A.t.val, pn, 4, lane);
+      if (kH) prefetch_chunk(A.h_in, pn, 8, lane);
+    }
     unsigned vm = 0, loc = 0;
     float v[kItems];
     int id[kItems];
