@@ -165,6 +165,25 @@ gbdt_status gbdt_comm_init(int32_t rank, int32_t world, const uint8_t id[128], i
                            gbdt_comm** out);
 void gbdt_comm_free(gbdt_comm* c); /* NULL-safe; must outlive the datasets that use it */
 
+/* Host-staged communicator with caller-supplied collectives, for testing the sharded path
+ * without NCCL (e.g. two processes sharing one GPU, exchanging over torch.distributed/gloo).
+ * The library synchronises its stream, copies the operand to a host buffer, calls the callback
+ * with HOST pointers and copies the result back.  allgather: every rank contributes `bytes`
+ * bytes, recv holds world * bytes in rank order.  allreduce_u8: element-wise uint8 sum in
+ * place.  Callbacks return 0 on success (else GBDT_E_NCCL).  Same semantics as gbdt_comm_init
+ * otherwise; `user` is passed through. */
+typedef int (*gbdt_allgather_fn)(const void* send, void* recv, size_t bytes, void* user);
+typedef int (*gbdt_allreduce_u8_fn)(void* buf, size_t n, void* user);
+gbdt_status gbdt_comm_init_callbacks(int32_t rank, int32_t world, gbdt_allgather_fn allgather,
+                                     gbdt_allreduce_u8_fn allreduce_u8, void* user, int32_t device,
+                                     gbdt_comm** out);
+
+/* Attribute ranges of a P-way sharding (host-only; no device is touched): shard i owns
+ * attributes [bounds[i], bounds[i+1]), contiguous ranges balanced by stored entries
+ * (col_counts[a] = entries of attribute a).  bounds: int32[P+1], caller-owned.  This is the
+ * partition gbdt_load_csr uses for n_shards = P or a world of P ranks. */
+gbdt_status gbdt_shard_ranges(int64_t n_cols, const int64_t* col_counts, int32_t P, int32_t* bounds);
+
 void gbdt_dataset_free(gbdt_dataset* ds); /* NULL-safe */
 void gbdt_model_free(gbdt_model* m);      /* NULL-safe */
 

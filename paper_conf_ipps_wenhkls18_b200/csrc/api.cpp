@@ -94,6 +94,22 @@ struct gbdt_comm {
   Comm* c = nullptr;
 };
 
+namespace gbdt {
+std::vector<int32_t> shard_ranges(int64_t n_cols, const int64_t* col_counts, int P) {
+  std::vector<int64_t> pre(n_cols + 1, 0);
+  for (int64_t a = 0; a < n_cols; ++a) pre[a + 1] = pre[a] + col_counts[a];
+  std::vector<int32_t> bnd(P + 1, 0);
+  bnd[P] = (int32_t)n_cols;
+  int64_t a = 0;
+  for (int i = 1; i < P; ++i) {
+    const double target = (double)pre[n_cols] * i / P;
+    while (a < n_cols && (double)pre[a] < target) ++a;
+    bnd[i] = (int32_t)std::max<int64_t>(a, bnd[i - 1]);
+  }
+  return bnd;
+}
+}  // namespace gbdt
+
 extern "C" {
 
 const char* gbdt_last_error(void) { return g_err.c_str(); }
@@ -163,16 +179,7 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
       const int P = comm ? world : nsh;
       ds.n_total_shards = P;
       // contiguous attribute ranges balanced by stored entries
-      std::vector<int64_t> pre(n_cols + 1, 0);
-      for (int64_t a = 0; a < n_cols; ++a) pre[a + 1] = pre[a] + col_counts[a];
-      std::vector<int32_t> bnd(P + 1, 0);
-      bnd[P] = (int32_t)n_cols;
-      int64_t a = 0;
-      for (int i = 1; i < P; ++i) {
-        const double target = (double)pre[n_cols] * i / P;
-        while (a < n_cols && (double)pre[a] < target) ++a;
-        bnd[i] = (int32_t)std::max<int64_t>(a, bnd[i - 1]);
-      }
+      const std::vector<int32_t> bnd = shard_ranges(n_cols, col_counts.data(), P);
       for (int i = 0; i < P; ++i) {
         if (comm && i != comm->rank) continue;
         auto sh = std::make_unique<Shard>();
@@ -317,6 +324,41 @@ gbdt_status gbdt_dataset_export_rle(const gbdt_dataset* d, int32_t shard, int64_
     if (run_ptr) GBDT_CUDA(cudaMemcpy(run_ptr, s.run_ptr.p, (size_t)(s.m + 1) * 8, cudaMemcpyDeviceToHost));
     if (run_val && s.runs) GBDT_CUDA(cudaMemcpy(run_val, s.run_val.p, (size_t)s.runs * 4, cudaMemcpyDeviceToHost));
     if (run_len && s.runs) GBDT_CUDA(cudaMemcpy(run_len, s.run_len.p, (size_t)s.runs * 4, cudaMemcpyDeviceToHost));
+  });
+}
+
+gbdt_status gbdt_shard_ranges(int64_t n_cols, const int64_t* col_counts, int32_t P, int32_t* bounds) {
+  return guarded([&] {
+    if ((!col_counts && n_cols > 0) || !bounds) fail(GBDT_E_INVAL, "NULL argument");
+    if (n_cols < 0 || n_cols >= (int64_t(1) << 31)) fail(GBDT_E_INVAL, "n_cols out of range");
+    if (P < 1 || P > 8 || (P & (P - 1))) fail(GBDT_E_RANGE, "P must be 1, 2, 4 or 8");
+    for (int64_t a = 0; a < n_cols; ++a)
+      if (col_counts[a] < 0) fail(GBDT_E_INVAL, "negative column count");
+    const std::vector<int32_t> b = shard_ranges(n_cols, col_counts, P);
+    std::copy(b.begin(), b.end(), bounds);
+  });
+}
+
+gbdt_status gbdt_comm_init_callbacks(int32_t rank, int32_t world, gbdt_allgather_fn allgather,
+                                     gbdt_allreduce_u8_fn allreduce_u8, void* user, int32_t device,
+                                     gbdt_comm** out) {
+  if (out) *out = nullptr;
+  return guarded([&] {
+    if (!allgather || !allreduce_u8 || !out) fail(GBDT_E_INVAL, "NULL argument");
+    if (world < 1 || world > 8 || (world & (world - 1))) fail(GBDT_E_RANGE, "world must be 1, 2, 4 or 8");
+    if (rank < 0 || rank >= world) fail(GBDT_E_RANGE, "rank out of range");
+    if (device >= 0) GBDT_CUDA(cudaSetDevice(device));
+    int dev = 0;
+    GBDT_CUDA(cudaGetDevice(&dev));
+    auto* c = new gbdt_comm();
+    c->c = new Comm();
+    c->c->rank = rank;
+    c->c->world = world;
+    c->c->device = dev;
+    c->c->cb_allgather = allgather;
+    c->c->cb_allreduce = allreduce_u8;
+    c->c->cb_user = user;
+    *out = c;
   });
 }
 

@@ -10,6 +10,7 @@
 #include <cstring>
 #include <mutex>
 #include <string>
+#include <vector>
 
 #include "internal.h"
 
@@ -56,11 +57,29 @@ void check(ncclResult_t r, const char* what) {
 }  // namespace
 
 void Comm::allgather(const void* send, void* recv, size_t bytes, cudaStream_t st) {
+  if (!nccl) {  // host-staged callback
+    std::vector<unsigned char> hs(bytes), hr(bytes * (size_t)world);
+    GBDT_CUDA(cudaMemcpyAsync(hs.data(), send, bytes, cudaMemcpyDeviceToHost, st));
+    GBDT_CUDA(cudaStreamSynchronize(st));
+    if (cb_allgather(hs.data(), hr.data(), bytes, cb_user) != 0) fail(GBDT_E_NCCL, "allgather callback failed");
+    GBDT_CUDA(cudaMemcpyAsync(recv, hr.data(), hr.size(), cudaMemcpyHostToDevice, st));
+    GBDT_CUDA(cudaStreamSynchronize(st));
+    return;
+  }
   count_launch();
   check(api().AllGather(send, recv, bytes, ncclUint8, (ncclComm_t)nccl, st), "ncclAllGather");
 }
 
 void Comm::allreduce_sum_u8(void* buf, size_t n, cudaStream_t st) {
+  if (!nccl) {
+    std::vector<unsigned char> hb(n);
+    GBDT_CUDA(cudaMemcpyAsync(hb.data(), buf, n, cudaMemcpyDeviceToHost, st));
+    GBDT_CUDA(cudaStreamSynchronize(st));
+    if (cb_allreduce(hb.data(), n, cb_user) != 0) fail(GBDT_E_NCCL, "allreduce callback failed");
+    GBDT_CUDA(cudaMemcpyAsync(buf, hb.data(), n, cudaMemcpyHostToDevice, st));
+    GBDT_CUDA(cudaStreamSynchronize(st));
+    return;
+  }
   count_launch();
   check(api().AllReduce(buf, buf, n, ncclUint8, ncclSum, (ncclComm_t)nccl, st), "ncclAllReduce");
 }

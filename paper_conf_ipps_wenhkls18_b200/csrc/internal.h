@@ -142,10 +142,16 @@ struct Model {
 struct Comm {
   int rank = 0, world = 1, device = 0;
   void* nccl = nullptr;  // ncclComm_t
+  // host-staged callback collectives (gbdt_comm_init_callbacks); used when nccl == nullptr
+  gbdt_allgather_fn cb_allgather = nullptr;
+  gbdt_allreduce_u8_fn cb_allreduce = nullptr;
+  void* cb_user = nullptr;
   void allgather(const void* send, void* recv, size_t bytes, cudaStream_t st);
   void allreduce_sum_u8(void* buf, size_t n, cudaStream_t st);
 };
 
+// api.cpp: contiguous attribute ranges balanced by entries
+std::vector<int32_t> shard_ranges(int64_t n_cols, const int64_t* col_counts, int P);
 // layout.cu
 void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices,
                   const float* d_values, const std::vector<int64_t>& col_counts,

@@ -75,11 +75,14 @@ def lib():
     L.gbdt_comm_unique_id.argtypes = [p]
     L.gbdt_comm_init.argtypes = [i32, i32, p, i32, C.POINTER(p)]
     L.gbdt_comm_free.argtypes = [p]
+    L.gbdt_comm_init_callbacks.argtypes = [i32, i32, _AG_FN, _AR_FN, p, i32, C.POINTER(p)]
+    L.gbdt_shard_ranges.argtypes = [i64, p, i32, p]
     L.gbdt_dataset_free.argtypes = [p]
     L.gbdt_model_free.argtypes = [p]
     for f in ("gbdt_load_csr", "gbdt_train", "gbdt_predict", "gbdt_model_num_trees", "gbdt_model_num_nodes",
               "gbdt_model_export", "gbdt_get_timings", "gbdt_dataset_info", "gbdt_dataset_export_layout",
-              "gbdt_dataset_export_rle", "gbdt_comm_unique_id", "gbdt_comm_init"):
+              "gbdt_dataset_export_rle", "gbdt_comm_unique_id", "gbdt_comm_init", "gbdt_comm_init_callbacks",
+              "gbdt_shard_ranges"):
         getattr(L, f).restype = C.c_int
     _lib = L
     return L
@@ -108,11 +111,16 @@ def last_launch_count() -> int:
     return int(lib().gbdt_last_launch_count())
 
 
+_AG_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_size_t, C.c_void_p)
+_AR_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_size_t, C.c_void_p)
+
+
 class Comm:
     """NCCL communicator (one process per GPU).  Use :func:`comm_from_torch` under torchrun."""
 
-    def __init__(self, handle):
+    def __init__(self, handle, keep=None):
         self._h = handle
+        self._keep = keep  # callback trampolines must outlive the handle
 
     def __del__(self):
         if getattr(self, "_h", None) and _lib is not None:
@@ -131,6 +139,56 @@ def comm_init(rank: int, world: int, uid: bytes, device: int = -1) -> Comm:
     h = C.c_void_p()
     _check(lib().gbdt_comm_init(rank, world, C.cast(buf, C.c_void_p), device, C.byref(h)))
     return Comm(h)
+
+
+def shard_ranges(col_counts, P: int) -> np.ndarray:
+    """Attribute ranges [b[i], b[i+1]) of a P-way sharding balanced by entries (host only)."""
+    cc = np.ascontiguousarray(col_counts, np.int64)
+    b = np.zeros(P + 1, np.int32)
+    _check(lib().gbdt_shard_ranges(cc.size, _p(cc), int(P), _p(b)))
+    return b
+
+
+def torch_collectives(group=None):
+    """(allgather, allreduce_u8) over host buffers given as addresses, run on a torch.distributed
+    group; the callbacks of :func:`comm_from_callbacks` (return 0 on success)."""
+    import torch
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+
+    def ag(send, recv, nbytes, user):
+        try:
+            src = torch.frombuffer((C.c_uint8 * nbytes).from_address(send), dtype=torch.uint8).clone()
+            out = torch.empty(nbytes * world, dtype=torch.uint8)
+            dist.all_gather_into_tensor(out, src, group=group)
+            C.memmove(recv, out.numpy().ctypes.data, nbytes * world)
+            return 0
+        except Exception:  # noqa: BLE001 - reported to the library as a failed collective
+            return 1
+
+    def ar(buf, n, user):
+        try:
+            t = torch.frombuffer((C.c_uint8 * n).from_address(buf), dtype=torch.uint8).to(torch.int32)
+            dist.all_reduce(t, group=group)
+            res = t.to(torch.uint8).numpy()  # keep alive across the copy
+            C.memmove(buf, res.ctypes.data, n)
+            return 0
+        except Exception:  # noqa: BLE001
+            return 1
+
+    return ag, ar
+
+
+def comm_from_callbacks(device: int = -1, group=None) -> Comm:
+    """Host-staged communicator whose collectives run over a torch.distributed group (e.g.
+    gloo).  For tests of the sharded path where NCCL cannot run (several ranks on one GPU)."""
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    ag, ar = torch_collectives(group)
+    fa, fr = _AG_FN(ag), _AR_FN(ar)
+    h = C.c_void_p()
+    _check(lib().gbdt_comm_init_callbacks(rank, world, fa, fr, None, device, C.byref(h)))
+    return Comm(h, keep=(fa, fr))
 
 
 def comm_from_torch(device: int = -1) -> Comm:
