@@ -32,7 +32,13 @@ sys.path.insert(0, ROOT)
 
 METRIC = "seconds per tree (depth 6) at 1/2/4/8 B200; split-find HBM GB/s vs peak"
 UNIT = "s/tree"
-BYTES_PER_ENTRY_SPLIT_FIND = 24  # val 4 + ins 4 + (g,h) fp64 gather 16
+# Algorithmic bytes of the two streaming kernels:
+#   k_split   (k_sf_fast + k_sf_gen) per entry of the level: value f32 4 + g-list fp64 8
+#             (+ h-list 8 when h is not a function of g; RLE: the runs replace the 4 value bytes)
+#   k_scatter per entry of the level: val 4 + ins 4 + g 8 + side 1 read; per kept entry (the
+#             next level's entries): val 4 + ins 4 + g 8 written
+BYTES_SPLIT_PER_ENTRY = 12
+BYTES_SCATTER_READ, BYTES_SCATTER_WRITE = 17, 16
 
 
 def parse():
@@ -43,6 +49,8 @@ def parse():
     ap.add_argument("--config", default="C3")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--rle", default="off")
+    ap.add_argument("--comm", default="nccl", choices=["nccl", "host"],
+                    help="host: gloo + host-staged callbacks (several ranks may share one GPU; testing only)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle CPU time for cpu_baseline")
@@ -174,17 +182,30 @@ def main():
         return
 
     import torch
+    host_comm = args.comm == "host"
+    if host_comm:
+        local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if host_comm:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     from paper_conf_ipps_wenhkls18_b200 import gbdt
+
+    def allmax(x):  # max over ranks of a host float
+        t = torch.tensor([x], device="cpu" if host_comm else "cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
 
     prob = synth.make(args.config)
     P = dict(prob.params)
     d = P["max_depth"]
-    comm = gbdt.comm_from_torch(local) if world > 1 else None
+    comm = None
+    if world > 1:
+        comm = gbdt.comm_from_callbacks(local) if host_comm else gbdt.comm_from_torch(local)
     stream = torch.cuda.current_stream()
     ds = gbdt.load_csr(prob.indptr, prob.indices, prob.values, prob.labels, prob.m, rle=args.rle,
                        stream=stream.cuda_stream, comm=comm)
@@ -210,24 +231,30 @@ def main():
     launches = gbdt.last_launch_count()
     ms = ev0.elapsed_time(ev1)
     if dist:
-        t = torch.tensor([ms], device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+        ms = allmax(ms)
         dist.barrier()
     torch.cuda.synchronize()
     tim = model.timings()
     nodes = model.nodes()
     ent = entries_per_level(nodes, m_local, d)       # summed over the K trees
-    sf_launches = args.steps * d
-    sf_bytes = float(ent.sum()) * BYTES_PER_ENTRY_SPLIT_FIND
-    sf_ms = tim["split_find"]
     peak, peak_kind = peaks()
-    achieved = (sf_bytes / 1e9) / (sf_ms / 1e3) if sf_ms > 0 else None
-    traffic = None
-    tp_path = os.path.join(ROOT, "profiles", f"ncu_split_find_{args.config}.json")
-    if os.path.exists(tp_path):
-        with open(tp_path) as f:
-            traffic = json.load(f).get("dram_bytes_per_launch")
+    kern = {
+        "k_split": dict(bytes=float(ent.sum()) * BYTES_SPLIT_PER_ENTRY, launches=args.steps * d,
+                        ms=tim["k_split"], bytes_per_entry=BYTES_SPLIT_PER_ENTRY),
+        "k_scatter": dict(bytes=float(ent[:-1].sum()) * BYTES_SCATTER_READ + float(ent[1:].sum()) * BYTES_SCATTER_WRITE,
+                          launches=args.steps * (d - 1), ms=tim["k_scatter"],
+                          bytes_per_entry=f"{BYTES_SCATTER_READ} read + {BYTES_SCATTER_WRITE} per kept entry"),
+    }
+    for kname, kv in kern.items():
+        kv["avg_launch_ms"] = kv["ms"] / kv["launches"]
+        kv["achieved"] = (kv["bytes"] / kv["launches"] / 1e9) / (kv["avg_launch_ms"] / 1e3) if kv["ms"] > 0 else None
+        kv["frac"] = kv["achieved"] / peak if kv["achieved"] else None
+        kv["traffic"] = None
+        tp_path = os.path.join(ROOT, "profiles", f"ncu_{kname}_{args.config}.json")
+        if os.path.exists(tp_path):
+            with open(tp_path) as f:
+                kv["traffic"] = json.load(f).get("dram_bytes_per_launch")
+    dom = max(kern, key=lambda k: kern[k]["ms"])
 
     # e2e through the C ABI from pinned host buffers
     e2e = None
@@ -243,9 +270,7 @@ def main():
         torch.cuda.synchronize()
         te = time.perf_counter() - t0
         if dist:
-            t = torch.tensor([te], device="cuda")
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            te = float(t.item())
+            te = allmax(te)
         h2d = hp.nbytes + hi.nbytes + hv.nbytes + hl.nbytes
         d2h = margin2.nbytes + nodes.nbytes
         e2e = {"value": te / args.steps, "unit": UNIT, "h2d_bytes_per_step": int(h2d / args.steps),
@@ -270,11 +295,11 @@ def main():
                        "max_depth": d, "trees_timed": args.steps, "lambda": P["lam"], "eta": P["eta"],
                        "rle": args.rle, "parallelism": f"attr-shard{world}",
                        "l2": "inputs larger than L2 (sorted lists %.2f GB)" % (prob.nnz * 8 / 1e9)},
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": (achieved / peak) if achieved else None, "traffic": traffic,
-                         "kernel": "k_split_find", "peak_kind": peak_kind,
-                         "bytes_per_entry": BYTES_PER_ENTRY_SPLIT_FIND, "launches": sf_launches,
-                         "avg_launch_ms": sf_ms / sf_launches},
+            "roofline": {"bound": "hbm", "achieved": kern[dom]["achieved"], "peak": peak, "unit": "GB/s",
+                         "frac": kern[dom]["frac"], "traffic": kern[dom]["traffic"], "kernel": dom,
+                         "peak_kind": peak_kind, "bytes_per_launch": kern[dom]["bytes"] / kern[dom]["launches"],
+                         "launches": kern[dom]["launches"], "avg_launch_ms": kern[dom]["avg_launch_ms"],
+                         "kernels": {k: {kk: vv for kk, vv in v.items() if kk != "bytes"} for k, v in kern.items()}},
             "phases_ms_per_tree": {k: v / args.steps for k, v in tim.items()},
             "cpu_baseline": cpu,
             "e2e": e2e,

@@ -105,7 +105,12 @@ enum {
   GBDT_PHASE_PARTITION = 4,  /* order-preserving partition */
   GBDT_PHASE_COMM = 5,       /* NCCL allgather of node bests + bitmap allreduce */
   GBDT_PHASE_TOTAL = 6,      /* whole gbdt_train on the device */
-  GBDT_N_PHASES = 7
+  /* kernel-level timers nested inside the phases above (profile = 1): */
+  GBDT_PHASE_K_CHUNK_AGG = 7, /* k_chunk_agg + exact carry scan (inside SPLIT_FIND) */
+  GBDT_PHASE_K_SPLIT = 8,     /* k_sf_fast + k_sf_gen: scan, gains, node bests (inside SPLIT_FIND) */
+  GBDT_PHASE_K_COUNT = 9,     /* k_part_count + count scan + plan (inside PARTITION) */
+  GBDT_PHASE_K_SCATTER = 10,  /* k_part_scatter (+ RLE run split) (inside PARTITION) */
+  GBDT_N_PHASES = 11
 };
 
 /* Copies a CSR matrix (indptr int64[n_rows+1], indices int32[nnz] strictly increasing per row,

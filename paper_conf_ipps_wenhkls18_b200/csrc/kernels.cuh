@@ -149,8 +149,9 @@ struct LevelKernels {
   void tile_prefix(const SplitArgs& A, int hmode, bool gather, unsigned groups, cudaStream_t st);
   void split_find(const SplitArgs& A, int hmode, bool missing, bool rle, cudaStream_t st);
   void seg_totals(const SplitArgs& A, int hmode, cudaStream_t st);
-  void partition(const PartArgs& A, const PlanArgs& P, bool counted, bool with_h, unsigned groups,
-                 const RunArgs* rle, cudaStream_t st);
+  // a8: count -> exact scan -> plan (next level's tables), then the stable scatter
+  void partition_count(const PartArgs& A, const PlanArgs& P, bool counted, unsigned groups, cudaStream_t st);
+  void partition_scatter(const PartArgs& A, bool with_h, const RunArgs* rle, cudaStream_t st);
 };
 
 }  // namespace gbdt

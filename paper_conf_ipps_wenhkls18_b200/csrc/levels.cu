@@ -1608,8 +1608,8 @@ void LevelKernels::seg_totals(const SplitArgs& A, int hmode, cudaStream_t st) {
   count_launch();
 }
 
-void LevelKernels::partition(const PartArgs& A, const PlanArgs& P, bool counted, bool with_h, unsigned groups,
-                             const RunArgs* rle, cudaStream_t st) {
+void LevelKernels::partition_count(const PartArgs& A, const PlanArgs& P, bool counted, unsigned groups,
+                                   cudaStream_t st) {
   k_part_count<<<grid_count, kThreads, 0, st>>>(A, counted ? 1 : 0);
   GBDT_LAUNCH_CHECK();
   count_launch();
@@ -1621,6 +1621,9 @@ void LevelKernels::partition(const PartArgs& A, const PlanArgs& P, bool counted,
   k_chunk_attr<<<(unsigned)(sms * 8), kThreads, 0, st>>>(P);
   GBDT_LAUNCH_CHECK();
   count_launch(3);
+}
+
+void LevelKernels::partition_scatter(const PartArgs& A, bool with_h, const RunArgs* rle, cudaStream_t st) {
   if (rle) {
     if (with_h) k_part_scatter<true, true><<<grid_scatter[1], kThreads, scatter_smem(true), st>>>(A);
     else k_part_scatter<false, true><<<grid_scatter[0], kThreads, scatter_smem(false), st>>>(A);
@@ -1637,7 +1640,7 @@ void LevelKernels::partition(const PartArgs& A, const PlanArgs& P, bool counted,
     else k_part_scatter<false, false><<<grid_scatter[0], kThreads, scatter_smem(false), st>>>(A);
   }
   GBDT_LAUNCH_CHECK();
-  count_launch(2);
+  count_launch();
 }
 
 }  // namespace gbdt

@@ -579,9 +579,9 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     w.tkey = tkey + (size_t)li * Kcap;
   }
 
-  PhaseTimer tm;
-  tm.on = P.profile != 0;
-  tm.st = st;
+  PhaseTimer tm, kt;  // phases; kernel-level timers nested inside them
+  tm.on = kt.on = P.profile != 0;
+  tm.st = kt.st = st;
   cudaEvent_t tot0 = nullptr, tot1 = nullptr;
   if (tm.on) {
     GBDT_CUDA(cudaEventCreate(&tot0));
@@ -630,10 +630,14 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         A.glist = w.glist[lvl & 1]; A.hlist = w.hlist[lvl & 1]; A.cagg = w.cagg; A.carry = w.carry;
         A.sgrp = w.sgrp; A.nrec = w.nrec; A.gkey = w.gkey; A.shard = sh.index;
         A.segPG_out = w.segPG; A.segPH_out = w.segPH;
+        kt.begin(GBDT_PHASE_K_CHUNK_AGG);
         LK.tile_prefix(A, hmode, /*gather=*/lvl == 0, w.groups, st);
+        kt.end();
         // present totals per segment first (needed for the missing direction)
         if (ds.has_missing) LK.seg_totals(A, hmode, st);
+        kt.begin(GBDT_PHASE_K_SPLIT);
         LK.split_find(A, hmode, ds.has_missing, sh.rle, st);
+        kt.end();
       }
       tm.end();
       tm.begin(GBDT_PHASE_DECIDE);
@@ -722,7 +726,12 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
           RA.slist = w.slist; RA.cpre = w.cpre; RA.run_seg = w.run_seg; RA.run_hl = w.run_hl; RA.cnt = w.rcnt; RA.fl = w.rfl;
           RA.Rp1 = w.Rp1; RA.sgrp = w.rsgrp; RA.groups = w.rgroups;
         }
-        LK.partition(PA, PL, ds.has_missing, hmode == kHGather, w.groups, sh.rle ? &RA : nullptr, st);
+        kt.begin(GBDT_PHASE_K_COUNT);
+        LK.partition_count(PA, PL, ds.has_missing, w.groups, st);
+        kt.end();
+        kt.begin(GBDT_PHASE_K_SCATTER);
+        LK.partition_scatter(PA, hmode == kHGather, sh.rle ? &RA : nullptr, st);
+        kt.end();
       }
       tm.end();
     }
@@ -752,6 +761,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   for (int i = 0; i < GBDT_N_PHASES; ++i) model.timings[i] = 0.0;
   if (tm.on) {
     tm.collect(model.timings);
+    kt.collect(model.timings);
     float tt = 0;
     GBDT_CUDA(cudaEventElapsedTime(&tt, tot0, tot1));
     model.timings[GBDT_PHASE_TOTAL] = tt;
