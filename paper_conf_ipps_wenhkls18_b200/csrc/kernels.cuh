@@ -66,8 +66,10 @@ struct SplitArgs {
   int* nrec;
   unsigned long long* gkey;  // [Kcap] per node max gain key
   int shard;
-  double* segPG_out;     // totals pass output
-  double* segPH_out;
+  double* segPG_out;     // present totals per segment (missing values), written by k_chunk_agg
+  double* segPH_out;     //   + k_seg_totals
+  int32_t* segEnd;       // [m*K] chunk holding the segment's last entry if the segment began in an
+                         // earlier chunk, else -1; nullptr: no missing values
 };
 
 // Decoupled look-back storage of the partition's (high, low) counts: integers, exact in any order.

@@ -344,6 +344,12 @@ __global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
         d.vnext = vnx;
         A.desc[c] = d;
         fxv_store(A.cagg + 5ll * c, FXV{to_fx(lg, Fg), to_fx(lh, Fh), len, s0 == M.p0 ? 1 : 0}, M.reset);
+        if (A.segEnd && p1 == se) {  // the segment ends here: its present totals (see k_seg_totals)
+          const long long s = M.sb + j0;
+          A.segPG_out[s] = lg;
+          A.segPH_out[s] = lh;
+          A.segEnd[s] = s0 == M.p0 ? -1 : c;
+        }
       }
       continue;
     }
@@ -376,6 +382,25 @@ __global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
     }
     if (lane == 31)
       fxv_store(A.cagg + 5ll * c, FXV{to_fx(run.g, Fg), to_fx(run.h, Fh), run.c, run.f}, M.reset);
+    if (A.segEnd) {
+      // present totals of the segments ending in this chunk: the in-chunk segmented sum at their
+      // last entry; k_seg_totals adds the carry when the segment began in an earlier chunk
+      SVf exc = shfl_up(run, 1);
+      if (lane == 0) exc = svf_zero();
+      SVf loc = svf_zero();
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) {
+        if (!((vm >> k) & 1)) continue;
+        if ((hm >> k) & 1) { loc.g = g[k]; loc.h = h[k]; loc.c = 1; loc.f = 1; }
+        else { loc.g = loc.g + g[k]; loc.h = loc.h + h[k]; loc.c += 1; }
+        if ((rem >> k) & 1) {
+          const long long s = M.sb + sj[k];
+          A.segPG_out[s] = loc.f ? loc.g : exc.g + loc.g;
+          A.segPH_out[s] = loc.f ? loc.h : exc.h + loc.h;
+          A.segEnd[s] = (loc.f || exc.f) ? -1 : c;
+        }
+      }
+    }
   }
 }
 
@@ -880,6 +905,10 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
   constexpr bool kH = HMODE == kHGather;
   __shared__ NodeBest B;
   __shared__ unsigned char flg[kWarps][kChunk];
+  // per-warp best per node: a chunk lies in one attribute, whose segments belong to distinct
+  // nodes, so a warp never posts two candidates for one node at once (no atomics, no locks)
+  __shared__ unsigned long long wgk[kTotals ? 1 : kWarps][kWarpK];
+  __shared__ Rec wrec[kTotals ? 1 : kWarps][kWarpK];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int K = *A.t.Kp;
   const int C = *A.t.tb.C;
@@ -888,6 +917,8 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
   const int Fg = A.fx[0], Fh = A.fx[1];
   const double lam = A.lam;
   nb_init(B, A, K);
+  if (!kTotals)
+    for (int j = threadIdx.x; j < kWarps * kWarpK; j += blockDim.x) wgk[j / kWarpK][j % kWarpK] = 0ull;
   __syncthreads();
   const int nw = (gridDim.x * blockDim.x) >> 5;
   // with missing values every chunk; else the chunks k_chunk_agg listed (they cross segments)
@@ -1075,11 +1106,28 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
         r.GL = g[k]; r.HL = h[k]; r.cntL = cnt[k];
       }
       r.gain = eq2_gain(r.GL, r.HL, nv.G, nv.H, lam, nv.P);
-      post_record(B, A, K, r);
+      if (K <= kWarpK) {
+        const unsigned long long gk = gain_key(r.gain);
+        if (rec_better(gk, r, wgk[wid][j], wrec[wid][j])) { wgk[wid][j] = gk; wrec[wid][j] = r; }
+      } else {
+        post_record(B, A, K, r);
+      }
     }
     __syncwarp();
   }
-  if (!kTotals) nb_flush(B, A, K);
+  if (!kTotals && K <= kWarpK) {  // merge the warp tables, one record per node and CTA
+    __syncthreads();
+    for (int j = threadIdx.x; j < K; j += blockDim.x) {
+      int bw = -1;
+      for (int w = 0; w < kWarps; ++w)
+        if (wgk[w][j] && (bw < 0 || rec_better(wgk[w][j], wrec[w][j], wgk[bw][j], wrec[bw][j]))) bw = w;
+      if (bw >= 0) {
+        const int gs = atomicAdd(A.nrec, 1);
+        A.rec[gs] = wrec[bw][j];
+        atomicMax(A.gkey + j, wgk[bw][j]);
+      }
+    }
+  }
 }
 
 // ============================================================================ a8: partition
@@ -1537,6 +1585,21 @@ void launch_scan(const int32_t* Cp, unsigned long long* in, unsigned long long* 
   count_launch(3);
 }
 
+// Present totals of every segment (missing values): the partial written by k_chunk_agg at the
+// segment's last entry, plus the exact carry of that chunk when the segment began before it.
+__global__ void __launch_bounds__(kThreads) k_seg_totals(SplitArgs A) {
+  const long long S = (long long)A.t.m * *A.t.Kp;
+  const int Fg = A.fx[0], Fh = A.fx[1];
+  for (long long s = blockIdx.x * (long long)blockDim.x + threadIdx.x; s < S; s += (long long)gridDim.x * blockDim.x) {
+    if (A.t.tb.seg_cnt[s] == 0) continue;
+    const int ce = A.segEnd[s];
+    if (ce < 0) continue;
+    const FXV cx = fxv_load(A.carry + 5ll * ce);
+    A.segPG_out[s] = from_fx(cx.g, Fg) + A.segPG_out[s];
+    A.segPH_out[s] = from_fx(cx.h, Fh) + A.segPH_out[s];
+  }
+}
+
 }  // namespace
 
 void LevelKernels::init(int device) {
@@ -1578,6 +1641,11 @@ void LevelKernels::tile_prefix(const SplitArgs& A, int hmode, bool gather, unsig
   GBDT_LAUNCH_CHECK();
   count_launch();
   launch_scan<true>(A.t.tb.C, A.cagg, A.sgrp, A.carry, groups, st);
+  if (A.segEnd) {
+    k_seg_totals<<<(unsigned)(sms * 4), kThreads, 0, st>>>(A);
+    GBDT_LAUNCH_CHECK();
+    count_launch();
+  }
 }
 
 void LevelKernels::split_find(const SplitArgs& A, int hmode, bool missing, bool rle, cudaStream_t st) {

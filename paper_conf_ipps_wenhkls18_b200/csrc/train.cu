@@ -353,6 +353,7 @@ struct ShardWork {
   Rec* rec;
   ChunkDesc* desc;
   int32_t* genlist;
+  int32_t* segEnd;
   int* nrec;
   unsigned long long *gkey, *tkey;
   int32_t *segH, *segL;
@@ -498,7 +499,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       q.take<unsigned long long>(2 * C0); q.take<unsigned long long>(2 * C0);
       q.take<unsigned long long>(5 * (size_t)LevelKernels::scan_groups(C0) + 8);
       q.take<int32_t>(T0); q.take<unsigned long long>(T0); q.take<unsigned long long>(T0);
-      q.take<Rec>(R); q.take<ChunkDesc>(C0); q.take<int32_t>(C0);
+      q.take<Rec>(R); q.take<ChunkDesc>(C0); q.take<int32_t>(C0); q.take<int32_t>(S);
       q.take<int32_t>(S); q.take<int32_t>(S); q.take<unsigned long long>(S); q.take<int64_t>(S); q.take<int64_t>(S);
       q.take<int64_t>(m); q.take<double>(S); q.take<double>(S); q.take<int>(4);
       q.take<unsigned long long>(2 * (size_t)(m + 1)); q.take<unsigned long long>(2 * (size_t)LevelKernels::scan_groups(m + 1) + 8);
@@ -531,6 +532,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     w.rec = q.take<Rec>(R);
     w.desc = q.take<ChunkDesc>(C0);
     w.genlist = q.take<int32_t>(C0);
+    w.segEnd = q.take<int32_t>(S);
     w.segH = q.take<int32_t>(S); w.segL = q.take<int32_t>(S);
     w.seg_pre = q.take<unsigned long long>(S);
     w.out_hi = q.take<int64_t>(S); w.out_lo = q.take<int64_t>(S);
@@ -630,11 +632,12 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         A.glist = w.glist[lvl & 1]; A.hlist = w.hlist[lvl & 1]; A.cagg = w.cagg; A.carry = w.carry;
         A.sgrp = w.sgrp; A.nrec = w.nrec; A.gkey = w.gkey; A.shard = sh.index;
         A.segPG_out = w.segPG; A.segPH_out = w.segPH;
+        // present totals per segment (needed for the missing direction), from the chunk pass
+        A.segEnd = ds.has_missing ? w.segEnd : nullptr;
         kt.begin(GBDT_PHASE_K_CHUNK_AGG);
         LK.tile_prefix(A, hmode, /*gather=*/lvl == 0, w.groups, st);
         kt.end();
-        // present totals per segment first (needed for the missing direction)
-        if (ds.has_missing) LK.seg_totals(A, hmode, st);
+
         kt.begin(GBDT_PHASE_K_SPLIT);
         LK.split_find(A, hmode, ds.has_missing, sh.rle, st);
         kt.end();
