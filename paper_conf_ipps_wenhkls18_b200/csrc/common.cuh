@@ -110,6 +110,10 @@ __device__ __forceinline__ unsigned long long gain_key(double g) {
   long long b = __double_as_longlong(g);
   return b < 0 ? ~(unsigned long long)b : ((unsigned long long)b | 0x8000000000000000ull);
 }
+// inverse of gain_key for a non-empty key
+__device__ __forceinline__ double key_gain(unsigned long long k) {
+  return __longlong_as_double((long long)((k & 0x8000000000000000ull) ? (k & 0x7fffffffffffffffull) : ~k));
+}
 // fp32 -> u32 ascending order key
 __device__ __forceinline__ unsigned int fkey(float v) {
   unsigned int b = __float_as_uint(v);

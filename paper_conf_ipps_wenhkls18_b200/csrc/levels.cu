@@ -122,7 +122,11 @@ __device__ __forceinline__ double hess_of(double g) {
   // logistic, 0/1 labels: y = [g < 0] (g = p - y with p in [0,1]); q = g + y; reading R5b
   const double q = g < 0.0 ? __dadd_rn(g, 1.0) : g;
   const double hh = __dmul_rn(q, __dsub_rn(1.0, q));
-  return hh > 1e-16 ? hh : 1e-16;
+  // max(hh, 1e-16); hh is never NaN (q in [0, 1]), so a plain compare-select (no fmax NaN rules)
+  double r;
+  asm("{\n .reg .pred p;\n setp.lt.f64 p, %1, 0d3C9CD2B297D889BC;\n selp.f64 %0, 0d3C9CD2B297D889BC, %1, p;\n}"
+      : "=d"(r) : "d"(hh));
+  return r;
 }
 
 // 1/x for x > 0 (normal): hardware seed + two Newton steps (~1 ulp).  Used only to RANK the
@@ -677,17 +681,17 @@ __device__ __forceinline__ void rle_values(const Tables& tb, int cg, long long p
 __device__ __forceinline__ void lds_blocked8(const double* chunk, int lane, double* out) {
   const double2* p = reinterpret_cast<const double2*>(chunk) + lane * 4;
   const int s = (lane >> 1) & 3;
-  double2 x[4];
+  double2 x[4], y[4];
 #pragma unroll
   for (int j = 0; j < 4; ++j) x[j] = p[(j + s) & 3];  // x[j] = piece (j + s) & 3
+  // piece r = x[(r - s) & 3]: rotate by s & 1, then by s & 2 (two select stages)
+#pragma unroll
+  for (int r = 0; r < 4; ++r) y[r] = (s & 1) ? x[(r + 3) & 3] : x[r];
 #pragma unroll
   for (int r = 0; r < 4; ++r) {
-    double2 y = x[0];
-#pragma unroll
-    for (int j = 1; j < 4; ++j)
-      if (((j + s) & 3) == r) y = x[j];
-    out[2 * r] = y.x;
-    out[2 * r + 1] = y.y;
+    const double2 z = (s & 2) ? y[(r + 2) & 3] : y[r];
+    out[2 * r] = z.x;
+    out[2 * r + 1] = z.y;
   }
 }
 __device__ __forceinline__ void lds_blocked8f(const float* chunk, int lane, float* out) {
@@ -785,48 +789,39 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
       const int j = jf & 0xffff;
       float* sv = W.val[st];
       const int q0 = lane * kItems;
-      // the lane's 8 consecutive entries into registers with bank-rotated 16-byte loads
-      double g[kItems], hh[kH ? kItems : 1];
+      double g[kItems], hk[kItems];
       float v[kItems], vn = 0.f;
+      if (!kRLE && lane == 0) sv[len] = d.vnext;  // the value after the chunk follows its last entry
+      __syncwarp();
       lds_blocked8(W.g[st], lane, g);
-      if (kH) lds_blocked8(W.h[st], lane, hh);
+      if (kH) lds_blocked8(W.h[st], lane, hk);
       if (kRLE) {
+        // rle_values also fills v[len - q0] (< kItems) or vn with the value after the chunk
         if (q0 < len) rle_values(A.t.tb, chunk(i), p0, len, (jf & kDescNext) != 0, p0 + q0, K, d.a * K + K, v, vn);
       } else {
         lds_blocked8f(sv, lane, v);
         vn = __shfl_down_sync(0xffffffffu, v[0], 1);
-        if (q0 + kItems >= len) vn = d.vnext;  // the entry after the chunk
+        if (lane == 31) vn = sv[kChunk];
       }
-      // value after item k (the chunk's last item: the value after the chunk, when there is one)
-      auto next_v = [&](int k) { return (k < kItems - 1 && q0 + k + 1 < len) ? v[k + 1] : vn; };
-      if (kRLE && q0 + kItems > len) {
-        // rle_values filled the value after the chunk into v[len - q0]
-        const int kl = len - q0;
+      if (!kH) {
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) hk[k] = hess_of<HMODE>(g[k]);
+      }
+      if (q0 + kItems > len) {  // the chunk's tail: items past its end contribute nothing
 #pragma unroll
         for (int k = 0; k < kItems; ++k)
-          if (k == kl) vn = v[k];
+          if (q0 + k >= len) { g[k] = 0.0; hk[k] = 0.0; }
       }
-      // pass 1: the lane's sums
-      double lg = 0.0, lh = 0.0;
-      int lc = 0;
-#pragma unroll
-      for (int k = 0; k < kItems; ++k) {
-        if (q0 + k < len) {
-          const double hk = kH ? hh[k] : hess_of<HMODE>(g[k]);
-          lg = lg + g[k]; lh = lh + hk; ++lc;
-        }
-      }
-      double wg = lg, wh = lh;
-      int wc = lc;
+      // pass 1: the lane's sums (fixed tree association), warp scan -> the lane's exclusive prefix
+      double wg = ((g[0] + g[1]) + (g[2] + g[3])) + ((g[4] + g[5]) + (g[6] + g[7]));
+      double wh = ((hk[0] + hk[1]) + (hk[2] + hk[3])) + ((hk[4] + hk[5]) + (hk[6] + hk[7]));
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         const double yg = __shfl_up_sync(0xffffffffu, wg, o), yh = __shfl_up_sync(0xffffffffu, wh, o);
-        const int yc = __shfl_up_sync(0xffffffffu, wc, o);
-        if (lane >= o) { wg = yg + wg; wh = yh + wh; wc += yc; }
+        if (lane >= o) { wg = yg + wg; wh = yh + wh; }
       }
       double eg = __shfl_up_sync(0xffffffffu, wg, 1), eh = __shfl_up_sync(0xffffffffu, wh, 1);
-      int ec = __shfl_up_sync(0xffffffffu, wc, 1);
-      if (lane == 0) { eg = 0.0; eh = 0.0; ec = 0; }
+      if (lane == 0) { eg = 0.0; eh = 0.0; }
       const bool head0 = (jf & kDescHead0) != 0;
       double bg, bh;
       int bc;
@@ -834,48 +829,59 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
         const FXV cx = fxv_load(W.carry[st]);
         bg = (head0 ? 0.0 : from_fx(cx.g, Fg)) + eg;
         bh = (head0 ? 0.0 : from_fx(cx.h, Fh)) + eh;
-        bc = (head0 ? 0 : cx.c) + ec;
+        bc = (head0 ? 0 : cx.c) + min(q0, len);  // entries of the segment before the lane's first item
       }
       const NodeV nv = node_v(S.B, A, K, j);
-      // pass 2: prefix at every run end, ranked inside the lane by the score num/den compared by
-      // cross-multiplication (no division), num = GL^2 (HR+l) + GR^2 (HL+l), den = (HL+l)(HR+l)
-      double bnum = 0.0, bden = 1.0, xg = 0.0, xh = 0.0;
-      int bq = INT_MAX, xc = 0;
-      float xv = 0.f;
-      double pg = 0.0, phh = 0.0;
-      int pc = 0;
-      const int se_q = (int)min(se - p0, (long long)kChunk + 1);  // segment end, chunk-relative
+      // Candidates are run ends (the next value differs) with a non-empty low side: there are no
+      // missing values on this path, so that excludes exactly the segment's last entry.
+      const int nc = min(((p0 + len == se) ? len - 1 : len) - q0, nv.C - 1 - bc);
+      // pass 2: prefix at every item, candidates ranked inside the lane by the score num/den
+      // compared by cross-multiplication (no division), num = GL^2 (HR+l) + GR^2 (HL+l),
+      // den = (HL+l)(HR+l); only the winning item index is carried
+      const double Hl = nv.H + lam;
+      double pg = bg, phh = bh, bnum = -1.0, bden = 1.0;
+      int bk = -1;
 #pragma unroll
       for (int k = 0; k < kItems; ++k) {
-        const int q = q0 + k;
-        if (q < len) {
-          const double hk = kH ? hh[k] : hess_of<HMODE>(g[k]);
-          pg = pg + g[k]; phh = phh + hk; ++pc;
-          const bool cand = (q + 1 == se_q) || (next_v(k) != v[k]);
-          const int cL = bc + pc;
-          if (cand && cL >= 1 && nv.C - cL >= 1) {
-            const double GL = bg + pg, HL = bh + phh;
-            const double dl = HL + lam, dr = (nv.H - HL) + lam, GR = nv.G - GL;
-            const double num = __fma_rn(GL * GL, dr, __dmul_rn(GR * GR, dl)), den = __dmul_rn(dl, dr);
-            if (bq == INT_MAX || __dmul_rn(num, bden) > __dmul_rn(bnum, den)) {
-              bnum = num; bden = den; bq = q; xg = GL; xh = HL; xc = cL; xv = v[k];
-            }
-          }
-        }
+        pg = pg + g[k];
+        phh = phh + hk[k];
+        const float nx = k < kItems - 1 ? v[k + 1] : vn;
+        const double dl = phh + lam, dr = Hl - phh, GR = nv.G - pg;
+        const double num = __fma_rn(__dmul_rn(pg, pg), dr, __dmul_rn(__dmul_rn(GR, GR), dl)), den = __dmul_rn(dl, dr);
+        if (k < nc && nx != v[k] && __dmul_rn(num, bden) > __dmul_rn(bnum, den)) { bnum = num; bden = den; bk = k; }
       }
-      double wb = bq == INT_MAX ? -INFINITY : __dmul_rn(bnum, rcp_nr(bden));
-      int wq = bq;
+      double wb = bk < 0 ? -INFINITY : __dmul_rn(bnum, rcp_nr(bden));
+      int wq = bk < 0 ? INT_MAX : q0 + bk;
 #pragma unroll
       for (int o = 16; o; o >>= 1) {
         const double ob = __shfl_xor_sync(0xffffffffu, wb, o);
         const int oq = __shfl_xor_sync(0xffffffffu, wq, o);
         if (ob > wb || (ob == wb && oq < wq)) { wb = ob; wq = oq; }
       }
-      if (wq != INT_MAX && wq == bq) {
+      // Can the chunk's best still beat node j's best so far in this CTA?  Its approximate gain
+      // (the ranking score, ~1e-15 relative) must come within a 1e-12 relative slack of it;
+      // otherwise the exact Eq. 2 evaluation and the post are skipped (warp-uniform test).
+      bool promising = wq != INT_MAX;
+      if (promising && K <= kWarpK) {
+        const unsigned long long cur = *reinterpret_cast<volatile unsigned long long*>(&S.B.gk[j]);
+        if (cur) {
+          const double ga = 0.5 * (wb - nv.P), slack = 1e-12 * (fabs(wb) + fabs(nv.P));
+          promising = ga + slack >= key_gain(cur);
+        }
+      }
+      if (promising && bk >= 0 && wq == q0 + bk) {
+        // the winner's prefix, by the same sequence of additions as pass 2
+        double xg = bg, xh = bh;
+        float xv = 0.f;
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+          if (k <= bk) { xg = xg + g[k]; xh = xh + hk[k]; }
+          if (k == bk) xv = v[k];
+        }
         Rec r;
         r.GL = xg;
         r.HL = xh;
-        r.cntL = xc;
+        r.cntL = bc + bk + 1;
         r.gain = eq2_gain(xg, xh, nv.G, nv.H, lam, nv.P);
         r.value = xv;
         r.attr = A.t.a_base + d.a;
@@ -883,7 +889,7 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
         r.node = j;
         r.epoch = epoch;
         r.shard = A.shard;
-        r.pos = p0 + bq;
+        r.pos = p0 + bk + q0;
         post_record(S.B, A, K, r);
       }
     }
