@@ -233,6 +233,35 @@ __device__ __forceinline__ void assign_segments(const long long* ss, const long 
   }
 }
 
+// Segment holding list position p0 (the largest j with ss[j] <= p0, as the binary searches find
+// it) and that segment's start/end, warp-cooperatively: with K <= 32 one coalesced load of the
+// attribute's segment table and a ballot instead of log2(K) dependent loads.  Warp-uniform result.
+struct SegOf {
+  int j;
+  long long s0, se;
+};
+__device__ __forceinline__ SegOf warp_seg(const long long* ss, const long long* sc, int K, long long p0, int lane) {
+  SegOf r;
+  if (K <= 32) {
+    const long long s = lane < K ? ss[lane] : LLONG_MAX;
+    const long long c = lane < K ? sc[lane] : 0;
+    const unsigned msk = __ballot_sync(0xffffffffu, s <= p0);
+    r.j = 31 - __clz(msk | 1u);
+    r.s0 = __shfl_sync(0xffffffffu, s, r.j);
+    r.se = r.s0 + __shfl_sync(0xffffffffu, c, r.j);
+  } else {
+    int lo = 0, hi = K - 1;
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (ss[mid] <= p0) lo = mid; else hi = mid - 1;
+    }
+    r.j = lo;
+    r.s0 = ss[lo];
+    r.se = r.s0 + sc[lo];
+  }
+  return r;
+}
+
 // ============================================================================ a4: chunk aggregates
 // One warp per chunk: g (h) of its entries -- gathered at the root (L2 evict-last) and laid out as
 // the chunk's g-list, read from the partition-carried g-list below -- and the chunk's segmented
@@ -295,38 +324,33 @@ __global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
             }
         }
       } else {
+        // every list is padded to 4 entries: the lane's two 4-entry halves are loaded whole
         const double2* gi = reinterpret_cast<const double2*>(A.glist + base);
         const double2* hi2 = reinterpret_cast<const double2*>(A.hlist + base);
+        const bool two = base + 4 < p1;
 #pragma unroll
         for (int q = 0; q < kItems / 2; ++q) {
-          const double2 x = __ldcs(gi + q);
-          g[2 * q] = x.x; g[2 * q + 1] = x.y;
-          if (HMODE == kHGather) { const double2 y = __ldcs(hi2 + q); h[2 * q] = y.x; h[2 * q + 1] = y.y; }
+          if (q < 2 || two) {
+            const double2 x = __ldcs(gi + q);
+            g[2 * q] = x.x; g[2 * q + 1] = x.y;
+            if (HMODE == kHGather) { const double2 y = __ldcs(hi2 + q); h[2 * q] = y.x; h[2 * q + 1] = y.y; }
+          }
         }
+        const int nv = (int)min((long long)kItems, p1 - base);
+        vm = (1u << nv) - 1u;
 #pragma unroll
         for (int k = 0; k < kItems; ++k) {
-          if (base + k < p1) {
-            vm |= 1u << k;
-            if (HMODE != kHGather) h[k] = hess_of<HMODE>(g[k]);
-          } else {
-            g[k] = 0.0; h[k] = 0.0;
-          }
+          if (HMODE != kHGather) h[k] = hess_of<HMODE>(g[k]);
+          if (k >= nv) { g[k] = 0.0; h[k] = 0.0; }
         }
       }
     }
     // segment of the chunk's first entry (warp-uniform search; the attribute's table is in L1)
     const long long* ss = (const long long*)(A.t.tb.seg_start + M.sb);
     const long long* sc = (const long long*)(A.t.tb.seg_cnt + M.sb);
-    int j0;
-    {
-      int lo = 0, hi = K - 1;
-      while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (ss[mid] <= M.p0) lo = mid; else hi = mid - 1;
-      }
-      j0 = lo;
-    }
-    const long long s0 = ss[j0], se = s0 + sc[j0];
+    const SegOf sg = warp_seg(ss, sc, K, M.p0, lane);
+    const int j0 = sg.j;
+    const long long s0 = sg.s0, se = sg.se;
     const int len = (int)(p1 - M.p0);
     if (p1 <= se) {
       // one segment: the aggregate is the whole chunk (a head can only be its first entry)
@@ -1148,17 +1172,29 @@ __global__ void __launch_bounds__(kThreads) k_part_count(PartArgs A, int counted
   tab_load(tc, A.t);
   __syncthreads();
   const int nw = (gridDim.x * blockDim.x) >> 5;
-  for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nw) {
+  // software pipeline: the instance ids of the warp's next chunk are loaded before the side
+  // gathers of the current one, so the list stream and the (L2) gathers overlap
+  int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  int4 n0 = make_int4(0, 0, 0, 0), n1 = n0;
+  auto load_ids = [&](int cc, int4& a0, int4& a1) {
+    const ChunkMeta Mx = chunk_meta(tc, A.t, K, cc);
+    const long long b = Mx.p0 + (long long)lane * kItems;
+    if (b < Mx.p1) {
+      a0 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + b));
+      if (b + 4 < Mx.p1) a1 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + b + 4));
+    }
+  };
+  if (c < C) load_ids(c, n0, n1);
+  for (; c < C; c += nw) {
     const ChunkMeta M = chunk_meta(tc, A.t, K, c);
     const long long base = M.p0 + (long long)lane * kItems;
-    if (c + nw < C) prefetch_chunk(A.t.ins, chunk_meta(tc, A.t, K, c + nw).p0, 4, lane);
+    const int4 i0 = n0, i1 = n1;
+    if (c + nw < C) load_ids(c + nw, n0, n1);
     unsigned vm = 0, loc = 0;
     uint8_t sd[kItems];
 #pragma unroll
     for (int k = 0; k < kItems; ++k) sd[k] = 0;
     if (base < M.p1) {
-      const int4 i0 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base));
-      const int4 i1 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base + 4));
       const int id[kItems] = {i0.x, i0.y, i0.z, i0.w, i1.x, i1.y, i1.z, i1.w};
 #pragma unroll
       for (int k = 0; k < kItems; ++k)
@@ -1306,35 +1342,26 @@ __global__ void __launch_bounds__(kThreads) k_chunk_attr(PlanArgs A) {
 
 // Stable scatter ("Scatter"), one warp per chunk: out(e) = out_base(seg, side) + rank of
 // e among the segment's same-side entries = C_side(e) - C_side(seg start), C counted within the
-// attribute (chunk prefix from the count scan + in-warp exclusive count).  The kept entries are
-// staged in shared memory in destination order (the chunk's high entries, then its low ones) so
-// that the stores go out as coalesced runs; g (h) move along.
-struct ScatterStage {
-  long long dst[kChunk];
-  double g[kChunk];
-  float v[kChunk];
-  int id[kChunk];
-};
-
+// attribute (chunk prefix from the count scan + in-chunk exclusive count).  The chunk is read in
+// the STRIPED arrangement (item k of lane l is entry p0 + 32 k + l): every load is one coalesced
+// row, and within a row the kept entries of one side are ranked by a ballot, so consecutive lanes
+// write consecutive destinations straight from registers (no staging, no bank conflicts).
+// g (h) move along with the entries.
 template <bool kH, bool kRLE>
-__global__ void __launch_bounds__(kThreads) k_part_scatter(PartArgs A) {
+__global__ void __launch_bounds__(kThreads, 3) k_part_scatter(PartArgs A) {
   __shared__ TabCache tc;
-  extern __shared__ __align__(16) unsigned char sc_raw[];
-  ScatterStage* stg = reinterpret_cast<ScatterStage*>(sc_raw);
-  double* stgh = reinterpret_cast<double*>(sc_raw + sizeof(ScatterStage) * kWarps);
+  __shared__ long long wss[kWarps][kWarpK];  // the attribute's segment starts (chunks crossing segments)
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int K = *A.t.Kp;
   const int C = *A.t.tb.C;
   if (K == 0 || C == 0) return;
   tab_load(tc, A.t);
   __syncthreads();
-  ScatterStage& W = stg[wid];
-  double* Wh = stgh + (size_t)wid * kChunk;
+  const unsigned lt = (1u << lane) - 1u;
   const int nw = (gridDim.x * blockDim.x) >> 5;
   for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nw) {
     const ChunkMeta M = chunk_meta(tc, A.t, K, c);
-    const long long p1 = M.p1;
-    const long long base = M.p0 + (long long)lane * kItems;
+    const long long p0 = M.p0, p1 = M.p1;
     if (c + nw < C) {  // the warp's next chunk streams into L2 meanwhile
       const long long pn = chunk_meta(tc, A.t, K, c + nw).p0;
       prefetch_chunk(A.t.ins, pn, 4, lane);
@@ -1342,82 +1369,69 @@ __global__ void __launch_bounds__(kThreads) k_part_scatter(PartArgs A) {
       if (!kRLE) prefetch_chunk(A.t.val, pn, 4, lane);
       if (kH) prefetch_chunk(A.h_in, pn, 8, lane);
     }
-    unsigned vm = 0, loc = 0;
-    float v[kItems];
-    int id[kItems];
-    double g[kItems], h[kItems];
     uint8_t sd[kItems];
-#pragma unroll
-    for (int k = 0; k < kItems; ++k) { sd[k] = 0; v[k] = 0.f; id[k] = 0; g[k] = 0.0; h[k] = 0.0; }
-    if (base < p1) {
-      const int4 i0 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base));
-      const int4 i1 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base + 4));
-      float4 v0 = make_float4(0.f, 0.f, 0.f, 0.f), v1 = v0;
-      if (!kRLE) {  // with RLE the values live in the runs, which are split separately
-        v0 = __ldcs(reinterpret_cast<const float4*>(A.t.val + base));
-        v1 = __ldcs(reinterpret_cast<const float4*>(A.t.val + base + 4));
-      }
-      const unsigned long long pk = (unsigned long long)__ldcs(reinterpret_cast<const unsigned*>(A.slist + base)) |
-                                    ((unsigned long long)__ldcs(reinterpret_cast<const unsigned*>(A.slist + base) + 1) << 32);
-      id[0] = i0.x; id[1] = i0.y; id[2] = i0.z; id[3] = i0.w; id[4] = i1.x; id[5] = i1.y; id[6] = i1.z; id[7] = i1.w;
-      v[0] = v0.x; v[1] = v0.y; v[2] = v0.z; v[3] = v0.w; v[4] = v1.x; v[5] = v1.y; v[6] = v1.z; v[7] = v1.w;
-      const double2* gi = reinterpret_cast<const double2*>(A.g_in + base);
-      const double2* hi2 = reinterpret_cast<const double2*>(A.h_in + base);
-#pragma unroll
-      for (int q = 0; q < kItems / 2; ++q) {
-        const double2 x = __ldcs(gi + q);
-        g[2 * q] = x.x; g[2 * q + 1] = x.y;
-        if (kH) { const double2 y = __ldcs(hi2 + q); h[2 * q] = y.x; h[2 * q + 1] = y.y; }
-      }
-#pragma unroll
-      for (int k = 0; k < kItems; ++k) {
-        if (base + k < p1) { vm |= 1u << k; sd[k] = (uint8_t)((pk >> (8 * k)) & 0xff); }
-        loc += sd[k] == 1 ? 1u : (sd[k] == 2 ? (1u << 16) : 0u);
-      }
-    }
-    int sj[kItems];
-    unsigned hm, pem, rem;
-    assign_segments<false>((const long long*)(A.t.tb.seg_start + M.sb), (const long long*)(A.t.tb.seg_cnt + M.sb),
-                           p1, K, base, vm, v, 0.f, sj, hm, pem, rem);
-    unsigned inc = loc;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const unsigned y = __shfl_up_sync(0xffffffffu, inc, o);
-      if (lane >= o) inc += y;
-    }
-    const unsigned tot = __shfl_sync(0xffffffffu, inc, 31);
-    const unsigned nhi = tot & 0xffffu, nkeep = nhi + (tot >> 16);
-    unsigned ex = inc - loc;
-    const unsigned long long cpv = A.cpre[2ll * c];
-    const long long chi0 = (long long)(cpv & 0xffffffffull), clo0 = (long long)(cpv >> 32);
-    __syncwarp();
+    int id[kItems];
+    float v[kItems];
+    double g[kItems], h[kItems];
 #pragma unroll
     for (int k = 0; k < kItems; ++k) {
-      if (sd[k]) {
-        const long long s = M.sb + sj[k];
-        const unsigned long long sp = A.seg_pre[s];
-        const unsigned rh = ex & 0xffffu, rl = ex >> 16;
-        long long dst;
-        int slot;
-        if (sd[k] == 1) { dst = A.out_hi[s] + (chi0 + (long long)rh - (long long)(sp & 0xffffffffull)); slot = (int)rh; }
-        else { dst = A.out_lo[s] + (clo0 + (long long)rl - (long long)(sp >> 32)); slot = (int)(nhi + rl); }
-        W.dst[slot] = dst;
-        W.v[slot] = v[k];
-        W.id[slot] = id[k];
-        W.g[slot] = g[k];
-        if (kH) Wh[slot] = h[k];
-        ex += sd[k] == 1 ? 1u : (1u << 16);
+      const long long p = p0 + 32 * k + lane;
+      sd[k] = 0; id[k] = 0; v[k] = 0.f; g[k] = 0.0; h[k] = 0.0;
+      if (p < p1) {
+        sd[k] = __ldcs(A.slist + p);
+        id[k] = __ldcs(A.t.ins + p);
+        if (!kRLE) v[k] = __ldcs(A.t.val + p);  // with RLE the values live in the runs
+        g[k] = __ldcs(A.g_in + p);
+        if (kH) h[k] = __ldcs(A.h_in + p);
       }
     }
-    __syncwarp();
-    for (int i = lane; i < (int)nkeep; i += 32) {
-      const long long d = W.dst[i];
-      if (!kRLE) A.val_out[d] = W.v[i];
-      A.ins_out[d] = W.id[i];
-      A.g_out[d] = W.g[i];
-      if (kH) A.h_out[d] = Wh[i];
+    const long long* ss = (const long long*)(A.t.tb.seg_start + M.sb);
+    const long long* scn = (const long long*)(A.t.tb.seg_cnt + M.sb);
+    const SegOf sg = warp_seg(ss, scn, K, p0, lane);
+    const bool single = p1 <= sg.se;  // warp-uniform; nearly always on dense data
+    const unsigned long long cpv = A.cpre[2ll * c];
+    const long long chi0 = (long long)(cpv & 0xffffffffull), clo0 = (long long)(cpv >> 32);
+    long long dh0 = 0, dl0 = 0;
+    if (single) {
+      const long long s = M.sb + sg.j;
+      const unsigned long long sp = A.seg_pre[s];
+      dh0 = A.out_hi[s] + chi0 - (long long)(sp & 0xffffffffull);
+      dl0 = A.out_lo[s] + clo0 - (long long)(sp >> 32);
+    } else if (K <= kWarpK) {
+      if (lane < K) wss[wid][lane] = ss[lane];
+      __syncwarp();
     }
-    __syncwarp();
+    unsigned nh = 0, nl = 0;  // kept entries of each side in the rows before
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) {
+      const unsigned bh = __ballot_sync(0xffffffffu, sd[k] == 1), bl = __ballot_sync(0xffffffffu, sd[k] == 2);
+      if (sd[k]) {
+        const bool hi = sd[k] == 1;
+        const long long rk = hi ? (long long)(nh + __popc(bh & lt)) : (long long)(nl + __popc(bl & lt));
+        long long d;
+        if (single) {
+          d = (hi ? dh0 : dl0) + rk;
+        } else {
+          const long long p = p0 + 32 * k + lane;
+          int lo = 0, hi2 = K - 1;  // largest j with ss[j] <= p
+          while (lo < hi2) {
+            const int mid = (lo + hi2 + 1) >> 1;
+            if ((K <= kWarpK ? wss[wid][mid] : ss[mid]) <= p) lo = mid; else hi2 = mid - 1;
+          }
+          const long long s = M.sb + lo;
+          const unsigned long long sp = A.seg_pre[s];
+          d = hi ? A.out_hi[s] + (chi0 + rk - (long long)(sp & 0xffffffffull))
+                 : A.out_lo[s] + (clo0 + rk - (long long)(sp >> 32));
+        }
+        if (!kRLE) A.val_out[d] = v[k];
+        A.ins_out[d] = id[k];
+        A.g_out[d] = g[k];
+        if (kH) A.h_out[d] = h[k];
+      }
+      nh += __popc(bh);
+      nl += __popc(bl);
+    }
+    if (!single) __syncwarp();  // wss is rewritten by the warp's next crossing chunk
   }
 }
 
@@ -1568,7 +1582,7 @@ unsigned grid_for(KernelT kern, size_t smem, int sms) {
   return (unsigned)(occ * sms);
 }
 
-size_t scatter_smem(bool h) { return sizeof(ScatterStage) * kWarps + (h ? sizeof(double) * kChunk * kWarps : 0); }
+size_t scatter_smem(bool) { return 0; }
 
 size_t fast_smem(int hmode) { return hmode == kHGather ? sizeof(FastSmem<true>) : sizeof(FastSmem<false>); }
 
