@@ -99,6 +99,11 @@ struct PartArgs {
   const int64_t* out_lo;
   float* val_out;
   int32_t* ins_out;
+  // Next level's chunk aggregates, accumulated by the scatter (no missing values): exact
+  // fixed-point (g, h) per chunk (words 0-3 of each 5-word record; k_desc writes word 4)
+  unsigned long long* cagg_next;  // nullptr: the next level runs k_chunk_agg instead
+  Tables nxt;                     // next level's tables (from the plan)
+  const int32_t* fx;              // [2] fixed-point scales of this tree
 };
 
 struct PlanArgs {
@@ -144,7 +149,7 @@ struct LevelKernels {
   unsigned grid_fast[3][2] = {{0}};  // [hmode][rle]
   unsigned grid_gen = 0;
   unsigned grid_agg[3] = {0};
-  unsigned grid_scatter[2] = {0}, grid_count = 0, grid_agg_list[3] = {0};
+  unsigned grid_scatter[3][2] = {{0}}, grid_count = 0, grid_agg_list[3] = {0};  // scatter: [hmode][agg]
   void init(int device);
   // a3/a4: tile aggregates (+ g/h lists) and the exact segmented carry scan
   static unsigned scan_groups(int64_t max_chunks);
@@ -153,7 +158,10 @@ struct LevelKernels {
   void seg_totals(const SplitArgs& A, int hmode, cudaStream_t st);
   // a8: count -> exact scan -> plan (next level's tables), then the stable scatter
   void partition_count(const PartArgs& A, const PlanArgs& P, bool counted, unsigned groups, cudaStream_t st);
-  void partition_scatter(const PartArgs& A, bool with_h, const RunArgs* rle, cudaStream_t st);
+  void partition_scatter(const PartArgs& A, int hmode, const RunArgs* rle, cudaStream_t st);
+  // a3: the level's chunk descriptors and scan flags when the previous scatter accumulated the
+  // chunk aggregates, then the exact carry scan
+  void chunk_desc(const SplitArgs& A, unsigned groups, cudaStream_t st);
 };
 
 }  // namespace gbdt

@@ -1347,21 +1347,62 @@ __global__ void __launch_bounds__(kThreads) k_chunk_attr(PlanArgs A) {
 // row, and within a row the kept entries of one side are ranked by a ballot, so consecutive lanes
 // write consecutive destinations straight from registers (no staging, no bank conflicts).
 // g (h) move along with the entries.
-template <bool kH, bool kRLE>
+// Exact fixed-point add of v into the 128-bit record word pair p[0] (lo), p[1] (hi): the low word's
+// carry is propagated by this contribution itself, so the total is exact in any order.
+__device__ __forceinline__ void fx_atomic_add(unsigned long long* p, __int128 v) {
+  const unsigned long long lo = (unsigned long long)v, hi = (unsigned long long)((unsigned __int128)v >> 64);
+  const unsigned long long old = atomicAdd(p, lo);
+  const unsigned long long c = (old + lo < old) ? 1ull : 0ull;
+  if (hi + c) atomicAdd(p + 1, hi + c);
+}
+
+// Does an entry of the child segment ending at child_end count in the segmented aggregate of the
+// next-level chunk x (attribute list [cs, ce))?  Yes iff no non-empty segment starts after it in
+// the chunk, i.e. the child reaches the chunk's end (or the end of the list).
+__device__ __forceinline__ bool agg_counts(long long child_end, long long cs, long long ce, long long xi) {
+  return child_end >= min(cs + ((xi + 1) << 8), ce);
+}
+
+// Sum of v[0..7] over the warp, transpose-reduced: afterwards lane l holds the total of value
+// ((l >> 2) & 7) (bit-reversed grouping below), so lanes 0, 4, ..., 28 hold the eight totals.
+__device__ __forceinline__ double warp_sum8(double (&v)[8], int lane) {
+  const bool u16 = lane & 16, u8 = lane & 8, u4 = lane & 4;
+  double w4[4], w2[2];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const double send = u16 ? v[i] : v[i + 4], keep = u16 ? v[i + 4] : v[i];
+    w4[i] = keep + __shfl_xor_sync(0xffffffffu, send, 16);
+  }
+#pragma unroll
+  for (int i = 0; i < 2; ++i) {
+    const double send = u8 ? w4[i] : w4[i + 2], keep = u8 ? w4[i + 2] : w4[i];
+    w2[i] = keep + __shfl_xor_sync(0xffffffffu, send, 8);
+  }
+  double w = (u4 ? w2[1] : w2[0]) + __shfl_xor_sync(0xffffffffu, u4 ? w2[0] : w2[1], 4);
+  w += __shfl_xor_sync(0xffffffffu, w, 2);
+  w += __shfl_xor_sync(0xffffffffu, w, 1);
+  return w;  // value index (u16 ? 4 : 0) + (u8 ? 2 : 0) + (u4 ? 1 : 0)
+}
+
+template <int HMODE, bool kRLE, bool kAgg>
 __global__ void __launch_bounds__(kThreads, 3) k_part_scatter(PartArgs A) {
+  constexpr bool kH = HMODE == kHGather;
+  constexpr int kHalf = kItems / 2;
   __shared__ TabCache tc;
   __shared__ long long wss[kWarps][kWarpK];  // the attribute's segment starts (chunks crossing segments)
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int K = *A.t.Kp;
   const int C = *A.t.tb.C;
   if (K == 0 || C == 0) return;
+  const int Fg = kAgg ? A.fx[0] : 0, Fh = kAgg ? A.fx[1] : 0;
   tab_load(tc, A.t);
   __syncthreads();
   const unsigned lt = (1u << lane) - 1u;
   const int nw = (gridDim.x * blockDim.x) >> 5;
   for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nw) {
     const ChunkMeta M = chunk_meta(tc, A.t, K, c);
-    const long long p0 = M.p0, p1 = M.p1;
+    const long long p0 = M.p0;
+    const int len = (int)(M.p1 - p0);
     if (c + nw < C) {  // the warp's next chunk streams into L2 meanwhile
       const long long pn = chunk_meta(tc, A.t, K, c + nw).p0;
       prefetch_chunk(A.t.ins, pn, 4, lane);
@@ -1369,69 +1410,173 @@ __global__ void __launch_bounds__(kThreads, 3) k_part_scatter(PartArgs A) {
       if (!kRLE) prefetch_chunk(A.t.val, pn, 4, lane);
       if (kH) prefetch_chunk(A.h_in, pn, 8, lane);
     }
-    uint8_t sd[kItems];
-    int id[kItems];
-    float v[kItems];
-    double g[kItems], h[kItems];
-#pragma unroll
-    for (int k = 0; k < kItems; ++k) {
-      const long long p = p0 + 32 * k + lane;
-      sd[k] = 0; id[k] = 0; v[k] = 0.f; g[k] = 0.0; h[k] = 0.0;
-      if (p < p1) {
-        sd[k] = __ldcs(A.slist + p);
-        id[k] = __ldcs(A.t.ins + p);
-        if (!kRLE) v[k] = __ldcs(A.t.val + p);  // with RLE the values live in the runs
-        g[k] = __ldcs(A.g_in + p);
-        if (kH) h[k] = __ldcs(A.h_in + p);
-      }
-    }
+    // chunk-relative lane pointers (item k of the lane is entry p0 + 32 k + lane)
+    const uint8_t* sp_ = A.slist + p0 + lane;
+    const int32_t* ip_ = A.t.ins + p0 + lane;
+    const float* vp_ = A.t.val + p0 + lane;
+    const double* gp_ = A.g_in + p0 + lane;
+    const double* hp_ = A.h_in + p0 + lane;
     const long long* ss = (const long long*)(A.t.tb.seg_start + M.sb);
     const long long* scn = (const long long*)(A.t.tb.seg_cnt + M.sb);
     const SegOf sg = warp_seg(ss, scn, K, p0, lane);
-    const bool single = p1 <= sg.se;  // warp-uniform; nearly always on dense data
+    const bool single = M.p1 <= sg.se;  // warp-uniform; nearly always on dense data
     const unsigned long long cpv = A.cpre[2ll * c];
     const long long chi0 = (long long)(cpv & 0xffffffffull), clo0 = (long long)(cpv >> 32);
-    long long dh0 = 0, dl0 = 0;
+    long long dh0 = 0, dl0 = 0, ehi = 0, elo = 0;
     if (single) {
       const long long s = M.sb + sg.j;
       const unsigned long long sp = A.seg_pre[s];
-      dh0 = A.out_hi[s] + chi0 - (long long)(sp & 0xffffffffull);
-      dl0 = A.out_lo[s] + clo0 - (long long)(sp >> 32);
+      const long long oh = A.out_hi[s], ol = A.out_lo[s];
+      dh0 = oh + chi0 - (long long)(sp & 0xffffffffull);
+      dl0 = ol + clo0 - (long long)(sp >> 32);
+      if (kAgg) { ehi = oh + A.segH[s]; elo = ol + A.segL[s]; }  // ends of the two child segments
     } else if (K <= kWarpK) {
       if (lane < K) wss[wid][lane] = ss[lane];
       __syncwarp();
     }
-    unsigned nh = 0, nl = 0;  // kept entries of each side in the rows before
+    // next level: the attribute's list and chunk origin; entries of each side before the
+    // destination chunk boundary that follows the side's first destination
+    long long ncs = 0, nce = 0;
+    int ncb = 0, cutH = 0, cutL = 0;
+    if (kAgg) {
+      ncs = A.nxt.col_start[M.a];
+      nce = ncs + A.nxt.col_len[M.a];
+      ncb = A.nxt.chunk_start[M.a];
+      cutH = kChunk - (int)((dh0 - ncs) & (kChunk - 1));
+      cutL = kChunk - (int)((dl0 - ncs) & (kChunk - 1));
+    }
+    double acc[8];  // (high A, high B, low A, low B) x (g, h); A: before the boundary
 #pragma unroll
-    for (int k = 0; k < kItems; ++k) {
-      const unsigned bh = __ballot_sync(0xffffffffu, sd[k] == 1), bl = __ballot_sync(0xffffffffu, sd[k] == 2);
-      if (sd[k]) {
-        const bool hi = sd[k] == 1;
-        const long long rk = hi ? (long long)(nh + __popc(bh & lt)) : (long long)(nl + __popc(bl & lt));
-        long long d;
-        if (single) {
-          d = (hi ? dh0 : dl0) + rk;
-        } else {
-          const long long p = p0 + 32 * k + lane;
-          int lo = 0, hi2 = K - 1;  // largest j with ss[j] <= p
-          while (lo < hi2) {
-            const int mid = (lo + hi2 + 1) >> 1;
-            if ((K <= kWarpK ? wss[wid][mid] : ss[mid]) <= p) lo = mid; else hi2 = mid - 1;
-          }
-          const long long s = M.sb + lo;
-          const unsigned long long sp = A.seg_pre[s];
-          d = hi ? A.out_hi[s] + (chi0 + rk - (long long)(sp & 0xffffffffull))
-                 : A.out_lo[s] + (clo0 + rk - (long long)(sp >> 32));
+    for (int i = 0; i < 8; ++i) acc[i] = 0.0;
+    int nh = 0, nl = 0;  // kept entries of each side in the rows before
+#pragma unroll
+    for (int half = 0; half < 2; ++half) {
+      uint8_t sd[kHalf];
+      int id[kHalf];
+      float v[kHalf];
+      double g[kHalf], h[kHalf];
+#pragma unroll
+      for (int kk = 0; kk < kHalf; ++kk) {
+        const int o = 32 * (half * kHalf + kk);
+        sd[kk] = 0; id[kk] = 0; v[kk] = 0.f; g[kk] = 0.0; h[kk] = 0.0;
+        if (o + lane < len) {
+          sd[kk] = __ldcs(sp_ + o);
+          id[kk] = __ldcs(ip_ + o);
+          if (!kRLE) v[kk] = __ldcs(vp_ + o);  // with RLE the values live in the runs
+          g[kk] = __ldcs(gp_ + o);
+          if (kH) h[kk] = __ldcs(hp_ + o);
         }
-        if (!kRLE) A.val_out[d] = v[k];
-        A.ins_out[d] = id[k];
-        A.g_out[d] = g[k];
-        if (kH) A.h_out[d] = h[k];
       }
-      nh += __popc(bh);
-      nl += __popc(bl);
+#pragma unroll
+      for (int kk = 0; kk < kHalf; ++kk) {
+        const int k = half * kHalf + kk;
+        const unsigned bh = __ballot_sync(0xffffffffu, sd[kk] == 1), bl = __ballot_sync(0xffffffffu, sd[kk] == 2);
+        if (sd[kk]) {
+          const bool hi = sd[kk] == 1;
+          const int rk = hi ? nh + __popc(bh & lt) : nl + __popc(bl & lt);
+          long long d;
+          if (single) {
+            d = (hi ? dh0 : dl0) + rk;
+            if (kAgg) {
+              const double hk = kH ? h[kk] : hess_of<HMODE>(g[kk]);
+              const int slot = (hi ? 0 : 4) + (rk < (hi ? cutH : cutL) ? 0 : 2);
+#pragma unroll
+              for (int i = 0; i < 8; i += 2)
+                if (slot == i) { acc[i] += g[kk]; acc[i + 1] += hk; }
+            }
+          } else {
+            const long long p = p0 + 32 * k + lane;
+            int lo = 0, hi2 = K - 1;  // largest j with ss[j] <= p
+            while (lo < hi2) {
+              const int mid = (lo + hi2 + 1) >> 1;
+              if ((K <= kWarpK ? wss[wid][mid] : ss[mid]) <= p) lo = mid; else hi2 = mid - 1;
+            }
+            const long long s = M.sb + lo;
+            const unsigned long long sp = A.seg_pre[s];
+            d = hi ? A.out_hi[s] + (chi0 + rk - (long long)(sp & 0xffffffffull))
+                   : A.out_lo[s] + (clo0 + rk - (long long)(sp >> 32));
+            if (kAgg) {  // rare (chunks crossing segments): the entry's own exact contribution
+              const double hk = kH ? h[kk] : hess_of<HMODE>(g[kk]);
+              const long long xi = (d - ncs) >> 8;
+              const long long cend = hi ? A.out_hi[s] + A.segH[s] : A.out_lo[s] + A.segL[s];
+              if (agg_counts(cend, ncs, nce, xi)) {
+                unsigned long long* rec = A.cagg_next + 5ll * (ncb + xi);
+                fx_atomic_add(rec, to_fx(g[kk], Fg));
+                fx_atomic_add(rec + 2, to_fx(hk, Fh));
+              }
+            }
+          }
+          if (!kRLE) A.val_out[d] = v[kk];
+          A.ins_out[d] = id[kk];
+          A.g_out[d] = g[kk];
+          if (kH) A.h_out[d] = h[kk];
+        }
+        nh += __popc(bh);
+        nl += __popc(bl);
+      }
+    }
+    if (kAgg && single) {
+      // warp totals of the four (side, destination chunk) parts, then one exact atomic add each
+      const double tot = warp_sum8(acc, lane);
+      const int vi = ((lane & 16) ? 4 : 0) + ((lane & 8) ? 2 : 0) + ((lane & 4) ? 1 : 0);
+      if ((lane & 3) == 0) {
+        const bool hiS = vi < 4, B = (vi >> 1) & 1, isH = vi & 1;
+        const int n = hiS ? nh : nl, cut = hiS ? cutH : cutL;
+        const int cnt = B ? n - min(n, cut) : min(n, cut);
+        const long long d0 = hiS ? dh0 : dl0;
+        const long long xi = ((d0 - ncs) >> 8) + (B ? 1 : 0);
+        if (cnt > 0 && agg_counts(hiS ? ehi : elo, ncs, nce, xi))
+          fx_atomic_add(A.cagg_next + 5ll * (ncb + xi) + (isH ? 2 : 0), to_fx(tot, isH ? Fh : Fg));
+      }
     }
     if (!single) __syncwarp();  // wss is rewritten by the warp's next crossing chunk
+  }
+}
+
+// Chunk descriptors and scan flags of a level whose chunk aggregates the previous scatter
+// accumulated (no missing values), one thread per chunk: the same descriptor k_chunk_agg writes,
+// and word 4 of the aggregate record: entries after the chunk's last segment head (all of them
+// when there is none) | head-inside << 32 | first-chunk-of-attribute << 33.
+__global__ void __launch_bounds__(kThreads) k_desc(SplitArgs A) {
+  const int K = *A.t.Kp;
+  const int C = *A.t.tb.C;
+  if (K == 0) return;
+  for (int c = blockIdx.x * blockDim.x + threadIdx.x; c < C; c += gridDim.x * blockDim.x) {
+    const int a = A.t.tb.chunk_attr[c];
+    const long long cs = A.t.tb.col_start[a], cl = A.t.tb.col_len[a];
+    const int k = c - A.t.tb.chunk_start[a];
+    const long long p0 = cs + (long long)k * kChunk, p1 = min(p0 + (long long)kChunk, cs + cl);
+    const bool more = p1 < cs + cl;
+    const long long* ss = (const long long*)(A.t.tb.seg_start + (long long)a * K);
+    const long long* sc = (const long long*)(A.t.tb.seg_cnt + (long long)a * K);
+    int lo = 0, hi = K - 1;  // largest j with ss[j] <= p0
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (ss[mid] <= p0) lo = mid; else hi = mid - 1;
+    }
+    const int j0 = lo;
+    const long long s0 = ss[j0], se = s0 + sc[j0];
+    const bool single = p1 <= se;
+    lo = j0; hi = K - 1;  // largest j with ss[j] < p1, then back over empty segments
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (ss[mid] < p1) lo = mid; else hi = mid - 1;
+    }
+    int j1 = lo;
+    while (j1 > 0 && sc[j1] == 0 && ss[j1] >= p0) --j1;
+    const bool head = sc[j1] > 0 && ss[j1] >= p0 && ss[j1] < p1;
+    const long long cnt = head ? p1 - ss[j1] : p1 - p0;
+    ChunkDesc d;
+    d.p0 = p0;
+    d.se = se;
+    d.len = (int)(p1 - p0);
+    d.a = a;
+    d.jf = j0 | (s0 == p0 ? kDescHead0 : 0) | (single ? kDescSingle : 0) | (more ? kDescNext : 0);
+    d.vnext = (more && !A.rle) ? A.t.val[p1] : 0.f;
+    A.desc[c] = d;
+    A.cagg[5ll * c + 4] = (unsigned long long)cnt | ((unsigned long long)(head ? 1 : 0) << 32) |
+                          ((unsigned long long)(k == 0 ? 1 : 0) << 33);
+    if (!single) A.genlist[atomicAdd(A.ngen, 1)] = c;
   }
 }
 
@@ -1582,7 +1727,6 @@ unsigned grid_for(KernelT kern, size_t smem, int sms) {
   return (unsigned)(occ * sms);
 }
 
-size_t scatter_smem(bool) { return 0; }
 
 size_t fast_smem(int hmode) { return hmode == kHGather ? sizeof(FastSmem<true>) : sizeof(FastSmem<false>); }
 
@@ -1637,10 +1781,12 @@ void LevelKernels::init(int device) {
   grid_agg_list[0] = grid_for(k_chunk_agg<0, false>, 0, sms);
   grid_agg_list[1] = grid_for(k_chunk_agg<1, false>, 0, sms);
   grid_agg_list[2] = grid_for(k_chunk_agg<2, false>, 0, sms);
-  grid_scatter[0] = grid_for(k_part_scatter<false, false>, scatter_smem(false), sms);
-  grid_scatter[1] = grid_for(k_part_scatter<true, false>, scatter_smem(true), sms);
-  grid_for(k_part_scatter<false, true>, scatter_smem(false), sms);
-  grid_for(k_part_scatter<true, true>, scatter_smem(true), sms);
+  grid_scatter[0][0] = grid_for(k_part_scatter<0, false, false>, 0, sms);
+  grid_scatter[1][0] = grid_for(k_part_scatter<1, false, false>, 0, sms);
+  grid_scatter[2][0] = grid_for(k_part_scatter<2, false, false>, 0, sms);
+  grid_scatter[0][1] = grid_for(k_part_scatter<0, false, true>, 0, sms);
+  grid_scatter[1][1] = grid_for(k_part_scatter<1, false, true>, 0, sms);
+  grid_scatter[2][1] = grid_for(k_part_scatter<2, false, true>, 0, sms);
   grid_count = grid_for(k_part_count, 0, sms);
 }
 
@@ -1711,10 +1857,17 @@ void LevelKernels::partition_count(const PartArgs& A, const PlanArgs& P, bool co
   count_launch(3);
 }
 
-void LevelKernels::partition_scatter(const PartArgs& A, bool with_h, const RunArgs* rle, cudaStream_t st) {
+template <int HM, bool kR>
+void launch_scatter(const LevelKernels& L, const PartArgs& A, cudaStream_t st) {
+  if (A.cagg_next) k_part_scatter<HM, kR, true><<<L.grid_scatter[HM][1], kThreads, 0, st>>>(A);
+  else k_part_scatter<HM, kR, false><<<L.grid_scatter[HM][0], kThreads, 0, st>>>(A);
+}
+
+void LevelKernels::partition_scatter(const PartArgs& A, int hmode, const RunArgs* rle, cudaStream_t st) {
   if (rle) {
-    if (with_h) k_part_scatter<true, true><<<grid_scatter[1], kThreads, scatter_smem(true), st>>>(A);
-    else k_part_scatter<false, true><<<grid_scatter[0], kThreads, scatter_smem(false), st>>>(A);
+    if (hmode == 0) launch_scatter<0, true>(*this, A, st);
+    else if (hmode == 1) launch_scatter<1, true>(*this, A, st);
+    else launch_scatter<2, true>(*this, A, st);
     GBDT_LAUNCH_CHECK();
     k_run_count<<<(unsigned)(sms * 8), kThreads, 0, st>>>(*rle);
     GBDT_LAUNCH_CHECK();
@@ -1724,11 +1877,19 @@ void LevelKernels::partition_scatter(const PartArgs& A, bool with_h, const RunAr
     k_run_scatter<<<(unsigned)(sms * 8), kThreads, 0, st>>>(*rle);
     count_launch();
   } else {
-    if (with_h) k_part_scatter<true, false><<<grid_scatter[1], kThreads, scatter_smem(true), st>>>(A);
-    else k_part_scatter<false, false><<<grid_scatter[0], kThreads, scatter_smem(false), st>>>(A);
+    if (hmode == 0) launch_scatter<0, false>(*this, A, st);
+    else if (hmode == 1) launch_scatter<1, false>(*this, A, st);
+    else launch_scatter<2, false>(*this, A, st);
   }
   GBDT_LAUNCH_CHECK();
   count_launch();
+}
+
+void LevelKernels::chunk_desc(const SplitArgs& A, unsigned groups, cudaStream_t st) {
+  k_desc<<<(unsigned)(sms * 8), kThreads, 0, st>>>(A);
+  GBDT_LAUNCH_CHECK();
+  count_launch();
+  launch_scan<true>(A.t.tb.C, A.cagg, A.sgrp, A.carry, groups, st);
 }
 
 }  // namespace gbdt

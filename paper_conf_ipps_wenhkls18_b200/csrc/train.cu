@@ -635,7 +635,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         // present totals per segment (needed for the missing direction), from the chunk pass
         A.segEnd = ds.has_missing ? w.segEnd : nullptr;
         kt.begin(GBDT_PHASE_K_CHUNK_AGG);
-        LK.tile_prefix(A, hmode, /*gather=*/lvl == 0, w.groups, st);
+        if (lvl > 0 && !ds.has_missing) LK.chunk_desc(A, w.groups, st);  // aggregates from the scatter
+        else LK.tile_prefix(A, hmode, /*gather=*/lvl == 0, w.groups, st);
         kt.end();
 
         kt.begin(GBDT_PHASE_K_SPLIT);
@@ -718,6 +719,10 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         PA.g_in = w.glist[lvl & 1]; PA.h_in = w.hlist[lvl & 1];
         PA.g_out = w.glist[(lvl + 1) & 1]; PA.h_out = w.hlist[(lvl + 1) & 1];
         PA.epochp = epoch; PA.lb = w.lb;
+        // without missing values the scatter accumulates the next level's chunk aggregates
+        PA.cagg_next = ds.has_missing ? nullptr : w.cagg;
+        PA.nxt = tn;
+        PA.fx = fxs;
         PlanArgs PL;
         PL.m = sh.m; PL.counted = ds.has_missing; PL.Kp = cur.K; PL.Knp = nxt.K; PL.cidx = cidx; PL.ncnt = nxt.cnt;
         PL.segH = w.segH; PL.segL = w.segL; PL.seg_pre = w.seg_pre;
@@ -733,7 +738,9 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         LK.partition_count(PA, PL, ds.has_missing, w.groups, st);
         kt.end();
         kt.begin(GBDT_PHASE_K_SCATTER);
-        LK.partition_scatter(PA, hmode == kHGather, sh.rle ? &RA : nullptr, st);
+        if (PA.cagg_next)
+          GBDT_CUDA(cudaMemsetAsync(w.cagg, 0, sizeof(unsigned long long) * 5 * (size_t)std::max<int64_t>(sh.C0, 1), st));
+        LK.partition_scatter(PA, hmode, sh.rle ? &RA : nullptr, st);
         kt.end();
       }
       tm.end();
