@@ -149,7 +149,7 @@ struct LevelKernels {
   unsigned grid_fast[3][2] = {{0}};  // [hmode][rle]
   unsigned grid_gen = 0;
   unsigned grid_agg[3] = {0};
-  unsigned grid_scatter[3][2] = {{0}}, grid_count = 0, grid_agg_list[3] = {0};  // scatter: [hmode][agg]
+  unsigned grid_scatter[3][2] = {{0}}, grid_count = 0, grid_count_dense = 0, grid_agg_list[3] = {0};  // scatter: [hmode][agg]
   void init(int device);
   // a3/a4: tile aggregates (+ g/h lists) and the exact segmented carry scan
   static unsigned scan_groups(int64_t max_chunks);

@@ -1243,6 +1243,69 @@ __global__ void __launch_bounds__(kThreads) k_part_count(PartArgs A, int counted
   }
 }
 
+// Dense variant (no per-segment counts needed): two chunks per warp iteration in the striped
+// arrangement, so 16 instance-id loads and then 16 side gathers per lane are in flight at once;
+// the side gathers ask L2 to keep the per-instance side array (evict-last) while the lists stream
+// past it.  Counts by ballot; the side-list rows are written as coalesced 32-byte rows.
+__device__ __forceinline__ uint8_t ld_keep_u8(const uint8_t* p, unsigned long long pol) {
+  unsigned short v;
+  asm volatile("ld.global.nc.L2::cache_hint.u8 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol));
+  return (uint8_t)v;
+}
+__global__ void __launch_bounds__(kThreads) k_part_count_dense(PartArgs A) {
+  __shared__ TabCache tc;
+  const int lane = threadIdx.x & 31;
+  const int K = *A.t.Kp;
+  const int C = *A.t.tb.C;
+  if (K == 0 || C == 0) return;
+  tab_load(tc, A.t);
+  __syncthreads();
+  const unsigned long long keep = policy_evict_last();
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += 2 * nw) {
+    long long p0[2];
+    int len[2], rs[2], id[2][kItems];
+    uint8_t sd[2][kItems];
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      const int cu = c + u * nw;
+      len[u] = 0;
+      p0[u] = 0;
+      rs[u] = 0;
+      if (cu < C) {
+        const ChunkMeta M = chunk_meta(tc, A.t, K, cu);
+        p0[u] = M.p0;
+        len[u] = (int)(M.p1 - M.p0);
+        rs[u] = M.reset;
+      }
+      const int32_t* ip = A.t.ins + p0[u] + lane;
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) id[u][k] = (32 * k + lane < len[u]) ? __ldcs(ip + 32 * k) : -1;
+    }
+#pragma unroll
+    for (int u = 0; u < 2; ++u)
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) sd[u][k] = id[u][k] >= 0 ? ld_keep_u8(A.side + id[u][k], keep) : (uint8_t)0;
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      const int cu = c + u * nw;
+      if (cu >= C) break;
+      unsigned nh = 0, nl = 0;
+      uint8_t* so = A.slist + p0[u] + lane;
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) {
+        nh += __popc(__ballot_sync(0xffffffffu, sd[u][k] == 1));
+        nl += __popc(__ballot_sync(0xffffffffu, sd[u][k] == 2));
+        if (32 * k + lane < len[u]) __stcs(so + 32 * k, sd[u][k]);
+      }
+      if (lane == 0) {
+        A.ccnt[2ll * cu] = (unsigned long long)nh | ((unsigned long long)nl << 32);
+        A.ccnt[2ll * cu + 1] = (unsigned long long)rs[u];
+      }
+    }
+  }
+}
+
 __device__ unsigned long long block_exscan_u64(unsigned long long x, unsigned long long& total) {
   __shared__ unsigned long long ws[32];
   __shared__ unsigned long long tot;
@@ -1788,6 +1851,7 @@ void LevelKernels::init(int device) {
   grid_scatter[1][1] = grid_for(k_part_scatter<1, false, true>, 0, sms);
   grid_scatter[2][1] = grid_for(k_part_scatter<2, false, true>, 0, sms);
   grid_count = grid_for(k_part_count, 0, sms);
+  grid_count_dense = grid_for(k_part_count_dense, 0, sms);
 }
 
 unsigned LevelKernels::scan_groups(int64_t max_chunks) {
@@ -1844,7 +1908,8 @@ void LevelKernels::seg_totals(const SplitArgs& A, int hmode, cudaStream_t st) {
 
 void LevelKernels::partition_count(const PartArgs& A, const PlanArgs& P, bool counted, unsigned groups,
                                    cudaStream_t st) {
-  k_part_count<<<grid_count, kThreads, 0, st>>>(A, counted ? 1 : 0);
+  if (counted) k_part_count<<<grid_count, kThreads, 0, st>>>(A, 1);
+  else k_part_count_dense<<<grid_count_dense, kThreads, 0, st>>>(A);
   GBDT_LAUNCH_CHECK();
   count_launch();
   launch_scan<false>(A.t.tb.C, A.ccnt, A.sgrp, A.cpre, groups, st);
