@@ -37,8 +37,10 @@ UNIT = "s/tree"
 #             (+ h-list 8 when h is not a function of g; RLE: the runs replace the 4 value bytes)
 #   k_scatter per entry of the level: val 4 + ins 4 + g 8 + side 1 read; per kept entry (the
 #             next level's entries): val 4 + ins 4 + g 8 written
-BYTES_SPLIT_PER_ENTRY = 12
-BYTES_SCATTER_READ, BYTES_SCATTER_WRITE = 17, 16
+#   with RLE the 4 value bytes are not streamed (values come from the runs, a few bytes per run)
+def byte_model(rle):
+    v = 0 if rle else 4
+    return 8 + v, 13 + v, 12 + v   # split per entry; scatter read per entry, write per kept entry
 
 
 def parse():
@@ -105,19 +107,6 @@ def clock_sampler_stop(proc, dev=0):
     if not sm:
         return None
     return {"sm_mhz": statistics.median(sm), "sm_max_mhz": smax, "reasons": sorted(reasons), "samples": len(sm)}
-
-
-def entries_per_level(nodes, m_local, d):
-    """Entries the split-find kernel reads per level, from the trees: a node at depth l is active at
-    level l and, for dense data, owns count x m_local entries of the shard's lists."""
-    out = np.zeros(d, np.int64)
-    present = nodes["heap_id"] >= 0
-    heap = np.arange(nodes.shape[1])
-    depth = np.floor(np.log2(heap + 1)).astype(int)
-    for lvl in range(d):
-        sel = present & (depth[None, :] == lvl)
-        out[lvl] = int(nodes["count"][sel].sum()) * m_local
-    return out
 
 
 def oracle_sample_rate(prob, target_s, trees=2):
@@ -236,14 +225,15 @@ def main():
     torch.cuda.synchronize()
     tim = model.timings()
     nodes = model.nodes()
-    ent = entries_per_level(nodes, m_local, d)       # summed over the K trees
+    ent = model.level_entries(d)                     # list entries per level, summed over the K trees
     peak, peak_kind = peaks()
+    b_split, b_sread, b_swrite = byte_model(args.rle != "off")
     kern = {
-        "k_split": dict(bytes=float(ent.sum()) * BYTES_SPLIT_PER_ENTRY, launches=args.steps * d,
-                        ms=tim["k_split"], bytes_per_entry=BYTES_SPLIT_PER_ENTRY),
-        "k_scatter": dict(bytes=float(ent[:-1].sum()) * BYTES_SCATTER_READ + float(ent[1:].sum()) * BYTES_SCATTER_WRITE,
+        "k_split": dict(bytes=float(ent.sum()) * b_split, launches=args.steps * d,
+                        ms=tim["k_split"], bytes_per_entry=b_split),
+        "k_scatter": dict(bytes=float(ent[:-1].sum()) * b_sread + float(ent[1:].sum()) * b_swrite,
                           launches=args.steps * (d - 1), ms=tim["k_scatter"],
-                          bytes_per_entry=f"{BYTES_SCATTER_READ} read + {BYTES_SCATTER_WRITE} per kept entry"),
+                          bytes_per_entry=f"{b_sread} read + {b_swrite} per kept entry"),
     }
     for kname, kv in kern.items():
         kv["avg_launch_ms"] = kv["ms"] / kv["launches"]

@@ -149,6 +149,12 @@ gbdt_status gbdt_model_export(const gbdt_model* m, int32_t tree, gbdt_node* node
  * ms_by_phase: caller-owned, n_phases entries (<= GBDT_N_PHASES filled). */
 gbdt_status gbdt_get_timings(const gbdt_model* m, double* ms_by_phase, int32_t n_phases);
 
+/* Entries of the local shards' attribute lists that split finding scanned at each level, summed
+ * over the trees of the gbdt_train that produced m (profile = 1; else zeros).  This is the unit of
+ * the bench's byte model (bytes per entry x entries).  entries: caller-owned, n_levels entries
+ * (level l < max_depth filled, the rest zeroed). */
+gbdt_status gbdt_get_level_entries(const gbdt_model* m, int64_t* entries, int32_t n_levels);
+
 /* Dataset inspection (tests): sizes and the built layout of one shard.
  * info: [n_rows, n_cols, nnz_stored, n_shards, attr_begin(shard), attr_end(shard), rle_runs(shard)]. */
 gbdt_status gbdt_dataset_info(const gbdt_dataset* ds, int32_t shard, int64_t info[7]);

@@ -281,6 +281,13 @@ gbdt_status gbdt_get_timings(const gbdt_model* m, double* ms, int32_t n) {
   });
 }
 
+gbdt_status gbdt_get_level_entries(const gbdt_model* m, int64_t* entries, int32_t n) {
+  return guarded([&] {
+    if (!m || !entries) fail(GBDT_E_INVAL, "NULL argument");
+    for (int i = 0; i < n; ++i) entries[i] = i < (int)m->m.level_entries.size() ? m->m.level_entries[i] : 0;
+  });
+}
+
 gbdt_status gbdt_dataset_info(const gbdt_dataset* d, int32_t shard, int64_t info[7]) {
   return guarded([&] {
     if (!d || !info) fail(GBDT_E_INVAL, "NULL argument");

@@ -135,6 +135,7 @@ struct Model {
   double eta = 0, base_margin = 0, lambda = 0;
   std::vector<gbdt_node> nodes;  // n_trees * NH
   double timings[GBDT_N_PHASES] = {0};
+  std::vector<int64_t> level_entries;  // [max_depth] list entries scanned per level (profile = 1)
   int device = 0;
   int64_t nh() const { return (int64_t(1) << (max_depth + 1)) - 1; }
 };

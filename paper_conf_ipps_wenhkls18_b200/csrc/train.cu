@@ -408,6 +408,14 @@ struct PhaseTimer {
 
 }  // namespace
 
+// sum of the level's attribute list lengths (profile = 1 only)
+__global__ void k_level_entries(const int64_t* col_len, int m, unsigned long long* out) {
+  unsigned long long s = 0;
+  for (int a = blockIdx.x * blockDim.x + threadIdx.x; a < m; a += gridDim.x * blockDim.x) s += (unsigned long long)col_len[a];
+  for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if ((threadIdx.x & 31) == 0 && s) atomicAdd(out, s);
+}
+
 // Level kernels are configured once per device (smem attributes, persistent grid sizes).
 static LevelKernels& level_kernels(int device) {
   static LevelKernels lk[16];
@@ -447,6 +455,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     c.take<int32_t>(Kcap); c.take<Rec>(Kcap); c.take<Rec>((size_t)nsh * Kcap); c.take<int>(1);
     c.take<unsigned long long>((size_t)nloc * Kcap); c.take<unsigned long long>((size_t)nloc * Kcap);
     c.take<int>(nloc);
+    c.take<unsigned long long>(16);
   };
   Carve probe{nullptr};
   sz_dev(probe);
@@ -477,6 +486,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   unsigned long long* gkey = c.take<unsigned long long>((size_t)nloc * Kcap);
   unsigned long long* tkey = c.take<unsigned long long>((size_t)nloc * Kcap);
   int* nrec = c.take<int>(nloc);
+  unsigned long long* lent = c.take<unsigned long long>(16);  // entries scanned per level (profile)
 
   // ---------------------------------------------------------------- per-shard state
   std::vector<ShardWork> sw(nloc);
@@ -642,6 +652,11 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         kt.begin(GBDT_PHASE_K_SPLIT);
         LK.split_find(A, hmode, ds.has_missing, sh.rle, st);
         kt.end();
+        if (P.profile) {  // the level's list entries (byte model of the bench), off the timed kernels
+          k_level_entries<<<(unsigned)std::min<int64_t>(ceil_div(sh.m, 256), sms * 4), 256, 0, st>>>(tb.col_len, sh.m, lent + lvl);
+          GBDT_LAUNCH_CHECK();
+          count_launch();
+        }
       }
       tm.end();
       tm.begin(GBDT_PHASE_DECIDE);
@@ -763,6 +778,13 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   model.lambda = P.lambda;
   model.device = ds.device;
   model.nodes.resize((size_t)P.n_trees * NH);
+  model.level_entries.assign(d, 0);
+  if (P.profile) {
+    std::vector<unsigned long long> le(16, 0);
+    GBDT_CUDA(cudaMemcpyAsync(le.data(), lent, sizeof(unsigned long long) * 16, cudaMemcpyDeviceToHost, st));
+    GBDT_CUDA(cudaStreamSynchronize(st));
+    for (int l = 0; l < d && l < 16; ++l) model.level_entries[l] = (int64_t)le[l];
+  }
   GBDT_CUDA(cudaMemcpyAsync(model.nodes.data(), trees, sizeof(gbdt_node) * model.nodes.size(),
                             cudaMemcpyDeviceToHost, st));
   if (margin_out)

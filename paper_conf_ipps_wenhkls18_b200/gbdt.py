@@ -70,6 +70,7 @@ def lib():
     L.gbdt_model_num_nodes.argtypes = [p, i32, C.POINTER(i32)]
     L.gbdt_model_export.argtypes = [p, i32, p]
     L.gbdt_get_timings.argtypes = [p, p, i32]
+    L.gbdt_get_level_entries.argtypes = [p, p, i32]
     L.gbdt_dataset_info.argtypes = [p, i32, p]
     L.gbdt_dataset_export_layout.argtypes = [p, i32, p, p, p]
     L.gbdt_dataset_export_rle.argtypes = [p, i32, p, p, p]
@@ -81,7 +82,7 @@ def lib():
     L.gbdt_dataset_free.argtypes = [p]
     L.gbdt_model_free.argtypes = [p]
     for f in ("gbdt_load_csr", "gbdt_train", "gbdt_predict", "gbdt_model_num_trees", "gbdt_model_num_nodes",
-              "gbdt_model_export", "gbdt_get_timings", "gbdt_dataset_info", "gbdt_dataset_export_layout",
+              "gbdt_model_export", "gbdt_get_timings", "gbdt_get_level_entries", "gbdt_dataset_info", "gbdt_dataset_export_layout",
               "gbdt_dataset_export_rle", "gbdt_comm_unique_id", "gbdt_comm_init", "gbdt_comm_init_callbacks",
               "gbdt_shard_ranges"):
         getattr(L, f).restype = C.c_int
@@ -273,6 +274,12 @@ class Model:
         a = np.zeros(len(PHASES), np.float64)
         _check(lib().gbdt_get_timings(self._h, _p(a), len(PHASES)))
         return dict(zip(PHASES, a.tolist()))
+
+    def level_entries(self, levels: int) -> np.ndarray:
+        """List entries split finding scanned per level, summed over the trees (profile=True)."""
+        a = np.zeros(levels, np.int64)
+        _check(lib().gbdt_get_level_entries(self._h, _p(a), levels))
+        return a
 
     def predict(self, indptr, indices, values, n_cols, output_margin=True) -> np.ndarray:
         return predict(self, indptr, indices, values, n_cols, output_margin)
