@@ -929,6 +929,158 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
   nb_flush(S.B, A, K);
 }
 
+// ---------------------------------------------------------------------------- short chunks
+// A chunk of at most 32 entries (the typical list of a sparse attribute, "many small
+// segments") with K <= 32 nodes: lane i holds entry p0 + i.  Segment heads come from the
+// attribute's segment table (lane l holds segment l), the segmented scan and the per-segment
+// argmax run over the lanes, so the work is ~1/8 of the 8-items-per-lane general path.
+template <int HMODE, bool kMissing, bool kRLE>
+__device__ __forceinline__ void sf_short(const SplitArgs& A, NodeBest& B, unsigned long long* wgk, Rec* wrec, int c,
+                                         const ChunkDesc& d, int K, int lane, int epoch, int Fg, int Fh, double lam) {
+  constexpr bool kH = HMODE == kHGather;
+  const long long p0 = d.p0;
+  const int len = d.len;
+  const long long sb = (long long)d.a * K;
+  const long long* ss = (const long long*)(A.t.tb.seg_start + sb);
+  const long long* sc = (const long long*)(A.t.tb.seg_cnt + sb);
+  const bool valid = lane < len;
+  const long long p = p0 + lane;
+  // the attribute's segment table: lane l holds segment l
+  const long long s_l = lane < K ? ss[lane] : LLONG_MAX;
+  const long long c_l = lane < K ? sc[lane] : 0;
+  double lPG = 0.0, lPH = 0.0;
+  if (kMissing && lane < K) { lPG = A.segPG[sb + lane]; lPH = A.segPH[sb + lane]; }
+  // head mask: the first entries of the non-empty segments that start inside the chunk
+  const bool starts = lane < K && c_l > 0 && s_l >= p0 && s_l < p0 + len;
+  unsigned hbit = starts ? (1u << (int)(s_l - p0)) : 0u;
+  const unsigned hm = __reduce_or_sync(0xffffffffu, hbit);
+  // segment of the chunk's first entry (largest j with ss[j] <= p0) and of every lane
+  const unsigned le0 = __ballot_sync(0xffffffffu, s_l <= p0);
+  const int j0 = 31 - __clz(le0 | 1u);
+  // lane -> segment: the head at or before the lane (its segment is the lane l that owns it)
+  const unsigned upto = hm & (0xffffffffu >> (31 - lane));
+  const int hpos = upto ? 31 - __clz(upto) : -1;  // position of the last head <= lane
+  // the segment starting at chunk position q is the largest l with s_l == p0 + q and c_l > 0
+  const unsigned own = __ballot_sync(0xffffffffu, starts);
+  int j = j0;
+  {
+    // find l with starts && s_l - p0 == hpos: scan the owners (at most K <= 32)
+    unsigned o = own;
+    while (o) {
+      const int l = __ffs(o) - 1;
+      o &= o - 1;
+      const long long sl = __shfl_sync(0xffffffffu, s_l, l);
+      if (hpos >= 0 && sl - p0 == hpos) j = l;
+    }
+  }
+  const long long sj0 = __shfl_sync(0xffffffffu, s_l, j & 31), cj0 = __shfl_sync(0xffffffffu, c_l, j & 31);
+  const long long se = sj0 + cj0;  // end of the lane's segment
+  const double PG = kMissing ? __shfl_sync(0xffffffffu, lPG, j & 31) : 0.0;
+  const double PH = kMissing ? __shfl_sync(0xffffffffu, lPH, j & 31) : 0.0;
+  // values, g, h
+  float v = 0.f;
+  double g = 0.0, h = 0.0;
+  if (valid) {
+    if (kRLE) {
+      int lo = A.t.tb.run_chunk[c];
+      int hi = (d.jf & kDescNext) ? A.t.tb.run_chunk[c + 1] : A.t.tb.seg_run[sb + K] - 1;
+      while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (A.t.tb.run_pos[mid] <= p) lo = mid; else hi = mid - 1;
+      }
+      v = A.t.tb.run_val[lo];
+    } else {
+      v = __ldcs(A.t.val + p);
+    }
+    g = __ldcs(A.glist + p);
+    h = kH ? __ldcs(A.hlist + p) : hess_of<HMODE>(g);
+  }
+  float vn = __shfl_down_sync(0xffffffffu, v, 1);
+  if (lane == len - 1) {
+    if (d.jf & kDescNext) {
+      if (kRLE) {
+        const int rc = A.t.tb.run_chunk[c + 1];
+        vn = A.t.tb.run_val[rc];
+      } else {
+        vn = d.vnext;
+      }
+    } else {
+      vn = v;  // no entry after the chunk: the segment ends here (seg_last below)
+    }
+  }
+  // segmented inclusive scan over the lanes; lanes before the first head continue the carry
+  const int sl = hpos >= 0 ? hpos : 0;  // first lane of the lane's segment piece
+  double ig = g, ih = h;
+  int icn = valid ? 1 : 0;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const double yg = __shfl_up_sync(0xffffffffu, ig, o), yh = __shfl_up_sync(0xffffffffu, ih, o);
+    const int yc = __shfl_up_sync(0xffffffffu, icn, o);
+    if (lane - o >= sl) { ig = yg + ig; ih = yh + ih; icn += yc; }
+  }
+  if (hpos < 0) {
+    const FXV cx = fxv_load(A.carry + 5ll * c);
+    ig = from_fx(cx.g, Fg) + ig;
+    ih = from_fx(cx.h, Fh) + ih;
+    icn = cx.c + icn;
+  }
+  // candidate: the end of a run of equal values (or of the segment), both directions when the
+  // segment has missing values
+  const bool seg_last = valid && (p + 1 == se);
+  const bool cand = valid && (seg_last || vn != v);
+  const NodeV nv = node_v(B, A, K, j);
+  double best = -INFINITY;
+  int bd = 0;
+  bool ok = false;
+  if (cand) {
+    if (icn >= 1 && nv.C - icn >= 1) { best = split_score(ig, ih, nv.G, nv.H, lam); ok = true; }
+    if (kMissing) {
+      const int cM = nv.C - (int)cj0;
+      const int cL1 = icn + cM;
+      if (cM > 0 && cL1 >= 1 && nv.C - cL1 >= 1) {
+        const double g1 = split_score(ig + (nv.G - PG), ih + (nv.H - PH), nv.G, nv.H, lam);
+        if (!ok || g1 > best) { best = g1; bd = 1; ok = true; }
+      }
+    }
+  }
+  // per-segment argmax: segmented max-scan of (score, lane); earlier lane = larger value (R12)
+  double lg = ok ? best : -INFINITY;
+  int lq = ok ? lane : INT_MAX;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const double yg = __shfl_up_sync(0xffffffffu, lg, o);
+    const int yq = __shfl_up_sync(0xffffffffu, lq, o);
+    if (lane - o >= sl && (yg > lg || (yg == lg && yq < lq))) { lg = yg; lq = yq; }
+  }
+  // the last lane of each segment piece posts its winner
+  const bool piece_end = valid && (lane == len - 1 || ((hm >> (lane + 1)) & 1u) || seg_last);
+  const int q = piece_end && lq != INT_MAX ? lq : lane;
+  const double wg = __shfl_sync(0xffffffffu, ig, q), wh = __shfl_sync(0xffffffffu, ih, q);
+  const int wc = __shfl_sync(0xffffffffu, icn, q), wd = __shfl_sync(0xffffffffu, bd, q);
+  const float wv = __shfl_sync(0xffffffffu, v, q);
+  if (piece_end && lq != INT_MAX) {
+    Rec r;
+    r.value = wv;
+    r.attr = A.t.a_base + d.a;
+    r.dir = wd;
+    r.node = j;
+    r.epoch = epoch;
+    r.shard = A.shard;
+    r.pos = p0 + lq;
+    if (wd) {
+      r.GL = wg + (nv.G - PG);
+      r.HL = wh + (nv.H - PH);
+      r.cntL = wc + (nv.C - (int)cj0);
+    } else {
+      r.GL = wg; r.HL = wh; r.cntL = wc;
+    }
+    r.gain = eq2_gain(r.GL, r.HL, nv.G, nv.H, lam, nv.P);
+    const unsigned long long gk = gain_key(r.gain);
+    if (rec_better(gk, r, wgk[j], wrec[j])) { wgk[j] = gk; wrec[j] = r; }
+  }
+  __syncwarp();
+}
+
 // ---------------------------------------------------------------------------- k_sf_gen
 template <int HMODE, bool kMissing, bool kTotals, bool kRLE>
 __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
@@ -960,6 +1112,10 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
     const long long p0 = d.p0;
     const long long cp1 = p0 + d.len;
     const long long sb = (long long)d.a * K;
+    if (!kTotals && d.len <= 32 && K <= kWarpK) {  // short chunk (sparse lists): one entry per lane
+      sf_short<HMODE, kMissing, kRLE>(A, B, wgk[wid], wrec[wid], c, d, K, lane, epoch, Fg, Fh, lam);
+      continue;
+    }
     const long long base = p0 + lane * kItems;
     const long long* ss = (const long long*)(A.t.tb.seg_start + sb);
     const long long* sc = (const long long*)(A.t.tb.seg_cnt + sb);
