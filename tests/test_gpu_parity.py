@@ -243,3 +243,44 @@ def test_rle_export_matches_oracle_encoding():
         assert np.array_equal(rv[run_ptr[a]:run_ptr[a + 1]].view(np.uint32), orv.view(np.uint32))
         assert np.array_equal(rl[run_ptr[a]:run_ptr[a + 1]], orl)
     assert run_ptr[-1] == rv.size
+
+
+# ------------------------------------------------------------------ path boundaries (round 1b)
+@pytest.mark.parametrize("n", [31, 32, 33, 255, 256, 257, 511, 513])
+def test_chunk_boundaries_dense_deep(n):
+    """Dense lists whose lengths straddle one warp (32, the short-chunk path) and one chunk (256);
+    depth 6 so that late levels have up to 32 segments per list and chunks that cross segments
+    (the scatter's per-entry aggregate path and k_desc's head/count flags)."""
+    p = synth.random_small(300 + n, n=n, m=5, nan_frac=0.0, n_distinct=max(3, n // 3), loss="logistic",
+                           d=6, T=3, eta=0.5)
+    model, margin = _train(p)
+    compare(p, model.nodes(), margin)
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_sparse_lists_around_32_entries(seed):
+    """Sparse attribute lists of ~25-40 entries with missing values: both the short-chunk split
+    path (<= 32) and the general one (> 32) on the same level, up to 32 nodes per level."""
+    p = synth.c4(seed=40 + seed, n=3000, m=120, density=0.011, T=2)
+    p.params["max_depth"] = 6
+    model, margin = _train(p)
+    compare(p, model.nodes(), margin)
+
+
+def test_scatter_aggregates_match_chunk_agg():
+    """The next-level chunk aggregates accumulated by the scatter (data without missing values)
+    and those k_chunk_agg computes (the same lists with one NaN column, which routes every level
+    through k_chunk_agg) give trees that both match the oracle."""
+    base = synth.random_small(909, n=6000, m=4, nan_frac=0.0, n_distinct=2000, loss="logistic", d=6, T=3)
+    model, margin = _train(base)
+    compare(base, model.nodes(), margin)
+    X = np.full((base.n, base.m + 1), np.nan, np.float32)
+    dense = np.zeros((base.n, base.m), np.float32)
+    for i in range(base.n):
+        cols = base.indices[base.indptr[i]:base.indptr[i + 1]]
+        dense[i, cols] = base.values[base.indptr[i]:base.indptr[i + 1]]
+    X[:, :base.m] = dense
+    X[::7, base.m] = 1.0  # a sparse extra column makes the dataset "has missing"
+    q = synth.from_dense("agg_missing", X, base.labels, dict(base.params))
+    model2, margin2 = _train(q)
+    compare(q, model2.nodes(), margin2)

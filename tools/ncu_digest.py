@@ -30,7 +30,7 @@ for r in R:
     op = s.split()[0].split(".")[0] if s else ""
     c[op] += e; T += e
 print("dynamic warp instructions", T)
-print("  " + "  ".join(f"{k}:{v/T*100:.1f}%" for k, v in c.most_common(16)))
+sys.stdout.flush(); print("  " + "  ".join(f"{k}:{v/T*100:.1f}%" for k, v in c.most_common(16)))
 if len(sys.argv) > 2:
     with open(sys.argv[2], "w") as f:
         for i, r in enumerate(R):
