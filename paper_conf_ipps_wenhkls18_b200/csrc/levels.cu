@@ -1604,9 +1604,15 @@ __device__ __forceinline__ double warp_sum8(double (&v)[8], int lane) {
 }
 
 template <int HMODE, bool kRLE, bool kAgg>
-__global__ void __launch_bounds__(kThreads, 3) k_part_scatter(PartArgs A) {
+#ifndef GBDT_SCATTER_CTAS
+#define GBDT_SCATTER_CTAS 3
+#endif
+#ifndef GBDT_SCATTER_ROWS
+#define GBDT_SCATTER_ROWS 4
+#endif
+__global__ void __launch_bounds__(kThreads, GBDT_SCATTER_CTAS) k_part_scatter(PartArgs A) {
   constexpr bool kH = HMODE == kHGather;
-  constexpr int kHalf = kItems / 2;
+  constexpr int kHalf = GBDT_SCATTER_ROWS;  // rows loaded per step
   __shared__ TabCache tc;
   __shared__ long long wss[kWarps][kWarpK];  // the attribute's segment starts (chunks crossing segments)
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -1669,7 +1675,7 @@ __global__ void __launch_bounds__(kThreads, 3) k_part_scatter(PartArgs A) {
     for (int i = 0; i < 8; ++i) acc[i] = 0.0;
     int nh = 0, nl = 0;  // kept entries of each side in the rows before
 #pragma unroll
-    for (int half = 0; half < 2; ++half) {
+    for (int half = 0; half < kItems / kHalf; ++half) {
       uint8_t sd[kHalf];
       int id[kHalf];
       float v[kHalf];

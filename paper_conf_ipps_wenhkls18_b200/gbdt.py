@@ -14,7 +14,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libgbdt.so")
+# GBDT_LIB: an alternative in-tree build of the same library (A/B measurements of kernel variants)
+LIB_PATH = os.environ.get("GBDT_LIB") or os.path.join(_HERE, "libgbdt.so")
 
 GBDT_OK = 0
 STATUS = {0: "OK", 1: "E_INVAL", 2: "E_NOMEM", 3: "E_CUDA", 4: "E_NCCL", 5: "E_STATE", 6: "E_RANGE"}
