@@ -53,6 +53,9 @@ def parse():
     ap.add_argument("--rle", default="off")
     ap.add_argument("--comm", default="nccl", choices=["nccl", "host"],
                     help="host: gloo + host-staged callbacks (several ranks may share one GPU; testing only)")
+    ap.add_argument("--depth", type=int, default=0, help="override the config's max_depth (sweeps, SURVEY §8(f2))")
+    ap.add_argument("--smartgd", default="on", choices=["on", "off"],
+                    help="off: SmartGD ablation, predictions recomputed by tree traversal (P:193-195, Fig. 9)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle CPU time for cpu_baseline")
@@ -191,17 +194,19 @@ def main():
 
     prob = synth.make(args.config)
     P = dict(prob.params)
+    if args.depth:
+        P["max_depth"] = args.depth
     d = P["max_depth"]
     comm = None
     if world > 1:
         comm = gbdt.comm_from_callbacks(local) if host_comm else gbdt.comm_from_torch(local)
     stream = torch.cuda.current_stream()
     ds = gbdt.load_csr(prob.indptr, prob.indices, prob.values, prob.labels, prob.m, rle=args.rle,
-                       stream=stream.cuda_stream, comm=comm)
+                       stream=stream.cuda_stream, comm=comm, keep_rows=args.smartgd == "off")
     info = ds.info(0)
     m_local = info["attr_end"] - info["attr_begin"]
     tp = dict(max_depth=d, lam=P["lam"], gamma=P["gamma"], eta=P["eta"], base_margin=P["base_margin"],
-              loss=P["loss"])
+              loss=P["loss"], smartgd=args.smartgd == "on")
 
     # warm-up (untimed)
     gbdt.train(ds, n_trees=max(args.warmup, 1), want_margin=False, **tp)
@@ -255,7 +260,8 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        ds2 = gbdt.load_csr(hp, hi, hv, hl, prob.m, rle=args.rle, stream=stream.cuda_stream, comm=comm)
+        ds2 = gbdt.load_csr(hp, hi, hv, hl, prob.m, rle=args.rle, stream=stream.cuda_stream, comm=comm,
+                            keep_rows=args.smartgd == "off")
         model2, margin2 = gbdt.train(ds2, n_trees=args.steps, want_margin=True, **tp)
         torch.cuda.synchronize()
         te = time.perf_counter() - t0
@@ -283,7 +289,7 @@ def main():
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": args.config, "n": prob.n, "m": prob.m, "nnz": prob.nnz, "loss": P["loss"],
                        "max_depth": d, "trees_timed": args.steps, "lambda": P["lam"], "eta": P["eta"],
-                       "rle": args.rle, "parallelism": f"attr-shard{world}",
+                       "rle": args.rle, "smartgd": args.smartgd, "parallelism": f"attr-shard{world}",
                        "l2": "inputs larger than L2 (sorted lists %.2f GB)" % (prob.nnz * 8 / 1e9)},
             "roofline": {"bound": "hbm", "achieved": kern[dom]["achieved"], "peak": peak, "unit": "GB/s",
                          "frac": kern[dom]["frac"], "traffic": kern[dom]["traffic"], "kernel": dom,

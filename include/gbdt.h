@@ -48,7 +48,17 @@ typedef enum {
   GBDT_E_RANGE = 6   /* a count outside the supported range (shards, devices, sizes) */
 } gbdt_status;
 
-typedef enum { GBDT_LOSS_SQUARED = 0, GBDT_LOSS_LOGISTIC = 1 } gbdt_loss;
+typedef enum { GBDT_LOSS_SQUARED = 0, GBDT_LOSS_LOGISTIC = 1, GBDT_LOSS_CUSTOM = 2 } gbdt_loss;
+
+/* User-defined loss (GBDT_LOSS_CUSTOM; the paper's "users can define their own loss function",
+ * P:193).  Called once per tree, after the cached prediction has been updated
+ * (SmartGD), with DEVICE pointers: yhat, labels (n each, read only) and g, h (n each, to be
+ * written: first and second derivative of the loss at yhat, h >= 0 and finite).  The callback
+ * must enqueue its work on `stream` (the library's cudaStream_t) or complete it before
+ * returning; the library reads g and h in stream order afterwards.  Returns 0 on success; any
+ * other value aborts the gbdt_train with GBDT_E_INVAL.  `user` is gbdt_params.grad_user. */
+typedef int (*gbdt_grad_fn)(int64_t n, const double* yhat, const float* labels, double* g, double* h,
+                            void* stream, void* user);
 typedef enum { GBDT_RLE_OFF = 0, GBDT_RLE_ON = 1, GBDT_RLE_AUTO = 2 } gbdt_rle;
 
 /* Options of gbdt_load_csr.  Zero-initialised means: no RLE, one shard, current device,
@@ -66,6 +76,7 @@ typedef struct {
   gbdt_comm* comm;        /* NULL: single process.  Else this process is rank r of a world of
                              size w and owns attribute range r of w (nnz-balanced, contiguous);
                              n_shards must then be 0 or 1. */
+  int32_t keep_rows;      /* 1: keep a device copy of the CSR rows (needed by smartgd_off) */
 } gbdt_load_opts;
 
 /* Training parameters, as the paper states them: d, T, gamma (Alg. 1 inputs),
@@ -79,6 +90,14 @@ typedef struct {
   double base_margin;     /* initial prediction (reading R7) */
   int32_t loss;           /* gbdt_loss */
   int32_t profile;        /* 1: record per-phase device times (gbdt_get_timings) */
+  int32_t smartgd_off;    /* 1: ablation of SmartGD (Fig. 9): before every tree each
+                             instance's prediction is recomputed by traversing all previous trees
+                             over its CSR row instead of adding its last leaf weight.  Same
+                             arithmetic in the same order, so the trees are bit-identical.  Needs
+                             a dataset loaded with keep_rows = 1 (else GBDT_E_STATE). */
+  int32_t reserved;       /* 0 */
+  gbdt_grad_fn grad_fn;   /* GBDT_LOSS_CUSTOM: the gradient callback (else ignored) */
+  void* grad_user;        /* passed through to grad_fn */
 } gbdt_params;
 
 /* One tree node in heap order: root 0, children of k are 2k+1 (high/left: x >= split_value)

@@ -200,9 +200,15 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
       ds.y.alloc((size_t)n_rows * 4, st);
       GBDT_CUDA(cudaMemcpyAsync(ds.y.p, labels, (size_t)n_rows * 4, cudaMemcpyHostToDevice, st));
       build_layout(ds, dptr.as<int64_t>(), didx.as<int32_t>(), dval.as<float>(), col_counts, o.rle_min_ratio);
-      dptr.release();
-      didx.release();
-      dval.release();
+      if (o.keep_rows) {
+        ds.rows_ptr = std::move(dptr);
+        ds.rows_idx = std::move(didx);
+        ds.rows_val = std::move(dval);
+      } else {
+        dptr.release();
+        didx.release();
+        dval.release();
+      }
       GBDT_CUDA(cudaStreamSynchronize(st));
     } catch (...) {
       delete h;
@@ -223,7 +229,10 @@ gbdt_status gbdt_train(gbdt_dataset* dsh, const gbdt_params* p, gbdt_model** out
     if (!(p->gamma >= 0) || !std::isfinite(p->gamma)) fail(GBDT_E_INVAL, "gamma must be finite and >= 0");
     if (!(p->eta > 0 && p->eta <= 1)) fail(GBDT_E_INVAL, "eta must be in (0, 1]");
     if (!std::isfinite(p->base_margin)) fail(GBDT_E_INVAL, "base_margin must be finite");
-    if (p->loss != GBDT_LOSS_SQUARED && p->loss != GBDT_LOSS_LOGISTIC) fail(GBDT_E_INVAL, "unknown loss");
+    if (p->loss != GBDT_LOSS_SQUARED && p->loss != GBDT_LOSS_LOGISTIC && p->loss != GBDT_LOSS_CUSTOM)
+      fail(GBDT_E_INVAL, "unknown loss");
+    if (p->loss == GBDT_LOSS_CUSTOM && !p->grad_fn) fail(GBDT_E_INVAL, "GBDT_LOSS_CUSTOM needs grad_fn");
+    if (p->smartgd_off && !ds.rows_ptr.p) fail(GBDT_E_STATE, "smartgd_off needs a dataset loaded with keep_rows = 1");
     if (p->loss == GBDT_LOSS_LOGISTIC && (ds.h_labels_minmax[0] < 0 || ds.h_labels_minmax[1] > 1))
       fail(GBDT_E_INVAL, "logistic loss needs labels in [0, 1]");
     if (p->lambda == 0 && p->loss == GBDT_LOSS_LOGISTIC) {

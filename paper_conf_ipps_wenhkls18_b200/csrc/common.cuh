@@ -163,4 +163,37 @@ __device__ __forceinline__ SV sv_add(const SV& a, const SV& b) {
   return SV{__dadd_rn(a.g, b.g), __dadd_rn(a.h, b.h), a.c + b.c};
 }
 
+// ----------------------------------------------------------------------------- tree traversal
+// Value of attribute a in CSR row i (binary search; rows have strictly increasing indices).
+// NaN = missing; -0.0 reads as +0.0 as in the layout.
+__device__ __forceinline__ bool csr_lookup(const int64_t* indptr, const int32_t* indices, const float* values,
+                                           int64_t i, int a, float& x) {
+  int64_t lo = indptr[i], hi = indptr[i + 1];
+  while (lo < hi) {
+    const int64_t mid = lo + ((hi - lo) >> 1);
+    if (indices[mid] < a) lo = mid + 1; else hi = mid;
+  }
+  if (lo < indptr[i + 1] && indices[lo] == a) {
+    const float v = values[lo];
+    if (isnan(v)) return false;
+    x = v == 0.0f ? 0.0f : v;
+    return true;
+  }
+  return false;
+}
+
+// Leaf weight of row i in tree T (heap order): present x >= split_value goes to the high child
+// 2k+1, else 2k+2; missing follows default_left (reading R11).
+__device__ __forceinline__ double tree_leaf_weight(const gbdt_node* T, const int64_t* indptr, const int32_t* indices,
+                                                   const float* values, int64_t i) {
+  int64_t k = 0;
+  while (!T[k].is_leaf) {
+    float x;
+    const bool high = csr_lookup(indptr, indices, values, i, T[k].attr, x) ? (x >= T[k].split_value)
+                                                                          : (T[k].default_left != 0);
+    k = high ? 2 * k + 1 : 2 * k + 2;
+  }
+  return T[k].weight;
+}
+
 }  // namespace gbdt

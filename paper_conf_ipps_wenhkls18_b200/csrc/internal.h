@@ -127,6 +127,7 @@ struct Dataset {
   int32_t n_total_shards = 1;    // across all ranks
   Comm* comm = nullptr;
   int rle = 0;
+  DBuf rows_ptr, rows_idx, rows_val;  // CSR rows (gbdt_load_opts.keep_rows; SmartGD-off ablation)
 };
 
 struct Model {

@@ -12,37 +12,13 @@
 namespace gbdt {
 namespace {
 
-__device__ __forceinline__ bool lookup(const int64_t* indptr, const int32_t* indices, const float* values,
-                                       int64_t i, int a, float& x) {
-  int64_t lo = indptr[i], hi = indptr[i + 1];
-  while (lo < hi) {
-    const int64_t mid = lo + ((hi - lo) >> 1);
-    if (indices[mid] < a) lo = mid + 1; else hi = mid;
-  }
-  if (lo < indptr[i + 1] && indices[lo] == a) {
-    const float v = values[lo];
-    if (isnan(v)) return false;
-    x = v == 0.0f ? 0.0f : v;
-    return true;
-  }
-  return false;
-}
-
 __global__ void k_predict(int64_t n, const int64_t* __restrict__ indptr, const int32_t* __restrict__ indices,
                           const float* __restrict__ values, const gbdt_node* __restrict__ nodes, int n_trees,
                           int64_t NH, double eta, double base, int sigmoid, double* __restrict__ out) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     double y = base;
     for (int t = 0; t < n_trees; ++t) {
-      const gbdt_node* T = nodes + (int64_t)t * NH;
-      int64_t k = 0;
-      while (!T[k].is_leaf) {
-        float x;
-        const bool high = lookup(indptr, indices, values, i, T[k].attr, x) ? (x >= T[k].split_value)
-                                                                           : (T[k].default_left != 0);
-        k = high ? 2 * k + 1 : 2 * k + 2;
-      }
-      y = __dadd_rn(y, __dmul_rn(eta, T[k].weight));
+      y = __dadd_rn(y, __dmul_rn(eta, tree_leaf_weight(nodes + (int64_t)t * NH, indptr, indices, values, i)));
     }
     if (sigmoid) y = __ddiv_rn(1.0, __dadd_rn(1.0, exp(-y)));
     out[i] = y;

@@ -20,6 +20,7 @@
 // in which pieces are reduced.
 #include <algorithm>
 #include <cstring>
+#include <string>
 #include <vector>
 
 #include "kernels.cuh"
@@ -33,18 +34,45 @@ thread_local int64_t g_launches = 0;
 // ============================================================================ a2: gradients
 // SmartGD: the instances are in leaf nodes at the end of a tree, so the prediction is
 // updated with the leaf weight of the node each instance ended in -- no tree traversal.
+// Rows of the SmartGD-off ablation: the prediction before tree t is recomputed by traversing
+// trees 0..t-1 over the instance's CSR row (the paper's baseline without SmartGD).
+struct RowsArgs {
+  const int64_t* indptr = nullptr;  // nullptr: SmartGD
+  const int32_t* indices = nullptr;
+  const float* values = nullptr;
+  const gbdt_node* trees = nullptr;
+  int64_t NH = 0;
+  int t = 0;                         // trees already built
+};
+__device__ __forceinline__ double traverse_margin(const RowsArgs& R, int64_t i, double base, double eta) {
+  double y = base;  // same operations in the same order as the SmartGD updates
+  for (int u = 0; u < R.t; ++u)
+    y = __dadd_rn(y, __dmul_rn(eta, tree_leaf_weight(R.trees + (int64_t)u * R.NH, R.indptr, R.indices, R.values, i)));
+  return y;
+}
+
+// mode 0: built-in loss; 1: custom loss, prediction update only (the callback writes g, h);
+// 2: custom loss, reduction of the callback's g, h only
 __global__ void k_grad(int64_t n, int loss, int first, double eta, double base,
                        const float* __restrict__ y, const double* __restrict__ wprev,
                        double* __restrict__ yhat, int32_t* __restrict__ pos,
                        double* __restrict__ gout, double* __restrict__ hout, int store_h,
-                       double* __restrict__ partial) {
+                       double* __restrict__ partial, RowsArgs R, int mode) {
   double sg = 0.0, sh = 0.0, mg = 0.0, mh = 0.0;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
-    double yh = first ? base : __dadd_rn(yhat[i], __dmul_rn(eta, wprev[pos[i]]));
-    yhat[i] = yh;
-    const double yi = (double)y[i];
     double g, h;
+    if (mode == 2) {
+      g = gout[i];
+      h = hout[i];
+    } else {
+      double yh;
+      if (R.indptr) yh = traverse_margin(R, i, base, eta);
+      else yh = first ? base : __dadd_rn(yhat[i], __dmul_rn(eta, wprev[pos[i]]));
+      yhat[i] = yh;
+      pos[i] = 0;
+      if (mode == 1) continue;
+      const double yi = (double)y[i];
     if (loss == GBDT_LOSS_SQUARED) {  // l = (y - yhat)^2: g = 2(yhat - y), h = 2 (R6)
       g = __dmul_rn(2.0, __dsub_rn(yh, yi));
       h = 2.0;
@@ -57,7 +85,7 @@ __global__ void k_grad(int64_t n, int loss, int first, double eta, double base,
     }
     gout[i] = g;
     if (store_h) hout[i] = h;
-    pos[i] = 0;
+    }
     sg += g;
     sh += h;
     mg = fmax(mg, fabs(g));
@@ -70,6 +98,7 @@ __global__ void k_grad(int64_t n, int loss, int first, double eta, double base,
     mg = fmax(mg, __shfl_xor_sync(0xffffffffu, mg, o));
     mh = fmax(mh, __shfl_xor_sync(0xffffffffu, mh, o));
   }
+  if (mode == 1) return;
   __shared__ double wg[32], wh[32], wmg[32], wmh[32];
   if ((threadIdx.x & 31) == 0) {
     wg[threadIdx.x >> 5] = sg; wh[threadIdx.x >> 5] = sh;
@@ -440,7 +469,14 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   const int nsh = ds.n_total_shards;
   const int sms = LK.sms;
   // gradient storage mode (kernels.cuh): squared -> h == 2; logistic with 0/1 labels -> h(g)
-  const int hmode = P.loss == GBDT_LOSS_SQUARED ? kHConst2 : (ds.binary_labels ? kHFromG : kHGather);
+  const int hmode = P.loss == GBDT_LOSS_SQUARED ? kHConst2
+                    : (P.loss == GBDT_LOSS_LOGISTIC && ds.binary_labels ? kHFromG : kHGather);
+  const bool custom = P.loss == GBDT_LOSS_CUSTOM;
+  RowsArgs rows;  // SmartGD-off ablation
+  if (P.smartgd_off) {
+    rows.indptr = ds.rows_ptr.as<int64_t>(); rows.indices = ds.rows_idx.as<int32_t>();
+    rows.values = ds.rows_val.as<float>(); rows.NH = NH;
+  }
   const unsigned inst_grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), (int64_t)sms * 8));
   const int grad_blocks = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), (int64_t)sms * 4));
   const int64_t npad = (n + 8) & ~int64_t(3);
@@ -607,9 +643,18 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     double* wcur = hweight + (size_t)(t & 1) * NH;
     gbdt_node* tree = trees + (size_t)t * NH;
     tm.begin(GBDT_PHASE_GRAD);
+    if (rows.indptr) { rows.trees = trees; rows.t = t; }
     k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, t == 0, P.eta, P.base_margin, ds.y.as<float>(), wprev,
-                                        yhat, pos, gv, hv, hmode == kHGather, partial);
+                                        yhat, pos, gv, hv, hmode == kHGather, partial, rows, custom ? 1 : 0);
     GBDT_LAUNCH_CHECK();
+    if (custom) {  // user-defined loss: g, h from the callback, on this stream
+      if (P.grad_fn(n, yhat, ds.y.as<float>(), gv, hv, (void*)st, P.grad_user) != 0)
+        fail(GBDT_E_INVAL, "grad_fn failed at tree " + std::to_string(t));
+      k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, 0, P.eta, P.base_margin, ds.y.as<float>(), wprev,
+                                          yhat, pos, gv, hv, 1, partial, RowsArgs{}, 2);
+      GBDT_LAUNCH_CHECK();
+      count_launch();
+    }
     k_tree_begin<<<1, 1024, 0, st>>>(grad_blocks, partial, n, P.lambda, nt[0], NH, wcur, hstate, tree, fxs);
     GBDT_LAUNCH_CHECK();
     count_launch(2);
@@ -764,7 +809,13 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   // final SmartGD step: the last tree's leaf weights
   {
     double* wlast = hweight + (size_t)((P.n_trees - 1) & 1) * NH;
-    k_apply<<<inst_grid, 256, 0, st>>>(n, P.eta, wlast, pos, yhat);
+    if (rows.indptr) {  // ablation: the final margin by traversal of all trees too
+      rows.trees = trees; rows.t = P.n_trees;
+      k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, 0, P.eta, P.base_margin, ds.y.as<float>(), wlast,
+                                          yhat, pos, gv, hv, 0, partial, rows, 1);
+    } else {
+      k_apply<<<inst_grid, 256, 0, st>>>(n, P.eta, wlast, pos, yhat);
+    }
     GBDT_LAUNCH_CHECK();
     count_launch();
   }

@@ -19,7 +19,7 @@ LIB_PATH = os.environ.get("GBDT_LIB") or os.path.join(_HERE, "libgbdt.so")
 
 GBDT_OK = 0
 STATUS = {0: "OK", 1: "E_INVAL", 2: "E_NOMEM", 3: "E_CUDA", 4: "E_NCCL", 5: "E_STATE", 6: "E_RANGE"}
-LOSS = {"squared": 0, "logistic": 1}
+LOSS = {"squared": 0, "logistic": 1, "custom": 2}
 RLE = {"off": 0, "on": 1, "auto": 2, False: 0, True: 1, None: 0}
 PHASES = ["grad", "split_find", "decide", "nodemap", "partition", "comm", "total",
           "k_chunk_agg", "k_split", "k_count", "k_scatter"]
@@ -41,13 +41,18 @@ class GbdtError(RuntimeError):
 
 class _LoadOpts(C.Structure):
     _fields_ = [("rle", C.c_int32), ("rle_min_ratio", C.c_double), ("n_shards", C.c_int32),
-                ("device", C.c_int32), ("stream", C.c_void_p), ("comm", C.c_void_p)]
+                ("device", C.c_int32), ("stream", C.c_void_p), ("comm", C.c_void_p), ("keep_rows", C.c_int32)]
+
+
+# gbdt_grad_fn(n, yhat, labels, g, h, stream, user): device pointers (GBDT_LOSS_CUSTOM)
+GRAD_FN = C.CFUNCTYPE(C.c_int, C.c_int64, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p)
 
 
 class _Params(C.Structure):
     _fields_ = [("max_depth", C.c_int32), ("n_trees", C.c_int32), ("lam", C.c_double),
                 ("gamma", C.c_double), ("eta", C.c_double), ("base_margin", C.c_double),
-                ("loss", C.c_int32), ("profile", C.c_int32)]
+                ("loss", C.c_int32), ("profile", C.c_int32), ("smartgd_off", C.c_int32),
+                ("reserved", C.c_int32), ("grad_fn", GRAD_FN), ("grad_user", C.c_void_p)]
 
 
 _lib = None
@@ -287,7 +292,7 @@ class Model:
 
 
 def load_csr(indptr, indices, values, labels, n_cols, rle="off", rle_min_ratio=0.0, n_shards=1,
-             device=-1, stream="current", comm: Comm | None = None) -> Dataset:
+             device=-1, stream="current", comm: Comm | None = None, keep_rows=False) -> Dataset:
     indptr = np.ascontiguousarray(indptr, np.int64)
     indices = np.ascontiguousarray(indices, np.int32)
     values = np.ascontiguousarray(values, np.float32)
@@ -296,7 +301,7 @@ def load_csr(indptr, indices, values, labels, n_cols, rle="off", rle_min_ratio=0
     if stream == "current":
         stream = _current_stream()
     o = _LoadOpts(RLE[rle], float(rle_min_ratio), int(n_shards), int(device), stream,
-                  comm._h if comm is not None else None)
+                  comm._h if comm is not None else None, int(bool(keep_rows)))
     h = C.c_void_p()
     _check(lib().gbdt_load_csr(n, int(n_cols), _p(indptr), _p(indices), _p(values), _p(labels), C.byref(o),
                                C.byref(h)))
@@ -304,9 +309,22 @@ def load_csr(indptr, indices, values, labels, n_cols, rle="off", rle_min_ratio=0
 
 
 def train(ds: Dataset, max_depth=6, n_trees=40, lam=1.0, gamma=0.0, eta=0.3, base_margin=0.0,
-          loss="squared", profile=False, want_margin=True):
+          loss="squared", profile=False, want_margin=True, smartgd=True, grad_fn=None):
+    """grad_fn (loss="custom"): python callable (n, yhat, labels, g, h, stream) -> None over
+    DEVICE addresses, run on the library's stream (see gbdt_grad_fn in include/gbdt.h)."""
+    cb = GRAD_FN()
+    if grad_fn is not None:
+        def _tramp(n, yh, y, g, h, st, user):
+            try:
+                grad_fn(int(n), yh, y, g, h, st)
+                return 0
+            except Exception:  # noqa: BLE001 - reported to the library as a failed callback
+                import traceback
+                traceback.print_exc()
+                return 1
+        cb = GRAD_FN(_tramp)
     prm = _Params(int(max_depth), int(n_trees), float(lam), float(gamma), float(eta), float(base_margin),
-                  LOSS[loss], int(bool(profile)))
+                  LOSS[loss], int(bool(profile)), int(not smartgd), 0, cb, None)
     h = C.c_void_p()
     margin = np.zeros(ds.n, np.float64) if want_margin else None
     _check(lib().gbdt_train(ds._h, C.byref(prm), C.byref(h), _p(margin)))
@@ -330,5 +348,7 @@ def train_problem(prob, **overrides):
     P.update(overrides)
     rle = P.pop("rle", "off")
     n_shards = P.pop("n_shards", 1)
-    ds = load_csr(prob.indptr, prob.indices, prob.values, prob.labels, prob.m, rle=rle, n_shards=n_shards)
+    keep_rows = not P.get("smartgd", True)  # the SmartGD-off ablation traverses the CSR rows
+    ds = load_csr(prob.indptr, prob.indices, prob.values, prob.labels, prob.m, rle=rle, n_shards=n_shards,
+                  keep_rows=keep_rows)
     return train(ds, **P)

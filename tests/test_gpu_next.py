@@ -1,0 +1,103 @@
+"""SURVEY §8(f) rows beyond the hot path, through the C ABI (-m gpu):
+
+f1  SmartGD ablation (Fig. 9): smartgd_off recomputes every prediction by traversing
+    all previous trees, with the same operations in the same order, so the model and the training
+    margin must be bit-identical to the SmartGD run.
+f4  user-defined loss hook ("users can define their own loss function"): a callback over
+    device pointers.  A callback computing the paper's squared loss must reproduce the built-in
+    squared-loss model; one computing the logistic loss is checked against the oracle.
+"""
+import ctypes as C
+
+import numpy as np
+import pytest
+
+from datagen import synth
+from paper_conf_ipps_wenhkls18_b200 import gbdt
+
+from parity import compare
+
+pytestmark = pytest.mark.gpu
+
+
+def _same_model(a, b):
+    na, nb = a.nodes(), b.nodes()
+    assert na.tobytes() == nb.tobytes()
+
+
+@pytest.mark.parametrize("maker", [
+    lambda: synth.c1(n=3000),
+    lambda: synth.random_small(4, n=2000, m=9, nan_frac=0.3, n_distinct=30, loss="logistic", d=5, T=4),
+    lambda: synth.c4(seed=7, n=700, m=2500, density=0.01),
+])
+def test_smartgd_off_bit_identical(maker):
+    p = maker()
+    m_on, y_on = gbdt.train_problem(p)
+    m_off, y_off = gbdt.train_problem(p, smartgd=False)
+    _same_model(m_on, m_off)
+    assert y_on.tobytes() == y_off.tobytes()
+
+
+def test_smartgd_off_needs_rows():
+    p = synth.c1(n=500)
+    ds = gbdt.load_csr(p.indptr, p.indices, p.values, p.labels, p.m)
+    with pytest.raises(gbdt.GbdtError, match="E_STATE"):
+        gbdt.train(ds, max_depth=3, n_trees=2, smartgd=False)
+
+
+def _host_grad(kind):
+    """A user loss over device pointers: copies yhat/labels to the host (cuda-python runtime),
+    computes g, h in numpy with the paper's formulas and copies them back, synchronously."""
+    from cuda.bindings import runtime as rt
+
+    def fn(n, yh, y, g, h, stream):
+        assert rt.cudaStreamSynchronize(stream)[0] == rt.cudaError_t.cudaSuccess
+        Y = np.empty(n, np.float64)
+        L = np.empty(n, np.float32)
+        assert rt.cudaMemcpy(Y.ctypes.data, yh, 8 * n, rt.cudaMemcpyKind.cudaMemcpyDeviceToHost)[0] == 0
+        assert rt.cudaMemcpy(L.ctypes.data, y, 4 * n, rt.cudaMemcpyKind.cudaMemcpyDeviceToHost)[0] == 0
+        yy = L.astype(np.float64)
+        if kind == "squared":  # g = 2(yhat - y), h = 2 (reading R6)
+            G = 2.0 * (Y - yy)
+            H = np.full(n, 2.0)
+        else:  # cross-entropy, readings R5/R5b
+            p = 1.0 / (1.0 + np.exp(-Y))
+            G = p - yy
+            q = G + yy
+            H = np.maximum(q * (1.0 - q), 1e-16)
+        assert rt.cudaMemcpy(g, G.ctypes.data, 8 * n, rt.cudaMemcpyKind.cudaMemcpyHostToDevice)[0] == 0
+        assert rt.cudaMemcpy(h, H.ctypes.data, 8 * n, rt.cudaMemcpyKind.cudaMemcpyHostToDevice)[0] == 0
+    return fn
+
+
+def test_custom_loss_squared_equals_builtin():
+    p = synth.c1(n=3000)
+    m_b, y_b = gbdt.train_problem(p)
+    m_c, y_c = gbdt.train_problem(p, loss="custom", grad_fn=_host_grad("squared"))
+    nb, nc = m_b.nodes(), m_c.nodes()
+    for f in ("heap_id", "is_leaf", "attr", "default_left", "split_value", "count"):
+        assert np.array_equal(nb[f], nc[f]), f
+    np.testing.assert_allclose(nc["weight"], nb["weight"], rtol=1e-12, atol=1e-15)
+    np.testing.assert_allclose(y_c, y_b, rtol=1e-12, atol=1e-15)
+
+
+@pytest.mark.parametrize("maker", [
+    lambda: synth.random_small(9, n=1500, m=6, nan_frac=0.25, n_distinct=25, loss="logistic", d=4, T=3),
+    lambda: synth.c2(n=4000, T=5),
+])
+def test_custom_loss_logistic_against_oracle(maker):
+    p = maker()
+    model, margin = gbdt.train_problem(p, loss="custom", grad_fn=_host_grad("logistic"))
+    compare(p, model.nodes(), margin)
+
+
+def test_custom_loss_errors():
+    p = synth.c1(n=300)
+    ds = gbdt.load_csr(p.indptr, p.indices, p.values, p.labels, p.m)
+    with pytest.raises(gbdt.GbdtError, match="E_INVAL"):
+        gbdt.train(ds, max_depth=2, n_trees=1, loss="custom")
+
+    def bad(n, yh, y, g, h, stream):
+        raise RuntimeError("user loss failed")
+    with pytest.raises(gbdt.GbdtError, match="grad_fn failed"):
+        gbdt.train(ds, max_depth=2, n_trees=1, loss="custom", grad_fn=bad)
