@@ -53,11 +53,17 @@ __device__ __forceinline__ double traverse_margin(const RowsArgs& R, int64_t i, 
 
 // mode 0: built-in loss; 1: custom loss, prediction update only (the callback writes g, h);
 // 2: custom loss, reduction of the callback's g, h only
-__global__ void k_grad(int64_t n, int loss, int first, double eta, double base,
-                       const float* __restrict__ y, const double* __restrict__ wprev,
+// tidx: the tree index t on the device (nullptr: R.t); the previous tree's leaf weights are
+// hweight + ((t + 1) & 1) * NH.
+__global__ void k_grad(int64_t n, int loss, const int32_t* __restrict__ tidx, double eta, double base,
+                       const float* __restrict__ y, const double* __restrict__ hweight, int64_t NH,
                        double* __restrict__ yhat, int32_t* __restrict__ pos,
                        double* __restrict__ gout, double* __restrict__ hout, int store_h,
                        double* __restrict__ partial, RowsArgs R, int mode) {
+  const int t = tidx ? *tidx : R.t;
+  const int first = t == 0;
+  const double* wprev = hweight + (size_t)((t + 1) & 1) * NH;
+  R.t = t;
   double sg = 0.0, sh = 0.0, mg = 0.0, mh = 0.0;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
@@ -127,8 +133,12 @@ __device__ int fx_scale(double n, double mx) {
 
 // Root node totals + per-tree reset (single thread block).
 __global__ void k_tree_begin(int nblk, const double* __restrict__ partial, int64_t n, double lam,
-                             NodeTab root, int64_t NH, double* __restrict__ wcur,
-                             uint8_t* __restrict__ hstate, gbdt_node* __restrict__ tree, int32_t* __restrict__ fx) {
+                             NodeTab root, int64_t NH, double* __restrict__ hweight,
+                             uint8_t* __restrict__ hstate, gbdt_node* __restrict__ trees, int32_t* __restrict__ fx,
+                             const int32_t* __restrict__ tidx) {
+  const int t = *tidx;
+  double* wcur = hweight + (size_t)(t & 1) * NH;
+  gbdt_node* tree = trees + (size_t)t * NH;
   for (int64_t k = threadIdx.x; k < NH; k += blockDim.x) {
     wcur[k] = 0.0;
     hstate[k] = 0;
@@ -153,6 +163,8 @@ __global__ void k_tree_begin(int nblk, const double* __restrict__ partial, int64
     root.pterm[0] = parent_term(G, H, lam);
   }
 }
+
+__global__ void k_tree_end(int32_t* __restrict__ tidx) { *tidx += 1; }
 
 __global__ void k_level_begin(int* __restrict__ epoch, int* __restrict__ counters, int ncounters,
                               int* __restrict__ nrec, int nshard, const int32_t* __restrict__ Kp,
@@ -228,8 +240,11 @@ struct DecideArgs {
   Rec* winner;          // [Kcap]
   uint8_t* hstate;      // by heap id: 1 split at this level, 2 leaf
   uint8_t* hdef;        // default side: 1 high
-  double* hweight;      // by heap id (this tree)
-  gbdt_node* tree;
+  double* hweight;      // by heap id, two trees (this one: + (t & 1) * NH)
+  gbdt_node* trees;     // all trees (this one: + t * NH)
+  gbdt_node* tree;      // set by k_decide
+  const int32_t* tidx;  // t
+  int64_t NH;
 };
 
 __device__ void write_leaf(const DecideArgs& A, int h, double G, double H, long long cnt) {
@@ -244,6 +259,11 @@ __device__ void write_leaf(const DecideArgs& A, int h, double G, double H, long 
 
 // Single thread block: merge the shards' node bests (strict total order), decide, emit.
 __global__ void k_decide(DecideArgs A) {
+  {
+    const int t = *A.tidx;
+    A.hweight += (size_t)(t & 1) * A.NH;
+    A.tree = A.trees + (size_t)t * A.NH;
+  }
   const int K = *A.cur.K;
   const int epoch = *A.epochp;
   unsigned long long carry = 0;
@@ -492,6 +512,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     c.take<unsigned long long>((size_t)nloc * Kcap); c.take<unsigned long long>((size_t)nloc * Kcap);
     c.take<int>(nloc);
     c.take<unsigned long long>(16);
+    c.take<int32_t>(4);
   };
   Carve probe{nullptr};
   sz_dev(probe);
@@ -523,6 +544,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   unsigned long long* tkey = c.take<unsigned long long>((size_t)nloc * Kcap);
   int* nrec = c.take<int>(nloc);
   unsigned long long* lent = c.take<unsigned long long>(16);  // entries scanned per level (profile)
+  int32_t* tidx = c.take<int32_t>(4);  // index of the tree being built (device side, for graph replays)
 
   // ---------------------------------------------------------------- per-shard state
   std::vector<ShardWork> sw(nloc);
@@ -638,24 +660,25 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   }
   const double thr = P.gamma > 0 ? P.gamma : 0.0;
 
-  for (int t = 0; t < P.n_trees; ++t) {
-    double* wprev = hweight + (size_t)((t + 1) & 1) * NH;
-    double* wcur = hweight + (size_t)(t & 1) * NH;
-    gbdt_node* tree = trees + (size_t)t * NH;
+  // One tree of Alg. 1 (every tree-dependent pointer is resolved on the device from tidx, so the
+  // same launch sequence builds any tree): captured once into a CUDA graph and replayed T times
+  // when nothing in it needs the host (no profiling events, no user-loss callback, no
+  // host-staged collectives); launched directly otherwise.
+  auto tree_body = [&](int t) {
     tm.begin(GBDT_PHASE_GRAD);
-    if (rows.indptr) { rows.trees = trees; rows.t = t; }
-    k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, t == 0, P.eta, P.base_margin, ds.y.as<float>(), wprev,
+    if (rows.indptr) rows.trees = trees;
+    k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, tidx, P.eta, P.base_margin, ds.y.as<float>(), hweight, NH,
                                         yhat, pos, gv, hv, hmode == kHGather, partial, rows, custom ? 1 : 0);
     GBDT_LAUNCH_CHECK();
     if (custom) {  // user-defined loss: g, h from the callback, on this stream
       if (P.grad_fn(n, yhat, ds.y.as<float>(), gv, hv, (void*)st, P.grad_user) != 0)
         fail(GBDT_E_INVAL, "grad_fn failed at tree " + std::to_string(t));
-      k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, 0, P.eta, P.base_margin, ds.y.as<float>(), wprev,
+      k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, tidx, P.eta, P.base_margin, ds.y.as<float>(), hweight, NH,
                                           yhat, pos, gv, hv, 1, partial, RowsArgs{}, 2);
       GBDT_LAUNCH_CHECK();
       count_launch();
     }
-    k_tree_begin<<<1, 1024, 0, st>>>(grad_blocks, partial, n, P.lambda, nt[0], NH, wcur, hstate, tree, fxs);
+    k_tree_begin<<<1, 1024, 0, st>>>(grad_blocks, partial, n, P.lambda, nt[0], NH, hweight, hstate, trees, fxs, tidx);
     GBDT_LAUNCH_CHECK();
     count_launch(2);
     tm.end();
@@ -724,7 +747,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       DecideArgs D;
       D.cur = cur; D.nxt = nxt; D.best_all = best_all; D.nshard = nsh; D.Kcap = Kcap; D.epochp = epoch;
       D.lam = P.lambda; D.thr = thr; D.last_level = last; D.cidx = cidx; D.winner = winner;
-      D.hstate = hstate; D.hdef = hdef; D.hweight = wcur; D.tree = tree;
+      D.hstate = hstate; D.hdef = hdef; D.hweight = hweight; D.trees = trees; D.tidx = tidx; D.NH = NH;
       k_decide<<<1, 1024, 0, st>>>(D);
       GBDT_LAUNCH_CHECK();
       count_launch();
@@ -805,13 +828,56 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       }
       tm.end();
     }
+    k_tree_end<<<1, 1, 0, st>>>(tidx);
+    GBDT_LAUNCH_CHECK();
+    count_launch();
+  };
+
+  const bool host_comm = ds.comm && ds.comm->world > 1 && !ds.comm->nccl;
+  const char* ge = getenv("GBDT_GRAPH");
+  const bool graph = !tm.on && !custom && !host_comm && P.n_trees > 1 && !(ge && ge[0] == '0');
+  if (!graph) {
+    for (int t = 0; t < P.n_trees; ++t) tree_body(t);
+  } else {
+    // capture on a private stream (the legacy default stream cannot be captured); nothing runs
+    // during the capture, the replays go to st in order
+    const cudaStream_t st0 = st;
+    cudaStream_t cs = nullptr;
+    GBDT_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+    cudaGraph_t g = nullptr;
+    cudaGraphExec_t gx = nullptr;
+    const int64_t before = launches_get();
+    st = cs;
+    GBDT_CUDA(cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
+    try {
+      tree_body(0);
+    } catch (...) {
+      cudaStreamEndCapture(cs, &g);
+      if (g) cudaGraphDestroy(g);
+      st = st0;
+      cudaStreamDestroy(cs);
+      throw;
+    }
+    GBDT_CUDA(cudaStreamEndCapture(cs, &g));
+    st = st0;
+    const int64_t per_tree = launches_get() - before;
+    launches_reset();
+    count_launch((int)before);
+    GBDT_CUDA(cudaGraphInstantiate(&gx, g, 0));
+    for (int t = 0; t < P.n_trees; ++t) {
+      GBDT_CUDA(cudaGraphLaunch(gx, st));
+      count_launch((int)per_tree);
+    }
+    GBDT_CUDA(cudaGraphExecDestroy(gx));
+    GBDT_CUDA(cudaGraphDestroy(g));
+    GBDT_CUDA(cudaStreamDestroy(cs));
   }
   // final SmartGD step: the last tree's leaf weights
   {
     double* wlast = hweight + (size_t)((P.n_trees - 1) & 1) * NH;
     if (rows.indptr) {  // ablation: the final margin by traversal of all trees too
       rows.trees = trees; rows.t = P.n_trees;
-      k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, 0, P.eta, P.base_margin, ds.y.as<float>(), wlast,
+      k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, nullptr, P.eta, P.base_margin, ds.y.as<float>(), hweight, NH,
                                           yhat, pos, gv, hv, 0, partial, rows, 1);
     } else {
       k_apply<<<inst_grid, 256, 0, st>>>(n, P.eta, wlast, pos, yhat);

@@ -101,3 +101,20 @@ def test_custom_loss_errors():
         raise RuntimeError("user loss failed")
     with pytest.raises(gbdt.GbdtError, match="grad_fn failed"):
         gbdt.train(ds, max_depth=2, n_trees=1, loss="custom", grad_fn=bad)
+
+
+@pytest.mark.parametrize("maker", [
+    lambda: synth.c1(n=3000),
+    lambda: synth.c4(seed=3, n=600, m=2000, density=0.01),
+    lambda: synth.c5(n=20000, T=3),
+])
+def test_graph_replay_bit_identical(maker, monkeypatch):
+    """the tree loop replayed as one CUDA graph per tree equals eager launches."""
+    p = maker()
+    monkeypatch.setenv("GBDT_GRAPH", "0")
+    m_e, y_e = gbdt.train_problem(p)
+    monkeypatch.setenv("GBDT_GRAPH", "1")
+    m_g, y_g = gbdt.train_problem(p)
+    _same_model(m_e, m_g)
+    assert y_e.tobytes() == y_g.tobytes()
+    compare(p, m_g.nodes(), y_g)
