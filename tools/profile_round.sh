@@ -6,7 +6,7 @@
 CFG=${CFG:-C3}
 mkdir -p gpurun_out
 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none \
-    -c 400 --csv --log-file gpurun_out/launches_$CFG.csv \
+    -c 1500 --csv --log-file gpurun_out/launches_$CFG.csv \
     python bench.py --config $CFG --steps 1 --warmup 0 --no-cpu-baseline --no-e2e > gpurun_out/ncu_launch_$CFG.log 2>&1
 for K in k_sf_fast k_part_scatter k_chunk_agg k_part_count; do
   ncu --set full --import-source on --clock-control none -k regex:$K -s 2 -c 1 -o gpurun_out/full_${K}_$CFG -f \
