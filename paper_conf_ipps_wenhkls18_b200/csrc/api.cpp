@@ -1,7 +1,11 @@
 // api.cpp -- the C ABI of libgbdt.so (include/gbdt.h): validation, handles, error reporting.
 #include <cmath>
+#include <atomic>
+#include <climits>
 #include <cstring>
+#include <thread>
 #include <exception>
+#include <algorithm>
 #include <limits>
 #include <new>
 #include <string>
@@ -55,7 +59,21 @@ static gbdt_status guarded(F&& f) {
   }
 }
 
+// Runs f(lo, hi) over [0, n) split into contiguous ranges on up to hardware_concurrency threads
+// (one range when n is small).
+template <class F>
+static void parallel_ranges(int64_t n, int64_t min_per_thread, F&& f) {
+  const int64_t hw = std::max<int64_t>(1, (int64_t)std::thread::hardware_concurrency());
+  const int64_t T = std::max<int64_t>(1, std::min<int64_t>(std::min<int64_t>(hw, 64), n / std::max<int64_t>(min_per_thread, 1)));
+  if (T == 1) { f(0, n, 0); return; }
+  std::vector<std::thread> th;
+  for (int64_t t = 0; t < T; ++t) th.emplace_back([&, t] { f(n * t / T, n * (t + 1) / T, (int)t); });
+  for (auto& x : th) x.join();
+}
+
 // CSR structure checks shared by load and predict (P:32 sparse rows; indices strictly increasing).
+// Row ranges are checked in parallel; the error reported is the one of the first bad row, as a
+// sequential scan would report it.
 static void validate_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr, const int32_t* indices,
                          const float* values, bool require_cols_in_range) {
   const int64_t kMax = (int64_t(1) << 31) - 1;
@@ -63,20 +81,40 @@ static void validate_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr, 
   if (n_cols < 1 || n_cols >= kMax) fail(GBDT_E_INVAL, "n_cols must be in [1, 2^31-1)");
   if (!indptr) fail(GBDT_E_INVAL, "indptr is NULL");
   if (indptr[0] != 0) fail(GBDT_E_INVAL, "indptr[0] must be 0");
-  for (int64_t i = 0; i < n_rows; ++i)
-    if (indptr[i + 1] < indptr[i]) fail(GBDT_E_INVAL, "indptr must be non-decreasing (row " + std::to_string(i) + ")");
+  std::atomic<int64_t> bad{INT64_MAX};
+  auto note = [&](int64_t i) {
+    int64_t cur = bad.load();
+    while (i < cur && !bad.compare_exchange_weak(cur, i)) {
+    }
+  };
+  parallel_ranges(n_rows, 1 << 16, [&](int64_t lo, int64_t hi, int) {
+    for (int64_t i = lo; i < hi; ++i)
+      if (indptr[i + 1] < indptr[i]) { note(i); return; }
+  });
+  if (bad.load() != INT64_MAX)
+    fail(GBDT_E_INVAL, "indptr must be non-decreasing (row " + std::to_string(bad.load()) + ")");
   const int64_t nnz = indptr[n_rows];
   if (nnz >= kMax) fail(GBDT_E_INVAL, "nnz must be < 2^31-1");
   if (nnz > 0 && (!indices || !values)) fail(GBDT_E_INVAL, "indices/values NULL with nnz > 0");
-  for (int64_t i = 0; i < n_rows; ++i) {
-    int32_t prev = -1;
-    for (int64_t p = indptr[i]; p < indptr[i + 1]; ++p) {
-      const int32_t a = indices[p];
-      if (a < 0 || (require_cols_in_range && a >= n_cols))
-        fail(GBDT_E_INVAL, "column index out of range in row " + std::to_string(i));
-      if (a <= prev) fail(GBDT_E_INVAL, "column indices must be strictly increasing in row " + std::to_string(i));
-      prev = a;
+  std::vector<int> kind(64, 0);  // per thread: 1 out of range, 2 not increasing (at its first bad row)
+  std::vector<int64_t> first(64, INT64_MAX);
+  parallel_ranges(n_rows, 1 << 14, [&](int64_t lo, int64_t hi, int t) {
+    for (int64_t i = lo; i < hi; ++i) {
+      int32_t prev = -1;
+      for (int64_t p = indptr[i]; p < indptr[i + 1]; ++p) {
+        const int32_t a = indices[p];
+        if (a < 0 || (require_cols_in_range && a >= n_cols)) { kind[t] = 1; first[t] = i; return; }
+        if (a <= prev) { kind[t] = 2; first[t] = i; return; }
+        prev = a;
+      }
     }
+  });
+  int bt = -1;
+  for (int t = 0; t < 64; ++t)
+    if (kind[t] && (bt < 0 || first[t] < first[bt])) bt = t;
+  if (bt >= 0) {
+    if (kind[bt] == 1) fail(GBDT_E_INVAL, "column index out of range in row " + std::to_string(first[bt]));
+    fail(GBDT_E_INVAL, "column indices must be strictly increasing in row " + std::to_string(first[bt]));
   }
 }
 
@@ -126,11 +164,27 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
     if (!labels) fail(GBDT_E_INVAL, "labels is NULL");
     float lmin = std::numeric_limits<float>::infinity(), lmax = -lmin;
     bool binary = true;
-    for (int64_t i = 0; i < n_rows; ++i) {
-      binary &= (labels[i] == 0.0f || labels[i] == 1.0f);
-      if (!std::isfinite(labels[i])) fail(GBDT_E_INVAL, "labels must be finite (row " + std::to_string(i) + ")");
-      lmin = std::min(lmin, labels[i]);
-      lmax = std::max(lmax, labels[i]);
+    {
+      struct LabelStats { float lo, hi; bool bin; int64_t bad; };
+      std::vector<LabelStats> ls(64, LabelStats{lmin, lmax, true, INT64_MAX});
+      parallel_ranges(n_rows, 1 << 16, [&](int64_t lo, int64_t hi, int t) {
+        LabelStats& L = ls[t];
+        for (int64_t i = lo; i < hi; ++i) {
+          const float y = labels[i];
+          if (!std::isfinite(y)) { L.bad = i; return; }
+          L.bin &= (y == 0.0f || y == 1.0f);
+          L.lo = std::min(L.lo, y);
+          L.hi = std::max(L.hi, y);
+        }
+      });
+      int64_t bad = INT64_MAX;
+      for (const LabelStats& L : ls) {
+        bad = std::min(bad, L.bad);
+        binary &= L.bin;
+        lmin = std::min(lmin, L.lo);
+        lmax = std::max(lmax, L.hi);
+      }
+      if (bad != INT64_MAX) fail(GBDT_E_INVAL, "labels must be finite (row " + std::to_string(bad) + ")");
     }
     gbdt_load_opts o;
     std::memset(&o, 0, sizeof o);
@@ -156,20 +210,29 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
     }
 
     const int64_t nnz = indptr[n_rows];
-    std::vector<int64_t> col_counts(n_cols, 0);
-    for (int64_t p = 0; p < nnz; ++p)
-      if (!std::isnan(values[p])) col_counts[indices[p]]++;
-    bool missing = false;
-    for (int64_t a = 0; a < n_cols; ++a) missing |= col_counts[a] != n_rows;
 
     auto* h = new gbdt_dataset();
     Dataset& ds = h->ds;
     try {
+      cudaStream_t st = (cudaStream_t)o.stream;
+      DBuf dptr((size_t)(n_rows + 1) * 8, st), didx((size_t)std::max<int64_t>(nnz, 1) * 4, st),
+          dval((size_t)std::max<int64_t>(nnz, 1) * 4, st);
+      GBDT_CUDA(cudaMemcpyAsync(dptr.p, indptr, (size_t)(n_rows + 1) * 8, cudaMemcpyHostToDevice, st));
+      if (nnz) {
+        GBDT_CUDA(cudaMemcpyAsync(didx.p, indices, (size_t)nnz * 4, cudaMemcpyHostToDevice, st));
+        GBDT_CUDA(cudaMemcpyAsync(dval.p, values, (size_t)nnz * 4, cudaMemcpyHostToDevice, st));
+      }
+      ds.y.alloc((size_t)n_rows * 4, st);
+      GBDT_CUDA(cudaMemcpyAsync(ds.y.p, labels, (size_t)n_rows * 4, cudaMemcpyHostToDevice, st));
+      // present entries per attribute, counted on the device
+      const std::vector<int64_t> col_counts = column_counts(nnz, n_cols, didx.as<int32_t>(), dval.as<float>(), st);
+      bool missing = false;
+      for (int64_t a = 0; a < n_cols; ++a) missing |= col_counts[a] != n_rows;
       ds.n = n_rows;
       ds.m = n_cols;
       ds.nnz = nnz;
       ds.device = dev;
-      ds.stream = (cudaStream_t)o.stream;
+      ds.stream = st;
       ds.has_missing = missing;
       ds.binary_labels = binary;
       ds.comm = comm;
@@ -189,16 +252,6 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
         sh->m = sh->a_end - sh->a_begin;
         ds.shards.push_back(std::move(sh));
       }
-      cudaStream_t st = ds.stream;
-      DBuf dptr((size_t)(n_rows + 1) * 8, st), didx((size_t)std::max<int64_t>(nnz, 1) * 4, st),
-          dval((size_t)std::max<int64_t>(nnz, 1) * 4, st);
-      GBDT_CUDA(cudaMemcpyAsync(dptr.p, indptr, (size_t)(n_rows + 1) * 8, cudaMemcpyHostToDevice, st));
-      if (nnz) {
-        GBDT_CUDA(cudaMemcpyAsync(didx.p, indices, (size_t)nnz * 4, cudaMemcpyHostToDevice, st));
-        GBDT_CUDA(cudaMemcpyAsync(dval.p, values, (size_t)nnz * 4, cudaMemcpyHostToDevice, st));
-      }
-      ds.y.alloc((size_t)n_rows * 4, st);
-      GBDT_CUDA(cudaMemcpyAsync(ds.y.p, labels, (size_t)n_rows * 4, cudaMemcpyHostToDevice, st));
       build_layout(ds, dptr.as<int64_t>(), didx.as<int32_t>(), dval.as<float>(), col_counts, o.rle_min_ratio);
       if (o.keep_rows) {
         ds.rows_ptr = std::move(dptr);

@@ -155,6 +155,8 @@ struct Comm {
 // api.cpp: contiguous attribute ranges balanced by entries
 std::vector<int32_t> shard_ranges(int64_t n_cols, const int64_t* col_counts, int P);
 // layout.cu
+std::vector<int64_t> column_counts(int64_t nnz, int64_t m, const int32_t* d_indices, const float* d_values,
+                                   cudaStream_t st);
 void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices,
                   const float* d_values, const std::vector<int64_t>& col_counts,
                   double rle_min_ratio);

@@ -236,7 +236,47 @@ __global__ void k_run_chunk_root(int m, Tables tb) {
   }
 }
 
+// Present (non-NaN) entries per attribute: block-private shared-memory histograms when the
+// attributes fit (one global add per attribute and block), plain global atomics otherwise.
+constexpr int kHistSmem = 8192;
+__global__ void k_col_hist(int64_t nnz, int64_t m, const int32_t* __restrict__ idx, const float* __restrict__ val,
+                           unsigned long long* __restrict__ cnt) {
+  __shared__ unsigned int hs[kHistSmem];
+  const bool priv = m <= kHistSmem;
+  if (priv)
+    for (int a = threadIdx.x; a < m; a += blockDim.x) hs[a] = 0u;
+  __syncthreads();
+  for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < nnz; p += (int64_t)gridDim.x * blockDim.x) {
+    if (isnan(val[p])) continue;
+    if (priv) atomicAdd(&hs[idx[p]], 1u);
+    else atomicAdd(cnt + idx[p], 1ull);
+  }
+  if (priv) {
+    __syncthreads();
+    for (int a = threadIdx.x; a < m; a += blockDim.x)
+      if (hs[a]) atomicAdd(cnt + a, (unsigned long long)hs[a]);
+  }
+}
+
 }  // namespace
+
+std::vector<int64_t> column_counts(int64_t nnz, int64_t m, const int32_t* d_indices, const float* d_values,
+                                   cudaStream_t st) {
+  int dev = 0, sms = 148;
+  GBDT_CUDA(cudaGetDevice(&dev));
+  GBDT_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  DBuf c((size_t)m * 8, st);
+  GBDT_CUDA(cudaMemsetAsync(c.p, 0, (size_t)m * 8, st));
+  if (nnz > 0) {
+    const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(nnz, 256), (int64_t)sms * 8));
+    k_col_hist<<<g, 256, 0, st>>>(nnz, m, d_indices, d_values, c.as<unsigned long long>());
+    GBDT_LAUNCH_CHECK();
+  }
+  std::vector<int64_t> h((size_t)m);
+  GBDT_CUDA(cudaMemcpyAsync(h.data(), c.p, (size_t)m * 8, cudaMemcpyDeviceToHost, st));
+  GBDT_CUDA(cudaStreamSynchronize(st));
+  return h;
+}
 
 static void radix_sort(unsigned long long*& keys, uint32_t*& ids, unsigned long long*& kalt,
                        uint32_t*& ialt, int64_t N, int bits, cudaStream_t st, int sms) {
