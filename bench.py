@@ -278,6 +278,19 @@ def main():
                "note": "one gbdt_load_csr (H2D + layout sort) + K-tree gbdt_train + margin D2H, amortised per tree"}
         del ds2, model2
 
+    # gbdt_predict on the training rows with the K trees: wall clock through the
+    # C ABI, the CSR's H2D copy included; must reproduce the training margin
+    pred = None
+    if rank == 0 and world == 1 and not args.no_e2e:
+        hp_, hi_, hv_ = [torch.from_numpy(np.ascontiguousarray(a)).pin_memory().numpy()
+                         for a in (prob.indptr, prob.indices, prob.values)]
+        model.predict(hp_, hi_, hv_, prob.m)  # warm-up
+        t0 = time.perf_counter()
+        model.predict(hp_, hi_, hv_, prob.m)
+        tp_s = time.perf_counter() - t0
+        pred = {"rows_per_s": prob.n / tp_s, "s": tp_s, "trees": args.steps,
+                "note": "gbdt_predict on the training rows, CSR H2D + D2H included"}
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         rate, cinfo, _ = oracle_sample_rate(prob, args.cpu_seconds)
@@ -305,6 +318,7 @@ def main():
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches,
+            "predict": pred,
             "clocks": clocks,
             "context": {"paper_gpu_gbdt_titanx_higgs10M_mse_s_per_tree": 5.50,
                         "paper_xgbst40_higgs10M_mse_s_per_tree": 9.66, "source": "PAPER.md P:478-487 /40"},

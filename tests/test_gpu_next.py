@@ -118,3 +118,44 @@ def test_graph_replay_bit_identical(maker, monkeypatch):
     _same_model(m_e, m_g)
     assert y_e.tobytes() == y_g.tobytes()
     compare(p, m_g.nodes(), y_g)
+
+
+def _traverse(nodes, eta, base, X):
+    """Host traversal of the model's trees (reading R11): present x >= split_value goes
+    high (2k+1), missing follows default_left; y accumulated in tree order in fp64."""
+    n = X.shape[0]
+    out = np.empty(n)
+    for i in range(n):
+        y = base
+        for t in range(nodes.shape[0]):
+            T = nodes[t]
+            k = 0
+            while not T[k]["is_leaf"]:
+                x = X[i, T[k]["attr"]]
+                high = bool(T[k]["default_left"]) if np.isnan(x) else bool(np.float32(x) >= T[k]["split_value"])
+                k = 2 * k + 1 if high else 2 * k + 2
+            y = y + eta * T[k]["weight"]
+        out[i] = y
+    return out
+
+
+@pytest.mark.parametrize("m_train", [6, 90])  # dense shared-memory kernel / CSR binary search
+def test_predict_kernels_match_host_traversal(m_train):
+    rng = np.random.default_rng(m_train)
+    p = synth.random_small(21, n=400, m=m_train, nan_frac=0.2, n_distinct=12, loss="logistic", d=4, T=3)
+    model, margin = gbdt.train_problem(p)
+    # new rows: NaN, -0.0 and columns past the training n_cols (ignored = missing)
+    n2, m2 = 300, m_train + 3
+    X = rng.integers(0, 12, size=(n2, m2)).astype(np.float32) / 4 - 1.0
+    X[rng.random((n2, m2)) < 0.25] = np.nan
+    X[rng.random((n2, m2)) < 0.05] = -0.0
+    mask = ~np.isnan(X) | (rng.random((n2, m2)) < 0.5)  # some NaNs stored explicitly, others absent
+    indptr = np.concatenate([[0], np.cumsum(mask.sum(1))]).astype(np.int64)
+    indices = np.nonzero(mask)[1].astype(np.int32)
+    values = X[mask].astype(np.float32)
+    got = model.predict(indptr, indices, values, m2)
+    Xd = np.where(mask, X, np.nan)[:, :m_train]
+    want = _traverse(model.nodes(), p.params.get("eta", 0.3), p.params.get("base_margin", 0.0), Xd)
+    assert got.tobytes() == want.tobytes()
+    # and the training rows reproduce the training margin
+    assert np.array_equal(model.predict(p.indptr, p.indices, p.values, p.m), margin)
