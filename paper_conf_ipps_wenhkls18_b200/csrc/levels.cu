@@ -863,24 +863,35 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
       // compared by cross-multiplication (no division), num = GL^2 (HR+l) + GR^2 (HL+l),
       // den = (HL+l)(HR+l); only the winning item index is carried
       const double Hl = nv.H + lam;
-      double pg = bg, phh = bh, bnum = -1.0, bden = 1.0;
-      int bk = -1;
+      unsigned cm = 0;  // the lane's candidates: run ends with a non-empty low side
 #pragma unroll
       for (int k = 0; k < kItems; ++k) {
-        pg = pg + g[k];
-        phh = phh + hk[k];
         const float nx = k < kItems - 1 ? v[k + 1] : vn;
-        const double dl = phh + lam, dr = Hl - phh, GR = nv.G - pg;
-        const double num = __fma_rn(__dmul_rn(pg, pg), dr, __dmul_rn(__dmul_rn(GR, GR), dl)), den = __dmul_rn(dl, dr);
-        if (k < nc && nx != v[k] && __dmul_rn(num, bden) > __dmul_rn(bnum, den)) { bnum = num; bden = den; bk = k; }
+        if (k < nc && nx != v[k]) cm |= 1u << k;
       }
-      double wb = bk < 0 ? -INFINITY : __dmul_rn(bnum, rcp_nr(bden));
-      int wq = bk < 0 ? INT_MAX : q0 + bk;
+      double pg = bg, phh = bh, bnum = -1.0, bden = 1.0;
+      int bk = -1;
+      double wb = -INFINITY;
+      int wq = INT_MAX;
+      // Low-cardinality lists (long runs of equal values, RLE-shaped data) have chunks without any
+      // run end: the whole warp skips the scoring (only run ends are candidates).
+      if (__any_sync(0xffffffffu, cm != 0u)) {
 #pragma unroll
-      for (int o = 16; o; o >>= 1) {
-        const double ob = __shfl_xor_sync(0xffffffffu, wb, o);
-        const int oq = __shfl_xor_sync(0xffffffffu, wq, o);
-        if (ob > wb || (ob == wb && oq < wq)) { wb = ob; wq = oq; }
+        for (int k = 0; k < kItems; ++k) {
+          pg = pg + g[k];
+          phh = phh + hk[k];
+          const double dl = phh + lam, dr = Hl - phh, GR = nv.G - pg;
+          const double num = __fma_rn(__dmul_rn(pg, pg), dr, __dmul_rn(__dmul_rn(GR, GR), dl)), den = __dmul_rn(dl, dr);
+          if (((cm >> k) & 1u) && __dmul_rn(num, bden) > __dmul_rn(bnum, den)) { bnum = num; bden = den; bk = k; }
+        }
+        wb = bk < 0 ? -INFINITY : __dmul_rn(bnum, rcp_nr(bden));
+        wq = bk < 0 ? INT_MAX : q0 + bk;
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+          const double ob = __shfl_xor_sync(0xffffffffu, wb, o);
+          const int oq = __shfl_xor_sync(0xffffffffu, wq, o);
+          if (ob > wb || (ob == wb && oq < wq)) { wb = ob; wq = oq; }
+        }
       }
       // Can the chunk's best still beat node j's best so far in this CTA?  Its approximate gain
       // (the ranking score, ~1e-15 relative) must come within a 1e-12 relative slack of it;
