@@ -522,31 +522,50 @@ __global__ void __launch_bounds__(kThreads) k_scan1(const int32_t* __restrict__ 
   }
 }
 
+// One block of kScan2Threads: every thread takes a contiguous run of group aggregates, so the
+// dependent chain is ceil(G / kScan2Threads) elements plus two warp scans (not G / 32 warp scans).
+constexpr int kScan2Threads = 1024;
 template <bool kFx>
-__global__ void k_scan2(const int32_t* __restrict__ Cp, unsigned long long* __restrict__ gagg) {
+__global__ void __launch_bounds__(kScan2Threads) k_scan2(const int32_t* __restrict__ Cp, unsigned long long* __restrict__ gagg) {
   using O = ScanOps<kFx>;
   using T = typename O::T;
+  __shared__ T wt[kScan2Threads / 32];
   const int C = *Cp;
   const int G = (C + kScanGroup - 1) / kScanGroup;
-  const int lane = threadIdx.x & 31;
-  T carry = O::zero();
-  for (int base = 0; base < G; base += 32) {
-    const int i = base + lane;
-    T x = O::zero();
-    if (i < G) x = O::load_plain(gagg, i);
-    T inc = x;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int per = (G + kScan2Threads - 1) / kScan2Threads;
+  const int i0 = threadIdx.x * per, i1 = min(G, i0 + per);
+  T run = O::zero();
+  for (int i = i0; i < i1; ++i) run = O::comb(run, O::load_plain(gagg, i));
+  T inc = run;
+  for (int o = 1; o < 32; o <<= 1) {
+    const T y = O::up(inc, o);
+    if (lane >= o) inc = O::comb(y, inc);
+  }
+  T ex = O::up(inc, 1);
+  if (lane == 0) ex = O::zero();
+  if (lane == 31) wt[wid] = inc;
+  __syncthreads();
+  if (wid == 0) {  // exclusive scan of the warp totals
+    const T x = wt[lane];
+    T wi = x;
     for (int o = 1; o < 32; o <<= 1) {
-      const T y = O::up(inc, o);
-      if (lane >= o) inc = O::comb(y, inc);
+      const T y = O::up(wi, o);
+      if (lane >= o) wi = O::comb(y, wi);
     }
-    T ex = O::up(inc, 1);
-    if (lane == 0) ex = O::zero();
-    const T e = O::comb(carry, ex);
-    if (i < G) O::store(gagg, i, e);
-    carry = O::comb(carry, O::idx(inc, 31));
+    T we = O::up(wi, 1);
+    if (lane == 0) we = O::zero();
+    __syncwarp();
+    wt[lane] = we;
+  }
+  __syncthreads();
+  T pre = O::comb(wt[wid], ex);  // everything before the thread's first element
+  for (int i = i0; i < i1; ++i) {
+    const T x = O::load_plain(gagg, i);
+    O::store(gagg, i, pre);
+    pre = O::comb(pre, x);
   }
 }
-
 template <bool kFx>
 __global__ void __launch_bounds__(kThreads) k_scan3(const int32_t* __restrict__ Cp, const unsigned long long* __restrict__ in,
                                                    const unsigned long long* __restrict__ gcar,
@@ -1979,7 +1998,7 @@ template <bool kFx>
 void launch_scan(const int32_t* Cp, unsigned long long* in, unsigned long long* gbuf, unsigned long long* out,
                  unsigned groups, cudaStream_t st) {
   k_scan1<kFx><<<groups, kThreads, 0, st>>>(Cp, in, gbuf);
-  k_scan2<kFx><<<1, 32, 0, st>>>(Cp, gbuf);
+  k_scan2<kFx><<<1, kScan2Threads, 0, st>>>(Cp, gbuf);
   k_scan3<kFx><<<groups, kThreads, 0, st>>>(Cp, in, gbuf, out);
   GBDT_LAUNCH_CHECK();
   count_launch(3);

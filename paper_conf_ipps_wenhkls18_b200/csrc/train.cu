@@ -833,9 +833,14 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     count_launch();
   };
 
-  const bool host_comm = ds.comm && ds.comm->world > 1 && !ds.comm->nccl;
+  // NCCL collectives inside the captured tree are supported by NCCL but not exercised on the
+  // single-GPU boxes this was built on: with a multi-rank communicator the graph is opt-in
+  // (GBDT_GRAPH=1); GBDT_GRAPH=0 forces eager launches everywhere
+  const bool multi = ds.comm && ds.comm->world > 1;
+  const bool host_comm = multi && !ds.comm->nccl;
   const char* ge = getenv("GBDT_GRAPH");
-  const bool graph = !tm.on && !custom && !host_comm && P.n_trees > 1 && !(ge && ge[0] == '0');
+  const bool graph_ok = ge ? ge[0] != '0' : !multi;
+  const bool graph = !tm.on && !custom && !host_comm && P.n_trees > 1 && graph_ok;
   if (!graph) {
     for (int t = 0; t < P.n_trees; ++t) tree_body(t);
   } else {
