@@ -1640,6 +1640,9 @@ template <int HMODE, bool kRLE, bool kAgg>
 #ifndef GBDT_SCATTER_ROWS
 #define GBDT_SCATTER_ROWS 4
 #endif
+#ifndef GBDT_SCATTER_STCS
+#define GBDT_SCATTER_STCS 1  // evict-first stores: 11.76 -> 11.38 ms/tree of scatter on C3
+#endif
 __global__ void __launch_bounds__(kThreads, GBDT_SCATTER_CTAS) k_part_scatter(PartArgs A) {
   constexpr bool kH = HMODE == kHGather;
   constexpr int kHalf = GBDT_SCATTER_ROWS;  // rows loaded per step
@@ -1761,10 +1764,17 @@ __global__ void __launch_bounds__(kThreads, GBDT_SCATTER_CTAS) k_part_scatter(Pa
               }
             }
           }
+#if GBDT_SCATTER_STCS
+          if (!kRLE) __stcs(A.val_out + d, v[kk]);
+          __stcs(A.ins_out + d, id[kk]);
+          __stcs(A.g_out + d, g[kk]);
+          if (kH) __stcs(A.h_out + d, h[kk]);
+#else
           if (!kRLE) A.val_out[d] = v[kk];
           A.ins_out[d] = id[kk];
           A.g_out[d] = g[kk];
           if (kH) A.h_out[d] = h[kk];
+#endif
         }
         nh += __popc(bh);
         nl += __popc(bl);
