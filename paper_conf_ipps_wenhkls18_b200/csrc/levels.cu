@@ -195,7 +195,9 @@ __device__ __forceinline__ ChunkMeta chunk_meta(const TabCache& tc, const TileAr
 // L2 prefetch of a chunk's list bytes [p0, p0 + 256) * elem (lanes take one 128-byte line each)
 __device__ __forceinline__ void prefetch_chunk(const void* list, long long p0, int elem, int lane) {
   const char* b = reinterpret_cast<const char*>(list) + p0 * elem;
-  if (lane * 128 < kChunk * elem) asm volatile("prefetch.global.L2 [%0];" ::"l"(b + lane * 128));
+  // evict-last: the prefetched lines must survive the streaming traffic until the warp reads them
+  // (C3 scatter 11.38 -> 11.22 ms/tree against a plain prefetch; 12.03 without prefetch)
+  if (lane * 128 < kChunk * elem) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(b + lane * 128));
 }
 
 // Segment (node) of each of the thread's items; head / piece-end / run-end masks.  ss/sc are the
