@@ -284,3 +284,22 @@ def test_scatter_aggregates_match_chunk_agg():
     q = synth.from_dense("agg_missing", X, base.labels, dict(base.params))
     model2, margin2 = _train(q)
     compare(q, model2.nodes(), margin2)
+
+
+def test_all_entries_missing_and_empty_rows():
+    """Degenerate inputs: no stored entry at all (every value missing) gives single-leaf
+    trees; rows without entries next to full rows still split on the present values."""
+    P = dict(loss="squared", max_depth=3, n_trees=2, lam=1.0, gamma=0.0, eta=0.5, base_margin=0.0)
+    X = np.full((50, 3), np.nan)
+    y = np.linspace(-1, 1, 50)
+    p = synth.from_dense("all-missing", X, y, P)
+    assert p.nnz == 0
+    model, margin = _train(p)
+    nodes = model.nodes()
+    assert (nodes["is_leaf"][:, 0] == 1).all() and (nodes["heap_id"][:, 1:] == -1).all()
+    compare(p, nodes, margin)
+    X = np.random.default_rng(3).normal(size=(200, 3))
+    X[::3] = np.nan  # a third of the rows are empty
+    p = synth.from_dense("empty-rows", X, np.nan_to_num(X[:, 1]), P)
+    model, margin = _train(p)
+    compare(p, model.nodes(), margin)
