@@ -72,13 +72,6 @@ struct SplitArgs {
                          // earlier chunk, else -1; nullptr: no missing values
 };
 
-// Decoupled look-back storage of the partition's (high, low) counts: integers, exact in any order.
-struct LookBack {
-  int32_t* flag;                 // 2*epoch+1: aggregate published, 2*epoch+2: inclusive prefix published
-  unsigned long long* agg;       // packed hi | lo << 32
-  unsigned long long* incl;
-};
-
 struct PartArgs {
   TileArgs t;
   const double* g_in;     // g-list (h-list) of this level, moved with the entries
@@ -86,7 +79,6 @@ struct PartArgs {
   double* g_out;
   double* h_out;
   const int32_t* epochp;
-  LookBack lb;
   const uint8_t* side;    // per instance: 0 drop, 1 high, 2 low
   uint8_t* slist;         // per list entry: side of its instance (k_part_count -> k_part_scatter)
   int32_t* segH;          // [m*K] counted (missing values) or derived from node counts (dense)

@@ -398,7 +398,6 @@ struct ShardWork {
   unsigned long long *ccnt, *cpre;    // [C0][2]
   unsigned long long* sgrp;           // scan scratch
   unsigned groups;
-  LookBack lb;                        // partition look-back
   Rec* rec;
   ChunkDesc* desc;
   int32_t* genlist;
@@ -553,7 +552,6 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     ShardWork& w = sw[li];
     const int m = sh.m;
     const int64_t S = (int64_t)m * Kcap;
-    const int64_t T0 = std::max(sh.T0, 1);
     const int64_t C0 = std::max(sh.C0, 1);
     // node-best records per level: one per CTA and node (K <= 32), else one per chunk and segment
     const int64_t R = (int64_t)(LK.grid_fast[2][1] + LK.grid_fast[1][1] + LK.grid_fast[0][1] + LK.grid_gen) * 64 +
@@ -566,7 +564,6 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       q.take<unsigned long long>(5 * C0); q.take<unsigned long long>(5 * C0);
       q.take<unsigned long long>(2 * C0); q.take<unsigned long long>(2 * C0);
       q.take<unsigned long long>(5 * (size_t)LevelKernels::scan_groups(C0) + 8);
-      q.take<int32_t>(T0); q.take<unsigned long long>(T0); q.take<unsigned long long>(T0);
       q.take<Rec>(R); q.take<ChunkDesc>(C0); q.take<int32_t>(C0); q.take<int32_t>(S);
       q.take<int32_t>(S); q.take<int32_t>(S); q.take<unsigned long long>(S); q.take<int64_t>(S); q.take<int64_t>(S);
       q.take<int64_t>(m); q.take<double>(S); q.take<double>(S); q.take<int>(4);
@@ -589,7 +586,6 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     w.ccnt = q.take<unsigned long long>(2 * C0); w.cpre = q.take<unsigned long long>(2 * C0);
     w.groups = LevelKernels::scan_groups(C0);
     w.sgrp = q.take<unsigned long long>(5 * (size_t)w.groups + 8);
-    w.lb.flag = q.take<int32_t>(T0); w.lb.agg = q.take<unsigned long long>(T0); w.lb.incl = q.take<unsigned long long>(T0);
     const int nl = hmode == kHGather ? 4 : 2;
     w.lists.alloc((size_t)sh.cap * 8 * nl + (size_t)sh.cap + 64, st);
     w.slist = reinterpret_cast<uint8_t*>(w.lists.as<double>() + (size_t)sh.cap * nl);
@@ -801,7 +797,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         PA.ccnt = w.ccnt; PA.cpre = w.cpre; PA.sgrp = w.sgrp;
         PA.g_in = w.glist[lvl & 1]; PA.h_in = w.hlist[lvl & 1];
         PA.g_out = w.glist[(lvl + 1) & 1]; PA.h_out = w.hlist[(lvl + 1) & 1];
-        PA.epochp = epoch; PA.lb = w.lb;
+        PA.epochp = epoch;
         // without missing values the scatter accumulates the next level's chunk aggregates
         PA.cagg_next = ds.has_missing ? nullptr : w.cagg;
         PA.nxt = tn;
