@@ -303,3 +303,19 @@ def test_all_entries_missing_and_empty_rows():
     p = synth.from_dense("empty-rows", X, np.nan_to_num(X[:, 1]), P)
     model, margin = _train(p)
     compare(p, model.nodes(), margin)
+
+
+@pytest.mark.parametrize("maker", [
+    lambda: synth.random_small(77, n=6000, m=6, nan_frac=0.0, n_distinct=400, loss="logistic", d=8, T=2),
+    lambda: synth.random_small(78, n=5000, m=5, nan_frac=0.25, n_distinct=60, loss="squared", d=9, T=2),
+    lambda: synth.c4(seed=13, n=3000, m=1500, density=0.02, T=2),
+])
+def test_deep_trees_more_than_32_nodes_per_level(maker):
+    """Depth >= 7: more than 32 active nodes per level, so node bests go through the global record
+    list (post_record, k_pick_tie/k_pick_best) and the scatter finds segments without the per-warp
+    table -- the paths depth-6 configs never take."""
+    p = maker()
+    if p.name.startswith("C4"):
+        p.params["max_depth"] = 8
+    model, margin = _train(p)
+    compare(p, model.nodes(), margin, params=p.params)
