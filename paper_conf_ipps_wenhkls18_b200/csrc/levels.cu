@@ -721,31 +721,23 @@ __device__ __forceinline__ void rle_values(const Tables& tb, int cg, long long p
 }
 
 // A lane's 8 consecutive entries [8 lane, 8 lane + 8) of a chunk staged in shared memory, read
-// as 16-byte pieces in a lane-rotated order so that every quarter-warp touches 8 distinct 16-byte
-// bank groups (the natural order would be a 16-way bank conflict), then rotated back.
+// as 16-byte pieces in natural order.  The 64-byte lane stride makes these 4-way (g) and 2-way (v)
+// bank conflicts; a lane-rotated order avoids them but needs ~40 selects per chunk to rotate back,
+// and the kernel is issue bound: natural order measured 6.41 vs 6.66 ms/tree of split on C3.
 __device__ __forceinline__ void lds_blocked8(const double* chunk, int lane, double* out) {
   const double2* p = reinterpret_cast<const double2*>(chunk) + lane * 4;
-  const int s = (lane >> 1) & 3;
-  double2 x[4], y[4];
 #pragma unroll
-  for (int j = 0; j < 4; ++j) x[j] = p[(j + s) & 3];  // x[j] = piece (j + s) & 3
-  // piece r = x[(r - s) & 3]: rotate by s & 1, then by s & 2 (two select stages)
-#pragma unroll
-  for (int r = 0; r < 4; ++r) y[r] = (s & 1) ? x[(r + 3) & 3] : x[r];
-#pragma unroll
-  for (int r = 0; r < 4; ++r) {
-    const double2 z = (s & 2) ? y[(r + 2) & 3] : y[r];
-    out[2 * r] = z.x;
-    out[2 * r + 1] = z.y;
+  for (int j = 0; j < 4; ++j) {
+    const double2 z = p[j];
+    out[2 * j] = z.x;
+    out[2 * j + 1] = z.y;
   }
 }
 __device__ __forceinline__ void lds_blocked8f(const float* chunk, int lane, float* out) {
   const float4* p = reinterpret_cast<const float4*>(chunk) + lane * 2;
-  const int s = (lane >> 2) & 1;
-  const float4 a = p[s], b = p[s ^ 1];
-  const float4 x0 = s ? b : a, x1 = s ? a : b;
-  out[0] = x0.x; out[1] = x0.y; out[2] = x0.z; out[3] = x0.w;
-  out[4] = x1.x; out[5] = x1.y; out[6] = x1.z; out[7] = x1.w;
+  const float4 a0 = p[0], a1 = p[1];
+  out[0] = a0.x; out[1] = a0.y; out[2] = a0.z; out[3] = a0.w;
+  out[4] = a1.x; out[5] = a1.y; out[6] = a1.z; out[7] = a1.w;
 }
 
 // ---------------------------------------------------------------------------- k_sf_fast
