@@ -116,6 +116,23 @@ __device__ __forceinline__ FXV fxv_load(const unsigned long long* src, int* rese
              (__int128)(((unsigned __int128)src[3] << 64) | src[2]), (int)(unsigned)w, (int)((w >> 32) & 1)};
 }
 
+// Carry record of a chunk as the split kernels read it: the exclusive segmented prefix converted
+// to fp64 once (k_scan3), and the entry count.
+struct CarryD {
+  double g, h;
+  int c;
+};
+__device__ __forceinline__ void carry_store(unsigned long long* dst5, long long i, const FXV& x, int Fg, int Fh) {
+  unsigned long long* d = dst5 + 5 * i;
+  d[0] = (unsigned long long)__double_as_longlong(from_fx(x.g, Fg));
+  d[2] = (unsigned long long)__double_as_longlong(from_fx(x.h, Fh));
+  d[4] = (unsigned long long)(unsigned)x.c | ((unsigned long long)(x.f & 1) << 32);
+}
+__device__ __forceinline__ CarryD carry_load(const unsigned long long* src5) {
+  return CarryD{__longlong_as_double((long long)src5[0]), __longlong_as_double((long long)src5[2]),
+                (int)(unsigned)src5[4]};
+}
+
 template <int HMODE>
 __device__ __forceinline__ double hess_of(double g) {
   if (HMODE == kHConst2) return 2.0;
@@ -568,10 +585,12 @@ __global__ void __launch_bounds__(kScan2Threads) k_scan2(const int32_t* __restri
     pre = O::comb(pre, x);
   }
 }
+// kFx: the carries are written as fp64 values (word 0: g, word 2: h, word 4: count | flags),
+// converted once here from the exact fixed-point prefix instead of in every consumer
 template <bool kFx>
 __global__ void __launch_bounds__(kThreads) k_scan3(const int32_t* __restrict__ Cp, const unsigned long long* __restrict__ in,
                                                    const unsigned long long* __restrict__ gcar,
-                                                   unsigned long long* __restrict__ out) {
+                                                   unsigned long long* __restrict__ out, const int32_t* __restrict__ fx) {
   using O = ScanOps<kFx>;
   using T = typename O::T;
   constexpr int kPer = kScanGroup / kThreads;
@@ -609,7 +628,10 @@ __global__ void __launch_bounds__(kThreads) k_scan3(const int32_t* __restrict__ 
 #pragma unroll
   for (int k = 0; k < kPer; ++k) {
     const long long i = g0 + (long long)threadIdx.x * kPer + k;
-    if (i < C) O::store(out, i, r[k] ? O::zero() : prev);
+    if (i < C) {
+      if constexpr (kFx) carry_store(out, i, r[k] ? O::zero() : prev, fx[0], fx[1]);
+      else O::store(out, i, r[k] ? O::zero() : prev);
+    }
     prev = O::comb(prev, x[k]);
   }
 }
@@ -863,9 +885,9 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
       double bg, bh;
       int bc;
       {
-        const FXV cx = fxv_load(W.carry[st]);
-        bg = (head0 ? 0.0 : from_fx(cx.g, Fg)) + eg;
-        bh = (head0 ? 0.0 : from_fx(cx.h, Fh)) + eh;
+        const CarryD cx = carry_load(W.carry[st]);
+        bg = (head0 ? 0.0 : cx.g) + eg;
+        bh = (head0 ? 0.0 : cx.h) + eh;
         bc = (head0 ? 0 : cx.c) + min(q0, len);  // entries of the segment before the lane's first item
       }
       const NodeV nv = node_v(S.B, A, K, j);
@@ -899,12 +921,17 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
         }
         wb = bk < 0 ? -INFINITY : __dmul_rn(bnum, rcp_nr(bden));
         wq = bk < 0 ? INT_MAX : q0 + bk;
-#pragma unroll
-        for (int o = 16; o; o >>= 1) {
-          const double ob = __shfl_xor_sync(0xffffffffu, wb, o);
-          const int oq = __shfl_xor_sync(0xffffffffu, wq, o);
-          if (ob > wb || (ob == wb && oq < wq)) { wb = ob; wq = oq; }
-        }
+        // warp argmax (largest score, then smallest position) by three integer reductions on the
+        // order-preserving bit pattern of the score (scores are >= +0 or -inf, never NaN)
+        unsigned long long kb = (unsigned long long)__double_as_longlong(wb);
+        kb = (kb >> 63) ? ~kb : (kb | 0x8000000000000000ull);
+        const unsigned mhi = __reduce_max_sync(0xffffffffu, (unsigned)(kb >> 32));
+        const unsigned mlo = __reduce_max_sync(0xffffffffu, (unsigned)(kb >> 32) == mhi ? (unsigned)kb : 0u);
+        const bool top = (unsigned)(kb >> 32) == mhi && (unsigned)kb == mlo;
+        wq = (int)__reduce_min_sync(0xffffffffu, top ? (unsigned)wq : 0xffffffffu);
+        unsigned long long km = ((unsigned long long)mhi << 32) | mlo;
+        km = (km >> 63) ? (km & 0x7fffffffffffffffull) : ~km;
+        wb = __longlong_as_double((long long)km);
       }
       // Can the chunk's best still beat node j's best so far in this CTA?  Its approximate gain
       // (the ranking score, ~1e-15 relative) must come within a 1e-12 relative slack of it;
@@ -1043,9 +1070,9 @@ __device__ __forceinline__ void sf_short(const SplitArgs& A, NodeBest& B, unsign
     if (lane - o >= sl) { ig = yg + ig; ih = yh + ih; icn += yc; }
   }
   if (hpos < 0) {
-    const FXV cx = fxv_load(A.carry + 5ll * c);
-    ig = from_fx(cx.g, Fg) + ig;
-    ih = from_fx(cx.h, Fh) + ih;
+    const CarryD cx = carry_load(A.carry + 5ll * c);
+    ig = cx.g + ig;
+    ih = cx.h + ih;
     icn = cx.c + icn;
   }
   // candidate: the end of a run of equal values (or of the segment), both directions when the
@@ -1179,8 +1206,8 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
         else { g[k] = 0.0; h[k] = 0.0; }
       }
     }
-    const FXV cx = fxv_load(A.carry + 5ll * c);
-    const SVf carry = SVf{from_fx(cx.g, Fg), from_fx(cx.h, Fh), cx.c, 0};
+    const CarryD cx = carry_load(A.carry + 5ll * c);
+    const SVf carry = SVf{cx.g, cx.h, cx.c, 0};
     int sj[kItems];
     unsigned hm, pem, rem;
     assign_segments<!kTotals>(ss, sc, cp1, K, base, vm, v, vnext, sj, hm, pem, rem);
@@ -2000,10 +2027,10 @@ void launch_gen(const SplitArgs& A, unsigned grid, cudaStream_t st) {
 
 template <bool kFx>
 void launch_scan(const int32_t* Cp, unsigned long long* in, unsigned long long* gbuf, unsigned long long* out,
-                 unsigned groups, cudaStream_t st) {
+                 unsigned groups, cudaStream_t st, const int32_t* fx = nullptr) {
   k_scan1<kFx><<<groups, kThreads, 0, st>>>(Cp, in, gbuf);
   k_scan2<kFx><<<1, kScan2Threads, 0, st>>>(Cp, gbuf);
-  k_scan3<kFx><<<groups, kThreads, 0, st>>>(Cp, in, gbuf, out);
+  k_scan3<kFx><<<groups, kThreads, 0, st>>>(Cp, in, gbuf, out, fx);
   GBDT_LAUNCH_CHECK();
   count_launch(3);
 }
@@ -2012,14 +2039,13 @@ void launch_scan(const int32_t* Cp, unsigned long long* in, unsigned long long* 
 // segment's last entry, plus the exact carry of that chunk when the segment began before it.
 __global__ void __launch_bounds__(kThreads) k_seg_totals(SplitArgs A) {
   const long long S = (long long)A.t.m * *A.t.Kp;
-  const int Fg = A.fx[0], Fh = A.fx[1];
   for (long long s = blockIdx.x * (long long)blockDim.x + threadIdx.x; s < S; s += (long long)gridDim.x * blockDim.x) {
     if (A.t.tb.seg_cnt[s] == 0) continue;
     const int ce = A.segEnd[s];
     if (ce < 0) continue;
-    const FXV cx = fxv_load(A.carry + 5ll * ce);
-    A.segPG_out[s] = from_fx(cx.g, Fg) + A.segPG_out[s];
-    A.segPH_out[s] = from_fx(cx.h, Fh) + A.segPH_out[s];
+    const CarryD cx = carry_load(A.carry + 5ll * ce);
+    A.segPG_out[s] = cx.g + A.segPG_out[s];
+    A.segPH_out[s] = cx.h + A.segPH_out[s];
   }
 }
 
@@ -2066,7 +2092,7 @@ void LevelKernels::tile_prefix(const SplitArgs& A, int hmode, bool gather, unsig
   }
   GBDT_LAUNCH_CHECK();
   count_launch();
-  launch_scan<true>(A.t.tb.C, A.cagg, A.sgrp, A.carry, groups, st);
+  launch_scan<true>(A.t.tb.C, A.cagg, A.sgrp, A.carry, groups, st, A.fx);
   if (A.segEnd) {
     k_seg_totals<<<(unsigned)(sms * 4), kThreads, 0, st>>>(A);
     GBDT_LAUNCH_CHECK();
@@ -2150,7 +2176,7 @@ void LevelKernels::chunk_desc(const SplitArgs& A, unsigned groups, cudaStream_t 
   k_desc<<<(unsigned)(sms * 8), kThreads, 0, st>>>(A);
   GBDT_LAUNCH_CHECK();
   count_launch();
-  launch_scan<true>(A.t.tb.C, A.cagg, A.sgrp, A.carry, groups, st);
+  launch_scan<true>(A.t.tb.C, A.cagg, A.sgrp, A.carry, groups, st, A.fx);
 }
 
 }  // namespace gbdt
