@@ -772,6 +772,7 @@ struct __align__(16) FastWarp {
   unsigned long long carry[kFS][6];
   ChunkDesc d[4];
   unsigned long long bar[kFS];
+  unsigned rend[kChunk / 32];  // RLE: bit p - p0 set iff entry p is the last entry of its run
 };
 template <bool kH>
 struct FastSmem {
@@ -854,9 +855,24 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
       __syncwarp();
       lds_blocked8(W.g[st], lane, g);
       if (kH) lds_blocked8(W.h[st], lane, hk);
+      unsigned rmask = 0;  // RLE: the lane's items that end a run (the runs are the candidates)
+      int rb = 0, re = 0;
       if (kRLE) {
-        // rle_values also fills v[len - q0] (< kItems) or vn with the value after the chunk
-        if (q0 < len) rle_values(A.t.tb, chunk(i), p0, len, (jf & kDescNext) != 0, p0 + q0, K, d.a * K + K, v, vn);
+        // the runs touching the chunk (one per lane, usually one or two in all): each marks its
+        // last entry, so no value is decompressed per entry
+        const int cg = chunk(i);
+        rb = A.t.tb.run_chunk[cg];
+        re = (jf & kDescNext) ? A.t.tb.run_chunk[cg + 1] : A.t.tb.seg_run[d.a * K + K] - 1;
+        if (lane < kChunk / 32) W.rend[lane] = 0u;
+        __syncwarp();
+        for (int r = rb + lane; r <= re; r += 32) {
+          const long long e = A.t.tb.run_pos[r] + A.t.tb.run_len[r] - 1 - p0;
+          if (e >= 0 && e < len) atomicOr(&W.rend[e >> 5], 1u << (e & 31));
+        }
+        __syncwarp();
+        rmask = (W.rend[lane >> 2] >> ((lane & 3) * 8)) & 0xffu;
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) v[k] = 0.f;
       } else {
         lds_blocked8f(sv, lane, v);
         vn = __shfl_down_sync(0xffffffffu, v[0], 1);
@@ -902,7 +918,7 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
 #pragma unroll
       for (int k = 0; k < kItems; ++k) {
         const float nx = k < kItems - 1 ? v[k + 1] : vn;
-        if (k < nc && nx != v[k]) cm |= 1u << k;
+        if (k < nc && (kRLE ? ((rmask >> k) & 1u) != 0u : nx != v[k])) cm |= 1u << k;
       }
       double pg = bg, phh = bh, bnum = -1.0, bden = 1.0;
       int bk = -1;
@@ -951,7 +967,12 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
 #pragma unroll
         for (int k = 0; k < kItems; ++k) {
           if (k <= bk) { xg = xg + g[k]; xh = xh + hk[k]; }
-          if (k == bk) xv = v[k];
+          if (!kRLE && k == bk) xv = v[k];
+        }
+        if (kRLE) {  // the winner ends a run of this chunk: that run's value
+          const long long pw = p0 + q0 + bk;
+          for (int r2 = rb; r2 <= re; ++r2)
+            if (A.t.tb.run_pos[r2] + A.t.tb.run_len[r2] - 1 == pw) { xv = A.t.tb.run_val[r2]; break; }
         }
         Rec r;
         r.GL = xg;
