@@ -80,6 +80,8 @@ struct PartArgs {
   double* h_out;
   const int32_t* epochp;
   const uint8_t* side;    // per instance: 0 drop, 1 high, 2 low
+  const uint32_t* hbit;   // per instance: bit = [side == 1] (dense count, chunks inside one segment)
+  const int32_t* cidx;    // [K] next-level index of node j's high child, -1 if j became a leaf
   uint8_t* slist;         // per list entry: side of its instance (k_part_count -> k_part_scatter)
   int32_t* segH;          // [m*K] counted (missing values) or derived from node counts (dense)
   int32_t* segL;

@@ -1480,6 +1480,11 @@ __device__ __forceinline__ uint8_t ld_keep_u8(const uint8_t* p, unsigned long lo
   asm volatile("ld.global.nc.L2::cache_hint.u8 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol));
   return (uint8_t)v;
 }
+__device__ __forceinline__ unsigned ld_keep_u32(const uint32_t* p, unsigned long long pol) {
+  unsigned v;
+  asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+  return v;
+}
 __global__ void __launch_bounds__(kThreads) k_part_count_dense(PartArgs A) {
   __shared__ TabCache tc;
   const int lane = threadIdx.x & 31;
@@ -1492,7 +1497,7 @@ __global__ void __launch_bounds__(kThreads) k_part_count_dense(PartArgs A) {
   const int nw = (gridDim.x * blockDim.x) >> 5;
   for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += 2 * nw) {
     long long p0[2];
-    int len[2], rs[2], id[2][kItems];
+    int len[2], rs[2], id[2][kItems], mode[2];
     uint8_t sd[2][kItems];
 #pragma unroll
     for (int u = 0; u < 2; ++u) {
@@ -1500,20 +1505,33 @@ __global__ void __launch_bounds__(kThreads) k_part_count_dense(PartArgs A) {
       len[u] = 0;
       p0[u] = 0;
       rs[u] = 0;
+      mode[u] = 0;
       if (cu < C) {
         const ChunkMeta M = chunk_meta(tc, A.t, K, cu);
         p0[u] = M.p0;
         len[u] = (int)(M.p1 - M.p0);
         rs[u] = M.reset;
+        // a chunk inside one segment: nothing to gather if its node became a leaf, else one bit
+        // per entry from the 1.4 MB high-child bitmap; a chunk crossing segments: side bytes
+        const SegOf sg = warp_seg((const long long*)(A.t.tb.seg_start + M.sb),
+                                  (const long long*)(A.t.tb.seg_cnt + M.sb), K, M.p0, lane);
+        mode[u] = M.p1 <= sg.se ? (A.cidx[sg.j] < 0 ? 0 : 1) : 2;
       }
       const int32_t* ip = A.t.ins + p0[u] + lane;
 #pragma unroll
-      for (int k = 0; k < kItems; ++k) id[u][k] = (32 * k + lane < len[u]) ? __ldcs(ip + 32 * k) : -1;
+      for (int k = 0; k < kItems; ++k) id[u][k] = (32 * k + lane < len[u] && mode[u]) ? __ldcs(ip + 32 * k) : -1;
     }
 #pragma unroll
     for (int u = 0; u < 2; ++u)
 #pragma unroll
-      for (int k = 0; k < kItems; ++k) sd[u][k] = id[u][k] >= 0 ? ld_keep_u8(A.side + id[u][k], keep) : (uint8_t)0;
+      for (int k = 0; k < kItems; ++k) {
+        uint8_t x = 0;
+        if (id[u][k] >= 0) {
+          if (mode[u] == 1) x = ((ld_keep_u32(A.hbit + (id[u][k] >> 5), keep) >> (id[u][k] & 31)) & 1u) ? 1 : 2;
+          else x = ld_keep_u8(A.side + id[u][k], keep);
+        }
+        sd[u][k] = x;
+      }
 #pragma unroll
     for (int u = 0; u < 2; ++u) {
       const int cu = c + u * nw;
