@@ -142,6 +142,16 @@ def _rows(prob, n_s):
                          prob.indices[:e], prob.values[:e], prob.labels[:n_s], prob.params)
 
 
+def arm_config(args, prob, P, d, world):
+    """The `config` object of the JSON line; identical for both arms."""
+    return {"workload": args.config, "n": prob.n, "m": prob.m, "nnz": prob.nnz, "loss": P["loss"],
+            "max_depth": d, "trees_timed": args.steps, "lambda": P["lam"], "eta": P["eta"],
+            "rle": args.rle, "smartgd": args.smartgd, "parallelism": f"attr-shard{world}",
+            "l2": ("inputs larger than L2 (sorted lists %.2f GB)" % (prob.nnz * 8 / 1e9)) if prob.nnz * 8 > 126e6
+                  else "inputs smaller than L2 (%.1f MB), not flushed between trees: latency-bound config"
+                  % (prob.nnz * 8 / 1e6)}
+
+
 def main():
     args = parse()
     rank = int(os.environ.get("RANK", "0"))
@@ -163,8 +173,7 @@ def main():
             "impl": "reference", "metric": METRIC, "value": rate, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": rate * 1e3, "higher_is_better": False,
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": args.config, "n": prob.n, "m": prob.m, "nnz": prob.nnz, "loss": P["loss"],
-                       "max_depth": P["max_depth"], "n_trees": P["n_trees"]},
+            "config": arm_config(args, prob, P, args.depth or P["max_depth"], world),
             "cpu_baseline": {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
                              "sample": f"first {info['n_rows']} rows ({info['entries']} entries), "
                                        f"{info['trees']} trees, presort excluded, scaled x{info['scale']:.1f} by entries"},
@@ -304,10 +313,7 @@ def main():
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": False,
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": args.config, "n": prob.n, "m": prob.m, "nnz": prob.nnz, "loss": P["loss"],
-                       "max_depth": d, "trees_timed": args.steps, "lambda": P["lam"], "eta": P["eta"],
-                       "rle": args.rle, "smartgd": args.smartgd, "parallelism": f"attr-shard{world}",
-                       "l2": "inputs larger than L2 (sorted lists %.2f GB)" % (prob.nnz * 8 / 1e9)},
+            "config": arm_config(args, prob, P, d, world),
             "roofline": {"bound": "hbm", "achieved": kern[dom]["achieved"], "peak": peak, "unit": "GB/s",
                          "frac": kern[dom]["frac"], "traffic": kern[dom]["traffic"], "kernel": dom,
                          "peak_kind": peak_kind, "bytes_per_launch": kern[dom]["bytes"] / kern[dom]["launches"],
