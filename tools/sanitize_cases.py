@@ -1,0 +1,21 @@
+"""Small trainings covering every kernel family (dense, missing values, sparse short lists, RLE,
+loopback shards, deep trees, SmartGD-off, prediction), for compute-sanitizer runs."""
+import sys
+
+sys.path.insert(0, ".")
+from datagen import synth  # noqa: E402
+from paper_conf_ipps_wenhkls18_b200 import gbdt  # noqa: E402
+
+cases = [
+    ("C1", synth.c1(n=3000), {}),
+    ("missing", synth.random_small(5, n=3000, m=6, nan_frac=0.3, n_distinct=40, loss="logistic", d=5, T=2), {}),
+    ("sparse", synth.c4(seed=9, n=1500, m=4000, density=0.01, T=2), {}),
+    ("rle", synth.c5(n=20000, T=2), {"rle": "on"}),
+    ("shards", synth.c1(n=2000), {"n_shards": 4}),
+    ("deep", synth.random_small(77, n=6000, m=6, nan_frac=0.0, n_distinct=400, loss="logistic", d=8, T=2), {}),
+    ("smartgd_off", synth.c1(n=1000), {"smartgd": False}),
+]
+for name, p, kw in cases:
+    model, margin = gbdt.train_problem(p, **kw)
+    model.predict(p.indptr, p.indices, p.values, p.m)
+    print(name, "ok", flush=True)
