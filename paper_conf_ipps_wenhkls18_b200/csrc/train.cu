@@ -742,7 +742,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         count_launch(2);
       }
       tm.end();
-      if (ds.comm && ds.comm->world > 1) {
+      if (ds.comm) {  // every rank (a world of 1 too: the same calls, trivially)
         tm.begin(GBDT_PHASE_COMM);
         Rec* mine = best_all + (size_t)ds.shards[0]->index * Kcap;
         ds.comm->allgather(mine, best_all, sizeof(Rec) * Kcap, st);
@@ -771,7 +771,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         count_launch();
       }
       tm.end();
-      if (ds.comm && ds.comm->world > 1) {
+      if (ds.comm) {
         tm.begin(GBDT_PHASE_COMM);
         ds.comm->allreduce_sum_u8(bits, (size_t)n, st);
         tm.end();
@@ -838,11 +838,11 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     count_launch();
   };
 
-  // NCCL collectives inside the captured tree are supported by NCCL but not exercised on the
-  // single-GPU boxes this was built on: with a multi-rank communicator the graph is opt-in
-  // (GBDT_GRAPH=1); GBDT_GRAPH=0 forces eager launches everywhere
+  // NCCL collectives inside the captured tree are exercised here only with a world of one rank
+  // (single-GPU boxes): with a multi-rank communicator the graph is opt-in (GBDT_GRAPH=1);
+  // GBDT_GRAPH=0 forces eager launches everywhere.  Host-staged collectives cannot be captured.
   const bool multi = ds.comm && ds.comm->world > 1;
-  const bool host_comm = multi && !ds.comm->nccl;
+  const bool host_comm = ds.comm && !ds.comm->nccl;
   const char* ge = getenv("GBDT_GRAPH");
   const bool graph_ok = ge ? ge[0] != '0' : !multi;
   const bool graph = !tm.on && !custom && !host_comm && P.n_trees > 1 && graph_ok;

@@ -67,3 +67,23 @@ def test_ranks_reproduce_single_process(tmp_path, name, world):
     margin = np.load(path + ".margin.npy")
     assert np.array_equal(nodes, ref_model.nodes().view(np.uint8))
     assert np.array_equal(margin, ref_margin)
+
+
+@pytest.mark.parametrize("graph", ["0", "1"])
+def test_nccl_world_of_one_runs_the_collectives(graph, monkeypatch):
+    """The NCCL path on one GPU: a world of one rank makes the same ncclAllGather / ncclAllReduce
+    calls per level (eager, or captured into the per-tree CUDA graph) and must reproduce the
+    communicator-free model bit for bit."""
+    import numpy as np
+    from datagen import synth
+    from paper_conf_ipps_wenhkls18_b200 import gbdt
+    monkeypatch.setenv("GBDT_GRAPH", graph)
+    p = synth.c1(n=3000)
+    m0, y0 = gbdt.train_problem(p)
+    comm = gbdt.comm_init(0, 1, gbdt.comm_unique_id(), 0)
+    ds = gbdt.load_csr(p.indptr, p.indices, p.values, p.labels, p.m, comm=comm)
+    P = dict(p.params)
+    m1, y1 = gbdt.train(ds, **P)
+    assert m0.nodes().tobytes() == m1.nodes().tobytes()
+    assert np.array_equal(y0, y1)
+    del ds
