@@ -160,11 +160,12 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
   if (out) *out = nullptr;
   return guarded([&] {
     if (!out) fail(GBDT_E_INVAL, "out is NULL");
-    validate_csr(n_rows, n_cols, indptr, indices, values, true);
-    if (!labels) fail(GBDT_E_INVAL, "labels is NULL");
     float lmin = std::numeric_limits<float>::infinity(), lmax = -lmin;
     bool binary = true;
-    {
+    // the full O(nnz) checks: run on the host cores while the H2D copies are in flight
+    auto validate_all = [&] {
+      validate_csr(n_rows, n_cols, indptr, indices, values, true);
+      if (!labels) fail(GBDT_E_INVAL, "labels is NULL");
       struct LabelStats { float lo, hi; bool bin; int64_t bad; };
       std::vector<LabelStats> ls(64, LabelStats{lmin, lmax, true, INT64_MAX});
       parallel_ranges(n_rows, 1 << 16, [&](int64_t lo, int64_t hi, int t) {
@@ -185,17 +186,31 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
         lmax = std::max(lmax, L.hi);
       }
       if (bad != INT64_MAX) fail(GBDT_E_INVAL, "labels must be finite (row " + std::to_string(bad) + ")");
-    }
+    };
+    // O(1) checks needed before anything is copied
+    const int64_t kMax = (int64_t(1) << 31) - 1;
+    if (n_rows < 1 || n_rows >= kMax) fail(GBDT_E_INVAL, "n_rows must be in [1, 2^31-1)");
+    if (n_cols < 1 || n_cols >= kMax) fail(GBDT_E_INVAL, "n_cols must be in [1, 2^31-1)");
+    if (!indptr) fail(GBDT_E_INVAL, "indptr is NULL");
+    if (indptr[0] != 0) fail(GBDT_E_INVAL, "indptr[0] must be 0");
     gbdt_load_opts o;
     std::memset(&o, 0, sizeof o);
     if (opts) o = *opts;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < 1) {
+      validate_all();  // argument errors are reported before the missing device
+      fail(GBDT_E_CUDA, "no CUDA device visible");
+    }
+    if (indptr[n_rows] < 0 || indptr[n_rows] >= kMax || !labels ||
+        (indptr[n_rows] > 0 && (!indices || !values))) {
+      validate_all();  // reports the precise error
+      fail(GBDT_E_INVAL, "malformed CSR");
+    }
     if (o.rle < 0 || o.rle > 2) fail(GBDT_E_INVAL, "rle must be OFF, ON or AUTO");
     int nsh = o.n_shards <= 0 ? 1 : o.n_shards;
     if (nsh != 1 && nsh != 2 && nsh != 4 && nsh != 8) fail(GBDT_E_RANGE, "n_shards must be 1, 2, 4 or 8");
     Comm* comm = o.comm ? o.comm->c : nullptr;
     if (comm && nsh != 1) fail(GBDT_E_RANGE, "n_shards must be 1 with a communicator");
-    int ndev = 0;
-    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < 1) fail(GBDT_E_CUDA, "no CUDA device visible");
     int dev = o.device;
     if (dev < 0) GBDT_CUDA(cudaGetDevice(&dev));
     if (dev >= ndev) fail(GBDT_E_RANGE, "device ordinal out of range");
@@ -224,6 +239,12 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
       }
       ds.y.alloc((size_t)n_rows * 4, st);
       GBDT_CUDA(cudaMemcpyAsync(ds.y.p, labels, (size_t)n_rows * 4, cudaMemcpyHostToDevice, st));
+      try {
+        validate_all();  // overlaps the copies (from pinned host memory they run asynchronously)
+      } catch (...) {
+        cudaStreamSynchronize(st);  // the copies still read the caller's buffers
+        throw;
+      }
       // present entries per attribute, counted on the device
       const std::vector<int64_t> col_counts = column_counts(nnz, n_cols, didx.as<int32_t>(), dval.as<float>(), st);
       bool missing = false;
