@@ -319,3 +319,13 @@ def test_deep_trees_more_than_32_nodes_per_level(maker):
         p.params["max_depth"] = 8
     model, margin = _train(p)
     compare(p, model.nodes(), margin, params=p.params)
+
+
+def test_deep_trees_rle_bit_identical():
+    """RLE run tables with more than 32 nodes per level (depth 8) equal the plain path."""
+    p = synth.random_small(79, n=8000, m=5, nan_frac=0.1, n_distinct=20, loss="logistic", d=8, T=2)
+    ref_model, ref_margin = _train(p)
+    model, margin = _train(p, rle="on")
+    assert np.array_equal(model.nodes().view(np.uint8), ref_model.nodes().view(np.uint8))
+    assert np.array_equal(margin, ref_margin)
+    compare(p, model.nodes(), margin)
