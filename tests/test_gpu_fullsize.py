@@ -86,3 +86,19 @@ def test_full_size_c5_rle_on_equals_off():
     b, mb = _run(prob, T=1, rle="on")
     assert np.array_equal(a.nodes().view(np.uint8), b.nodes().view(np.uint8))
     assert np.array_equal(ma, mb)
+
+
+def test_full_size_c3_forty_trees_as_benched():
+    """C3 at its full size and the bench's configuration (40 trees in one gbdt_train, one CUDA
+    graph per tree): every tree satisfies the structural invariants, the first tree equals the
+    one a 1-tree run builds, and prediction by traversal reproduces the SmartGD margin."""
+    prob = synth.make("C3")
+    model, margin = _run(prob, T=40)
+    nodes = model.nodes()
+    P = prob.params
+    structural_invariants(nodes, prob.n, P["max_depth"], P["lam"], P["gamma"])
+    one, _ = _run(prob, T=1)
+    assert nodes[0].tobytes() == one.nodes()[0].tobytes()
+    pred = gbdt.predict(model, prob.indptr, prob.indices, prob.values, prob.m)
+    assert np.array_equal(pred, margin)
+    assert np.isfinite(margin).all()
