@@ -142,6 +142,7 @@ struct LevelKernels {
   int sms = 148;
   unsigned grid_fast[3][2] = {{0}};  // [hmode][rle]
   unsigned grid_gen = 0;
+  unsigned grid_short = 0;
   unsigned grid_agg[3] = {0};
   unsigned grid_scatter[3][2] = {{0}}, grid_count = 0, grid_count_dense = 0, grid_agg_list[3] = {0};  // scatter: [hmode][agg]
   void init(int device);

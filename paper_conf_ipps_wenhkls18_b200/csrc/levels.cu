@@ -282,6 +282,117 @@ __device__ __forceinline__ SegOf warp_seg(const long long* ss, const long long* 
 }
 
 // ============================================================================ a4: chunk aggregates
+#ifndef GBDT_AGG_SHORT
+#define GBDT_AGG_SHORT 1
+#endif
+// Short chunk (<= 32 entries, K <= 32: the typical sparse list): lane i holds entry
+// p0 + i, the segment structure comes from the attribute's segment table held one segment per
+// lane (as in sf_short), and the segmented sums run over the lanes instead of the 8-items-per-lane
+// layout, whose loops and scans a 20-entry list pays in full.  Same outputs as the general path:
+// descriptor, exact chunk aggregate, g-list at the root, present totals of the ending segments.
+template <int HMODE, bool kGather>
+__device__ __forceinline__ void agg_short(const SplitArgs& A, const ChunkMeta& M, int c, int K, int lane, int Fg,
+                                          int Fh, unsigned long long pol_keep, float vnx) {
+  const long long p0 = M.p0;
+  const int len = (int)(M.p1 - p0);
+  const bool valid = lane < len;
+  const long long p = p0 + lane;
+  double g = 0.0, h = 0.0;
+  if (valid) {
+    if (kGather) {
+      const int id = __ldcs(A.t.ins + p);
+      g = ld_keep(A.g + id, pol_keep);
+      h = HMODE == kHGather ? ld_keep(A.h + id, pol_keep) : hess_of<HMODE>(g);
+      __stcs(A.glist + p, g);
+      if (HMODE == kHGather) __stcs(A.hlist + p, h);
+    } else {
+      g = __ldcs(A.glist + p);
+      h = HMODE == kHGather ? __ldcs(A.hlist + p) : hess_of<HMODE>(g);
+    }
+  }
+  const long long* ss = (const long long*)(A.t.tb.seg_start + M.sb);
+  const long long* sc = (const long long*)(A.t.tb.seg_cnt + M.sb);
+  const long long s_l = lane < K ? ss[lane] : LLONG_MAX;
+  const long long c_l = lane < K ? sc[lane] : 0;
+  // segment of the chunk's first entry: the largest j with ss[j] <= p0 (warp_seg's choice)
+  const unsigned le0 = __ballot_sync(0xffffffffu, s_l <= p0);
+  const int j0 = 31 - __clz(le0 | 1u);
+  const long long s0 = __shfl_sync(0xffffffffu, s_l, j0);
+  const long long se0 = s0 + __shfl_sync(0xffffffffu, c_l, j0);
+  const int head0 = s0 == p0 ? 1 : 0;
+  if (M.p1 <= se0) {  // one segment: the aggregate is the whole chunk
+    double lg = g, lh = h;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+      lg = lg + __shfl_xor_sync(0xffffffffu, lg, o);
+      lh = lh + __shfl_xor_sync(0xffffffffu, lh, o);
+    }
+    if (lane == 0) {
+      ChunkDesc d;
+      d.p0 = p0;
+      d.se = se0;
+      d.len = len;
+      d.a = M.a;
+      d.jf = j0 | (head0 ? kDescHead0 : 0) | kDescSingle | (M.more ? kDescNext : 0);
+      d.vnext = vnx;
+      A.desc[c] = d;
+      fxv_store(A.cagg + 5ll * c, FXV{to_fx(lg, Fg), to_fx(lh, Fh), len, head0}, M.reset);
+      if (A.segEnd && M.p1 == se0) {
+        const long long s = M.sb + j0;
+        A.segPG_out[s] = lg;
+        A.segPH_out[s] = lh;
+        A.segEnd[s] = head0 ? -1 : c;
+      }
+    }
+    return;
+  }
+  if (lane == 0) {  // the chunk crosses a segment boundary: k_sf_gen's
+    ChunkDesc d;
+    d.p0 = p0;
+    d.se = se0;
+    d.len = len;
+    d.a = M.a;
+    d.jf = j0 | (head0 ? kDescHead0 : 0) | (M.more ? kDescNext : 0);
+    d.vnext = vnx;
+    A.desc[c] = d;
+    A.genlist[atomicAdd(A.ngen, 1)] = c;
+  }
+  // heads inside the chunk (first entries of non-empty segments) and the lane's segment piece
+  const bool starts = lane < K && c_l > 0 && s_l >= p0 && s_l < p0 + len;
+  const unsigned hm = __reduce_or_sync(0xffffffffu, starts ? (1u << (int)(s_l - p0)) : 0u);
+  const unsigned upto = hm & (0xffffffffu >> (31 - lane));
+  const int hpos = upto ? 31 - __clz(upto) : -1;  // last head at or before the lane
+  const int sl = hpos >= 0 ? hpos : 0;
+  double ig = g, ih = h;
+  int icn = valid ? 1 : 0;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const double yg = __shfl_up_sync(0xffffffffu, ig, o), yh = __shfl_up_sync(0xffffffffu, ih, o);
+    const int yc = __shfl_up_sync(0xffffffffu, icn, o);
+    if (lane - o >= sl) { ig = yg + ig; ih = yh + ih; icn += yc; }
+  }
+  // lanes past the end hold zeros in the last piece: lane 31 has the aggregate since the last head
+  if (lane == 31) fxv_store(A.cagg + 5ll * c, FXV{to_fx(ig, Fg), to_fx(ih, Fh), icn, hm != 0u}, M.reset);
+  if (A.segEnd) {
+    // the lane's segment: the owner of the head at hpos (unique: heads are non-empty segments)
+    int j = j0;
+    unsigned o = __ballot_sync(0xffffffffu, starts);
+    while (o) {
+      const int l = __ffs(o) - 1;
+      o &= o - 1;
+      const long long sll = __shfl_sync(0xffffffffu, s_l, l);
+      if (hpos >= 0 && sll - p0 == hpos) j = l;
+    }
+    const long long se = __shfl_sync(0xffffffffu, s_l, j & 31) + __shfl_sync(0xffffffffu, c_l, j & 31);
+    if (valid && p + 1 == se) {  // present totals of the segments ending here (see k_seg_totals)
+      const long long s = M.sb + j;
+      A.segPG_out[s] = ig;
+      A.segPH_out[s] = ih;
+      A.segEnd[s] = hpos >= 0 ? -1 : c;
+    }
+  }
+}
+
 // One warp per chunk: g (h) of its entries -- gathered at the root (L2 evict-last) and laid out as
 // the chunk's g-list, read from the partition-carried g-list below -- and the chunk's segmented
 // aggregate (sum since its last segment head, fixed association) as an exact fixed-point value.
@@ -308,6 +419,12 @@ __global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
     }
     // value after the chunk (same attribute), for the descriptor; loaded early
     const float vnx = (lane == 0 && M.more && !A.rle) ? __ldg(A.t.val + p1) : 0.f;
+#if GBDT_AGG_SHORT
+    if (p1 - M.p0 <= 32 && K <= 32) {
+      agg_short<HMODE, kGather>(A, M, c, K, lane, Fg, Fh, pol_keep, vnx);
+      continue;
+    }
+#endif
     unsigned vm = 0;
     double g[kItems], h[kItems];
 #pragma unroll
@@ -1153,6 +1270,65 @@ __device__ __forceinline__ void sf_short(const SplitArgs& A, NodeBest& B, unsign
   __syncwarp();
 }
 
+// ---------------------------------------------------------------------------- k_sf_short
+// The short chunks of k_sf_gen's chunk set in a kernel of their own.  In the general kernel the
+// ~6 k-instruction body stalled on instruction fetch ("no_instructions") a third of the time on
+// C4a, whose ~1.35 M lists per level are nearly all short, at 2 CTAs per SM (128 registers); here
+// the loop runs from sf_short's small footprint at the occupancy its registers allow.
+#ifndef GBDT_SF_SHORT_KERNEL
+#define GBDT_SF_SHORT_KERNEL 1
+#endif
+template <int HMODE, bool kMissing, bool kRLE>
+__global__ void __launch_bounds__(kThreads) k_sf_short(SplitArgs A) {
+  __shared__ NodeBest B;
+  __shared__ unsigned long long wgk[kWarps][kWarpK];
+  __shared__ Rec wrec[kWarps][kWarpK];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int K = *A.t.Kp;
+  const int C = *A.t.tb.C;
+  if (K == 0 || C == 0 || K > kWarpK) return;
+  const int epoch = *A.epochp;
+  const int Fg = A.fx[0], Fh = A.fx[1];
+  nb_init(B, A, K);
+  for (int j = threadIdx.x; j < kWarps * kWarpK; j += blockDim.x) wgk[j / kWarpK][j % kWarpK] = 0ull;
+  __syncthreads();
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  const int n = kMissing ? C : *A.ngen;  // k_sf_gen's chunk set
+  // 32 chunks per warp step, lane l testing chunk bt + l * nbat (strided, so the chunks of one long
+  // list spread over the warps); the warp then runs the short ones
+  // (only when the chunks outnumber the warps 32 to 1: a short list of heavy chunks, e.g. the
+  // segment-crossing chunks of dense data, stays one chunk per warp)
+  const int bw = n >= 32 * nw ? 32 : 1;
+  const int nbat = (n + bw - 1) / bw;
+  for (int bt = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; bt < nbat; bt += nw) {
+    const int ii = bt + lane * nbat;
+    int cc = 0;
+    bool take = false;
+    if (lane < bw && ii < n) {
+      cc = kMissing ? ii : A.genlist[ii];
+      take = A.desc[cc].len <= 32;
+    }
+    unsigned todo = __ballot_sync(0xffffffffu, take);
+    while (todo) {
+      const int c = __shfl_sync(0xffffffffu, cc, __ffs(todo) - 1);
+      todo &= todo - 1;
+      const ChunkDesc d = A.desc[c];
+      sf_short<HMODE, kMissing, kRLE>(A, B, wgk[wid], wrec[wid], c, d, K, lane, epoch, Fg, Fh, A.lam);
+    }
+  }
+  __syncthreads();  // merge the warp tables, one record per node and CTA
+  for (int j = threadIdx.x; j < K; j += blockDim.x) {
+    int bw = -1;
+    for (int w = 0; w < kWarps; ++w)
+      if (wgk[w][j] && (bw < 0 || rec_better(wgk[w][j], wrec[w][j], wgk[bw][j], wrec[bw][j]))) bw = w;
+    if (bw >= 0) {
+      const int gs = atomicAdd(A.nrec, 1);
+      A.rec[gs] = wrec[bw][j];
+      atomicMax(A.gkey + j, wgk[bw][j]);
+    }
+  }
+}
+
 // ---------------------------------------------------------------------------- k_sf_gen
 template <int HMODE, bool kMissing, bool kTotals, bool kRLE>
 __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
@@ -1178,15 +1354,33 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
   // with missing values every chunk; else the chunks k_chunk_agg listed (they cross segments)
   constexpr bool kAll = kMissing || kTotals;
   const int n = kAll ? C : *A.ngen;
-  for (int i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < n; i += nw) {
-    const int c = kAll ? i : A.genlist[i];
+  // 32 chunks per warp step (lane l tests chunk bt + l * nbat); the short ones are k_sf_short's,
+  // so they cost one descriptor word here instead of a dependent descriptor load each
+  // (only when the chunks outnumber the warps 32 to 1: a short list of heavy chunks, e.g. the
+  // segment-crossing chunks of dense data, stays one chunk per warp)
+  const int bw = n >= 32 * nw ? 32 : 1;
+  const int nbat = (n + bw - 1) / bw;
+  for (int bt = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; bt < nbat; bt += nw) {
+    const int ii = bt + lane * nbat;
+    int cc = 0;
+    bool take = false;
+    if (lane < bw && ii < n) {
+      cc = kAll ? ii : A.genlist[ii];
+      take = kTotals || !GBDT_SF_SHORT_KERNEL || !(A.desc[cc].len <= 32 && K <= kWarpK);
+    }
+    unsigned todo = __ballot_sync(0xffffffffu, take);
+    while (todo) {
+    const int c = __shfl_sync(0xffffffffu, cc, __ffs(todo) - 1);
+    todo &= todo - 1;
     const ChunkDesc d = A.desc[c];
     const long long p0 = d.p0;
     const long long cp1 = p0 + d.len;
     const long long sb = (long long)d.a * K;
     if (!kTotals && d.len <= 32 && K <= kWarpK) {  // short chunk (sparse lists): one entry per lane
+#if !GBDT_SF_SHORT_KERNEL
       sf_short<HMODE, kMissing, kRLE>(A, B, wgk[wid], wrec[wid], c, d, K, lane, epoch, Fg, Fh, lam);
-      continue;
+#endif
+      continue;  // else k_sf_short's
     }
     const long long base = p0 + lane * kItems;
     const long long* ss = (const long long*)(A.t.tb.seg_start + sb);
@@ -1372,6 +1566,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
       }
     }
     __syncwarp();
+    }
   }
   if (!kTotals && K <= kWarpK) {  // merge the warp tables, one record per node and CTA
     __syncthreads();
@@ -1391,6 +1586,60 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
 // ============================================================================ a8: partition
 // One warp per chunk: (high, low) entry counts (packed hi | lo << 32) + reset flag; with missing
 // values also the per-segment counts (the plan needs them).
+// Short chunk of k_part_count (<= 32 entries, K <= 32, per-segment counts wanted): lane i on
+// entry p0 + i, side counts by ballots over the lanes, one atomic pair per segment piece (the
+// piece's last lane), the side-list written in the same 4-entry words.  The ids were streamed into
+// L1/L2 by the warp's prefetch, so the reload here hits.
+__device__ __forceinline__ void count_short(const PartArgs& A, const ChunkMeta& M, int c, int K, int lane) {
+  const long long p0 = M.p0;
+  const int len = (int)(M.p1 - p0);
+  const bool valid = lane < len;
+  const long long p = p0 + lane;
+  unsigned sd = 0;
+  if (valid) sd = __ldg(A.side + __ldg(A.t.ins + p));
+  const unsigned bh = __ballot_sync(0xffffffffu, sd == 1), bl = __ballot_sync(0xffffffffu, sd == 2);
+  // side-list words: lane 4q packs lanes 4q .. 4q+3 (invalid lanes hold 0, as in the general path)
+  unsigned w = sd;
+  w |= __shfl_down_sync(0xffffffffu, sd, 1) << 8;
+  w |= __shfl_down_sync(0xffffffffu, sd, 2) << 16;
+  w |= __shfl_down_sync(0xffffffffu, sd, 3) << 24;
+  if ((lane & 3) == 0 && valid) reinterpret_cast<unsigned*>(A.slist + p)[0] = w;
+  // segment pieces (as in sf_short): heads from the attribute's segment table, one segment per lane
+  const long long* ss = (const long long*)(A.t.tb.seg_start + M.sb);
+  const long long* sc = (const long long*)(A.t.tb.seg_cnt + M.sb);
+  const long long s_l = lane < K ? ss[lane] : LLONG_MAX;
+  const long long c_l = lane < K ? sc[lane] : 0;
+  const unsigned le0 = __ballot_sync(0xffffffffu, s_l <= p0);
+  const int j0 = 31 - __clz(le0 | 1u);
+  const bool starts = lane < K && c_l > 0 && s_l >= p0 && s_l < p0 + len;
+  const unsigned hm = __reduce_or_sync(0xffffffffu, starts ? (1u << (int)(s_l - p0)) : 0u);
+  const unsigned upto = hm & (0xffffffffu >> (31 - lane));
+  const int hpos = upto ? 31 - __clz(upto) : -1;
+  int j = j0;
+  unsigned o = __ballot_sync(0xffffffffu, starts);
+  while (o) {
+    const int l = __ffs(o) - 1;
+    o &= o - 1;
+    const long long sll = __shfl_sync(0xffffffffu, s_l, l);
+    if (hpos >= 0 && sll - p0 == hpos) j = l;
+  }
+  const bool piece_end = valid && (lane == len - 1 || ((hm >> (lane + 1)) & 1u));
+  if (piece_end) {
+    const int sl = hpos >= 0 ? hpos : 0;
+    const unsigned pm = (0xffffffffu >> (31 - lane)) & (0xffffffffu << sl);
+    const int ch = __popc(bh & pm), cl = __popc(bl & pm);
+    if (ch) atomicAdd(A.segH + M.sb + j, ch);
+    if (cl) atomicAdd(A.segL + M.sb + j, cl);
+  }
+  if (lane == 0) {
+    A.ccnt[2ll * c] = (unsigned long long)__popc(bh) | ((unsigned long long)__popc(bl) << 32);
+    A.ccnt[2ll * c + 1] = (unsigned long long)M.reset;
+  }
+}
+
+#ifndef GBDT_COUNT_SHORT
+#define GBDT_COUNT_SHORT 1
+#endif
 __global__ void __launch_bounds__(kThreads) k_part_count(PartArgs A, int counted) {
   __shared__ TabCache tc;
   const int lane = threadIdx.x & 31;
@@ -1418,6 +1667,12 @@ __global__ void __launch_bounds__(kThreads) k_part_count(PartArgs A, int counted
     const long long base = M.p0 + (long long)lane * kItems;
     const int4 i0 = n0, i1 = n1;
     if (c + nw < C) load_ids(c + nw, n0, n1);
+#if GBDT_COUNT_SHORT
+    if (counted && M.p1 - M.p0 <= 32 && K <= 32) {
+      count_short(A, M, c, K, lane);
+      continue;
+    }
+#endif
     unsigned vm = 0, loc = 0;
     uint8_t sd[kItems];
 #pragma unroll
@@ -1585,59 +1840,112 @@ __device__ unsigned long long block_exscan_u64(unsigned long long x, unsigned lo
 //   k_plan_attr  per attribute: (high, low) counts before each segment and the child list length
 //   (exact integer scan over the attributes of (padded length | chunks << 32))
 //   k_plan_seg   per attribute: list start, chunk start, every child segment's start and count
+// A group of G lanes per attribute (G = K rounded up to a power of two, at most 32; tiles of 32
+// segments when K > 32), lane j of the group on segment j: the segment tables are read and written
+// in coalesced rows, all lanes busy whatever K, and the running offsets are group scans.  (A thread
+// per attribute looping over its K segments strided every write by K words: on C4a, 1.35 M
+// attributes x up to 32 segments, k_plan_seg moved 3x its algorithmic bytes in partial sectors.)
+__device__ __forceinline__ int plan_group(int K) {
+  int G = 1;
+  while (G < K && G < 32) G <<= 1;
+  return G;
+}
+
 __global__ void __launch_bounds__(kThreads) k_plan_attr(PlanArgs A) {
   const int K = *A.Kp, m = A.m;
-  const int stride = gridDim.x * blockDim.x;
-  for (int a = blockIdx.x * blockDim.x + threadIdx.x; a <= m; a += stride) {
-    if (a == m) { A.el[2ll * m] = 0ull; A.el[2ll * m + 1] = 0ull; continue; }
+  const int lane = threadIdx.x & 31;
+  const int G = plan_group(K), per = 32 / G, sub = lane / G, jj = lane % G;
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int a0 = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * per; a0 <= m; a0 += nw * per) {
+    const int a = a0 + sub;
+    const bool act = a < m;
+    if (a == m && jj == 0) { A.el[2ll * m] = 0ull; A.el[2ll * m + 1] = 0ull; }
     unsigned long long pre = 0;
     long long L = 0;
-    for (int j = 0; j < K; ++j) {
+    for (int j0 = 0; j0 < K; j0 += G) {
+      const int j = j0 + jj;
       const long long s = (long long)a * K + j;
-      const int c = A.cidx[j];
-      if (!A.counted) {  // no missing values: every instance of a node is in every attribute list
-        A.segH[s] = c >= 0 ? A.ncnt[c] : 0;
-        A.segL[s] = c >= 0 ? A.ncnt[c + 1] : 0;
+      unsigned long long x = 0;
+      long long l = 0;
+      if (act && j < K) {
+        const int c = A.cidx[j];
+        unsigned hi, lo;
+        if (!A.counted) {  // no missing values: every instance of a node is in every attribute list
+          hi = c >= 0 ? (unsigned)A.ncnt[c] : 0u;
+          lo = c >= 0 ? (unsigned)A.ncnt[c + 1] : 0u;
+          A.segH[s] = (int32_t)hi;
+          A.segL[s] = (int32_t)lo;
+        } else {
+          hi = (unsigned)A.segH[s];
+          lo = (unsigned)A.segL[s];
+        }
+        x = (unsigned long long)hi | ((unsigned long long)lo << 32);
+        if (c >= 0) l = (long long)hi + lo;
       }
-      const unsigned hi = (unsigned)A.segH[s], lo = (unsigned)A.segL[s];
-      A.seg_pre[s] = pre;
-      pre += (unsigned long long)hi | ((unsigned long long)lo << 32);
-      if (c >= 0) L += (long long)hi + lo;
+      unsigned long long inc = x;
+      for (int o = 1; o < G; o <<= 1) {
+        const unsigned long long y = __shfl_up_sync(0xffffffffu, inc, o, G);
+        if (jj >= o) inc += y;
+      }
+      if (act && j < K) A.seg_pre[s] = pre + (inc - x);
+      pre += __shfl_sync(0xffffffffu, inc, G - 1, G);
+      for (int o = G >> 1; o; o >>= 1) l += __shfl_xor_sync(0xffffffffu, l, o, G);
+      L += l;
     }
-    A.nxt.col_len[a] = L;
-    A.el[2ll * a] = (unsigned long long)((L + 3) & ~3ll) | ((unsigned long long)((L + kChunk - 1) / kChunk) << 32);
-    A.el[2ll * a + 1] = 0ull;
+    if (act && jj == 0) {
+      A.nxt.col_len[a] = L;
+      A.el[2ll * a] = (unsigned long long)((L + 3) & ~3ll) | ((unsigned long long)((L + kChunk - 1) / kChunk) << 32);
+      A.el[2ll * a + 1] = 0ull;
+    }
   }
 }
 
 __global__ void __launch_bounds__(kThreads) k_plan_seg(PlanArgs A) {
   const int K = *A.Kp, Kn = *A.Knp, m = A.m;
-  const int stride = gridDim.x * blockDim.x;
-  for (int a = blockIdx.x * blockDim.x + threadIdx.x; a <= m; a += stride) {
-    const unsigned long long ex = A.el[2ll * a];
-    const long long cs = (long long)(ex & 0xffffffffull);
-    const int ch = (int)(ex >> 32);
-    A.nxt.col_start[a] = cs;
-    A.nxt.chunk_start[a] = ch;
-    if (a == m) {
-      *A.nxt.C = ch;
-      *A.nxt.T = (ch + kChunksPerTile - 1) / kChunksPerTile;
-      continue;
+  const int lane = threadIdx.x & 31;
+  const int G = plan_group(K), per = 32 / G, sub = lane / G, jj = lane % G;
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int a0 = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * per; a0 <= m; a0 += nw * per) {
+    const int a = a0 + sub;
+    const bool act = a < m;
+    long long cs = 0;
+    if (a <= m) {
+      const unsigned long long ex = A.el[2ll * a];
+      cs = (long long)(ex & 0xffffffffull);
+      const int ch = (int)(ex >> 32);
+      if (jj == 0) {
+        A.nxt.col_start[a] = cs;
+        A.nxt.chunk_start[a] = ch;
+        if (a == m) {
+          *A.nxt.C = ch;
+          *A.nxt.T = (ch + kChunksPerTile - 1) / kChunksPerTile;
+        }
+      }
     }
     long long r = cs;
-    for (int j = 0; j < K; ++j) {
-      const int c = A.cidx[j];
-      if (c < 0) continue;
+    for (int j0 = 0; j0 < K; j0 += G) {
+      const int j = j0 + jj;
+      const int c = (act && j < K) ? A.cidx[j] : -1;
       const long long s = (long long)a * K + j;
-      const long long hi = A.segH[s], lo = A.segL[s];
-      A.out_hi[s] = r;
-      A.nxt.seg_start[(long long)a * Kn + c] = r;
-      A.nxt.seg_cnt[(long long)a * Kn + c] = hi;
-      r += hi;
-      A.out_lo[s] = r;
-      A.nxt.seg_start[(long long)a * Kn + c + 1] = r;
-      A.nxt.seg_cnt[(long long)a * Kn + c + 1] = lo;
-      r += lo;
+      long long hi = 0, lo = 0;
+      if (c >= 0) { hi = A.segH[s]; lo = A.segL[s]; }
+      const long long x = hi + lo;
+      long long inc = x;
+      for (int o = 1; o < G; o <<= 1) {
+        const long long y = __shfl_up_sync(0xffffffffu, inc, o, G);
+        if (jj >= o) inc += y;
+      }
+      if (c >= 0) {
+        const long long st = r + (inc - x);
+        const long long sn = (long long)a * Kn + c;
+        A.out_hi[s] = st;
+        A.nxt.seg_start[sn] = st;
+        A.nxt.seg_cnt[sn] = hi;
+        A.out_lo[s] = st + hi;
+        A.nxt.seg_start[sn + 1] = st + hi;
+        A.nxt.seg_cnt[sn + 1] = lo;
+      }
+      r += __shfl_sync(0xffffffffu, inc, G - 1, G);
     }
   }
 }
@@ -2064,6 +2372,12 @@ void launch_gen(const SplitArgs& A, unsigned grid, cudaStream_t st) {
   k_sf_gen<HM, kM, kT, kR><<<grid, kThreads, 0, st>>>(A);
 }
 
+template <int HM>
+void launch_short(const SplitArgs& A, bool missing, bool rle, unsigned grid, cudaStream_t st) {
+  if (missing) { if (rle) k_sf_short<HM, true, true><<<grid, kThreads, 0, st>>>(A); else k_sf_short<HM, true, false><<<grid, kThreads, 0, st>>>(A); }
+  else { if (rle) k_sf_short<HM, false, true><<<grid, kThreads, 0, st>>>(A); else k_sf_short<HM, false, false><<<grid, kThreads, 0, st>>>(A); }
+}
+
 template <bool kFx>
 void launch_scan(const int32_t* Cp, unsigned long long* in, unsigned long long* gbuf, unsigned long long* out,
                  unsigned groups, cudaStream_t st, const int32_t* fx = nullptr) {
@@ -2099,6 +2413,7 @@ void LevelKernels::init(int device) {
   grid_fast[2][0] = grid_for(k_sf_fast<2, false>, fast_smem(2), sms);
   grid_fast[2][1] = grid_for(k_sf_fast<2, true>, fast_smem(2), sms);
   grid_gen = grid_for(k_sf_gen<2, true, false, true>, 0, sms);  // the largest variant
+  grid_short = grid_for(k_sf_short<2, true, true>, 0, sms);
   grid_agg[0] = grid_for(k_chunk_agg<0, true>, 0, sms);
   grid_agg[1] = grid_for(k_chunk_agg<1, true>, 0, sms);
   grid_agg[2] = grid_for(k_chunk_agg<2, true>, 0, sms);
@@ -2141,6 +2456,13 @@ void LevelKernels::tile_prefix(const SplitArgs& A, int hmode, bool gather, unsig
 
 void LevelKernels::split_find(const SplitArgs& A, int hmode, bool missing, bool rle, cudaStream_t st) {
   const unsigned gg = grid_gen;
+#if GBDT_SF_SHORT_KERNEL
+  if (hmode == 0) launch_short<0>(A, missing, rle, grid_short, st);
+  else if (hmode == 1) launch_short<1>(A, missing, rle, grid_short, st);
+  else launch_short<2>(A, missing, rle, grid_short, st);
+  GBDT_LAUNCH_CHECK();
+  count_launch();
+#endif
   if (!missing) {  // single-segment chunks stream through k_sf_fast; the rest go through k_sf_gen
     const unsigned gf = grid_fast[hmode][rle];
     if (hmode == 0) { if (rle) launch_fast<0, true>(A, gf, st); else launch_fast<0, false>(A, gf, st); }
@@ -2174,7 +2496,7 @@ void LevelKernels::partition_count(const PartArgs& A, const PlanArgs& P, bool co
   GBDT_LAUNCH_CHECK();
   count_launch();
   launch_scan<false>(A.t.tb.C, A.ccnt, A.sgrp, A.cpre, groups, st);
-  const unsigned pg = (unsigned)std::max(1, std::min((P.m + kThreads) / kThreads, sms * 8));
+  const unsigned pg = (unsigned)std::max(1, std::min((P.m + kWarps) / kWarps, sms * 8));  // a warp per attribute
   k_plan_attr<<<pg, kThreads, 0, st>>>(P);
   launch_scan<false>(P.mp1, P.el, P.egrp, P.el, P.egroups, st);
   k_plan_seg<<<pg, kThreads, 0, st>>>(P);

@@ -563,7 +563,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     const int64_t S = (int64_t)m * Kcap;
     const int64_t C0 = std::max(sh.C0, 1);
     // node-best records per level: one per CTA and node (K <= 32), else one per chunk and segment
-    const int64_t R = (int64_t)(LK.grid_fast[2][1] + LK.grid_fast[1][1] + LK.grid_fast[0][1] + LK.grid_gen) * 64 +
+    const int64_t R = (int64_t)(LK.grid_fast[2][1] + LK.grid_fast[1][1] + LK.grid_fast[0][1] + LK.grid_gen + LK.grid_short) * 64 +
                       2 * C0 + S + 64;
     auto sz = [&](Carve& q) {
       for (int b = 0; b < 2; ++b) {
