@@ -1366,7 +1366,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
     bool take = false;
     if (lane < bw && ii < n) {
       cc = kAll ? ii : A.genlist[ii];
-      take = kTotals || !GBDT_SF_SHORT_KERNEL || !(A.desc[cc].len <= 32 && K <= kWarpK);
+      take = kTotals || !GBDT_SF_SHORT_KERNEL || !kMissing || !(A.desc[cc].len <= 32 && K <= kWarpK);
     }
     unsigned todo = __ballot_sync(0xffffffffu, take);
     while (todo) {
@@ -1376,12 +1376,14 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
     const long long p0 = d.p0;
     const long long cp1 = p0 + d.len;
     const long long sb = (long long)d.a * K;
+#if GBDT_SF_SHORT_KERNEL
+    if (kMissing && !kTotals && d.len <= 32 && K <= kWarpK) continue;  // k_sf_short's (sparse lists)
+#else
     if (!kTotals && d.len <= 32 && K <= kWarpK) {  // short chunk (sparse lists): one entry per lane
-#if !GBDT_SF_SHORT_KERNEL
       sf_short<HMODE, kMissing, kRLE>(A, B, wgk[wid], wrec[wid], c, d, K, lane, epoch, Fg, Fh, lam);
-#endif
-      continue;  // else k_sf_short's
+      continue;
     }
+#endif
     const long long base = p0 + lane * kItems;
     const long long* ss = (const long long*)(A.t.tb.seg_start + sb);
     const long long* sc = (const long long*)(A.t.tb.seg_cnt + sb);
@@ -2077,6 +2079,7 @@ __global__ void __launch_bounds__(kThreads, GBDT_SCATTER_CTAS) k_part_scatter(Pa
     int nh = 0, nl = 0;  // kept entries of each side in the rows before
 #pragma unroll
     for (int half = 0; half < kItems / kHalf; ++half) {
+      if (half > 0 && 32 * half * kHalf >= len) break;  // short lists: no empty rows (warp-uniform)
       uint8_t sd[kHalf];
       int id[kHalf];
       float v[kHalf];
@@ -2096,6 +2099,7 @@ __global__ void __launch_bounds__(kThreads, GBDT_SCATTER_CTAS) k_part_scatter(Pa
 #pragma unroll
       for (int kk = 0; kk < kHalf; ++kk) {
         const int k = half * kHalf + kk;
+        if (kk > 0 && 32 * k >= len) break;
         const unsigned bh = __ballot_sync(0xffffffffu, sd[kk] == 1), bl = __ballot_sync(0xffffffffu, sd[kk] == 2);
         if (sd[kk]) {
           const bool hi = sd[kk] == 1;
@@ -2457,11 +2461,15 @@ void LevelKernels::tile_prefix(const SplitArgs& A, int hmode, bool gather, unsig
 void LevelKernels::split_find(const SplitArgs& A, int hmode, bool missing, bool rle, cudaStream_t st) {
   const unsigned gg = grid_gen;
 #if GBDT_SF_SHORT_KERNEL
-  if (hmode == 0) launch_short<0>(A, missing, rle, grid_short, st);
-  else if (hmode == 1) launch_short<1>(A, missing, rle, grid_short, st);
-  else launch_short<2>(A, missing, rle, grid_short, st);
-  GBDT_LAUNCH_CHECK();
-  count_launch();
+  // sparse lists (missing values): their short chunks go through k_sf_short; without missing
+  // values the only short chunks are segment-crossing list tails, which k_sf_gen takes
+  if (missing) {
+    if (hmode == 0) launch_short<0>(A, missing, rle, grid_short, st);
+    else if (hmode == 1) launch_short<1>(A, missing, rle, grid_short, st);
+    else launch_short<2>(A, missing, rle, grid_short, st);
+    GBDT_LAUNCH_CHECK();
+    count_launch();
+  }
 #endif
   if (!missing) {  // single-segment chunks stream through k_sf_fast; the rest go through k_sf_gen
     const unsigned gf = grid_fast[hmode][rle];
