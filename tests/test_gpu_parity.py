@@ -267,6 +267,17 @@ def test_sparse_lists_around_32_entries(seed):
     compare(p, model.nodes(), margin)
 
 
+def test_sparse_many_chunks_batched_split():
+    """More chunks than 32 x the split kernels' warps (~189 k lists, most <= 32 entries, a Zipf head
+    of lists up to ~7.8 k entries, missing values): k_sf_short and k_sf_gen test 32 descriptors
+    per warp step only in this regime (and in the bench's C4a), so it needs a case of its own."""
+    p = synth.c4(seed=50, n=8000, m=240_000, density=0.0015, T=2)
+    p.params["max_depth"] = 6
+    model, margin = _train(p)
+    compare(p, model.nodes(), margin)
+    structural_invariants(model.nodes(), p.n, 6, p.params["lam"], p.params["gamma"])
+
+
 def test_scatter_aggregates_match_chunk_agg():
     """The next-level chunk aggregates accumulated by the scatter (data without missing values)
     and those k_chunk_agg computes (the same lists with one NaN column, which routes every level
