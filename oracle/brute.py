@@ -21,9 +21,7 @@ def _grad(loss, yhat, y):
     if loss == "squared":
         return 2.0 * (yhat - y), np.full_like(yhat, 2.0)
     p = 1.0 / (1.0 + np.exp(-yhat))
-    g = p - y
-    q = g + y  # reading R5b
-    return g, np.maximum(q * (1.0 - q), 1e-16)
+    return p - y, np.maximum(p * (1.0 - p), 1e-16)  # Eq. 1, reading R5
 
 
 def _gain_exact(GL, HL, G, H, lam):

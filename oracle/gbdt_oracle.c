@@ -12,9 +12,8 @@
  *   R1  Eq. 2 parent denominator is H_L + H_R + lambda (P:128 prints "- lambda": garble).
  *   R2  split iff best gain > max(gamma, 0), strictly (Alg. 1 l.15-17).
  *   R3  leaf weight w = -G / (H + lambda) (never printed; "weight of the leaf node").
- *   R5  logistic: p = 1/(1+exp(-yhat)), g = p - y, h = max(q(1-q), 1e-16) with q = g + y
- *       (R5b: the hessian sigma(1-sigma) is evaluated at the probability recovered from the
- *       stored gradient; q == p exactly for y = 0 and for p >= 0.5, else within 2^-54).
+ *   R5  logistic (cross-entropy; Eq. 1): p = 1/(1+exp(-yhat)), g = p - y,
+ *       h = max(p(1-p), 1e-16), both derivatives taken at p itself.
  *   R6  squared: g = 2(yhat - y), h = 2.
  *   R8  attribute lists sorted descending; high/left = prefix side.
  *   R9  equal values ordered by ascending instance id.
@@ -130,8 +129,7 @@ void orc_gradients(int32_t loss, int64_t n, const double* yhat, const float* y, 
     } else {
       double p = 1.0 / (1.0 + exp(-yhat[i]));
       g[i] = p - (double)y[i];
-      double q = g[i] + (double)y[i]; /* R5b: p recovered from the stored gradient */
-      double hh = q * (1.0 - q);
+      double hh = p * (1.0 - p);  /* second derivative of the cross-entropy at p (Eq. 1) */
       h[i] = hh > 1e-16 ? hh : 1e-16;
     }
   }

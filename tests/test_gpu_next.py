@@ -60,11 +60,10 @@ def _host_grad(kind):
         if kind == "squared":  # g = 2(yhat - y), h = 2 (reading R6)
             G = 2.0 * (Y - yy)
             H = np.full(n, 2.0)
-        else:  # cross-entropy, readings R5/R5b
+        else:  # cross-entropy, Eq. 1, reading R5
             p = 1.0 / (1.0 + np.exp(-Y))
             G = p - yy
-            q = G + yy
-            H = np.maximum(q * (1.0 - q), 1e-16)
+            H = np.maximum(p * (1.0 - p), 1e-16)
         assert rt.cudaMemcpy(g, G.ctypes.data, 8 * n, rt.cudaMemcpyKind.cudaMemcpyHostToDevice)[0] == 0
         assert rt.cudaMemcpy(h, H.ctypes.data, 8 * n, rt.cudaMemcpyKind.cudaMemcpyHostToDevice)[0] == 0
     return fn

@@ -234,3 +234,166 @@ def test_follow_mode_flags_a_wrong_split():
     bad[0, 0]["split_value"] = np.float32(0.5)
     _, _, st = oracle.train(p, follow=bad)
     assert st["mismatch"] >= 1
+
+
+# ------------------------------------------------------------------ follow-mode acceptance bands
+# The north_star exempts only near-ties: a different (attr, value, dir) is accepted iff its gain is
+# within 1e-6 relative of the oracle's best; a different split/leaf decision iff the best gain is
+# within max(1e-6 |gain|, 1e-12 S) of gamma (SURVEY §8(c) "Follow mode").  These pins construct
+# gaps just inside and just outside each band, priced by exact rational Eq. 2 (brute force), so a
+# band set 10x too wide or too narrow fails one of them.
+from fractions import Fraction
+
+
+def _exact_gain(g, h, hi, lam):
+    G, H = sum(g), sum(h)
+    GL = sum(g[i] for i in hi)
+    HL = sum(h[i] for i in hi)
+    GR, HR = G - GL, H - HL
+    return Fraction(1, 2) * (GL * GL / (HL + lam) + GR * GR / (HR + lam) - G * G / (H + lam))
+
+
+def _two_split_problem(delta, K=1000):
+    """Squared loss, lambda=1, depth 1, yhat=0.  a0 sends {0..K-1} high; a1 sends {0..K-1, 2K}
+    high.  Instances 0..K-1 have y=1, K..2K-1 y=0, instance 2K has y=delta: delta moves the gain
+    of a1 relative to a0 continuously (delta=0 favours a0, delta=1 favours a1)."""
+    n = 2 * K + 1
+    y = np.zeros(n, np.float32)
+    y[:K] = 1.0
+    y[2 * K] = np.float32(delta)
+    X = np.zeros((n, 2))
+    X[:K, 0] = 1.0
+    X[:K, 1] = 1.0
+    X[2 * K, 1] = 1.0
+    p = synth.from_dense("ties", X, y, dict(loss="squared", max_depth=1, n_trees=1, lam=1.0,
+                                             gamma=0.0, eta=1.0, base_margin=0.0))
+    g = [Fraction(-2.0 * float(v)) for v in p.labels]    # P:193 at yhat = 0
+    h = [Fraction(2)] * n
+    lam = Fraction(1)
+    ga0 = _exact_gain(g, h, range(K), lam)
+    ga1 = _exact_gain(g, h, list(range(K)) + [2 * K], lam)
+    return p, ga0, ga1
+
+
+def _delta_for_gap(gap):
+    """float32 delta with exact gain(a1) = gain(a0) * (1 - rel), rel as close to `gap` as fp32 allows."""
+    lo, hi = 0.0, 1.0
+    for _ in range(60):
+        mid = float(np.float32((lo + hi) / 2))
+        _, a0, a1 = _two_split_problem(mid)
+        if 1 - a1 / a0 > gap:
+            lo = mid
+        else:
+            hi = mid
+        if lo == hi or mid in (lo, hi) and hi - lo < 1e-7:
+            break
+    return lo
+
+
+def _follow_with(nodes, **root):
+    f = nodes.copy()
+    for k, v in root.items():
+        f[0, 0][k] = v
+    return f
+
+
+@pytest.mark.parametrize("gap,status", [(1e-7, 1), (5e-7, 1), (2e-6, 2), (1e-5, 2)])
+def test_follow_near_tie_band(gap, status):
+    p, a0, a1 = _two_split_problem(_delta_for_gap(gap))
+    rel = float(1 - a1 / a0)
+    assert 0.5 * gap <= rel <= 2.0 * gap, rel            # the construction hit the intended gap
+    nodes, _, st = oracle.train(p)
+    assert (nodes[0, 0]["attr"], nodes[0, 0]["is_leaf"]) == (0, 0) and st["mismatch"] == 0
+    follow = _follow_with(nodes, attr=1, split_value=np.float32(1.0), default_left=0)
+    fn, _, st = oracle.train(p, follow=follow)
+    assert fn[0, 0]["follow_status"] == status, (rel, fn[0, 0]["follow_status"])
+    if status == 1:                                      # accepted: training continues with a1
+        assert st["near_tie"] == 1 and fn[0, 0]["attr"] == 1 and fn[0, 1]["count"] == 1001
+
+
+def _table1_root():
+    p = synth.table1(loss="squared", d=1, T=1, lam=1.0, eta=1.0)
+    nodes, _, _ = oracle.train(p)
+    return p, nodes, Fraction(32, 45)                    # Appendix A root gain
+
+
+@pytest.mark.parametrize("rel,status", [(1e-8, 1), (5e-7, 1), (3e-6, 2), (1e-4, 2)])
+def test_follow_gamma_band_oracle_splits_follower_leaf(rel, status):
+    """gamma just below the best gain: the oracle splits, the followed model made a leaf."""
+    p, nodes, g = _table1_root()
+    leaf = nodes.copy()
+    leaf[0] = np.zeros_like(leaf[0])
+    leaf[0]["heap_id"] = -1
+    leaf[0, 0] = nodes[0, 0]
+    leaf[0, 0]["is_leaf"] = 1
+    fn, _, _ = oracle.train(p, params=dict(gamma=float(g) * (1 - rel)), follow=leaf)
+    assert fn[0, 0]["follow_status"] == status
+
+
+@pytest.mark.parametrize("rel,status", [(1e-8, 1), (5e-7, 1), (3e-6, 2), (1e-4, 2)])
+def test_follow_gamma_band_oracle_leaf_follower_splits(rel, status):
+    """gamma just above the best gain: the oracle makes a leaf, the followed model split."""
+    p, nodes, g = _table1_root()
+    own, _, _ = oracle.train(p, params=dict(gamma=float(g) * (1 + rel)))
+    assert own[0, 0]["is_leaf"] == 1
+    fn, _, _ = oracle.train(p, params=dict(gamma=float(g) * (1 + rel)), follow=nodes)
+    assert fn[0, 0]["follow_status"] == status
+
+
+def _flat_problem(eps):
+    """gamma = 0 and one admissible split whose gain is a tiny remnant of cancellation: the high
+    half has y = 1 + eps, the low half y = 1 (squared loss, lambda = 0, so the gain is the SSE
+    reduction).  S = GL^2/HL + GR^2/HR ~ 4000 while the gain ~ 1000 eps^2."""
+    K = 1000
+    y = np.ones(2 * K, np.float32)
+    y[:K] = np.float32(1.0 + eps)
+    X = np.zeros((2 * K, 1))
+    X[:K, 0] = 1.0
+    return synth.from_dense("flat", X, y, dict(loss="squared", max_depth=1, n_trees=1, lam=0.0,
+                                                gamma=0.0, eta=1.0, base_margin=0.0))
+
+
+@pytest.mark.parametrize("eps,status", [(2.0 ** -23, 1), (1.5e-6, 1), (5e-6, 2), (2.0 ** -13, 2)])
+def test_follow_gamma_band_cancellation_floor(eps, status):
+    """The 1e-12 S floor of the gamma band: gains of ~2e-15 S (one fp32 ulp of label difference)
+    and ~3e-13 S are within the band whichever way the followed model decided; gains of ~3e-12 S
+    and ~7e-9 S are real splits and a followed leaf is a mismatch."""
+    p = _flat_problem(eps)
+    nodes, _, _ = oracle.train(p)
+    g = [Fraction(-2.0 * float(v)) for v in p.labels]
+    h = [Fraction(2)] * p.n
+    gain = _exact_gain(g, h, range(1000), Fraction(0))
+    GL, G = sum(g[:1000]), sum(g)
+    S = GL * GL / 2000 + (G - GL) ** 2 / 2000
+    ratio = float(gain / S)
+    assert (ratio < 0.5e-12) if status == 1 else (2e-12 < ratio < 1e-6), ratio
+    ref = synth.from_dense("ref", np.array([[1.0], [0.0]]), np.array([1.0, 0.0]), dict(p.params))
+    split_tree, _, _ = oracle.train(ref)                 # a 1-split tree on a0 >= 1 (same heap shape)
+    if nodes[0, 0]["is_leaf"]:                           # fp64 rounding decided "leaf": follow a split
+        follow = split_tree.copy()
+        follow[0, 0]["split_value"] = np.float32(1.0)
+    else:                                                # it decided "split": follow a leaf
+        follow = nodes.copy()
+        follow[0, 1:] = np.zeros_like(follow[0, 1:])
+        follow[0, 1:]["heap_id"] = -1
+        follow[0, 0]["is_leaf"] = 1
+    assert status == 1 or nodes[0, 0]["is_leaf"] == 0    # a 1e-9 S gain survives fp64 rounding
+    fn, _, _ = oracle.train(p, follow=follow)
+    assert fn[0, 0]["follow_status"] == status
+
+
+@pytest.mark.parametrize("off,status", [(0.3e-12, 1), (3e-12, 2)])
+def test_follow_gamma_band_cancellation_floor_follower_splits(off, status):
+    """The same floor from the other side: gamma sits `off` S above a tiny gain (~3e-12 S, so
+    1e-6 |gain| is far below 1e-12 S): the oracle makes a leaf, the followed model split."""
+    p = _flat_problem(5e-6)
+    nodes, _, _ = oracle.train(p)
+    assert nodes[0, 0]["is_leaf"] == 0
+    g = [Fraction(-2.0 * float(v)) for v in p.labels]
+    GL, G = sum(g[:1000]), sum(g)
+    S = float(GL * GL / 2000 + (G - GL) ** 2 / 2000)
+    gamma = float(nodes[0, 0]["gain"]) + off * S
+    own, _, _ = oracle.train(p, params=dict(gamma=gamma))
+    assert own[0, 0]["is_leaf"] == 1
+    fn, _, _ = oracle.train(p, params=dict(gamma=gamma), follow=nodes)
+    assert fn[0, 0]["follow_status"] == status
