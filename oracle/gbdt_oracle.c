@@ -27,8 +27,10 @@
  *
  * Parity pins for every exported function live in tests/test_oracle_pins.py.
  */
+#define _POSIX_C_SOURCE 199309L
 #include <math.h>
 #include <stdint.h>
+#include <time.h>
 #include <stdlib.h>
 #include <string.h>
 
@@ -150,6 +152,25 @@ double orc_gain(double GL, double HL, double G, double H, double lam) {
   return eq2_gain(GL, HL, G, H, lam, NULL);
 }
 
+/* ------------------------------------------------------------------ timing (bench / tests only) */
+/* Wall-clock seconds of the last orc_train on this thread: [0] presort, [1 + t] tree t.  No part
+ * of the method; lets the cpu_baseline report per-tree time with the presort excluded. */
+#define ORC_MAX_TIMED 4096
+static _Thread_local double orc_times[ORC_MAX_TIMED + 1];
+static _Thread_local int orc_n_times;
+
+static double now_s(void) {
+  struct timespec ts;
+  clock_gettime(CLOCK_MONOTONIC, &ts);
+  return (double)ts.tv_sec + 1e-9 * (double)ts.tv_nsec;
+}
+
+int orc_last_timings(double* out, int cap) {
+  int k = orc_n_times < cap ? orc_n_times : cap;
+  for (int i = 0; i < k; ++i) out[i] = orc_times[i];
+  return orc_n_times;
+}
+
 /* ------------------------------------------------------------------ training */
 typedef struct {
   int valid;
@@ -228,10 +249,14 @@ int orc_train(int64_t n, int64_t m, const int64_t* indptr, const int32_t* indice
   const double thr = P->gamma > 0.0 ? P->gamma : 0.0;
   int64_t nnz = indptr[n];
 
+  double t_start = now_s();
+  orc_n_times = 0;
   int64_t* col_ptr = (int64_t*)malloc(sizeof(int64_t) * (size_t)(m + 1));
   float* cval = (float*)malloc(sizeof(float) * (size_t)(nnz > 0 ? nnz : 1));
   int32_t* cins = (int32_t*)malloc(sizeof(int32_t) * (size_t)(nnz > 0 ? nnz : 1));
   orc_presort(n, m, indptr, indices, values, col_ptr, cval, cins);
+  double t_prev = now_s();
+  orc_times[orc_n_times++] = t_prev - t_start;
 
   double* yhat = (double*)malloc(sizeof(double) * (size_t)n);
   double* g = (double*)malloc(sizeof(double) * (size_t)n);
@@ -392,6 +417,9 @@ int orc_train(int64_t n, int64_t m, const int64_t* indptr, const int32_t* indice
       }
     }
     for (int64_t i = 0; i < n; ++i) yhat[i] = yhat[i] + P->eta * wleaf[node_of[i]];
+    double t_now = now_s();
+    if (orc_n_times <= ORC_MAX_TIMED) orc_times[orc_n_times++] = t_now - t_prev;
+    t_prev = t_now;
   }
   if (out_margin) memcpy(out_margin, yhat, sizeof(double) * (size_t)n);
 

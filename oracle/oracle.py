@@ -59,6 +59,8 @@ def lib():
         _lib.orc_train.restype = C.c_int
         _lib.orc_train.argtypes = [i64, i64, p, p, p, p, C.POINTER(_Params), p, p, p, C.POINTER(_Stats)]
         _lib.orc_predict.argtypes = [i64, p, p, p, p, C.c_int32, C.c_int32, C.c_double, C.c_double, p]
+        _lib.orc_last_timings.restype = C.c_int
+        _lib.orc_last_timings.argtypes = [p, C.c_int]
     return _lib
 
 
@@ -137,6 +139,13 @@ def train(prob, params=None, follow=None):
     if rc != 0:
         raise ValueError(f"orc_train failed ({rc})")
     return nodes, margin, dict(exact=st.nodes_exact, near_tie=st.nodes_near_tie, mismatch=st.nodes_mismatch)
+
+
+def last_timings():
+    """Wall-clock seconds of the calling thread's last train(): (presort_s, [tree_s, ...])."""
+    buf = np.zeros(4097, np.float64)
+    k = min(lib().orc_last_timings(_ptr(buf), buf.size), buf.size)
+    return float(buf[0]), buf[1:k].tolist()
 
 
 def predict(nodes, indptr, indices, values, eta, base_margin=0.0):

@@ -5,9 +5,18 @@ direction, leaf/internal) must match exactly except where the oracle's top two g
 1e-6 relative (follow mode accepts and counts those), and leaf weights / predictions must match
 within 1e-5 relative (+1e-9 absolute floor, reading R23).
 """
+import functools
+
 import numpy as np
 
+from datagen import synth
 from oracle import oracle
+
+
+@functools.lru_cache(maxsize=None)
+def full_problem(name):
+    """BASELINE.json config `name` at full size, generated once per test session."""
+    return synth.make(name)
 
 RTOL = 1e-5
 ATOL = 1e-9
@@ -15,7 +24,13 @@ ATOL = 1e-9
 
 def compare(prob, nodes, margin, params=None, allow_near_ties=True):
     """Returns the oracle follow-mode stats; asserts parity."""
-    onodes, omargin, st = oracle.train(prob, params=params, follow=nodes)
+    return check(prob, nodes, margin, oracle.train(prob, params=params, follow=nodes), allow_near_ties)
+
+
+def check(prob, nodes, margin, oracle_out, allow_near_ties=True):
+    """Asserts parity of a CUDA model against an oracle follow-mode run (nodes, margin, stats)
+    already computed on the same inputs with follow=nodes; returns the stats."""
+    onodes, omargin, st = oracle_out
     assert st["mismatch"] == 0, f"{prob.name}: {st['mismatch']} node(s) differ from the oracle beyond near-ties: {st}"
     if not allow_near_ties:
         assert st["near_tie"] == 0, st

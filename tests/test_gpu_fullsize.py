@@ -1,56 +1,19 @@
 """Parity at BASELINE.json's full sizes, in the launch configuration bench.py times (-m gpu).
 
-The oracle cannot train a whole full-size tree in seconds, so each full-size run is checked on
-outputs it CAN compute one by one, plus properties that hold at any size:
-  * the root split (first tree, gradients at base_margin): the oracle trains a depth-1 tree on
-    the full rows restricted to a seeded sample of attributes that includes the CUDA path's root
-    attribute; its best split over that sample must be the CUDA root split (same attribute,
-    value, default direction, gain within 1e-6 relative), or an oracle near-tie of it;
+Tree-for-tree oracle parity at full size is tests/test_gpu_fullsize_parity.py.  This module
+checks what holds at any size, on the bench's own 40-tree C3 run and across code paths:
   * structural invariants of every tree (counts, child totals, leaf weights, gains > gamma);
   * gbdt_predict on the training rows reproduces the training margin bit for bit;
-  * C3: a 2-shard (loopback) run gives bit-identical trees; C5: RLE on == RLE off.
+  * C3: a 2-shard (loopback) run gives bit-identical trees.
 """
 import numpy as np
 import pytest
 
-from datagen import synth
-from oracle import oracle
 from paper_conf_ipps_wenhkls18_b200 import gbdt
 
-from parity import structural_invariants
+from parity import full_problem, structural_invariants
 
 pytestmark = pytest.mark.gpu
-
-
-def _columns(prob, cols):
-    """The full rows of `prob` restricted to attributes `cols` (renumbered 0..k-1 in order)."""
-    cols = np.asarray(sorted(cols), np.int64)
-    remap = np.full(prob.m, -1, np.int64)
-    remap[cols] = np.arange(cols.size)
-    keep = remap[prob.indices] >= 0
-    row = np.repeat(np.arange(prob.n), np.diff(prob.indptr))[keep]
-    indptr = np.zeros(prob.n + 1, np.int64)
-    np.add.at(indptr, row + 1, 1)
-    indptr = np.cumsum(indptr)
-    return synth.Problem(prob.name + "-cols", prob.n, int(cols.size), indptr,
-                         remap[prob.indices[keep]].astype(np.int32), prob.values[keep], prob.labels,
-                         dict(prob.params)), cols
-
-
-def _check_root(prob, root, n_other=5, seed=0):
-    rng = np.random.default_rng(seed)
-    a_star = int(root["attr"])
-    others = rng.choice(np.setdiff1d(np.arange(prob.m), [a_star]), size=min(n_other, prob.m - 1), replace=False)
-    sub, cols = _columns(prob, np.concatenate([[a_star], others]))
-    on, _, _ = oracle.train(sub, params=dict(max_depth=1, n_trees=1))
-    o = on[0][0]
-    assert not o["is_leaf"], "oracle finds no split where the CUDA path split"
-    o_attr = int(cols[o["attr"]])
-    assert o["G"] == pytest.approx(root["G"], rel=1e-9, abs=1e-6)
-    if o_attr == a_star and o["split_value"] == root["split_value"] and o["default_left"] == root["default_left"]:
-        assert root["gain"] == pytest.approx(o["gain"], rel=1e-6)
-    else:  # only an oracle near-tie may differ (north_star exemption)
-        assert root["gain"] == pytest.approx(o["gain"], rel=1e-6), (o_attr, a_star, o["gain"], root["gain"])
 
 
 def _run(prob, T=1, **kw):
@@ -60,30 +23,10 @@ def _run(prob, T=1, **kw):
     return gbdt.train_problem(prob, **P)
 
 
-@pytest.mark.parametrize("name", ["C2", "C3", "C4b", "C5", "C4a"])
-def test_full_size_root_and_invariants(name):
-    prob = synth.make(name)
-    model, margin = _run(prob, T=2)
-    nodes = model.nodes()
-    P = prob.params
-    structural_invariants(nodes, prob.n, P["max_depth"], P["lam"], P["gamma"])
-    _check_root(prob, nodes[0][0])
-    pred = gbdt.predict(model, prob.indptr, prob.indices, prob.values, prob.m)
-    assert np.array_equal(pred, margin)
-
-
 def test_full_size_c3_shards_bit_identical():
-    prob = synth.make("C3")
+    prob = full_problem("C3")
     a, ma = _run(prob, T=1)
     b, mb = _run(prob, T=1, n_shards=2)
-    assert np.array_equal(a.nodes().view(np.uint8), b.nodes().view(np.uint8))
-    assert np.array_equal(ma, mb)
-
-
-def test_full_size_c5_rle_on_equals_off():
-    prob = synth.make("C5")
-    a, ma = _run(prob, T=1)
-    b, mb = _run(prob, T=1, rle="on")
     assert np.array_equal(a.nodes().view(np.uint8), b.nodes().view(np.uint8))
     assert np.array_equal(ma, mb)
 
@@ -92,7 +35,7 @@ def test_full_size_c3_forty_trees_as_benched():
     """C3 at its full size and the bench's configuration (40 trees in one gbdt_train, one CUDA
     graph per tree): every tree satisfies the structural invariants, the first tree equals the
     one a 1-tree run builds, and prediction by traversal reproduces the SmartGD margin."""
-    prob = synth.make("C3")
+    prob = full_problem("C3")
     model, margin = _run(prob, T=40)
     nodes = model.nodes()
     P = prob.params
