@@ -129,7 +129,9 @@ enum {
   GBDT_PHASE_K_SPLIT = 8,     /* k_sf_fast + k_sf_gen: scan, gains, node bests (inside SPLIT_FIND) */
   GBDT_PHASE_K_COUNT = 9,     /* k_part_count + count scan + plan (inside PARTITION) */
   GBDT_PHASE_K_SCATTER = 10,  /* k_part_scatter (+ RLE run split) (inside PARTITION) */
-  GBDT_N_PHASES = 11
+  GBDT_PHASE_K_FUSED = 11,    /* dense data: k_fused, the partition of level l and the split find
+                                 of level l+1 in one pass (inside PARTITION) */
+  GBDT_N_PHASES = 12
 };
 
 /* Copies a CSR matrix (indptr int64[n_rows+1], indices int32[nnz] strictly increasing per row,

@@ -152,6 +152,47 @@ __device__ __forceinline__ void fill_run_chunks(int32_t* run_chunk, const Tables
   for (long long q = cs + k0 * kChunk; q < P + L; q += kChunk) run_chunk[c0 + (q - cs) / kChunk] = o;
 }
 
+// ============================================================================ exact fixed point
+// x -> trunc(x * 2^F) as a 128-bit integer.  A pure function of x, and integer addition is
+// associative, so sums of converted values are bit-identical in any order.
+__device__ __forceinline__ __int128 to_fx(double x, int F) {
+  if (x == 0.0) return 0;
+  const long long b = __double_as_longlong(x);
+  const int e = (int)((b >> 52) & 0x7ff);
+  const unsigned long long mant = (unsigned long long)(b & 0xfffffffffffffll) | (e ? (1ull << 52) : 0ull);
+  const int sh = (e ? e : 1) - 1075 + F;
+  unsigned __int128 v;
+  if (sh >= 0) v = (unsigned __int128)mant << (sh > 74 ? 74 : sh);
+  else v = (sh > -64) ? (unsigned __int128)(mant >> (-sh)) : (unsigned __int128)0;
+  return b < 0 ? -(__int128)v : (__int128)v;
+}
+__device__ __forceinline__ double from_fx(__int128 v, int F) {
+  const bool neg = v < 0;
+  const unsigned __int128 u = neg ? (unsigned __int128)(-v) : (unsigned __int128)v;
+  const double hi = (double)(unsigned long long)(u >> 64), lo = (double)(unsigned long long)u;
+  double r = __dadd_rn(__dmul_rn(hi, 18446744073709551616.0), lo);
+  r = __dmul_rn(r, __longlong_as_double((long long)(1023 - F) << 52));  // exact power of two
+  return neg ? -r : r;
+}
+// ----------------------------------------------------------------------------- hessian
+// Gradient storage mode of the split-find kernels:
+//   0: squared loss, h == 2 (only g is gathered)
+//   1: logistic loss with 0/1 labels, h = max(q(1-q), 1e-16), q = g + [g < 0] (K1)
+//   2: general: h gathered too
+enum { kHConst2 = 0, kHFromG = 1, kHGather = 2 };
+template <int HMODE>
+__device__ __forceinline__ double hess_of(double g) {
+  if (HMODE == kHConst2) return 2.0;
+  // logistic, 0/1 labels: y = [g < 0] (g = p - y with p in [0,1]); q = g + y (K1)
+  const double q = g < 0.0 ? __dadd_rn(g, 1.0) : g;
+  const double hh = __dmul_rn(q, __dsub_rn(1.0, q));
+  // max(hh, 1e-16); hh is never NaN (q in [0, 1]), so a plain compare-select (no fmax NaN rules)
+  double r;
+  asm("{\n .reg .pred p;\n setp.lt.f64 p, %1, 0d3C9CD2B297D889BC;\n selp.f64 %0, 0d3C9CD2B297D889BC, %1, p;\n}"
+      : "=d"(r) : "d"(hh));
+  return r;
+}
+
 // ----------------------------------------------------------------------------- scan value
 struct SV {
   double g, h;

@@ -25,11 +25,7 @@ struct TileArgs {
   int* counter;        // dynamic tile claim counter (reset per level)
 };
 
-// Gradient storage mode of the split-find kernels:
-//   0: squared loss, h == 2 (only g is gathered)
-//   1: logistic loss with 0/1 labels, h = max(q(1-q), 1e-16), q = g + [g < 0] (reading R5b)
-//   2: general: h gathered too
-enum { kHConst2 = 0, kHFromG = 1, kHGather = 2 };
+
 
 // Per-chunk descriptor written by k_chunk_agg for the split-find kernels (32 bytes).
 struct ChunkDesc {
@@ -137,6 +133,53 @@ struct RunArgs {
   unsigned groups;
 };
 
+// fused.cu: dense levels below the root, partition of level l + split find of level l+1 in one
+// pass (no missing values, g-list only, K <= kFusedMaxK nodes per level, i.e. max_depth <= 8)
+constexpr int kFusedMaxK = 64;
+struct FusedPlan {            // device, written by k_fused_plan
+  long long n_act;            // entries per attribute list at level l (instances in active nodes)
+  long long stride;           // padded list length at level l (attribute a starts at a * stride)
+  long long n_next, stride_next;
+  int tpa;                    // 2048-entry tiles per attribute
+  int T;                      // tiles of the level (0: no child to scan)
+  int K, Kn;                  // nodes at level l, l+1
+  int epoch;                  // the level epoch of the records / look-back status words
+  int off[kFusedMaxK + 1];    // segment start of node j within an attribute list, off[K] = n_act
+  int cidx[kFusedMaxK];       // high child of node j at level l+1 (low = +1), -1: became a leaf
+  int offn[2 * kFusedMaxK + 1];  // child segment starts in the next level's lists
+  int pj[2 * kFusedMaxK];     // parent of child c
+};
+struct FusedArgs {
+  const float* val;           // level l lists (val, ins, g-list)
+  const int32_t* ins;
+  const double* gl;
+  float* val_out;             // level l+1 lists (when the children are partitioned again)
+  int32_t* ins_out;
+  double* g_out;
+  const uint32_t* hbit;       // instance -> high-child bit of level l's splits
+  const FusedPlan* plan;
+  NodeTab nxt;                // the children: G, H, pterm
+  unsigned* lb_status;        // [tiles] look-back status (epoch << 2 | 1 aggregate / 2 inclusive)
+  void* lb_agg_;              // [tiles] look-back records (fused.cu LBRec)
+  void* lb_inc_;
+  int* ticket;                // tile claim counter (reset by the plan)
+  const int32_t* fx;          // [2] fixed-point scales of this tree
+  double lam;
+  int m, a_base, shard;
+  Rec* rec;                   // node-best records of level l+1 (appended)
+  int* nrec;
+  unsigned long long* gkey;
+};
+size_t fused_lb_bytes(int64_t max_tiles);
+int64_t fused_tiles(int64_t n, int m);
+void fused_init(int sms);
+unsigned fused_grid(int hmode);
+void fused_plan(FusedPlan* P, const NodeTab& cur, const NodeTab& nxt, const int32_t* cidx, const int* epoch, int m,
+                int* ticket, unsigned long long* lent, int lvl, cudaStream_t st);
+void fused_pass(const FusedArgs& A, int hmode, bool write, cudaStream_t st);
+void fused_mark(const FusedPlan* P, const int32_t* Kp, const int32_t* cidx, const Rec* winner, int shard, int a_base,
+                const int32_t* ins, const uint32_t* hbit, uint8_t* bits, int64_t n, int Kl, int sms, cudaStream_t st);
+
 // levels.cu launchers
 struct LevelKernels {
   int sms = 148;
@@ -144,6 +187,7 @@ struct LevelKernels {
   unsigned grid_gen = 0;
   unsigned grid_short = 0;
   unsigned grid_agg[3] = {0};
+  unsigned grid_fused = 0;
   unsigned grid_scatter[3][2] = {{0}}, grid_count = 0, grid_count_dense = 0, grid_agg_list[3] = {0};  // scatter: [hmode][agg]
   void init(int device);
   // a3/a4: tile aggregates (+ g/h lists) and the exact segmented carry scan

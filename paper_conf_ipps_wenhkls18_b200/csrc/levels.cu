@@ -58,28 +58,6 @@ __device__ __forceinline__ SVf shfl_up(const SVf& x, int o) {
              __shfl_up_sync(0xffffffffu, x.c, o), __shfl_up_sync(0xffffffffu, x.f, o)};
 }
 
-// ============================================================================ exact fixed point
-// x -> trunc(x * 2^F) as a 128-bit integer.  A pure function of x, and integer addition is
-// associative, so sums of converted values are bit-identical in any order.
-__device__ __forceinline__ __int128 to_fx(double x, int F) {
-  if (x == 0.0) return 0;
-  const long long b = __double_as_longlong(x);
-  const int e = (int)((b >> 52) & 0x7ff);
-  const unsigned long long mant = (unsigned long long)(b & 0xfffffffffffffll) | (e ? (1ull << 52) : 0ull);
-  const int sh = (e ? e : 1) - 1075 + F;
-  unsigned __int128 v;
-  if (sh >= 0) v = (unsigned __int128)mant << (sh > 74 ? 74 : sh);
-  else v = (sh > -64) ? (unsigned __int128)(mant >> (-sh)) : (unsigned __int128)0;
-  return b < 0 ? -(__int128)v : (__int128)v;
-}
-__device__ __forceinline__ double from_fx(__int128 v, int F) {
-  const bool neg = v < 0;
-  const unsigned __int128 u = neg ? (unsigned __int128)(-v) : (unsigned __int128)v;
-  const double hi = (double)(unsigned long long)(u >> 64), lo = (double)(unsigned long long)u;
-  double r = __dadd_rn(__dmul_rn(hi, 18446744073709551616.0), lo);
-  r = __dmul_rn(r, __longlong_as_double((long long)(1023 - F) << 52));  // exact power of two
-  return neg ? -r : r;
-}
 __device__ __forceinline__ __int128 shfl_up128(__int128 v, int o) {
   const unsigned long long lo = __shfl_up_sync(0xffffffffu, (unsigned long long)v, o);
   const unsigned long long hi = __shfl_up_sync(0xffffffffu, (unsigned long long)((unsigned __int128)v >> 64), o);
@@ -131,19 +109,6 @@ __device__ __forceinline__ void carry_store(unsigned long long* dst5, long long 
 __device__ __forceinline__ CarryD carry_load(const unsigned long long* src5) {
   return CarryD{__longlong_as_double((long long)src5[0]), __longlong_as_double((long long)src5[2]),
                 (int)(unsigned)src5[4]};
-}
-
-template <int HMODE>
-__device__ __forceinline__ double hess_of(double g) {
-  if (HMODE == kHConst2) return 2.0;
-  // logistic, 0/1 labels: y = [g < 0] (g = p - y with p in [0,1]); q = g + y; reading R5b
-  const double q = g < 0.0 ? __dadd_rn(g, 1.0) : g;
-  const double hh = __dmul_rn(q, __dsub_rn(1.0, q));
-  // max(hh, 1e-16); hh is never NaN (q in [0, 1]), so a plain compare-select (no fmax NaN rules)
-  double r;
-  asm("{\n .reg .pred p;\n setp.lt.f64 p, %1, 0d3C9CD2B297D889BC;\n selp.f64 %0, 0d3C9CD2B297D889BC, %1, p;\n}"
-      : "=d"(r) : "d"(hh));
-  return r;
 }
 
 // 1/x for x > 0 (normal): hardware seed + two Newton steps (~1 ulp).  Used only to RANK the
@@ -2432,6 +2397,8 @@ void LevelKernels::init(int device) {
   grid_scatter[2][1] = grid_for(k_part_scatter<2, false, true>, 0, sms);
   grid_count = grid_for(k_part_count, 0, sms);
   grid_count_dense = grid_for(k_part_count_dense, 0, sms);
+  fused_init(sms);
+  grid_fused = std::max(fused_grid(0), fused_grid(1));
 }
 
 unsigned LevelKernels::scan_groups(int64_t max_chunks) {

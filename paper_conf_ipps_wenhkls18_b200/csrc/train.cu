@@ -422,6 +422,12 @@ struct ShardWork {
   unsigned long long *run_hl = nullptr, *rcnt = nullptr, *rfl = nullptr, *rsgrp = nullptr;
   int32_t* Rp1 = nullptr;
   unsigned rgroups = 1;
+  // fused dense levels: plans of two levels, look-back records, tile ticket
+  DBuf fz;
+  FusedPlan* fplan[2] = {nullptr, nullptr};
+  unsigned* lb_status = nullptr;
+  void *lb_agg = nullptr, *lb_inc = nullptr;
+  int* ticket = nullptr;
   // attribute-parallel partition plan
   unsigned long long *pel = nullptr, *pgrp = nullptr;
   int32_t* mp1 = nullptr;
@@ -520,6 +526,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     c.take<unsigned long long>(16);
     c.take<int32_t>(4);
     c.take<uint32_t>((size_t)(n + 31) / 32 + 1);
+    c.take<uint32_t>((size_t)(n + 31) / 32 + 1);
   };
   Carve probe{nullptr};
   sz_dev(probe);
@@ -553,6 +560,22 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   unsigned long long* lent = c.take<unsigned long long>(16);  // entries scanned per level (profile)
   int32_t* tidx = c.take<int32_t>(4);  // index of the tree being built (device side, for graph replays)
   uint32_t* hbit = c.take<uint32_t>((size_t)(n + 31) / 32 + 1);  // instance -> high child bit
+  uint32_t* hbit2 = c.take<uint32_t>((size_t)(n + 31) / 32 + 1);  // the fused path's second level
+  uint32_t* hbitF[2] = {hbit, hbit2};
+
+  // Fused dense levels (fused.cu): no missing values, g-list only, K <= kFusedMaxK at the last
+  // partitioned level, plain lists with the dense root layout (attribute a at a * pad4(n))
+  bool fused = !ds.has_missing && hmode != kHGather && d >= 2 && d <= 8;
+  for (auto& shp : ds.shards) {
+    const Shard& sh = *shp;
+    if (sh.rle) fused = false;
+    for (int a = 0; a < sh.m && fused; ++a)
+      if (sh.h_col_len[a] != n || sh.h_col_start[a] != (int64_t)a * pad4(n)) fused = false;
+  }
+  {  // opt-in while the fused pass is being tuned (GBDT_FUSED=1)
+    const char* fe = getenv("GBDT_FUSED");
+    fused = fused && fe && fe[0] != '0';
+  }
 
   // ---------------------------------------------------------------- per-shard state
   std::vector<ShardWork> sw(nloc);
@@ -564,7 +587,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     const int64_t C0 = std::max(sh.C0, 1);
     // node-best records per level: one per CTA and node (K <= 32), else one per chunk and segment
     const int64_t R = (int64_t)(LK.grid_fast[2][1] + LK.grid_fast[1][1] + LK.grid_fast[0][1] + LK.grid_gen + LK.grid_short) * 64 +
-                      2 * C0 + S + 64;
+                      (int64_t)LK.grid_fused * 2 * kFusedMaxK + 2 * C0 + S + 64;
     auto sz = [&](Carve& q) {
       for (int b = 0; b < 2; ++b) {
         q.take<int64_t>(m + 1); q.take<int64_t>(m); q.take<int32_t>(m + 1); q.take<int32_t>(m + 1);
@@ -649,6 +672,19 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       w.rcnt = r.take<unsigned long long>(2 * Rcap); w.rfl = r.take<unsigned long long>(2 * (Rcap + 1));
       w.Rp1 = r.take<int32_t>(1); w.rsgrp = r.take<unsigned long long>(2 * (size_t)w.rgroups + 8);
     }
+    if (fused && m > 0) {
+      const int64_t tiles = fused_tiles(n, m);
+      const size_t lbb = fused_lb_bytes(tiles);
+      w.fz.alloc(2 * sizeof(FusedPlan) + 256 + lbb + 1024, st);
+      GBDT_CUDA(cudaMemsetAsync(w.fz.p, 0, w.fz.bytes, st));
+      Carve f{w.fz.as<char>()};
+      w.fplan[0] = f.take<FusedPlan>(1);
+      w.fplan[1] = f.take<FusedPlan>(1);
+      w.ticket = f.take<int>(4);
+      w.lb_agg = f.take<char>(96 * (size_t)tiles);
+      w.lb_inc = f.take<char>(96 * (size_t)tiles);
+      w.lb_status = f.take<unsigned>((size_t)tiles);
+    }
     w.nrec = nrec + li;
     w.gkey = gkey + (size_t)li * Kcap;
     w.tkey = tkey + (size_t)li * Kcap;
@@ -693,14 +729,18 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       NodeTab& nxt = nt[(lvl + 1) & 1];
       const bool last = (lvl == d - 1);
       const int Kl = 1 << lvl;  // upper bound of active nodes at this level
+      // fz: this level's node bests were found by the previous level's fused pass
+      const bool fz = fused && lvl >= 1;
+      if (!fz) {
       tm.begin(GBDT_PHASE_DECIDE);
       k_level_begin<<<1, 1024, 0, st>>>(epoch, sw[0].counters, 0, nrec, nloc, cur.K, gkey, tkey, Kcap);
       GBDT_LAUNCH_CHECK();
       count_launch();
       for (int li = 0; li < nloc; ++li) GBDT_CUDA(cudaMemsetAsync(sw[li].counters, 0, 4 * sizeof(int), st));
       tm.end();
+      }
       tm.begin(GBDT_PHASE_SPLIT_FIND);
-      for (int li = 0; li < nloc; ++li) {
+      for (int li = 0; li < nloc && !fz; ++li) {
         Shard& sh = *ds.shards[li];
         ShardWork& w = sw[li];
         if (sh.m == 0) continue;
@@ -763,6 +803,12 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       for (int li = 0; li < nloc; ++li) {
         Shard& sh = *ds.shards[li];
         if (sh.m == 0) continue;
+        if (fz) {  // the winners' child segments, read from the parent level's lists
+          const int32_t* pins = lvl == 1 ? sh.ins0.as<int32_t>() : sh.insw[(lvl - 1) & 1].as<int32_t>();
+          fused_mark(sw[li].fplan[(lvl - 1) & 1], cur.K, cidx, winner, sh.index, sh.a_begin, pins,
+                     hbitF[(lvl - 1) & 1], bits, n, Kl, sms, st);
+          continue;
+        }
         const Tables tb = lvl == 0 ? sh.root : sw[li].tab[lvl & 1];
         const int32_t* ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
         dim3 grid((unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256 * (int64_t)Kl), (int64_t)sms * 4)), (unsigned)Kl);
@@ -777,13 +823,42 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         tm.end();
       }
       tm.begin(GBDT_PHASE_NODEMAP);
-      k_nodemap<<<inst_grid, 256, 0, st>>>(n, bits, hstate, hdef, pos, side, hbit);
+      k_nodemap<<<inst_grid, 256, 0, st>>>(n, bits, hstate, hdef, pos, side, fused ? hbitF[lvl & 1] : hbit);
       GBDT_LAUNCH_CHECK();
       count_launch();
       tm.end();
 
       if (last) break;
       tm.begin(GBDT_PHASE_PARTITION);
+      if (fused) {  // partition of this level + split find of the next, one pass (fused.cu)
+        k_level_begin<<<1, 1024, 0, st>>>(epoch, sw[0].counters, 0, nrec, nloc, nxt.K, gkey, tkey, Kcap);
+        GBDT_LAUNCH_CHECK();
+        count_launch();
+        for (int li = 0; li < nloc; ++li) {
+          Shard& sh = *ds.shards[li];
+          ShardWork& w = sw[li];
+          if (sh.m == 0) continue;
+          fused_plan(w.fplan[lvl & 1], cur, nxt, cidx, epoch, sh.m, w.ticket, P.profile ? lent : nullptr, lvl, st);
+          FusedArgs FA;
+          FA.val = lvl == 0 ? sh.val0.as<float>() : sh.valw[lvl & 1].as<float>();
+          FA.ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
+          FA.gl = w.glist[lvl & 1];
+          FA.val_out = sh.valw[(lvl + 1) & 1].as<float>();
+          FA.ins_out = sh.insw[(lvl + 1) & 1].as<int32_t>();
+          FA.g_out = w.glist[(lvl + 1) & 1];
+          FA.hbit = hbitF[lvl & 1];
+          FA.plan = w.fplan[lvl & 1];
+          FA.nxt = nxt;
+          FA.lb_status = w.lb_status; FA.lb_agg_ = w.lb_agg; FA.lb_inc_ = w.lb_inc; FA.ticket = w.ticket;
+          FA.fx = fxs; FA.lam = P.lambda; FA.m = sh.m; FA.a_base = sh.a_begin; FA.shard = sh.index;
+          FA.rec = w.rec; FA.nrec = w.nrec; FA.gkey = w.gkey;
+          kt.begin(GBDT_PHASE_K_FUSED);
+          fused_pass(FA, hmode, /*write=*/lvl + 1 < d - 1, st);
+          kt.end();
+        }
+        tm.end();
+        continue;
+      }
       for (int li = 0; li < nloc; ++li) {
         Shard& sh = *ds.shards[li];
         ShardWork& w = sw[li];

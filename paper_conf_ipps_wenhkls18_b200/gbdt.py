@@ -22,7 +22,7 @@ STATUS = {0: "OK", 1: "E_INVAL", 2: "E_NOMEM", 3: "E_CUDA", 4: "E_NCCL", 5: "E_S
 LOSS = {"squared": 0, "logistic": 1, "custom": 2}
 RLE = {"off": 0, "on": 1, "auto": 2, False: 0, True: 1, None: 0}
 PHASES = ["grad", "split_find", "decide", "nodemap", "partition", "comm", "total",
-          "k_chunk_agg", "k_split", "k_count", "k_scatter"]
+          "k_chunk_agg", "k_split", "k_count", "k_scatter", "k_fused"]
 
 NODE_DTYPE = np.dtype([
     ("heap_id", np.int32), ("is_leaf", np.int32), ("attr", np.int32), ("default_left", np.int32),

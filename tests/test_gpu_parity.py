@@ -200,8 +200,9 @@ def test_deterministic_across_runs():
 
 # ------------------------------------------------------------------ a8 RLE: direct split
 # The RLE path reads values from the runs and splits the runs themselves (no decompression in HBM);
-# it sees the same entry streams, so its trees and margins must be bit-identical to the plain path,
-# and both match the oracle.
+# it sees the same entry streams, so its trees and margins must be bit-identical to the plain
+# level-by-level path (GBDT_FUSED=0: dense data otherwise takes the fused pass of fused.cu, whose
+# sums associate differently), and both match the oracle.
 @pytest.mark.parametrize("maker", [
     lambda: synth.c5(n=40000, T=3),
     lambda: synth.table1(),
@@ -210,8 +211,9 @@ def test_deterministic_across_runs():
     lambda: synth.c4(seed=9, n=1500, m=2000, density=0.01, T=2),
     lambda: synth.c1(n=5000),
 ])
-def test_rle_direct_split_bit_identical(maker):
+def test_rle_direct_split_bit_identical(maker, monkeypatch):
     p = maker()
+    monkeypatch.setenv("GBDT_FUSED", "0")
     ref_model, ref_margin = _train(p)
     model, margin = _train(p, rle="on")
     assert np.array_equal(model.nodes().view(np.uint8), ref_model.nodes().view(np.uint8))
@@ -225,8 +227,9 @@ def test_rle_c5_against_oracle():
 
 
 @pytest.mark.parametrize("k", [2, 4])
-def test_rle_with_shards(k):
+def test_rle_with_shards(k, monkeypatch):
     p = synth.c5(n=30000, T=2)
+    monkeypatch.setenv("GBDT_FUSED", "0")
     ref_model, ref_margin = _train(p)
     model, margin = _train(p, rle="on", n_shards=k)
     assert np.array_equal(model.nodes().view(np.uint8), ref_model.nodes().view(np.uint8))
@@ -332,11 +335,56 @@ def test_deep_trees_more_than_32_nodes_per_level(maker):
     compare(p, model.nodes(), margin, params=p.params)
 
 
-def test_deep_trees_rle_bit_identical():
+def test_deep_trees_rle_bit_identical(monkeypatch):
     """RLE run tables with more than 32 nodes per level (depth 8) equal the plain path."""
     p = synth.random_small(79, n=8000, m=5, nan_frac=0.1, n_distinct=20, loss="logistic", d=8, T=2)
+    monkeypatch.setenv("GBDT_FUSED", "0")
     ref_model, ref_margin = _train(p)
     model, margin = _train(p, rle="on")
     assert np.array_equal(model.nodes().view(np.uint8), ref_model.nodes().view(np.uint8))
     assert np.array_equal(margin, ref_margin)
     compare(p, model.nodes(), margin)
+
+
+# ------------------------------------------------------------------ fused dense levels (fused.cu)
+# Dense data below the root takes one pass per level (partition of level l + split find of level
+# l+1).  Against the oracle on shapes that exercise its tile machinery: many tiles per segment
+# (look-back chains), segments ending inside tiles, tiles holding several segments at depth 7-8
+# (up to 64 parent nodes), long runs of equal values crossing tiles (C5/C2-shaped), both losses,
+# and the non-writing last pass.
+@pytest.mark.parametrize("maker", [
+    lambda: synth.c3(n=60000, T=3),
+    lambda: synth.c5(n=50000, T=3),
+    lambda: synth.c2(n=30000, T=4),
+    lambda: synth.random_small(31, n=20000, m=4, nan_frac=0.0, n_distinct=7, loss="squared", d=8, T=2),
+    lambda: synth.random_small(32, n=12000, m=3, nan_frac=0.0, n_distinct=5000, loss="logistic", d=7, T=2),
+    lambda: synth.random_small(33, n=2049, m=3, nan_frac=0.0, n_distinct=2, loss="squared", d=2, T=3),
+])
+def test_fused_dense_against_oracle(maker, monkeypatch):
+    monkeypatch.setenv("GBDT_FUSED", "1")
+    p = maker()
+    model, margin = _train(p)
+    compare(p, model.nodes(), margin)
+
+
+@pytest.mark.parametrize("k", [2, 4])
+def test_fused_shards_bit_identical(k, monkeypatch):
+    monkeypatch.setenv("GBDT_FUSED", "1")
+    p = synth.c3(n=50000, T=2)
+    a, ma = _train(p)
+    b, mb = _train(p, n_shards=k)
+    assert np.array_equal(a.nodes().view(np.uint8), b.nodes().view(np.uint8))
+    assert np.array_equal(ma, mb)
+
+
+def test_fused_equals_level_by_level_up_to_rounding(monkeypatch):
+    p = synth.c3(n=40000, T=3)
+    monkeypatch.setenv("GBDT_FUSED", "1")
+    a, ma = _train(p)
+    monkeypatch.setenv("GBDT_FUSED", "0")
+    b, mb = _train(p)
+    na, nb = a.nodes(), b.nodes()
+    for f in ("heap_id", "is_leaf", "attr", "default_left", "split_value", "count"):
+        assert np.array_equal(na[f], nb[f]), f
+    np.testing.assert_allclose(na["weight"], nb["weight"], rtol=1e-10, atol=1e-14)
+    np.testing.assert_allclose(ma, mb, rtol=1e-10, atol=1e-14)
