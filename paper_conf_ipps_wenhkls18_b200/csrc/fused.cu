@@ -1,34 +1,33 @@
-// fused.cu -- dense levels below the root in ONE streaming pass per level.
+// fused.cu -- dense levels below the root: the partition of level l and the split
+// finding of level l+1 in one streaming pass over the level's lists.
 //
 // For data without missing values every (node, attribute) segment of node j holds exactly the
-// node's cnt[j] instances, so the partition of level l and the split finding of
-// level l+1 can share one read of the level's lists:
+// node's cnt[j] instances, so a child's segment is its side of the parent's segment, in the
+// parent's order (order preserving), and the child's segmented prefix sums (P:197-208,
+// Fig. 1) can be formed while the parent's entries stream past.  A level is cut into 2048-entry
+// TILES (attribute-aligned; tile k of an attribute covers its list positions [2048 k, 2048 k +
+// 2048) at that level, whatever the sharding) and runs in three steps:
 //
-//   k_fused   persistent CTAs claim 2048-entry tiles in order (a ticket counter) and stream each
-//             tile's values, instance ids and g-list into shared memory with TMA 1-D bulk copies
-//             (2-stage ring).  Per tile:
-//               1. every entry's child side: the node's decision (leaf -> dropped) and, for a
-//                  split node, one bit gathered from the instance -> high-child bitmap
-//               2. a stable in-tile partition by (segment, side), ranked by a block scan of the
-//                  packed side counts: the tile becomes contiguous runs of CHILD entries in child
-//                  order (order preserving)
-//               3. a segmented prefix sum of (g, h) over those runs (Fig. 1); the
-//                  child segment's prefix from earlier tiles arrives through a decoupled look-back
-//                  over per-tile records (counts and exact 128-bit fixed-point sums, so any
-//                  look-back path gives bit-identical carries)
-//               4. Eq. 2 (+lambda per reading R1) at every boundary between two distinct
-//                  values of a child segment (run ends), exact IEEE divisions; per
-//                  child node argmax in the R12 total order, merged per CTA, flushed once
-//               5. the child runs written to the next level's lists (coalesced), unless the
-//                  children are the last level that splits
-//   k_mark_fused   the instance -> child bits of a level found by k_fused: the winner's child
-//             segment is the winner's side of its parent segment in the PARENT level's lists,
-//             and the high part of it is every such entry at a parent position <= Rec.pos
+//   k_tile_agg   per tile: every entry's child side -- the node's decision (leaf -> dropped) and,
+//                for a split node, one bit gathered from the instance -> high-child bitmap
+//                -- kept as a bit per entry, and the tile's per-side count, exact fixed-point
+//                (g, h) sums and last entry of its LAST segment piece
+//   k_tscan1/2/3 the exact segmented inclusive scan of those records over the tiles (integer sums:
+//                any decomposition gives the same carries)
+//   k_fused      per tile, TMA-staged in shared memory (2-stage ring): a stable in-tile partition by
+//                (segment, side) ranked by a block scan of the packed side counts (the tile becomes
+//                contiguous runs of CHILD entries in child order), the segmented prefix sums of
+//                (g, h) over those runs from the carry of the tiles before, Eq. 2 (+lambda,
+//                reading R1) at every boundary between two distinct values of a child segment (run
+//                ends), the per-child-node argmax in the R12 total order, and the child
+//                runs written to the next level's lists (coalesced) unless the children are the
+//                last level that splits
+//   k_mark_fused the instance -> child bits of a level found by k_fused: the winner's child
+//                segment is the winner's side of its parent segment in the PARENT level's lists,
+//                and the high part of it is every such entry at a parent position <= Rec.pos
 //
-// Determinism: tiles are attribute-aligned (tile k of an attribute covers its list positions
-// [2048 k, 2048 k + 2048) at that level), inside a tile every sum has a fixed association, and
-// carries are exact integer sums, so every gain -- hence every tree -- is bit-identical for any
-// attribute sharding and any schedule.
+// Determinism: inside a tile every sum has a fixed association, and carries are exact integer
+// sums, so every gain -- hence every tree -- is bit-identical for any attribute sharding.
 #include <algorithm>
 #include <climits>
 
@@ -41,162 +40,78 @@ constexpr int kFT = 256;            // threads per CTA
 constexpr int kFI = 8;              // items per thread (blocked arrangement)
 constexpr int kFTile = kFT * kFI;   // entries per tile
 constexpr int kFW = kFT / 32;
-// One tile in flight per CTA.  A CTA that also held the ticket of its next tile (a 2-stage TMA
-// ring) would publish that tile's look-back record a whole tile later than it could, and the tiles
-// of its chain behind it would wait (measured: C3 148 vs 49 ms/tree, 84 % of stall samples at the
-// barrier behind the look-back).  The load latency is hidden by the other CTAs of the SM instead.
+constexpr int kTSGroup = 256;       // tiles per CTA in the tile scan
+constexpr int kFusedMaxCTAs = 148 * 8;  // persistent k_fused CTAs (node-best scratch per CTA)
+#ifndef GBDT_FUSED_STAGES
+#define GBDT_FUSED_STAGES 1
+#endif
 #ifndef GBDT_FUSED_CTAS
 #define GBDT_FUSED_CTAS 3
 #endif
+constexpr int kFS = GBDT_FUSED_STAGES;
 
-// The look-back record of one tile: per child side (0 high, 1 low) the entries of its LAST
-// segment piece, their exact fixed-point sums, and the value / parent position of the last one.
-struct __align__(16) LBSide {
-  unsigned long long g_lo, g_hi, h_lo, h_hi;
-  long long pos;
-  int cnt;
-  float val;
-};
-struct __align__(16) LBRec {
-  LBSide s[2];
-};
-static_assert(sizeof(LBRec) == 96, "look-back record");
-constexpr unsigned kLBAgg = 1, kLBInc = 2;
-__device__ __forceinline__ LBRec* lb_agg(const FusedArgs& A) { return static_cast<LBRec*>(A.lb_agg_); }
-__device__ __forceinline__ LBRec* lb_inc(const FusedArgs& A) { return static_cast<LBRec*>(A.lb_inc_); }
-
-struct FusedSmem {
-  float val[kFTile];                // the tile as loaded (TMA), never reordered in place
-  int32_t ins[kFTile];
-  double g[kFTile];
-  unsigned short src[kFTile];       // child order: slot r holds tile entry src[r]
-  unsigned long long bar;
-  int tile;
-  // plan copy
-  int off[kFusedMaxK + 1];
-  int cidx[kFusedMaxK];
-  int offn[2 * kFusedMaxK + 1];
-  double cG[2 * kFusedMaxK], cH[2 * kFusedMaxK], cHl[2 * kFusedMaxK], cP[2 * kFusedMaxK];
-  // CTA node-best table (children)
-  unsigned long long ngk[2 * kFusedMaxK];
-  Rec nrec[2 * kFusedMaxK];
-  // per tile
-  int j0, nseg, nk, cont;
-  int pq[kFusedMaxK + 1];           // tile-relative start of piece s (pq[nseg] = tile length)
-  int base[kFusedMaxK + 1];         // packed exclusive (high | low << 16) count at piece start
-  int gb[2 * kFusedMaxK + 1];       // child-order group starts: group 2s = piece s high, 2s+1 low
-  unsigned long long gk[2 * kFusedMaxK];
-  int wr[2 * kFusedMaxK];
-  int wsum[kFW];
-  double wg[kFW], wh[kFW];
-  int wf[kFW];
-  double lg[2], lh[2];              // sums of the last piece's two groups
-  float lv[2];
-  int ls[2];                        // tile entry of the groups' last members
-  LBSide ex[2];                     // carry of the first piece (look-back)
-};
-
-__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
-  unsigned v;
-  asm volatile("ld.global.acquire.gpu.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_release_u32(unsigned* p, unsigned v) {
-  asm volatile("st.global.release.gpu.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
+static_assert(sizeof(TRec) == 96, "tile record");
 
 __device__ __forceinline__ unsigned __int128 u128(unsigned long long lo, unsigned long long hi) {
   return ((unsigned __int128)hi << 64) | lo;
 }
-__device__ __forceinline__ unsigned __int128 warp_sum128(unsigned __int128 v) {
-#pragma unroll
-  for (int o = 16; o; o >>= 1) {
-    const unsigned long long lo = __shfl_xor_sync(0xffffffffu, (unsigned long long)v, o);
-    const unsigned long long hi = __shfl_xor_sync(0xffffffffu, (unsigned long long)(v >> 64), o);
-    v += u128(lo, hi);
-  }
-  return v;
+// x (+) y: y follows x in list order
+__device__ __forceinline__ TSide tside_add(const TSide& x, const TSide& y) {
+  TSide r;
+  const unsigned __int128 G = u128(x.g_lo, x.g_hi) + u128(y.g_lo, y.g_hi);
+  const unsigned __int128 H = u128(x.h_lo, x.h_hi) + u128(y.h_lo, y.h_hi);
+  r.g_lo = (unsigned long long)G; r.g_hi = (unsigned long long)(G >> 64);
+  r.h_lo = (unsigned long long)H; r.h_hi = (unsigned long long)(H >> 64);
+  r.cnt = x.cnt + y.cnt;
+  r.val = y.cnt ? y.val : x.val;
+  r.pos = y.cnt ? y.pos : x.pos;
+  return r;
 }
-
-__device__ __forceinline__ void lb_store(LBRec* dst, const LBSide* s) {
+__device__ __forceinline__ TRec trec_add(const TRec& x, const TRec& y) {
+  TRec r;
+  r.s[0] = tside_add(x.s[0], y.s[0]);
+  r.s[1] = tside_add(x.s[1], y.s[1]);
+  return r;
+}
+__device__ __forceinline__ TRec trec_zero() {
+  TRec r;
   for (int q = 0; q < 2; ++q) {
-    dst->s[q].g_lo = s[q].g_lo; dst->s[q].g_hi = s[q].g_hi;
-    dst->s[q].h_lo = s[q].h_lo; dst->s[q].h_hi = s[q].h_hi;
-    dst->s[q].pos = s[q].pos; dst->s[q].cnt = s[q].cnt; dst->s[q].val = s[q].val;
+    r.s[q].g_lo = r.s[q].g_hi = r.s[q].h_lo = r.s[q].h_hi = 0ull;
+    r.s[q].pos = 0; r.s[q].cnt = 0; r.s[q].val = 0.f;
   }
+  return r;
+}
+__device__ __forceinline__ TRec trec_shfl_up(const TRec& x, int o) {
+  TRec r;
+  const unsigned* p = reinterpret_cast<const unsigned*>(&x);
+  unsigned* d = reinterpret_cast<unsigned*>(&r);
+#pragma unroll
+  for (int i = 0; i < 24; ++i) d[i] = __shfl_up_sync(0xffffffffu, p[i], o);
+  return r;
+}
+__device__ __forceinline__ TRec trec_ld(const TRec* p) {
+  TRec r;
+  const uint4* s = reinterpret_cast<const uint4*>(p);
+  uint4* d = reinterpret_cast<uint4*>(&r);
+#pragma unroll
+  for (int i = 0; i < 6; ++i) d[i] = __ldcg(s + i);
+  return r;
+}
+__device__ __forceinline__ void trec_st(TRec* p, const TRec& x) {
+  const uint4* s = reinterpret_cast<const uint4*>(&x);
+  uint4* d = reinterpret_cast<uint4*>(p);
+#pragma unroll
+  for (int i = 0; i < 6; ++i) __stcg(d + i, s[i]);
 }
 
-// Exclusive carry of tile t's first segment piece from the tiles before it (one warp).  Lane i
-// inspects tile t-1-i; the chain ends at the closest tile whose record is inclusive (the tile in
-// which the segment starts publishes an inclusive record at once).
-// Only tiles >= tmin (the tile holding the segment's start, whose record is inclusive) are read:
-// with tickets dealt round-robin over the attributes, tiles before tmin may belong to a later
-// ticket, and waiting on them could deadlock.
-__device__ void lookback(const FusedArgs& A, int t, int tmin, unsigned ep, LBSide* out, int lane) {
-  unsigned __int128 G[2] = {0, 0}, H[2] = {0, 0};
-  long long cnt[2] = {0, 0};
-  float lv[2] = {0.f, 0.f};
-  long long lp[2] = {0, 0};
-  bool have[2] = {false, false};
-  int base = t - 1;
-  while (true) {
-    const int idx = base - lane;
-    unsigned s = (ep << 2) | kLBInc;
-    if (idx >= tmin) {
-      do {
-        s = ld_acquire_u32(A.lb_status + idx);
-      } while ((s >> 2) != ep || (s & 3u) == 0u);
-    }
-    const bool inc = (s & 3u) == kLBInc;
-    const unsigned incm = __ballot_sync(0xffffffffu, inc);
-    const int lim = incm ? __ffs(incm) - 1 : 31;
-    const bool use = lane <= lim && idx >= tmin;
-    const LBRec* src = use ? ((inc ? lb_inc(A) : lb_agg(A)) + idx) : nullptr;
-#pragma unroll
-    for (int q = 0; q < 2; ++q) {
-      unsigned __int128 g = 0, h = 0;
-      int c = 0;
-      float v = 0.f;
-      long long p = 0;
-      if (use) {
-        const unsigned long long* w = reinterpret_cast<const unsigned long long*>(&src->s[q]);
-        g = u128(__ldcg(w + 0), __ldcg(w + 1));
-        h = u128(__ldcg(w + 2), __ldcg(w + 3));
-        p = (long long)__ldcg(w + 4);
-        const unsigned long long cv = __ldcg(w + 5);
-        c = (int)(unsigned)cv;
-        v = __uint_as_float((unsigned)(cv >> 32));
-      }
-      const unsigned nz = __ballot_sync(0xffffffffu, use && c > 0);
-      if (!have[q] && nz) {  // the last value of this side: the closest tile that has one
-        const int l = __ffs(nz) - 1;
-        lv[q] = __shfl_sync(0xffffffffu, v, l);
-        lp[q] = __shfl_sync(0xffffffffu, p, l);
-        have[q] = true;
-      }
-      int cs = c;
-#pragma unroll
-      for (int o = 16; o; o >>= 1) cs += __shfl_xor_sync(0xffffffffu, cs, o);
-      cnt[q] += cs;
-      G[q] += warp_sum128(g);
-      H[q] += warp_sum128(h);
-    }
-    if (incm) break;
-    base -= 32;
+// largest j with off[j] <= q
+__device__ __forceinline__ int seg_of(const int* off, int K, int q) {
+  int lo = 0, hi = K - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (off[mid] <= q) lo = mid; else hi = mid - 1;
   }
-  if (lane == 0) {
-    for (int q = 0; q < 2; ++q) {
-      out[q].g_lo = (unsigned long long)G[q]; out[q].g_hi = (unsigned long long)(G[q] >> 64);
-      out[q].h_lo = (unsigned long long)H[q]; out[q].h_hi = (unsigned long long)(H[q] >> 64);
-      out[q].cnt = (int)cnt[q];
-      out[q].val = lv[q];
-      out[q].pos = lp[q];
-    }
-  }
-}
-
-__device__ __forceinline__ bool rec_better_f(unsigned long long gk, const Rec& r, unsigned long long gk0, const Rec& r0) {
-  return gk > gk0 || (gk == gk0 && tie_key(r.attr, r.value, r.dir) < tie_key(r0.attr, r0.value, r0.dir));
+  return lo;
 }
 
 // exclusive block scan of an int (all threads); returns the total too
@@ -219,6 +134,279 @@ __device__ __forceinline__ int block_exscan_int(int x, int& total, int* wsum, in
   total = tot;
   return wex + incl - x;
 }
+
+__device__ __forceinline__ bool rec_better_f(unsigned long long gk, const Rec& r, unsigned long long gk0, const Rec& r0) {
+  return gk > gk0 || (gk == gk0 && tie_key(r.attr, r.value, r.dir) < tie_key(r0.attr, r0.value, r0.dir));
+}
+
+// ============================================================================ k_tile_agg
+struct AggSmem {
+  int off[kFusedMaxK + 1];
+  int cidx[kFusedMaxK];
+  double wg[2][2][kFW], wh[2][2][kFW];  // [tile parity][side][warp]
+  int wc[2][2][kFW], wi[2][2][kFW];
+};
+
+template <int HMODE>
+__global__ void __launch_bounds__(kFT) k_tile_agg(FusedArgs A) {
+  __shared__ AggSmem S;
+  const FusedPlan* P = A.plan;
+  const int T = P->T;
+  if (T == 0) return;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int K = P->K, tpa = P->tpa, n_act = (int)P->n_act;
+  const long long stride = P->stride;
+  const int Fg = A.fx[0], Fh = A.fx[1];
+  for (int i = tid; i <= K; i += kFT) S.off[i] = P->off[i];
+  for (int i = tid; i < K; i += kFT) S.cidx[i] = P->cidx[i];
+  __syncthreads();
+  const int qi = tid * kFI;
+  int par = 0;
+  for (int t = blockIdx.x; t < T; t += gridDim.x, par ^= 1) {
+    const int a = t / tpa;
+    const int q0 = (t - a * tpa) * kFTile;
+    const int len = min(kFTile, n_act - q0);
+    const long long tbase = (long long)a * stride + q0;
+    const int jf = seg_of(S.off, K, q0);              // the tile's first piece
+    const int jl = seg_of(S.off, K, q0 + len - 1);    // its last piece
+    const bool live_l = S.cidx[jl] >= 0;
+    const int ql = S.off[jl] - q0;                    // the last piece's start, tile-relative
+    int id[kFI];
+    double g[kFI];
+    if (qi + kFI <= len) {
+      const int4 i0 = __ldcs(reinterpret_cast<const int4*>(A.ins + tbase + qi));
+      const int4 i1 = __ldcs(reinterpret_cast<const int4*>(A.ins + tbase + qi) + 1);
+      id[0] = i0.x; id[1] = i0.y; id[2] = i0.z; id[3] = i0.w; id[4] = i1.x; id[5] = i1.y; id[6] = i1.z; id[7] = i1.w;
+      const double2* pg = reinterpret_cast<const double2*>(A.gl + tbase + qi);
+#pragma unroll
+      for (int k = 0; k < kFI / 2; ++k) {
+        const double2 z = __ldcs(pg + k);
+        g[2 * k] = z.x;
+        g[2 * k + 1] = z.y;
+      }
+    } else {  // the list's tail: scalar loads, nothing past its end
+#pragma unroll
+      for (int k = 0; k < kFI; ++k) {
+        const bool in = qi + k < len;
+        id[k] = in ? A.ins[tbase + qi + k] : 0;
+        g[k] = in ? A.gl[tbase + qi + k] : 0.0;
+      }
+    }
+    // items whose node split (their side is looked up) and items of the last piece (summed)
+    unsigned livem = 0, lastm = 0;
+    const unsigned validm = qi >= len ? 0u : (qi + kFI <= len ? 0xffu : ((1u << (len - qi)) - 1u));
+    if (jf == jl) {  // one segment piece: the common case
+      livem = live_l ? validm : 0u;
+      lastm = livem;
+    } else {
+      int j = seg_of(S.off, K, q0 + min(qi, len - 1));
+#pragma unroll
+      for (int k = 0; k < kFI; ++k) {
+        while (j + 1 < K && S.off[j + 1] <= q0 + qi + k) ++j;
+        if (S.cidx[j] >= 0) livem |= 1u << k;
+        if (j == jl) lastm |= 1u << k;
+      }
+      livem &= validm;
+      lastm &= livem;
+    }
+    unsigned w[kFI];
+#pragma unroll
+    for (int k = 0; k < kFI; ++k) w[k] = ((livem >> k) & 1u) ? __ldg(A.hbit + (id[k] >> 5)) : 0u;
+    unsigned bits = 0;
+#pragma unroll
+    for (int k = 0; k < kFI; ++k) bits |= ((w[k] >> (id[k] & 31)) & 1u) << k;
+    bits &= livem;
+    A.tbits[(size_t)t * kFT + tid] = (unsigned char)bits;
+    // the last piece's sums per side, in entry order; last entry per side
+    double sg[2] = {0.0, 0.0}, sh[2] = {0.0, 0.0};
+#pragma unroll
+    for (int k = 0; k < kFI; ++k) {
+      if ((lastm >> k) & 1u) {
+        const double h = hess_of<HMODE>(g[k]);
+        if ((bits >> k) & 1u) { sg[0] = sg[0] + g[k]; sh[0] = sh[0] + h; }
+        else { sg[1] = sg[1] + g[k]; sh[1] = sh[1] + h; }
+      }
+    }
+    const unsigned hm = bits & lastm, lm = ~bits & lastm;
+    int sc[2] = {__popc(hm), __popc(lm)};
+    int si[2] = {hm ? qi + 31 - __clz(hm) : -1, lm ? qi + 31 - __clz(lm) : -1};
+    // block sums: a fixed tree (xor shuffles, then warps in order)
+#pragma unroll
+    for (int s = 0; s < 2; ++s) {
+#pragma unroll
+      for (int o = 16; o; o >>= 1) {
+        sg[s] = sg[s] + __shfl_xor_sync(0xffffffffu, sg[s], o);
+        sh[s] = sh[s] + __shfl_xor_sync(0xffffffffu, sh[s], o);
+        sc[s] += __shfl_xor_sync(0xffffffffu, sc[s], o);
+        si[s] = max(si[s], __shfl_xor_sync(0xffffffffu, si[s], o));
+      }
+      if (lane == 0) {
+        S.wg[par][s][wid] = sg[s]; S.wh[par][s][wid] = sh[s];
+        S.wc[par][s][wid] = sc[s]; S.wi[par][s][wid] = si[s];
+      }
+    }
+    __syncthreads();  // (the other parity's slots are free: one barrier per tile)
+    if (tid < 2) {
+      const int s = tid;
+      double G = 0.0, H = 0.0;
+      int c = 0, ix = -1;
+#pragma unroll
+      for (int w2 = 0; w2 < kFW; ++w2) {
+        G = G + S.wg[par][s][w2]; H = H + S.wh[par][s][w2];
+        c += S.wc[par][s][w2]; ix = max(ix, S.wi[par][s][w2]);
+      }
+      TSide r;
+      const __int128 Gx = c ? to_fx(G, Fg) : 0, Hx = c ? to_fx(H, Fh) : 0;
+      r.g_lo = (unsigned long long)Gx; r.g_hi = (unsigned long long)((unsigned __int128)Gx >> 64);
+      r.h_lo = (unsigned long long)Hx; r.h_hi = (unsigned long long)((unsigned __int128)Hx >> 64);
+      r.cnt = c;
+      r.val = 0.f;  // k_fused reads the value at pos itself
+      r.pos = c ? tbase + ix : 0;
+      const uint4* src4 = reinterpret_cast<const uint4*>(&r);
+      uint4* d4 = reinterpret_cast<uint4*>(&A.tagg[t].s[s]);
+#pragma unroll
+      for (int i = 0; i < 3; ++i) __stcg(d4 + i, src4[i]);
+      if (s == 0) A.treset[t] = (unsigned char)(ql >= 0 || !live_l);  // the piece starts in this tile
+    }
+  }
+}
+
+// ============================================================================ tile scan
+// S1: per group of kTSGroup tiles, the segmented inclusive scan (reset = the tile's last piece
+// starts in it); the group's aggregate and whether a reset occurred up to each tile
+__global__ void __launch_bounds__(kTSGroup) k_tscan1(FusedArgs A) {
+  __shared__ TRec wtot[kTSGroup / 32];
+  __shared__ int wf[kTSGroup / 32];
+  const int T = A.plan->T;
+  const int t = blockIdx.x * kTSGroup + threadIdx.x;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if ((int)(blockIdx.x * kTSGroup) >= T) return;
+  TRec x = t < T ? trec_ld(A.tagg + t) : trec_zero();
+  int f = t < T ? A.treset[t] : 0;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const TRec y = trec_shfl_up(x, o);
+    const int yf = __shfl_up_sync(0xffffffffu, f, o);
+    if (lane >= o) {
+      if (!f) x = trec_add(y, x);
+      f |= yf;
+    }
+  }
+  if (lane == 31) { wtot[wid] = x; wf[wid] = f; }
+  __syncthreads();
+  if (!f) {
+    TRec p = trec_zero();
+    int pf = 0;
+    for (int w = 0; w < wid; ++w) {
+      p = wf[w] ? wtot[w] : trec_add(p, wtot[w]);
+      pf |= wf[w];
+    }
+    x = trec_add(p, x);
+    f = pf;
+  }
+  if (t < T) {
+    trec_st(A.tinc + t, x);
+    A.tseen[t] = (unsigned char)f;
+  }
+  if (threadIdx.x == kTSGroup - 1 || t == T - 1) {
+    trec_st(A.tgagg + blockIdx.x, x);
+    A.tgf[blockIdx.x] = (unsigned char)f;
+  }
+}
+
+// S2: carries between groups: the same segmented scan over the group aggregates, one CTA, in
+// chunks of kTSGroup with a running carry
+__global__ void __launch_bounds__(kTSGroup) k_tscan2(FusedArgs A) {
+  __shared__ TRec wtot[kTSGroup / 32];
+  __shared__ int wf[kTSGroup / 32];
+  __shared__ TRec run;
+  const int T = A.plan->T;
+  const int ng = (T + kTSGroup - 1) / kTSGroup;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if (threadIdx.x == 0) run = trec_zero();
+  __syncthreads();
+  for (int b0 = 0; b0 < ng; b0 += kTSGroup) {
+    const int gi = b0 + threadIdx.x;
+    TRec x = gi < ng ? trec_ld(A.tgagg + gi) : trec_zero();
+    int f = gi < ng ? A.tgf[gi] : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const TRec y = trec_shfl_up(x, o);
+      const int yf = __shfl_up_sync(0xffffffffu, f, o);
+      if (lane >= o) {
+        if (!f) x = trec_add(y, x);
+        f |= yf;
+      }
+    }
+    if (lane == 31) { wtot[wid] = x; wf[wid] = f; }
+    __syncthreads();
+    if (!f) {
+      TRec p = run;
+      for (int w = 0; w < wid; ++w) p = wf[w] ? wtot[w] : trec_add(p, wtot[w]);
+      x = trec_add(p, x);
+    }
+    // exclusive: the inclusive value of the previous group
+    const TRec prev = trec_shfl_up(x, 1);
+    __syncthreads();
+    if (gi < ng) {
+      TRec ex = prev;
+      if (lane == 0) {  // from the previous warp (or the previous chunk)
+        TRec p = run;
+        for (int w = 0; w < wid; ++w) p = wf[w] ? wtot[w] : trec_add(p, wtot[w]);
+        ex = p;
+      }
+      trec_st(A.tgcarry + gi, ex);
+    }
+    __syncthreads();
+    if (gi == min(ng, b0 + kTSGroup) - 1) run = x;
+    __syncthreads();
+  }
+}
+
+// S3: tiles before their group's first reset take the group's carry; the value of each side's
+// last entry is read here once (k_fused's carry then needs no dependent load)
+__global__ void __launch_bounds__(kTSGroup) k_tscan3(FusedArgs A) {
+  const int T = A.plan->T;
+  const int t = blockIdx.x * kTSGroup + threadIdx.x;
+  if (t >= T) return;
+  TRec x = trec_ld(A.tinc + t);
+  if (blockIdx.x > 0 && !A.tseen[t]) x = trec_add(trec_ld(A.tgcarry + blockIdx.x), x);
+  for (int q = 0; q < 2; ++q) x.s[q].val = x.s[q].cnt ? A.val[x.s[q].pos] : 0.f;
+  trec_st(A.tinc + t, x);
+}
+
+// ============================================================================ k_fused
+struct FusedSmem {
+  float val[kFS][kFTile];
+  int32_t ins[kFS][kFTile];
+  double g[kFS][kFTile];
+  unsigned short src[kFTile];       // child order: slot r holds tile entry src[r]
+  float cval[kFTile];               // single-piece tiles: the entries moved into child order
+  int32_t cins[kFTile];
+  double cg[kFTile];
+  int rowc[kFTile / 32];            // per 32-entry row: packed (high | low << 16) counts, then their scan
+  int tot;
+  unsigned long long bar[kFS];
+  // plan copy
+  int off[kFusedMaxK + 1];
+  int cidx[kFusedMaxK];
+  int offn[2 * kFusedMaxK + 1];
+  double cG[2 * kFusedMaxK], cH[2 * kFusedMaxK], cHl[2 * kFusedMaxK], cP[2 * kFusedMaxK];
+  // CTA node-best table (children)
+  unsigned long long ngk[2 * kFusedMaxK];
+  // per tile
+  int j0, nseg, nk, cont;
+  int pq[kFusedMaxK + 1];           // tile-relative start of piece s (pq[nseg] = tile length)
+  int base[kFusedMaxK + 1];         // packed exclusive (high | low << 16) count at piece start
+  int gb[2 * kFusedMaxK + 1];       // child-order group starts: group 2s = piece s high, 2s+1 low
+  unsigned long long gk[2 * kFusedMaxK];
+  int wr[2 * kFusedMaxK];
+  int wsum[kFW];
+  double wg[kFW], wh[kFW];
+  int wf[kFW];
+  TSide ex[2];                      // carry of the first piece (the tile scan's record of t - 1)
+  double cgx[2], chx[2];            // the carry's sums as fp64 (single-piece path)
+};
 
 // rank score of a split, GL^2/(HL+l) + GR^2/(HR+l) = 2 Eq.2 + const, kept as num / den:
 // candidates of a thread's run are compared by cross-multiplication (no division); the run's
@@ -250,47 +438,42 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
     S.cG[c] = A.nxt.G[c]; S.cH[c] = A.nxt.H[c]; S.cHl[c] = __dadd_rn(A.nxt.H[c], lam); S.cP[c] = A.nxt.pterm[c];
     S.ngk[c] = 0ull;
   }
+  Rec* const nrec = A.cta_rec + (size_t)blockIdx.x * (2 * kFusedMaxK);  // CTA node-best records (global, L1)
   const unsigned long long pol = policy_evict_first();
-  // Tickets are dealt round-robin over the attributes (ticket u -> tile u / m of attribute u % m):
-  // every attribute's segments form their own look-back chains, so a chain has ~1/m of the tiles
-  // in flight and a look-back rarely reads more than one 32-tile window.  Tile index t = a * tpa + k
-  // (the look-back predecessor of t is t - 1).
-  const int mm = A.m;
-  auto tile_of = [&](int u) { return (u % mm) * tpa + u / mm; };
-  auto issue = [&](int t) {  // TMA of tile t's lists
+  auto issue = [&](int st, int t) {  // TMA of tile t's lists into stage st
     const int a = t / tpa;
     const int q0 = (t - a * tpa) * kFTile;
     const long long p0 = (long long)a * stride + q0;
     const uint32_t n = (uint32_t)((min(kFTile, n_act - q0) + 3) & ~3);
-    mbar_arrive_expect_tx(&S.bar, 16u * n);
-    tma_load_1d(S.val, A.val + p0, 4u * n, &S.bar, pol);
-    tma_load_1d(S.ins, A.ins + p0, 4u * n, &S.bar, pol);
-    tma_load_1d(S.g, A.gl + p0, 8u * n, &S.bar, pol);
+    mbar_arrive_expect_tx(&S.bar[st], 16u * n);
+    tma_load_1d(S.val[st], A.val + p0, 4u * n, &S.bar[st], pol);
+    tma_load_1d(S.ins[st], A.ins + p0, 4u * n, &S.bar[st], pol);
+    tma_load_1d(S.g[st], A.gl + p0, 8u * n, &S.bar[st], pol);
   };
   if (tid == 0) {
-    mbar_init(&S.bar, 1);
+    for (int st = 0; st < kFS; ++st) mbar_init(&S.bar[st], 1);
     fence_mbar_init();
-    const int u = atomicAdd(A.ticket, 1);
-    S.tile = u;
-    if (u < T) issue(tile_of(u));
+    for (int st = 0; st < kFS; ++st) {
+      const int t = blockIdx.x + st * gridDim.x;
+      if (t < T) issue(st, t);
+    }
   }
   __syncthreads();
   uint32_t phase = 0;
   const int qi = tid * kFI;
-  while (true) {
-    const int u = S.tile;
-    if (u >= T) break;
-    const int t = tile_of(u);
+  for (int it = 0;; ++it) {
+    const int t = blockIdx.x + it * gridDim.x;
+    if (t >= T) break;
+    const int st = it % kFS;
     const int a = t / tpa;
     const int q0 = (t - a * tpa) * kFTile;
     const int len = min(kFTile, n_act - q0);
     const long long tbase = (long long)a * stride + q0;
+    const float* sval = S.val[st];
+    const int32_t* sins = S.ins[st];
+    const double* sg = S.g[st];
     if (tid == 0) {  // the tile's pieces (parent segments), while the copy is in flight
-      int lo = 0, hi = K - 1;
-      while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (S.off[mid] <= q0) lo = mid; else hi = mid - 1;
-      }
+      const int lo = seg_of(S.off, K, q0);
       int s = 0;
       S.pq[0] = 0;
       while (S.off[lo + s + 1] < q0 + len) { ++s; S.pq[s] = S.off[lo + s] - q0; }
@@ -298,24 +481,248 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
       S.j0 = lo;
       S.nseg = s + 1;
       S.cont = S.off[lo] < q0 && S.cidx[lo] >= 0;
+    } else if (tid >= 32 && tid < 38) {  // carry of the first piece: the scanned record of t - 1
+      const int lo = seg_of(S.off, K, q0);
+      const bool c = S.off[lo] < q0 && S.cidx[lo] >= 0;
+      uint4* d = reinterpret_cast<uint4*>(S.ex);
+      d[tid - 32] = c ? __ldcg(reinterpret_cast<const uint4*>(A.tinc + (t - 1)) + (tid - 32)) : make_uint4(0, 0, 0, 0);
     }
-    mbar_wait(&S.bar, phase);
-    phase ^= 1u;
+    const unsigned tb = A.tbits[(size_t)t * kFT + tid];
+    mbar_wait(&S.bar[st], (phase >> st) & 1);
+    phase ^= 1u << st;
     __syncthreads();
     const int j0 = S.j0, nseg = S.nseg;
     const bool cont = S.cont != 0;
+    bool issued = false;  // thread 0: the next tile's copy into this stage has been started
 
-    // ---- 1. child side of every entry; stable in-tile partition by (piece, side) -> src[]
-    int sidx[kFI];
+    if (nseg == 1) {
+      // ================= one segment piece (the common case): two child runs, high then low.
+      //  1. striped (entry k*256 + 32 w + lane): side bits per 32-entry row from k_tile_agg's
+      //     words, ranks by popc, the rows' counts scanned by one warp; entries MOVED into the
+      //     child-order buffer (consecutive lanes -> consecutive slots, no bank conflicts), after
+      //     which the stage is free and the next tile's copy starts
+      //  2. blocked (child slots 8 tid .. 8 tid + 7, 16-byte loads): segmented scans, candidates
+      //  3. striped: coalesced stores of the child runs
+      const int c0 = S.cidx[j0];
+      if (c0 >= 0) {
+        const unsigned* words = reinterpret_cast<const unsigned*>(A.tbits) + (size_t)t * (kFTile / 32);
+        const unsigned myw = lane < kFI ? __ldg(words + lane * kFW + wid) : 0u;
+        const unsigned ltm = (1u << lane) - 1u;
+        const bool full = len == kFTile;
+        unsigned wk[kFI];
+#pragma unroll
+        for (int k = 0; k < kFI; ++k) {
+          const int e0 = k * kFT + 32 * wid;  // the row's first entry
+          const unsigned vm = full ? 0xffffffffu : (e0 >= len ? 0u : (e0 + 32 <= len ? 0xffffffffu : ((1u << (len - e0)) - 1u)));
+          wk[k] = __shfl_sync(0xffffffffu, myw, k) & vm;
+          if (lane == 0) S.rowc[k * kFW + wid] = __popc(wk[k]) | ((__popc(vm) - __popc(wk[k])) << 16);
+        }
+        __syncthreads();
+        if (wid == 0) {  // exclusive scan of the 64 row counts (2 per lane), in tile order
+          const int x0 = S.rowc[2 * lane], x1 = S.rowc[2 * lane + 1];
+          int incl = x0 + x1;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += y;
+          }
+          const int exl = incl - x0 - x1;
+          S.rowc[2 * lane] = exl;
+          S.rowc[2 * lane + 1] = exl + x0;
+          if (lane == 31) S.tot = incl;
+          if (lane == 0) {
+            S.gk[0] = S.gk[1] = 0ull;
+            S.wr[0] = S.wr[1] = INT_MAX;
+            for (int q = 0; q < 2; ++q) {  // the carries as fp64, once
+              S.cgx[q] = cont ? from_fx((__int128)u128(S.ex[q].g_lo, S.ex[q].g_hi), Fg) : 0.0;
+              S.chx[q] = cont ? from_fx((__int128)u128(S.ex[q].h_lo, S.ex[q].h_hi), Fh) : 0.0;
+            }
+          }
+        }
+        __syncthreads();
+        const int NH = S.tot & 0xffff, NK = NH + (S.tot >> 16);
+#pragma unroll
+        for (int k = 0; k < kFI; ++k) {  // move into child order
+          const int e = k * kFT + 32 * wid + lane;
+          if (full || e < len) {
+            const int b = S.rowc[k * kFW + wid];
+            const bool hi = (wk[k] >> lane) & 1u;
+            const int rh = __popc(wk[k] & ltm);  // high entries before this lane in the row
+            const int r = hi ? (b & 0xffff) + rh : NH + (b >> 16) + (lane - rh);  // all lanes < e are valid
+            S.cval[r] = sval[e];
+            S.cins[r] = sins[e];
+            S.cg[r] = sg[e];
+            S.src[r] = (unsigned short)e;
+          }
+        }
+        __syncthreads();
+        if (tid == 0) {  // the stage is drained: start the next tile's copy now
+          const int t2 = t + kFS * gridDim.x;
+          if (t2 < T) {
+            fence_proxy_async();
+            issue(st, t2);
+          }
+          issued = true;
+        }
+        // child-order slots r = qi .. qi + 7: high run [0, NH), low run [NH, NK); heads at 0, NH
+        double gv[kFI], hv[kFI];
+        float vv[kFI];
+        {
+          const double2* pg = reinterpret_cast<const double2*>(S.cg + qi);
+          const float4* pv = reinterpret_cast<const float4*>(S.cval + qi);
+#pragma unroll
+          for (int k = 0; k < kFI / 2; ++k) {
+            const double2 z = pg[k];
+            gv[2 * k] = z.x;
+            gv[2 * k + 1] = z.y;
+          }
+          const float4 a0 = pv[0], a1 = pv[1];
+          vv[0] = a0.x; vv[1] = a0.y; vv[2] = a0.z; vv[3] = a0.w; vv[4] = a1.x; vv[5] = a1.y; vv[6] = a1.z; vv[7] = a1.w;
+        }
+        const int kh = NH - qi;  // item index of slot NH in this thread, if 0 <= kh < kFI
+        const unsigned headm = (qi == 0 ? 1u : 0u) | ((kh >= 0 && kh < kFI && NH < NK) ? (1u << kh) : 0u);
+        const int nin = min(kFI, NK - qi);  // slots of this thread (may be <= 0)
+        double ag = 0.0, ah = 0.0;
+#pragma unroll
+        for (int k = 0; k < kFI; ++k) {
+          hv[k] = hess_of<HMODE>(gv[k]);
+          if (k < nin) {
+            if ((headm >> k) & 1u) { ag = gv[k]; ah = hv[k]; }
+            else { ag = ag + gv[k]; ah = ah + hv[k]; }
+          }
+        }
+        double ig = ag, ih = ah;
+        int iflag = headm != 0u;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const double yg = __shfl_up_sync(0xffffffffu, ig, o), yh = __shfl_up_sync(0xffffffffu, ih, o);
+          const int yf = __shfl_up_sync(0xffffffffu, iflag, o);
+          if (lane >= o) {
+            if (!iflag) { ig = yg + ig; ih = yh + ih; }
+            iflag |= yf;
+          }
+        }
+        if (lane == 31) { S.wg[wid] = ig; S.wh[wid] = ih; S.wf[wid] = iflag; }
+        double eg = __shfl_up_sync(0xffffffffu, ig, 1), eh = __shfl_up_sync(0xffffffffu, ih, 1);
+        int ef = __shfl_up_sync(0xffffffffu, iflag, 1);
+        if (lane == 0) { eg = 0.0; eh = 0.0; ef = 0; }
+        __syncthreads();
+        if (!ef) {
+          double pg = 0.0, ph = 0.0;
+          for (int w = 0; w < wid; ++w) {
+            if (S.wf[w]) { pg = S.wg[w]; ph = S.wh[w]; }
+            else { pg = pg + S.wg[w]; ph = ph + S.wh[w]; }
+          }
+          eg = pg + eg;
+          eh = ph + eh;
+        }
+        // GL, HL of a slot = carry of its run + the tile's sum over the run's earlier slots,
+        // associated as (carry + eg) + g_k ... (fixed, so ranking and record agree)
+        const int q0s = qi < NH ? 0 : 1;  // run of the thread's first slot
+        const double sg0 = S.cgx[q0s] + eg, sh0 = S.chx[q0s] + eh;
+        int ra_g = -1, rb_g = -1, ra_r = -1, rb_r = -1;
+        unsigned long long ra_k = 0ull, rb_k = 0ull;
+        double aGL = 0, aHL = 0, bGL = 0, bHL = 0;
+        if (nin > 0) {
+          int q = q0s;
+          int c = c0 + q;
+          double Gc = S.cG[c], Hl = S.cHl[c];
+          double rg = sg0, rh = sh0;
+          double bnum = -1.0, bden = 1.0, bGLc = 0.0, bHLc = 0.0;
+          int br = -1;
+          float pv;
+          bool prev;
+          if (qi != 0 && qi != NH) { pv = S.cval[qi - 1]; prev = true; }
+          else { prev = cont && S.ex[q].cnt > 0; pv = S.ex[q].val; }
+#pragma unroll
+          for (int k = 0; k < kFI; ++k) {
+            if (k < nin) {
+              const int r = qi + k;
+              if ((headm >> k) & 1u) {
+                if (k > 0) {  // the low run starts inside this thread: close the high one
+                  if (br >= 0) { ra_g = 0; ra_r = br; aGL = bGLc; aHL = bHLc; }
+                  q = 1; c = c0 + 1; Gc = S.cG[c]; Hl = S.cHl[c];
+                  bnum = -1.0; bden = 1.0; br = -1;
+                  prev = cont && S.ex[1].cnt > 0;
+                  pv = S.ex[1].val;
+                }
+                rg = S.cgx[q];
+                rh = S.chx[q];
+              }
+              const float cv = vv[k];
+              if (prev && pv != cv) {
+                const double dl = rh + lam, dr = Hl - rh, GR = Gc - rg;
+                const double num = __fma_rn(rg * rg, dr, (GR * GR) * dl), den = dl * dr;
+                if (num * bden > bnum * den) { bnum = num; bden = den; br = r; bGLc = rg; bHLc = rh; }
+              }
+              rg = rg + gv[k];
+              rh = rh + hv[k];
+              pv = cv;
+              prev = true;
+            }
+          }
+          if (br >= 0) {
+            if (ra_g < 0 && !(q == 1 && qi < NH)) { ra_g = q; ra_r = br; aGL = bGLc; aHL = bHLc; }
+            else { rb_g = q; rb_r = br; bGL = bGLc; bHL = bHLc; }
+          }
+        }
+        if (ra_g >= 0) { const int c = c0 + ra_g; ra_k = gain_key(eq2_gain(aGL, aHL, S.cG[c], S.cH[c], lam, S.cP[c])); }
+        if (rb_g >= 0) { const int c = c0 + rb_g; rb_k = gain_key(eq2_gain(bGL, bHL, S.cG[c], S.cH[c], lam, S.cP[c])); }
+        {  // group maxima: the first run through a warp reduction, the other one directly
+          const unsigned peers = __match_any_sync(0xffffffffu, ra_g);
+          const unsigned hi = __reduce_max_sync(peers, (unsigned)(ra_k >> 32));
+          const unsigned lo = __reduce_max_sync(peers, (unsigned)(ra_k >> 32) == hi ? (unsigned)ra_k : 0u);
+          if (ra_g >= 0 && lane == __ffs(peers) - 1) atomicMax(&S.gk[ra_g], ((unsigned long long)hi << 32) | lo);
+          if (rb_g >= 0) atomicMax(&S.gk[rb_g], rb_k);
+        }
+        __syncthreads();
+        if (ra_g >= 0 && ra_k == S.gk[ra_g]) atomicMin(&S.wr[ra_g], ra_r);  // ties: the larger value
+        if (rb_g >= 0 && rb_k == S.gk[rb_g]) atomicMin(&S.wr[rb_g], rb_r);
+        __syncthreads();
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+          const int gq = i ? rb_g : ra_g, r = i ? rb_r : ra_r;
+          const unsigned long long key = i ? rb_k : ra_k;
+          if (gq < 0 || S.wr[gq] != r || key != S.gk[gq]) continue;
+          const int gs = gq ? NH : 0;
+          const int c = c0 + gq;
+          Rec rc;
+          rc.GL = i ? bGL : aGL;
+          rc.HL = i ? bHL : aHL;
+          rc.cntL = (cont ? S.ex[gq].cnt : 0) + (r - gs);
+          rc.gain = eq2_gain(rc.GL, rc.HL, S.cG[c], S.cH[c], lam, S.cP[c]);
+          rc.value = r > gs ? S.cval[r - 1] : S.ex[gq].val;
+          rc.pos = r > gs ? tbase + S.src[r - 1] : S.ex[gq].pos;
+          rc.attr = A.a_base + a;
+          rc.dir = 0;
+          rc.node = c;
+          rc.epoch = (int)ep;
+          rc.shard = A.shard;
+          if (rec_better_f(key, rc, S.ngk[c], nrec[c])) {  // one writer per child node per tile
+            nrec[c] = rc;
+            S.ngk[c] = key;
+          }
+        }
+        if (kWrite) {  // child runs -> the next level's lists, 32 consecutive slots per warp
+          const long long bh = (long long)a * stride_n + S.offn[c0] + (cont ? S.ex[0].cnt : 0);
+          const long long bl = (long long)a * stride_n + S.offn[c0 + 1] + (cont ? S.ex[1].cnt : 0) - NH;
+          for (int r = tid; r < NK; r += kFT) {
+            const long long d = (r < NH ? bh : bl) + r;
+            __stcs(A.val_out + d, S.cval[r]);
+            __stcs(A.ins_out + d, S.cins[r]);
+            __stcs(A.g_out + d, S.cg[r]);
+          }
+        }
+      }
+    } else {
+#ifndef GBDT_FUSED_NO_GENERAL
+    // ---- 1. stable in-tile partition by (piece, side) -> src[]
+    int sidx[kFI];  // piece << 2 | side (1 high, 2 low); -1 dropped
     {
-      const int4 i0 = reinterpret_cast<const int4*>(S.ins + qi)[0];
-      const int4 i1 = reinterpret_cast<const int4*>(S.ins + qi)[1];
-      const int id[kFI] = {i0.x, i0.y, i0.z, i0.w, i1.x, i1.y, i1.z, i1.w};
       int s = 0;
       while (s + 1 < nseg && qi >= S.pq[s + 1]) ++s;
       int nb = S.pq[s + 1];
       bool live = S.cidx[j0 + s] >= 0;
-      unsigned w[kFI];
 #pragma unroll
       for (int k = 0; k < kFI; ++k) {
         if (qi + k >= nb && s + 1 < nseg) {
@@ -323,12 +730,8 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
           nb = S.pq[s + 1];
           live = S.cidx[j0 + s] >= 0;
         }
-        sidx[k] = (qi + k < len && live) ? s : -1;
-        w[k] = sidx[k] >= 0 ? __ldg(A.hbit + (id[k] >> 5)) : 0u;
+        sidx[k] = (qi + k < len && live) ? ((s << 2) | (((tb >> k) & 1u) ? 1 : 2)) : -1;
       }
-#pragma unroll
-      for (int k = 0; k < kFI; ++k)  // piece index << 2 | side (1 high, 2 low); -1 dropped
-        sidx[k] = sidx[k] < 0 ? -1 : ((sidx[k] << 2) | (((w[k] >> (id[k] & 31)) & 1u) ? 1 : 2));
     }
     int pc = 0;
 #pragma unroll
@@ -402,7 +805,7 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
             if (k) gstep |= 1u << k;
           }
           if (r == S.gb[gg]) headm |= 1u << k;
-          xg[k] = S.g[sr[k]];
+          xg[k] = sg[sr[k]];
           xh[k] = hess_of<HMODE>(xg[k]);
         }
       }
@@ -439,77 +842,20 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
       eg = pg + eg;
       eh = ph + eh;
     }
-    // exclusive in-tile prefix per slot (replaces g, h); the last piece's group totals
-    {
+    {  // exclusive in-tile prefix per slot (replaces g, h)
       double rg = eg, rh = eh;
-      int gg = grp0;
 #pragma unroll
       for (int k = 0; k < kFI; ++k) {
-        const int r = qi + k;
-        if (r < nk) {
-          if ((gstep >> k) & 1u) { while (r >= S.gb[gg + 1]) ++gg; }
-          if ((headm >> k) & 1u) { rg = 0.0; rh = 0.0; }
-          const double ng_ = rg + xg[k], nh_ = rh + xh[k];
-          if ((gg >> 1) == nseg - 1 && r + 1 == S.gb[gg + 1]) {
-            S.lg[gg & 1] = ng_;
-            S.lh[gg & 1] = nh_;
-            S.lv[gg & 1] = S.val[sr[k]];
-            S.ls[gg & 1] = sr[k];
-          }
-          xg[k] = rg;
-          xh[k] = rh;
-          rg = ng_;
-          rh = nh_;
-        }
+        if ((headm >> k) & 1u) { rg = 0.0; rh = 0.0; }
+        const double ng_ = rg + xg[k], nh_ = rh + xh[k];
+        xg[k] = rg;
+        xh[k] = rh;
+        rg = ng_;
+        rh = nh_;
       }
     }
-    __syncthreads();
 
-    // ---- 3. publish this tile's record; look back for the first piece's carry
-    if (wid == 0) {
-      const int jl = j0 + nseg - 1;
-      LBSide rec[2];
-      if (lane == 0) {
-        const bool live = S.cidx[jl] >= 0;
-        for (int q = 0; q < 2; ++q) {
-          const int cnt = live ? S.gb[2 * (nseg - 1) + q + 1] - S.gb[2 * (nseg - 1) + q] : 0;
-          const __int128 G = cnt ? to_fx(S.lg[q], Fg) : 0, H = cnt ? to_fx(S.lh[q], Fh) : 0;
-          rec[q].g_lo = (unsigned long long)G; rec[q].g_hi = (unsigned long long)((unsigned __int128)G >> 64);
-          rec[q].h_lo = (unsigned long long)H; rec[q].h_hi = (unsigned long long)((unsigned __int128)H >> 64);
-          rec[q].cnt = cnt;
-          rec[q].val = cnt ? S.lv[q] : 0.f;
-          rec[q].pos = cnt ? tbase + S.ls[q] : 0;
-        }
-        const bool last_cont = live && S.off[jl] < q0;  // the last piece began in an earlier tile
-        lb_store((last_cont ? lb_agg(A) : lb_inc(A)) + t, rec);
-        __threadfence();
-        st_release_u32(A.lb_status + t, (ep << 2) | (last_cont ? kLBAgg : kLBInc));
-      }
-      if (cont) {
-        lookback(A, t, a * tpa + S.off[j0] / kFTile, ep, S.ex, lane);
-        if (lane == 0 && nseg == 1) {  // the first piece is the last one: inclusive = carry + own
-          LBSide inc[2];
-          for (int q = 0; q < 2; ++q) {
-            const unsigned __int128 G = u128(S.ex[q].g_lo, S.ex[q].g_hi) + u128(rec[q].g_lo, rec[q].g_hi);
-            const unsigned __int128 H = u128(S.ex[q].h_lo, S.ex[q].h_hi) + u128(rec[q].h_lo, rec[q].h_hi);
-            inc[q].g_lo = (unsigned long long)G; inc[q].g_hi = (unsigned long long)(G >> 64);
-            inc[q].h_lo = (unsigned long long)H; inc[q].h_hi = (unsigned long long)(H >> 64);
-            inc[q].cnt = S.ex[q].cnt + rec[q].cnt;
-            inc[q].val = rec[q].cnt ? rec[q].val : S.ex[q].val;
-            inc[q].pos = rec[q].cnt ? rec[q].pos : S.ex[q].pos;
-          }
-          lb_store(lb_inc(A) + t, inc);
-          __threadfence();
-          st_release_u32(A.lb_status + t, (ep << 2) | kLBInc);
-        }
-      } else if (lane < 2) {
-        S.ex[lane].g_lo = S.ex[lane].g_hi = S.ex[lane].h_lo = S.ex[lane].h_hi = 0ull;
-        S.ex[lane].cnt = 0; S.ex[lane].val = 0.f; S.ex[lane].pos = 0;
-      }
-    }
-    __syncthreads();
-
-    // ---- 4. candidates: the boundary before every child entry whose predecessor in its child
+    // ---- 3. candidates: the boundary before every child entry whose predecessor in its child
     // segment has another value (the predecessor ends a run); GL, HL = sums over the
     // predecessor and everything before it.  Per run of the thread's slots in one group: the
     // best by score, then its exact Eq. 2 gain.
@@ -536,7 +882,7 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
       Cand b{-1.0, 1.0, 0.0, 0.0, -1};
       float pv;
       bool prev;
-      if (qi > gs) { pv = S.val[S.src[qi - 1]]; prev = true; }
+      if (qi > gs) { pv = sval[S.src[qi - 1]]; prev = true; }
       else { prev = carry && S.ex[q].cnt > 0; pv = S.ex[q].val; }
 #pragma unroll
       for (int k = 0; k < kFI; ++k) {
@@ -560,7 +906,7 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
             prev = carry && S.ex[q].cnt > 0;
             pv = S.ex[q].val;
           }
-          const float cv = S.val[sr[k]];
+          const float cv = sval[sr[k]];
           if (prev && pv != cv) {
             const double GL = carry ? __dadd_rn(q ? cgx[1] : cgx[0], xg[k]) : xg[k];
             const double HL = carry ? __dadd_rn(q ? chx[1] : chx[0], xh[k]) : xh[k];
@@ -606,25 +952,24 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
       rc.cntL = (carry ? S.ex[q].cnt : 0) + (r - gs);
       rc.gain = eq2_gain(rc.GL, rc.HL, S.cG[c], S.cH[c], lam, S.cP[c]);
       const int ps = r > gs ? S.src[r - 1] : -1;
-      rc.value = ps >= 0 ? S.val[ps] : S.ex[q].val;
+      rc.value = ps >= 0 ? sval[ps] : S.ex[q].val;
       rc.pos = ps >= 0 ? tbase + ps : S.ex[q].pos;
       rc.attr = A.a_base + a;
       rc.dir = 0;
       rc.node = c;
       rc.epoch = (int)ep;
       rc.shard = A.shard;
-      if (rec_better_f(rkey[i], rc, S.ngk[c], S.nrec[c])) {  // one writer per child node per tile
-        S.nrec[c] = rc;
+      if (rec_better_f(rkey[i], rc, S.ngk[c], nrec[c])) {  // one writer per child node per tile
+        nrec[c] = rc;
         S.ngk[c] = rkey[i];
       }
     }
-    // ---- 5. child runs -> the next level's lists (coalesced: 32 consecutive slots per warp)
+    // ---- 4. child runs -> the next level's lists (coalesced: 32 consecutive slots per warp)
     if (kWrite) {
-      int gg = -1, gn = 0;
+      int gg = 0, gn = -1;
       long long dbase = 0;
       for (int r = tid; r < nk; r += kFT) {
         if (r >= gn) {
-          if (gg < 0) gg = 0;
           while (r >= S.gb[gg + 1]) ++gg;
           gn = S.gb[gg + 1];
           const int s = gg >> 1, q = gg & 1;
@@ -632,35 +977,37 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
                   S.gb[gg];
         }
         const int e = S.src[r];
-        __stcs(A.val_out + dbase + r, S.val[e]);
-        __stcs(A.ins_out + dbase + r, S.ins[e]);
-        __stcs(A.g_out + dbase + r, S.g[e]);
+        __stcs(A.val_out + dbase + r, sval[e]);
+        __stcs(A.ins_out + dbase + r, sins[e]);
+        __stcs(A.g_out + dbase + r, sg[e]);
       }
     }
-    __syncthreads();  // the tile and its scratch are free
-    if (tid == 0) {
-      const int u2 = atomicAdd(A.ticket, 1);
-      S.tile = u2;
-      if (u2 < T) {
+#endif
+    }  // general path
+    __syncthreads();  // stage st and the tile scratch are free
+    if (tid == 0 && !issued) {
+      const int t2 = t + kFS * gridDim.x;
+      if (t2 < T) {
         fence_proxy_async();
-        issue(tile_of(u2));
+        issue(st, t2);
       }
     }
-    __syncthreads();
   }
+  __syncthreads();
   // flush the CTA's node bests (R12 merge across CTAs by k_pick_tie / k_pick_best)
   for (int c = tid; c < Kn; c += kFT) {
     if (S.ngk[c]) {
       const int gs = atomicAdd(A.nrec, 1);
-      A.rec[gs] = S.nrec[c];
+      A.rec[gs] = nrec[c];
       atomicMax(A.gkey + c, S.ngk[c]);
     }
   }
 }
 
-// One block: the level's segment offsets, child offsets / parents, tile count; resets the ticket.
+// ============================================================================ plan + mark
+// One thread: the level's segment offsets, child offsets / parents, tile count.
 __global__ void k_fused_plan(FusedPlan* P, NodeTab cur, NodeTab nxt, const int32_t* __restrict__ cidx,
-                             const int* __restrict__ epoch, int m, int* ticket, unsigned long long* lent, int lvl) {
+                             const int* __restrict__ epoch, int m, unsigned long long* lent, int lvl) {
   if (threadIdx.x != 0) return;
   const int K = *cur.K, Kn = *nxt.K;
   P->K = K;
@@ -686,7 +1033,6 @@ __global__ void k_fused_plan(FusedPlan* P, NodeTab cur, NodeTab nxt, const int32
   P->tpa = (o + kFTile - 1) / kFTile;
   P->T = Kn > 0 ? m * P->tpa : 0;
   P->epoch = *epoch;
-  *ticket = 0;
   if (lent) lent[lvl + 1] += (unsigned long long)on * (unsigned long long)m;
 }
 
@@ -715,6 +1061,7 @@ __global__ void k_mark_fused(const FusedPlan* __restrict__ P, const int32_t* __r
 }
 
 unsigned g_fused_grid[2][2] = {{0, 0}, {0, 0}};
+unsigned g_agg_grid = 0;
 
 template <int HM, bool W>
 void set_fused(int sms) {
@@ -723,31 +1070,61 @@ void set_fused(int sms) {
   int occ = 0;
   GBDT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fused<HM, W>, kFT, smem));
   if (occ < 1) fail(GBDT_E_CUDA, "k_fused does not fit on an SM");
-  g_fused_grid[HM][W ? 1 : 0] = (unsigned)(occ * sms);
+  g_fused_grid[HM][W ? 1 : 0] = (unsigned)std::min(occ * sms, kFusedMaxCTAs);
 }
 
 }  // namespace
 
-size_t fused_lb_bytes(int64_t max_tiles) { return (size_t)max_tiles * (sizeof(LBRec) * 2 + 4); }
+size_t fused_tile_bytes(int64_t max_tiles) {
+  const int64_t groups = (max_tiles + kTSGroup - 1) / kTSGroup + 1;
+  return (size_t)max_tiles * (2 * sizeof(TRec) + 2 + kFT) + (size_t)groups * (2 * sizeof(TRec) + 1) + 8192 +
+         sizeof(Rec) * 2 * kFusedMaxK * (size_t)kFusedMaxCTAs;
+}
 int64_t fused_tiles(int64_t n, int m) { return (int64_t)m * ((n + kFTile - 1) / kFTile); }
+
+void fused_carve(FusedArgs& A, void* base, int64_t max_tiles) {
+  const int64_t groups = (max_tiles + kTSGroup - 1) / kTSGroup + 1;
+  char* p = static_cast<char*>(base);
+  auto take = [&](size_t b) { char* r = p; p += (b + 255) & ~size_t(255); return r; };
+  A.cta_rec = reinterpret_cast<Rec*>(take(sizeof(Rec) * 2 * kFusedMaxK * (size_t)kFusedMaxCTAs));
+  A.tagg = reinterpret_cast<TRec*>(take(sizeof(TRec) * max_tiles));
+  A.tinc = reinterpret_cast<TRec*>(take(sizeof(TRec) * max_tiles));
+  A.tgagg = reinterpret_cast<TRec*>(take(sizeof(TRec) * groups));
+  A.tgcarry = reinterpret_cast<TRec*>(take(sizeof(TRec) * groups));
+  A.treset = reinterpret_cast<unsigned char*>(take(max_tiles));
+  A.tseen = reinterpret_cast<unsigned char*>(take(max_tiles));
+  A.tgf = reinterpret_cast<unsigned char*>(take(groups));
+  A.tbits = reinterpret_cast<unsigned char*>(take((size_t)kFT * max_tiles));
+}
 
 void fused_init(int sms) {
   set_fused<kHConst2, true>(sms);
   set_fused<kHConst2, false>(sms);
   set_fused<kHFromG, true>(sms);
   set_fused<kHFromG, false>(sms);
+  int occ = 0;
+  GBDT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tile_agg<kHFromG>, kFT, 0));
+  g_agg_grid = (unsigned)(std::max(occ, 1) * sms);
 }
 
 unsigned fused_grid(int hmode) { return std::max(g_fused_grid[hmode][0], g_fused_grid[hmode][1]); }
 
 void fused_plan(FusedPlan* P, const NodeTab& cur, const NodeTab& nxt, const int32_t* cidx, const int* epoch, int m,
-                int* ticket, unsigned long long* lent, int lvl, cudaStream_t st) {
-  k_fused_plan<<<1, 32, 0, st>>>(P, cur, nxt, cidx, epoch, m, ticket, lent, lvl);
+                unsigned long long* lent, int lvl, cudaStream_t st) {
+  k_fused_plan<<<1, 32, 0, st>>>(P, cur, nxt, cidx, epoch, m, lent, lvl);
   GBDT_LAUNCH_CHECK();
   count_launch();
 }
 
-void fused_pass(const FusedArgs& A, int hmode, bool write, cudaStream_t st) {
+void fused_pass(const FusedArgs& A, int hmode, bool write, int64_t max_tiles, cudaStream_t st) {
+  // tile sides + aggregates, the exact tile scan, then the fused pass itself
+  const unsigned ga = (unsigned)std::max<int64_t>(1, std::min<int64_t>(max_tiles, g_agg_grid));
+  if (hmode == kHConst2) k_tile_agg<kHConst2><<<ga, kFT, 0, st>>>(A);
+  else k_tile_agg<kHFromG><<<ga, kFT, 0, st>>>(A);
+  const unsigned gs = (unsigned)std::max<int64_t>(1, (max_tiles + kTSGroup - 1) / kTSGroup);
+  k_tscan1<<<gs, kTSGroup, 0, st>>>(A);
+  k_tscan2<<<1, kTSGroup, 0, st>>>(A);
+  k_tscan3<<<gs, kTSGroup, 0, st>>>(A);
   const size_t smem = sizeof(FusedSmem);
   const unsigned grid = g_fused_grid[hmode][write ? 1 : 0];
   if (hmode == kHConst2) {
@@ -758,7 +1135,7 @@ void fused_pass(const FusedArgs& A, int hmode, bool write, cudaStream_t st) {
     else k_fused<kHFromG, false><<<grid, kFT, smem, st>>>(A);
   }
   GBDT_LAUNCH_CHECK();
-  count_launch();
+  count_launch(5);
 }
 
 void fused_mark(const FusedPlan* P, const int32_t* Kp, const int32_t* cidx, const Rec* winner, int shard, int a_base,

@@ -149,6 +149,17 @@ struct FusedPlan {            // device, written by k_fused_plan
   int offn[2 * kFusedMaxK + 1];  // child segment starts in the next level's lists
   int pj[2 * kFusedMaxK];     // parent of child c
 };
+// Per child side (0 high, 1 low) of a tile's last segment piece: entries, exact fixed-point
+// (g, h) sums, value and level position of the last one (fused.cu tile records / carries)
+struct __align__(16) TSide {
+  unsigned long long g_lo, g_hi, h_lo, h_hi;
+  long long pos;
+  int cnt;
+  float val;
+};
+struct __align__(16) TRec {
+  TSide s[2];
+};
 struct FusedArgs {
   const float* val;           // level l lists (val, ins, g-list)
   const int32_t* ins;
@@ -159,10 +170,16 @@ struct FusedArgs {
   const uint32_t* hbit;       // instance -> high-child bit of level l's splits
   const FusedPlan* plan;
   NodeTab nxt;                // the children: G, H, pterm
-  unsigned* lb_status;        // [tiles] look-back status (epoch << 2 | 1 aggregate / 2 inclusive)
-  void* lb_agg_;              // [tiles] look-back records (fused.cu LBRec)
-  void* lb_inc_;
-  int* ticket;                // tile claim counter (reset by the plan)
+  // per tile (fused_carve): records, scanned carries, side bits
+  TRec* tagg;
+  TRec* tinc;
+  TRec* tgagg;
+  TRec* tgcarry;
+  unsigned char* treset;
+  unsigned char* tseen;
+  unsigned char* tgf;
+  unsigned char* tbits;       // [tiles][256]: bit k of byte i = entry 8 i + k goes high
+  Rec* cta_rec;               // [CTAs][2 kFusedMaxK] node-best records of each k_fused CTA
   const int32_t* fx;          // [2] fixed-point scales of this tree
   double lam;
   int m, a_base, shard;
@@ -170,13 +187,14 @@ struct FusedArgs {
   int* nrec;
   unsigned long long* gkey;
 };
-size_t fused_lb_bytes(int64_t max_tiles);
+size_t fused_tile_bytes(int64_t max_tiles);
 int64_t fused_tiles(int64_t n, int m);
+void fused_carve(FusedArgs& A, void* base, int64_t max_tiles);
 void fused_init(int sms);
 unsigned fused_grid(int hmode);
 void fused_plan(FusedPlan* P, const NodeTab& cur, const NodeTab& nxt, const int32_t* cidx, const int* epoch, int m,
-                int* ticket, unsigned long long* lent, int lvl, cudaStream_t st);
-void fused_pass(const FusedArgs& A, int hmode, bool write, cudaStream_t st);
+                unsigned long long* lent, int lvl, cudaStream_t st);
+void fused_pass(const FusedArgs& A, int hmode, bool write, int64_t max_tiles, cudaStream_t st);
 void fused_mark(const FusedPlan* P, const int32_t* Kp, const int32_t* cidx, const Rec* winner, int shard, int a_base,
                 const int32_t* ins, const uint32_t* hbit, uint8_t* bits, int64_t n, int Kl, int sms, cudaStream_t st);
 

@@ -422,12 +422,11 @@ struct ShardWork {
   unsigned long long *run_hl = nullptr, *rcnt = nullptr, *rfl = nullptr, *rsgrp = nullptr;
   int32_t* Rp1 = nullptr;
   unsigned rgroups = 1;
-  // fused dense levels: plans of two levels, look-back records, tile ticket
+  // fused dense levels: plans of two levels, per-tile records / carries / side bits
   DBuf fz;
   FusedPlan* fplan[2] = {nullptr, nullptr};
-  unsigned* lb_status = nullptr;
-  void *lb_agg = nullptr, *lb_inc = nullptr;
-  int* ticket = nullptr;
+  void* tilemem = nullptr;
+  int64_t tiles = 0;
   // attribute-parallel partition plan
   unsigned long long *pel = nullptr, *pgrp = nullptr;
   int32_t* mp1 = nullptr;
@@ -673,17 +672,14 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       w.Rp1 = r.take<int32_t>(1); w.rsgrp = r.take<unsigned long long>(2 * (size_t)w.rgroups + 8);
     }
     if (fused && m > 0) {
-      const int64_t tiles = fused_tiles(n, m);
-      const size_t lbb = fused_lb_bytes(tiles);
-      w.fz.alloc(2 * sizeof(FusedPlan) + 256 + lbb + 1024, st);
+      w.tiles = fused_tiles(n, m);
+      const size_t tb = fused_tile_bytes(w.tiles);
+      w.fz.alloc(2 * sizeof(FusedPlan) + 1024 + tb, st);
       GBDT_CUDA(cudaMemsetAsync(w.fz.p, 0, w.fz.bytes, st));
       Carve f{w.fz.as<char>()};
       w.fplan[0] = f.take<FusedPlan>(1);
       w.fplan[1] = f.take<FusedPlan>(1);
-      w.ticket = f.take<int>(4);
-      w.lb_agg = f.take<char>(96 * (size_t)tiles);
-      w.lb_inc = f.take<char>(96 * (size_t)tiles);
-      w.lb_status = f.take<unsigned>((size_t)tiles);
+      w.tilemem = f.take<char>(tb);
     }
     w.nrec = nrec + li;
     w.gkey = gkey + (size_t)li * Kcap;
@@ -838,7 +834,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
           Shard& sh = *ds.shards[li];
           ShardWork& w = sw[li];
           if (sh.m == 0) continue;
-          fused_plan(w.fplan[lvl & 1], cur, nxt, cidx, epoch, sh.m, w.ticket, P.profile ? lent : nullptr, lvl, st);
+          fused_plan(w.fplan[lvl & 1], cur, nxt, cidx, epoch, sh.m, P.profile ? lent : nullptr, lvl, st);
           FusedArgs FA;
           FA.val = lvl == 0 ? sh.val0.as<float>() : sh.valw[lvl & 1].as<float>();
           FA.ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
@@ -849,11 +845,11 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
           FA.hbit = hbitF[lvl & 1];
           FA.plan = w.fplan[lvl & 1];
           FA.nxt = nxt;
-          FA.lb_status = w.lb_status; FA.lb_agg_ = w.lb_agg; FA.lb_inc_ = w.lb_inc; FA.ticket = w.ticket;
+          fused_carve(FA, w.tilemem, w.tiles);
           FA.fx = fxs; FA.lam = P.lambda; FA.m = sh.m; FA.a_base = sh.a_begin; FA.shard = sh.index;
           FA.rec = w.rec; FA.nrec = w.nrec; FA.gkey = w.gkey;
           kt.begin(GBDT_PHASE_K_FUSED);
-          fused_pass(FA, hmode, /*write=*/lvl + 1 < d - 1, st);
+          fused_pass(FA, hmode, /*write=*/lvl + 1 < d - 1, w.tiles, st);
           kt.end();
         }
         tm.end();
