@@ -160,6 +160,11 @@ gbdt_status gbdt_train(gbdt_dataset* ds, const gbdt_params* p, gbdt_model** out,
 gbdt_status gbdt_predict(const gbdt_model* m, int64_t n_rows, int64_t n_cols,
                          const int64_t* indptr, const int32_t* indices, const float* values,
                          int32_t output_margin, double* out);
+/* gbdt_predict with every copy and launch on the caller's cudaStream_t `stream` (NULL = the legacy
+ * default stream, which is what gbdt_predict uses).  Returns after the result is in `out`. */
+gbdt_status gbdt_predict_on_stream(const gbdt_model* m, int64_t n_rows, int64_t n_cols,
+                                   const int64_t* indptr, const int32_t* indices, const float* values,
+                                   int32_t output_margin, double* out, void* stream);
 
 /* Model inspection.  Nodes are returned in heap order, 2^(max_depth+1)-1 slots per tree. */
 gbdt_status gbdt_model_num_trees(const gbdt_model* m, int32_t* out);

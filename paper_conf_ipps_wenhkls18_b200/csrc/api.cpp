@@ -7,6 +7,7 @@
 #include <exception>
 #include <algorithm>
 #include <limits>
+#include <mutex>
 #include <new>
 #include <string>
 #include <vector>
@@ -21,11 +22,38 @@ thread_local std::string g_err;
 
 void fail(gbdt_status st, const std::string& msg) { throw Error{st, msg}; }
 
+// The library's own stream-ordered memory pool per device: freed allocations stay cached in it
+// across gbdt_train / gbdt_load_csr calls (release threshold = max), without touching the
+// process-wide default pool that other libraries (PyTorch) allocate from.
+static cudaMemPool_t lib_pool(int dev) {
+  static std::once_flag once[kMaxDevices];
+  static cudaMemPool_t pools[kMaxDevices];
+  static cudaError_t errs[kMaxDevices];
+  if (dev < 0 || dev >= kMaxDevices) fail(GBDT_E_RANGE, "device ordinal >= " + std::to_string(kMaxDevices));
+  std::call_once(once[dev], [dev] {
+    cudaMemPoolProps props;
+    std::memset(&props, 0, sizeof props);
+    props.allocType = cudaMemAllocationTypePinned;
+    props.handleTypes = cudaMemHandleTypeNone;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    errs[dev] = cudaMemPoolCreate(&pools[dev], &props);
+    if (errs[dev] == cudaSuccess) {
+      uint64_t thr = UINT64_MAX;
+      errs[dev] = cudaMemPoolSetAttribute(pools[dev], cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  });
+  GBDT_CUDA(errs[dev]);
+  return pools[dev];
+}
+
 void DBuf::alloc(size_t b, cudaStream_t s) {
   release();
   st = s;
   bytes = b ? b : 16;
-  GBDT_CUDA(cudaMallocAsync(&p, bytes, st));
+  int dev = 0;
+  GBDT_CUDA(cudaGetDevice(&dev));
+  GBDT_CUDA(cudaMallocFromPoolAsync(&p, bytes, lib_pool(dev), st));
 }
 
 void DBuf::release() {
@@ -216,13 +244,6 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
     if (dev >= ndev) fail(GBDT_E_RANGE, "device ordinal out of range");
     if (comm) dev = comm->device;
     GBDT_CUDA(cudaSetDevice(dev));
-    {
-      // keep freed stream-ordered allocations cached in the pool across gbdt_train calls
-      cudaMemPool_t pool;
-      GBDT_CUDA(cudaDeviceGetDefaultMemPool(&pool, dev));
-      uint64_t thr = UINT64_MAX;
-      GBDT_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
-    }
 
     const int64_t nnz = indptr[n_rows];
 
@@ -329,7 +350,18 @@ gbdt_status gbdt_predict(const gbdt_model* mh, int64_t n_rows, int64_t n_cols, c
     if (!mh || !out) fail(GBDT_E_INVAL, "NULL argument");
     if (mh->m.n_trees < 1) fail(GBDT_E_STATE, "model has no trees");
     validate_csr(n_rows, n_cols, indptr, indices, values, false);
-    predict(mh->m, n_rows, n_cols, indptr, indices, values, output_margin, out);
+    predict(mh->m, n_rows, n_cols, indptr, indices, values, output_margin, out, nullptr);
+  });
+}
+
+gbdt_status gbdt_predict_on_stream(const gbdt_model* mh, int64_t n_rows, int64_t n_cols, const int64_t* indptr,
+                                   const int32_t* indices, const float* values, int32_t output_margin, double* out,
+                                   void* stream) {
+  return guarded([&] {
+    if (!mh || !out) fail(GBDT_E_INVAL, "NULL argument");
+    if (mh->m.n_trees < 1) fail(GBDT_E_STATE, "model has no trees");
+    validate_csr(n_rows, n_cols, indptr, indices, values, false);
+    predict(mh->m, n_rows, n_cols, indptr, indices, values, output_margin, out, (cudaStream_t)stream);
   });
 }
 

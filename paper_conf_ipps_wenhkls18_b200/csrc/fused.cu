@@ -1042,7 +1042,7 @@ __global__ void k_fused_plan(FusedPlan* P, NodeTab cur, NodeTab nxt, const int32
 __global__ void k_mark_fused(const FusedPlan* __restrict__ P, const int32_t* __restrict__ Kp,
                              const int32_t* __restrict__ cidx_now, const Rec* __restrict__ winner, int shard,
                              int a_base, const int32_t* __restrict__ ins, const uint32_t* __restrict__ hbit,
-                             uint8_t* __restrict__ bits) {
+                             uint32_t* __restrict__ bits) {
   const int c = blockIdx.y;
   if (c >= *Kp || cidx_now[c] < 0) return;
   const Rec& w = winner[c];
@@ -1056,7 +1056,7 @@ __global__ void k_mark_fused(const FusedPlan* __restrict__ P, const int32_t* __r
     const int i = ins[p];
     if (((hbit[i >> 5] >> (i & 31)) & 1u) != want) continue;
     const int high = p <= w.pos;
-    if (high != w.dir) bits[i] = 1;
+    if (high != w.dir) atomicOr(bits + (i >> 5), 1u << (i & 31));
   }
 }
 
@@ -1139,7 +1139,7 @@ void fused_pass(const FusedArgs& A, int hmode, bool write, int64_t max_tiles, cu
 }
 
 void fused_mark(const FusedPlan* P, const int32_t* Kp, const int32_t* cidx, const Rec* winner, int shard, int a_base,
-                const int32_t* ins, const uint32_t* hbit, uint8_t* bits, int64_t n, int Kl, int sms, cudaStream_t st) {
+                const int32_t* ins, const uint32_t* hbit, uint32_t* bits, int64_t n, int Kl, int sms, cudaStream_t st) {
   dim3 grid((unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256 * (int64_t)Kl), (int64_t)sms * 4)),
             (unsigned)Kl);
   k_mark_fused<<<grid, 256, 0, st>>>(P, Kp, cidx, winner, shard, a_base, ins, hbit, bits);

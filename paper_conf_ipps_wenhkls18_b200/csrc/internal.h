@@ -11,6 +11,8 @@
 
 namespace gbdt {
 
+constexpr int kMaxDevices = 64;  // device ordinals the library keeps per-device state for
+
 struct Error {
   gbdt_status st;
   std::string msg;
@@ -164,7 +166,7 @@ void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices
 void train(Dataset& ds, const gbdt_params& p, Model& model, double* margin_out);
 // predict.cu
 void predict(const Model& m, int64_t n_rows, int64_t n_cols, const int64_t* indptr,
-             const int32_t* indices, const float* values, int output_margin, double* out);
+             const int32_t* indices, const float* values, int output_margin, double* out, cudaStream_t st);
 
 inline int64_t pad4(int64_t x) { return (x + 3) & ~int64_t(3); }
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }

@@ -196,7 +196,7 @@ void fused_plan(FusedPlan* P, const NodeTab& cur, const NodeTab& nxt, const int3
                 unsigned long long* lent, int lvl, cudaStream_t st);
 void fused_pass(const FusedArgs& A, int hmode, bool write, int64_t max_tiles, cudaStream_t st);
 void fused_mark(const FusedPlan* P, const int32_t* Kp, const int32_t* cidx, const Rec* winner, int shard, int a_base,
-                const int32_t* ins, const uint32_t* hbit, uint8_t* bits, int64_t n, int Kl, int sms, cudaStream_t st);
+                const int32_t* ins, const uint32_t* hbit, uint32_t* bits, int64_t n, int Kl, int sms, cudaStream_t st);
 
 // levels.cu launchers
 struct LevelKernels {

@@ -733,11 +733,8 @@ __global__ void __launch_bounds__(kThreads) k_scan3(const int32_t* __restrict__ 
 constexpr int kWarpK = 32;  // CTA node tables when K <= kWarpK (d <= 6); else global records
 
 struct NodeBest {
-  unsigned long long gk[kWarpK];
-  Rec rec[kWarpK];
   double G[kWarpK], H[kWarpK], P[kWarpK];
   int C[kWarpK];
-  int lock[kWarpK];
 };
 
 struct NodeV {
@@ -751,8 +748,6 @@ __device__ __forceinline__ NodeV node_v(const NodeBest& B, const SplitArgs& A, i
 
 __device__ __forceinline__ void nb_init(NodeBest& B, const SplitArgs& A, int K) {
   for (int j = threadIdx.x; j < kWarpK; j += blockDim.x) {
-    B.gk[j] = 0ull;
-    B.lock[j] = 0;
     if (j < K) { B.G[j] = A.nodes.G[j]; B.H[j] = A.nodes.H[j]; B.P[j] = A.nodes.pterm[j]; B.C[j] = A.nodes.cnt[j]; }
   }
 }
@@ -761,36 +756,27 @@ __device__ __forceinline__ bool rec_better(unsigned long long gk, const Rec& r, 
   return gk > gk0 || (gk == gk0 && tie_key(r.attr, r.value, r.dir) < tie_key(r0.attr, r0.value, r0.dir));
 }
 
-// R12 order merge of one candidate record into the CTA table (or the global record list)
-__device__ __forceinline__ void post_record(NodeBest& B, const SplitArgs& A, int K, const Rec& r) {
-  const unsigned long long gk = gain_key(r.gain);
-  if (K > kWarpK) {
-    const int gs = atomicAdd(A.nrec, 1);
-    A.rec[gs] = r;
-    atomicMax(A.gkey + r.node, gk);
-    return;
-  }
-  const int j = r.node;
-  if (gk < *reinterpret_cast<volatile unsigned long long*>(&B.gk[j])) return;  // keys only grow
-  while (atomicCAS(&B.lock[j], 0, 1) != 0) {
-  }
-  __threadfence_block();
-  if (rec_better(gk, r, B.gk[j], B.rec[j])) {
-    B.rec[j] = r;
-    B.gk[j] = gk;
-  }
-  __threadfence_block();
-  atomicExch(&B.lock[j], 0);
+// One candidate record into the global record list (K > kWarpK: too many nodes for the per-warp
+// tables); k_pick_tie / k_pick_best merge them in the R12 order.
+__device__ __forceinline__ void post_global(const SplitArgs& A, const Rec& r) {
+  const int gs = atomicAdd(A.nrec, 1);
+  A.rec[gs] = r;
+  atomicMax(A.gkey + r.node, gain_key(r.gain));
 }
 
-__device__ __forceinline__ void nb_flush(NodeBest& B, const SplitArgs& A, int K) {
-  if (K > kWarpK) return;
+// With K <= kWarpK every warp keeps its own best record per node (one writer: no lock, no race);
+// at the end the CTA merges its warps' tables in the R12 order and posts one record per node.
+__device__ __forceinline__ void merge_warp_tables(const SplitArgs& A, int K, unsigned long long (*wgk)[kWarpK],
+                                                  Rec (*wrec)[kWarpK]) {
   __syncthreads();
   for (int j = threadIdx.x; j < K; j += blockDim.x) {
-    if (B.gk[j]) {
+    int bw = -1;
+    for (int w = 0; w < kWarps; ++w)
+      if (wgk[w][j] && (bw < 0 || rec_better(wgk[w][j], wrec[w][j], wgk[bw][j], wrec[bw][j]))) bw = w;
+    if (bw >= 0) {
       const int gs = atomicAdd(A.nrec, 1);
-      A.rec[gs] = B.rec[j];
-      atomicMax(A.gkey + j, B.gk[j]);
+      A.rec[gs] = wrec[bw][j];
+      atomicMax(A.gkey + j, wgk[bw][j]);
     }
   }
 }
@@ -860,6 +846,8 @@ template <bool kH>
 struct FastSmem {
   FastWarp<kH> w[kWarps];
   NodeBest B;
+  unsigned long long wgk[kWarps][kWarpK];  // per-warp node bests (K <= kWarpK)
+  Rec wrec[kWarps][kWarpK];
 };
 
 template <int HMODE, bool kRLE>
@@ -876,6 +864,7 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
   const double lam = A.lam;
   FastWarp<kH>& W = S.w[wid];
   nb_init(S.B, A, K);
+  for (int j = threadIdx.x; j < kWarps * kWarpK; j += blockDim.x) S.wgk[j / kWarpK][j % kWarpK] = 0ull;
   if (lane == 0) {
     for (int s = 0; s < kFS; ++s) mbar_init(&W.bar[s], 1);
     fence_mbar_init();
@@ -1036,7 +1025,7 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
       // otherwise the exact Eq. 2 evaluation and the post are skipped (warp-uniform test).
       bool promising = wq != INT_MAX;
       if (promising && K <= kWarpK) {
-        const unsigned long long cur = *reinterpret_cast<volatile unsigned long long*>(&S.B.gk[j]);
+        const unsigned long long cur = S.wgk[wid][j];  // this warp's best so far (written by it only)
         if (cur) {
           const double ga = 0.5 * (wb - nv.P), slack = 1e-12 * (fabs(wb) + fabs(nv.P));
           promising = ga + slack >= key_gain(cur);
@@ -1068,7 +1057,12 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
         r.epoch = epoch;
         r.shard = A.shard;
         r.pos = p0 + bk + q0;
-        post_record(S.B, A, K, r);
+        if (K <= kWarpK) {
+          const unsigned long long gk = gain_key(r.gain);
+          if (rec_better(gk, r, S.wgk[wid][j], S.wrec[wid][j])) { S.wgk[wid][j] = gk; S.wrec[wid][j] = r; }
+        } else {
+          post_global(A, r);
+        }
       }
     }
     __syncwarp();  // stage st and descriptor slot i & 3 are free
@@ -1080,7 +1074,7 @@ __global__ void __launch_bounds__(kThreads, 3) k_sf_fast(SplitArgs A) {
     cp_async_commit();
   }
   cp_async_wait<0>();
-  nb_flush(S.B, A, K);
+  if (K <= kWarpK) merge_warp_tables(A, K, S.wgk, S.wrec);
 }
 
 // ---------------------------------------------------------------------------- short chunks
@@ -1529,25 +1523,13 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
         const unsigned long long gk = gain_key(r.gain);
         if (rec_better(gk, r, wgk[wid][j], wrec[wid][j])) { wgk[wid][j] = gk; wrec[wid][j] = r; }
       } else {
-        post_record(B, A, K, r);
+        post_global(A, r);
       }
     }
     __syncwarp();
     }
   }
-  if (!kTotals && K <= kWarpK) {  // merge the warp tables, one record per node and CTA
-    __syncthreads();
-    for (int j = threadIdx.x; j < K; j += blockDim.x) {
-      int bw = -1;
-      for (int w = 0; w < kWarps; ++w)
-        if (wgk[w][j] && (bw < 0 || rec_better(wgk[w][j], wrec[w][j], wgk[bw][j], wrec[bw][j]))) bw = w;
-      if (bw >= 0) {
-        const int gs = atomicAdd(A.nrec, 1);
-        A.rec[gs] = wrec[bw][j];
-        atomicMax(A.gkey + j, wgk[bw][j]);
-      }
-    }
-  }
+  if (!kTotals && K <= kWarpK) merge_warp_tables(A, K, wgk, wrec);  // one record per node and CTA
 }
 
 // ============================================================================ a8: partition

@@ -81,9 +81,8 @@ __global__ void __launch_bounds__(kPredRows) k_predict_dense(int64_t n, int m, c
 }  // namespace
 
 void predict(const Model& m, int64_t n_rows, int64_t n_cols, const int64_t* indptr, const int32_t* indices,
-             const float* values, int output_margin, double* out) {
+             const float* values, int output_margin, double* out, cudaStream_t st) {
   GBDT_CUDA(cudaSetDevice(m.device));
-  cudaStream_t st = nullptr;
   const int64_t nnz = indptr[n_rows];
   const int64_t NH = m.nh();
   DBuf dptr((size_t)(n_rows + 1) * 8, st), didx((size_t)std::max<int64_t>(nnz, 1) * 4, st),

@@ -20,6 +20,7 @@
 // in which pieces are reduced.
 #include <algorithm>
 #include <cstring>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -59,7 +60,7 @@ __global__ void k_grad(int64_t n, int loss, const int32_t* __restrict__ tidx, do
                        const float* __restrict__ y, const double* __restrict__ hweight, int64_t NH,
                        double* __restrict__ yhat, int32_t* __restrict__ pos,
                        double* __restrict__ gout, double* __restrict__ hout, int store_h,
-                       double* __restrict__ partial, RowsArgs R, int mode) {
+                       double* __restrict__ partial, RowsArgs R, int mode, int* __restrict__ bad) {
   const int t = tidx ? *tidx : R.t;
   const int first = t == 0;
   const double* wprev = hweight + (size_t)((t + 1) & 1) * NH;
@@ -71,6 +72,7 @@ __global__ void k_grad(int64_t n, int loss, const int32_t* __restrict__ tidx, do
     if (mode == 2) {
       g = gout[i];
       h = hout[i];
+      if (!(isfinite(g) && isfinite(h) && h >= 0.0)) atomicOr(bad, 1);  // the callback's contract
     } else {
       double yh;
       if (R.indptr) yh = traverse_margin(R, i, base, eta);
@@ -82,10 +84,12 @@ __global__ void k_grad(int64_t n, int loss, const int32_t* __restrict__ tidx, do
     if (loss == GBDT_LOSS_SQUARED) {  // l = (y - yhat)^2: g = 2(yhat - y), h = 2 (R6)
       g = __dmul_rn(2.0, __dsub_rn(yh, yi));
       h = 2.0;
-    } else {  // cross-entropy, readings R5/R5b
+    } else {  // cross-entropy, Eq. 1: g = p - y, h = max(p(1-p), 1e-16) (reading R5)
       const double p = __ddiv_rn(1.0, __dadd_rn(1.0, exp(-yh)));
       g = __dsub_rn(p, yi);
-      const double q = __dadd_rn(g, yi);
+      // h is stored (labels not all 0/1): p(1-p) itself; otherwise the split kernels recompute h
+      // from the stored g (K1), so the node totals use that same form: q = g + y
+      const double q = store_h ? p : __dadd_rn(g, yi);
       const double hh = __dmul_rn(q, __dsub_rn(1.0, q));
       h = hh > 1e-16 ? hh : 1e-16;
     }
@@ -95,7 +99,7 @@ __global__ void k_grad(int64_t n, int loss, const int32_t* __restrict__ tidx, do
     sg += g;
     sh += h;
     mg = fmax(mg, fabs(g));
-    mh = fmax(mh, h);
+    mh = fmax(mh, fabs(h));
   }
   // fixed-shape block reduction (deterministic for a fixed grid)
   for (int o = 16; o; o >>= 1) {
@@ -330,7 +334,7 @@ __global__ void k_decide(DecideArgs A) {
 // ============================================================================ a7: node map
 __global__ void k_mark(const int32_t* __restrict__ Kp, const int32_t* __restrict__ cidx,
                        const Rec* __restrict__ winner, int shard, int a_base, Tables tb,
-                       const int32_t* __restrict__ ins, uint8_t* __restrict__ bits) {
+                       const int32_t* __restrict__ ins, uint32_t* __restrict__ bits) {
   const int K = *Kp;
   const int j = blockIdx.y;
   if (j >= K || cidx[j] < 0) return;
@@ -342,13 +346,16 @@ __global__ void k_mark(const int32_t* __restrict__ Kp, const int32_t* __restrict
   for (long long q = (long long)blockIdx.x * blockDim.x + threadIdx.x; q < n; q += (long long)gridDim.x * blockDim.x) {
     const long long p = s0 + q;
     const int high = p <= w.pos;   // prefix of the descending list = values >= split value
-    if (high != defhi) bits[ins[p]] = 1;  // goes to the non-default side
+    if (high != defhi) {  // goes to the non-default side: bit i of the n-bit map (multi-GPU: OR-allreduced)
+      const int i = ins[p];
+      atomicOr(bits + (i >> 5), 1u << (i & 31));
+    }
   }
 }
 
 // side[i]: 0 (node became a leaf), 1 (high child), 2 (low child); hbit: bit i = [side[i] == 1],
 // packed by warp ballots (the dense partition count gathers these 1.4 MB instead of 11 MB)
-__global__ void k_nodemap(int64_t n, const uint8_t* __restrict__ bits, const uint8_t* __restrict__ hstate,
+__global__ void k_nodemap(int64_t n, const uint32_t* __restrict__ bits, const uint8_t* __restrict__ hstate,
                           const uint8_t* __restrict__ hdef, int32_t* __restrict__ pos,
                           uint8_t* __restrict__ side, uint32_t* __restrict__ hbit) {
   const int64_t n32 = (n + 31) & ~int64_t(31);
@@ -358,7 +365,7 @@ __global__ void k_nodemap(int64_t n, const uint8_t* __restrict__ bits, const uin
       const int h = pos[i];
       if (hstate[h] == 1) {
         const int defhi = hdef[h];
-        const int hi = bits[i] ? !defhi : defhi;
+        const int hi = ((bits[i >> 5] >> (i & 31)) & 1u) ? !defhi : defhi;
         pos[i] = hi ? 2 * h + 1 : 2 * h + 2;
         sd = hi ? 1 : 2;
       }
@@ -476,14 +483,24 @@ __global__ void k_level_entries(const int64_t* col_len, int m, unsigned long lon
   if ((threadIdx.x & 31) == 0 && s) atomicAdd(out, s);
 }
 
-// Level kernels are configured once per device (smem attributes, persistent grid sizes).
+// Level kernels are configured once per device (smem attributes, persistent grid sizes); safe
+// when several host threads train different handles at once.
 static LevelKernels& level_kernels(int device) {
-  static LevelKernels lk[16];
-  static bool done[16] = {false};
-  if (!done[device]) {
-    lk[device].init(device);
-    done[device] = true;
-  }
+  static LevelKernels lk[kMaxDevices];
+  static std::once_flag once[kMaxDevices];
+  static std::string err[kMaxDevices];
+  static gbdt_status est[kMaxDevices];
+  if (device < 0 || device >= kMaxDevices) fail(GBDT_E_RANGE, "device ordinal >= " + std::to_string(kMaxDevices));
+  std::call_once(once[device], [device] {
+    try {
+      lk[device].init(device);
+      est[device] = GBDT_OK;
+    } catch (const Error& e) {
+      est[device] = e.st;
+      err[device] = e.msg;
+    }
+  });
+  if (est[device] != GBDT_OK) fail(est[device], err[device]);
   return lk[device];
 }
 
@@ -515,7 +532,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   // ---------------------------------------------------------------- per-device state
   auto sz_dev = [&](Carve& c) {
     c.take<double>(n); c.take<double>(hmode == kHGather ? n : 1); c.take<double>(n); c.take<int32_t>(n);
-    c.take<uint8_t>(npad); c.take<uint8_t>(npad);
+    c.take<uint8_t>(npad); c.take<uint32_t>((size_t)(n + 31) / 32 + 1);
     c.take<double>(2 * NH); c.take<uint8_t>(NH); c.take<uint8_t>(NH);
     c.take<gbdt_node>((size_t)P.n_trees * NH); c.take<double>(4 * grad_blocks); c.take<int32_t>(2);
     for (int b = 0; b < 2; ++b) { c.take<int32_t>(1); c.take<int32_t>(Kcap); c.take<double>(Kcap); c.take<double>(Kcap); c.take<int32_t>(Kcap); c.take<double>(Kcap); }
@@ -537,7 +554,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   double* yhat = c.take<double>(n);
   int32_t* pos = c.take<int32_t>(n);
   uint8_t* side = c.take<uint8_t>(npad);
-  uint8_t* bits = c.take<uint8_t>(npad);
+  uint32_t* bits = c.take<uint32_t>((size_t)(n + 31) / 32 + 1);  // instance -> non-default side (n bits)
   double* hweight = c.take<double>(2 * NH);
   uint8_t* hstate = c.take<uint8_t>(NH);
   uint8_t* hdef = c.take<uint8_t>(NH);
@@ -705,15 +722,20 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     tm.begin(GBDT_PHASE_GRAD);
     if (rows.indptr) rows.trees = trees;
     k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, tidx, P.eta, P.base_margin, ds.y.as<float>(), hweight, NH,
-                                        yhat, pos, gv, hv, hmode == kHGather, partial, rows, custom ? 1 : 0);
+                                        yhat, pos, gv, hv, hmode == kHGather, partial, rows, custom ? 1 : 0, tidx + 2);
     GBDT_LAUNCH_CHECK();
     if (custom) {  // user-defined loss: g, h from the callback, on this stream
       if (P.grad_fn(n, yhat, ds.y.as<float>(), gv, hv, (void*)st, P.grad_user) != 0)
         fail(GBDT_E_INVAL, "grad_fn failed at tree " + std::to_string(t));
+      GBDT_CUDA(cudaMemsetAsync(tidx + 2, 0, sizeof(int32_t), st));
       k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, tidx, P.eta, P.base_margin, ds.y.as<float>(), hweight, NH,
-                                          yhat, pos, gv, hv, 1, partial, RowsArgs{}, 2);
+                                          yhat, pos, gv, hv, 1, partial, RowsArgs{}, 2, tidx + 2);
       GBDT_LAUNCH_CHECK();
       count_launch();
+      int32_t bad = 0;  // the custom path runs eagerly: check the callback's g, h before using them
+      GBDT_CUDA(cudaMemcpyAsync(&bad, tidx + 2, sizeof bad, cudaMemcpyDeviceToHost, st));
+      GBDT_CUDA(cudaStreamSynchronize(st));
+      if (bad) fail(GBDT_E_INVAL, "grad_fn returned a non-finite g or h, or h < 0, at tree " + std::to_string(t));
     }
     k_tree_begin<<<1, 1024, 0, st>>>(grad_blocks, partial, n, P.lambda, nt[0], NH, hweight, hstate, trees, fxs, tidx);
     GBDT_LAUNCH_CHECK();
@@ -795,7 +817,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       tm.end();
 
       tm.begin(GBDT_PHASE_NODEMAP);
-      GBDT_CUDA(cudaMemsetAsync(bits, 0, (size_t)n, st));
+      const size_t bit_bytes = ((size_t)n + 31) / 32 * 4;
+      GBDT_CUDA(cudaMemsetAsync(bits, 0, bit_bytes, st));
       for (int li = 0; li < nloc; ++li) {
         Shard& sh = *ds.shards[li];
         if (sh.m == 0) continue;
@@ -815,7 +838,9 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       tm.end();
       if (ds.comm) {
         tm.begin(GBDT_PHASE_COMM);
-        ds.comm->allreduce_sum_u8(bits, (size_t)n, st);
+        // the ranks' bits are disjoint (one owner shard per node), so a byte-wise sum is their OR:
+        // n/8 bytes on the wire (1.4 MB for C3)
+        ds.comm->allreduce_sum_u8(bits, bit_bytes, st);
         tm.end();
       }
       tm.begin(GBDT_PHASE_NODEMAP);
@@ -909,13 +934,12 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     count_launch();
   };
 
-  // NCCL collectives inside the captured tree are exercised here only with a world of one rank
-  // (single-GPU boxes): with a multi-rank communicator the graph is opt-in (GBDT_GRAPH=1);
-  // GBDT_GRAPH=0 forces eager launches everywhere.  Host-staged collectives cannot be captured.
-  const bool multi = ds.comm && ds.comm->world > 1;
+  // One CUDA graph per tree, NCCL collectives included (captured on the library's stream; a world
+  // of one rank exercises the same captured calls on single-GPU boxes).  GBDT_GRAPH=0 forces eager
+  // launches.  Host-staged collectives (callbacks) cannot be captured.
   const bool host_comm = ds.comm && !ds.comm->nccl;
   const char* ge = getenv("GBDT_GRAPH");
-  const bool graph_ok = ge ? ge[0] != '0' : !multi;
+  const bool graph_ok = ge ? ge[0] != '0' : true;
   const bool graph = !tm.on && !custom && !host_comm && P.n_trees > 1 && graph_ok;
   if (!graph) {
     for (int t = 0; t < P.n_trees; ++t) tree_body(t);
@@ -959,7 +983,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     if (rows.indptr) {  // ablation: the final margin by traversal of all trees too
       rows.trees = trees; rows.t = P.n_trees;
       k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, nullptr, P.eta, P.base_margin, ds.y.as<float>(), hweight, NH,
-                                          yhat, pos, gv, hv, 0, partial, rows, 1);
+                                          yhat, pos, gv, hv, 0, partial, rows, 1, tidx + 2);
     } else {
       k_apply<<<inst_grid, 256, 0, st>>>(n, P.eta, wlast, pos, yhat);
     }

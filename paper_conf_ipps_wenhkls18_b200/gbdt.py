@@ -72,6 +72,7 @@ def lib():
     L.gbdt_load_csr.argtypes = [i64, i64, p, p, p, p, C.POINTER(_LoadOpts), C.POINTER(p)]
     L.gbdt_train.argtypes = [p, C.POINTER(_Params), C.POINTER(p), p]
     L.gbdt_predict.argtypes = [p, i64, i64, p, p, p, i32, p]
+    L.gbdt_predict_on_stream.argtypes = [p, i64, i64, p, p, p, i32, p, p]
     L.gbdt_model_num_trees.argtypes = [p, C.POINTER(i32)]
     L.gbdt_model_num_nodes.argtypes = [p, i32, C.POINTER(i32)]
     L.gbdt_model_export.argtypes = [p, i32, p]
@@ -87,7 +88,7 @@ def lib():
     L.gbdt_shard_ranges.argtypes = [i64, p, i32, p]
     L.gbdt_dataset_free.argtypes = [p]
     L.gbdt_model_free.argtypes = [p]
-    for f in ("gbdt_load_csr", "gbdt_train", "gbdt_predict", "gbdt_model_num_trees", "gbdt_model_num_nodes",
+    for f in ("gbdt_load_csr", "gbdt_train", "gbdt_predict", "gbdt_predict_on_stream", "gbdt_model_num_trees", "gbdt_model_num_nodes",
               "gbdt_model_export", "gbdt_get_timings", "gbdt_get_level_entries", "gbdt_dataset_info", "gbdt_dataset_export_layout",
               "gbdt_dataset_export_rle", "gbdt_comm_unique_id", "gbdt_comm_init", "gbdt_comm_init_callbacks",
               "gbdt_shard_ranges"):
@@ -331,14 +332,16 @@ def train(ds: Dataset, max_depth=6, n_trees=40, lam=1.0, gamma=0.0, eta=0.3, bas
     return Model(h), margin
 
 
-def predict(model: Model, indptr, indices, values, n_cols, output_margin=True) -> np.ndarray:
+def predict(model: Model, indptr, indices, values, n_cols, output_margin=True, stream="current") -> np.ndarray:
     indptr = np.ascontiguousarray(indptr, np.int64)
     indices = np.ascontiguousarray(indices, np.int32)
     values = np.ascontiguousarray(values, np.float32)
     n = indptr.size - 1
     out = np.zeros(n, np.float64)
-    _check(lib().gbdt_predict(model._h, n, int(n_cols), _p(indptr), _p(indices), _p(values),
-                              int(bool(output_margin)), _p(out)))
+    if stream == "current":
+        stream = _current_stream()
+    _check(lib().gbdt_predict_on_stream(model._h, n, int(n_cols), _p(indptr), _p(indices), _p(values),
+                                        int(bool(output_margin)), _p(out), stream))
     return out
 
 

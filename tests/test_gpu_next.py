@@ -102,6 +102,32 @@ def test_custom_loss_errors():
         gbdt.train(ds, max_depth=2, n_trees=1, loss="custom", grad_fn=bad)
 
 
+@pytest.mark.parametrize("poison", ["nan_g", "inf_h", "neg_h"])
+def test_custom_loss_rejects_invalid_derivatives(poison):
+    """The callback's contract (gbdt.h: h >= 0 and finite) is checked before the sums use it."""
+    from cuda.bindings import runtime as rt
+    p = synth.c1(n=400)
+    ds = gbdt.load_csr(p.indptr, p.indices, p.values, p.labels, p.m)
+    good = _host_grad("squared")
+
+    def fn(n, yh, y, g, h, stream):
+        good(n, yh, y, g, h, stream)
+        H = np.empty(n, np.float64)
+        G = np.empty(n, np.float64)
+        assert rt.cudaMemcpy(G.ctypes.data, g, 8 * n, rt.cudaMemcpyKind.cudaMemcpyDeviceToHost)[0] == 0
+        assert rt.cudaMemcpy(H.ctypes.data, h, 8 * n, rt.cudaMemcpyKind.cudaMemcpyDeviceToHost)[0] == 0
+        if poison == "nan_g":
+            G[7] = np.nan
+        elif poison == "inf_h":
+            H[3] = np.inf
+        else:
+            H[11] = -1.0
+        assert rt.cudaMemcpy(g, G.ctypes.data, 8 * n, rt.cudaMemcpyKind.cudaMemcpyHostToDevice)[0] == 0
+        assert rt.cudaMemcpy(h, H.ctypes.data, 8 * n, rt.cudaMemcpyKind.cudaMemcpyHostToDevice)[0] == 0
+    with pytest.raises(gbdt.GbdtError, match="non-finite g or h"):
+        gbdt.train(ds, max_depth=2, n_trees=1, loss="custom", grad_fn=fn)
+
+
 @pytest.mark.parametrize("maker", [
     lambda: synth.c1(n=3000),
     lambda: synth.c4(seed=3, n=600, m=2000, density=0.01),

@@ -388,3 +388,61 @@ def test_fused_equals_level_by_level_up_to_rounding(monkeypatch):
         assert np.array_equal(na[f], nb[f]), f
     np.testing.assert_allclose(na["weight"], nb["weight"], rtol=1e-10, atol=1e-14)
     np.testing.assert_allclose(ma, mb, rtol=1e-10, atol=1e-14)
+
+
+# ------------------------------------------------------------------ P:116 edge values, CART
+# Values as gbdt.h states them ("missing values"): NaN stored in the CSR is missing, -0.0 is
+# +0.0, +-Inf are ordinary values; each case against the oracle (which reads the same CSR bytes).
+def _edge_problem(kind, seed=17, n=3000, m=5, loss="logistic"):
+    rng = np.random.default_rng(seed)
+    X = rng.integers(-3, 4, size=(n, m)).astype(np.float64)
+    if kind == "nan":
+        X[rng.uniform(size=X.shape) < 0.2] = np.nan       # stored NaN entries (from_dense drops them)
+    elif kind == "negzero":
+        X[X == 0] = -0.0
+        X[:, 0] = np.where(rng.uniform(size=n) < 0.5, -0.0, 0.0)  # a column of +-0 only
+    elif kind == "inf":
+        X[rng.uniform(size=X.shape) < 0.1] = np.inf
+        X[rng.uniform(size=X.shape) < 0.1] = -np.inf
+    Xf = np.nan_to_num(X, nan=0.0, posinf=5.0, neginf=-5.0)
+    y = (np.sin(Xf[:, 1]) + 0.3 * rng.normal(size=n) > 0).astype(np.float64) if loss == "logistic" else \
+        Xf[:, 2] + rng.normal(size=n)
+    p = synth.from_dense(kind, X, y,
+                         dict(loss=loss, max_depth=4, n_trees=3, lam=1.0, gamma=0.0, eta=0.3, base_margin=0.0))
+    if kind == "nan":  # store the NaNs explicitly in the CSR (not dropped): the library must treat them as missing
+        indptr = np.arange(0, n * m + 1, m, dtype=np.int64)
+        p = synth.Problem(kind, n, m, indptr, np.tile(np.arange(m, dtype=np.int32), n), X.reshape(-1).astype(np.float32),
+                          p.labels, p.params)
+    return p
+
+
+@pytest.mark.parametrize("kind", ["nan", "negzero", "inf"])
+def test_edge_values_against_oracle(kind):
+    p = _edge_problem(kind)
+    if kind == "nan":
+        assert np.isnan(p.values).any()
+    if kind == "negzero":
+        assert np.signbit(p.values[p.values == 0]).any()
+    if kind == "inf":
+        assert np.isinf(p.values).any()
+    model, margin = _train(p)
+    compare(p, model.nodes(), margin)
+
+
+def test_lambda0_squared_is_cart_on_gpu():
+    """Squared loss, lambda = 0, eta = 1, one tree: the GPU tree is scikit-learn's CART tree
+    (same leaf partition, leaf value = mean target), a library routine the method reduces to."""
+    from sklearn.tree import DecisionTreeRegressor
+    rng = np.random.default_rng(4)
+    n, m, d = 2000, 6, 4
+    X = rng.uniform(-1, 1, size=(n, m)).astype(np.float32).astype(np.float64)
+    y = np.sin(3 * X[:, 0]) + X[:, 1] * X[:, 2] + 0.1 * rng.normal(size=n)
+    p = synth.from_dense("cart", X, y, dict(loss="squared", max_depth=d, n_trees=1, lam=0.0, gamma=0.0,
+                                            eta=1.0, base_margin=0.0))
+    model, margin = _train(p)
+    sk = DecisionTreeRegressor(max_depth=d, random_state=0).fit(X.astype(np.float32), p.labels.astype(np.float64))
+    leaves_sk = sk.apply(X.astype(np.float32))
+    groups_sk = {frozenset(np.where(leaves_sk == l)[0]) for l in np.unique(leaves_sk)}
+    groups_gpu = {frozenset(np.where(margin == v)[0]) for v in np.unique(margin)}
+    assert groups_sk == groups_gpu
+    np.testing.assert_allclose(margin, sk.predict(X.astype(np.float32)), rtol=0, atol=1e-9)
