@@ -13,9 +13,18 @@ ABI from pinned host buffers: gbdt_load_csr (H2D + layout build) + gbdt_train + 
 For N > 1 (torchrun) the attributes are sharded over the ranks (NCCL allgather of node bests +
 bitmap allreduce per level) and the total work is fixed ("strong" scaling).
 
---impl reference times the CPU oracle (oracle/, single thread) on a bounded row sample of the
-same workload and scales it to the full workload's entries (the paper's cost model is linear in
-the number of entries per level).
+--impl reference times the CPU oracle (oracle/, single thread pinned to one core) on the FULL
+rows of the same workload: presort once (excluded, reported), then the first K' trees (K' =
+min(--steps, --ref-trees)); `steps` reports K' (the trees actually run).  cpu_baseline (our arm,
+rank 0, N=1) is the same measurement with --cpu-trees trees.
+
+roofline: SURVEY.md §8(d)'s algorithmic bytes per unit (one active entry at one level):
+split find 24 B (logistic: val 4 + ins 4 + g/h 16; squared 16), partition 16 B (read 8 + write 8,
+levels < d-1), node map 12 B per instance per level, gradient 40 B per instance per tree; the
+level entries N_l come from the library (gbdt_get_level_entries).  `roofline` is the partition
+phase (the phase furthest below its bound), per level: bytes / (phase ms per level); the split
+phase and the whole tree are reported beside it.  The design's own streaming bytes and the ncu
+DRAM bytes are side fields.
 """
 import argparse
 import json
@@ -32,15 +41,21 @@ sys.path.insert(0, ROOT)
 
 METRIC = "seconds per tree (depth 6) at 1/2/4/8 B200; split-find HBM GB/s vs peak"
 UNIT = "s/tree"
-# Algorithmic bytes of the two streaming kernels:
-#   k_split   (k_sf_fast + k_sf_gen) per entry of the level: value f32 4 + g-list fp64 8
-#             (+ h-list 8 when h is not a function of g; RLE: the runs replace the 4 value bytes)
-#   k_scatter per entry of the level: val 4 + ins 4 + g 8 + side 1 read; per kept entry (the
-#             next level's entries): val 4 + ins 4 + g 8 written
-#   with RLE the 4 value bytes are not streamed (values come from the runs, a few bytes per run)
-def byte_model(rle):
+# SURVEY.md §8(d) algorithmic bytes (the unit: one active entry at one level)
+def s8d_bytes(loss, rle):
+    """(split B/entry, partition B/entry, nodemap B/instance/level, gradient B/instance/tree)."""
+    gh = 8 if loss == "squared" else 16
+    split = (4 + gh) if rle else (4 + 4 + gh)   # RLE: ins 4 + g/h (+ 8 B per run, not counted here)
+    part = 8 if rle else 16                      # RLE: ins r/w (+ per-run bytes, not counted here)
+    return split, part, 12, 40
+
+
+# The design's own streaming bytes (DESIGN.md §6; g travels with the entries):
+#   split find reads val 4 + g-list 8 per entry (+ h-list 8 when h is stored; RLE: no val)
+#   partition reads val 4 + ins 4 + g 8 + side 1 per entry and writes val 4 + ins 4 + g 8 per kept entry
+def design_bytes(rle):
     v = 0 if rle else 4
-    return 8 + v, 13 + v, 12 + v   # split per entry; scatter read per entry, write per kept entry
+    return 8 + v, 13 + v, 12 + v
 
 
 def parse():
@@ -58,7 +73,8 @@ def parse():
                     help="off: SmartGD ablation, predictions recomputed by tree traversal (P:193-195, Fig. 9)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle CPU time for cpu_baseline")
+    ap.add_argument("--cpu-trees", type=int, default=1, help="oracle trees (full rows) timed for cpu_baseline")
+    ap.add_argument("--ref-trees", type=int, default=2, help="--impl reference: at most this many full-row trees")
     return ap.parse_args()
 
 
@@ -112,34 +128,35 @@ def clock_sampler_stop(proc, dev=0):
     return {"sm_mhz": statistics.median(sm), "sm_max_mhz": smax, "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def oracle_sample_rate(prob, target_s, trees=2):
-    """Oracle seconds per tree on the full workload, estimated from a bounded row sample."""
-    from datagen import synth
+def host_info():
+    model = ""
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"cpu_model": model, "nproc": os.cpu_count()}
+
+
+def oracle_full_rows(prob, trees, depth):
+    """The CPU oracle (single thread, pinned to one core) on the workload's full rows: presort once,
+    then `trees` trees at `depth`.  Returns (seconds per tree, info)."""
     from oracle import oracle
-    n_s = min(prob.n, 20000)
-    while True:
-        sub = _rows(prob, n_s)
+    old = os.sched_getaffinity(0)
+    core = max(old)
+    os.sched_setaffinity(0, {core})  # this (calling) thread only
+    try:
         t0 = time.perf_counter()
-        oracle.presort(sub.indptr, sub.indices, sub.values, sub.n, sub.m)
-        t1 = time.perf_counter()
-        oracle.train(sub, params=dict(n_trees=trees))
-        t2 = time.perf_counter()
-        per_tree = max((t2 - t1) - (t1 - t0), 1e-9) / trees
-        if t2 - t0 > target_s / 4 or n_s >= prob.n:
-            break
-        n_s = min(prob.n, int(n_s * min(8.0, max(2.0, (target_s / 4) / max(t2 - t0, 1e-3)))))
-    scale = prob.nnz / sub.nnz
-    return per_tree * scale, dict(n_rows=n_s, entries=sub.nnz, trees=trees, per_tree_s=per_tree,
-                                  scale=scale, presort_s=t1 - t0), synth
-
-
-def _rows(prob, n_s):
-    from datagen import synth
-    if n_s >= prob.n:
-        return prob
-    e = int(prob.indptr[n_s])
-    return synth.Problem(prob.name + f"[:{n_s}]", n_s, prob.m, prob.indptr[:n_s + 1].copy(),
-                         prob.indices[:e], prob.values[:e], prob.labels[:n_s], prob.params)
+        oracle.train(prob, params=dict(n_trees=trees, max_depth=depth))
+        wall = time.perf_counter() - t0
+        presort, per_tree = oracle.last_timings()
+    finally:
+        os.sched_setaffinity(0, old)
+    info = dict(trees=trees, presort_s=presort, tree_s=per_tree, wall_s=wall, core=core, **host_info())
+    return sum(per_tree) / max(len(per_tree), 1), info
 
 
 def arm_config(args, prob, P, d, world):
@@ -164,19 +181,19 @@ def main():
             return
         prob = synth.make(args.config)
         P = prob.params
-        from oracle import oracle
-        # warm-up: W trees on a small sample (untimed), then the bounded timed sample
-        sub = _rows(prob, min(prob.n, 2000))
-        oracle.train(sub, params=dict(n_trees=max(1, min(args.warmup, 3))))
-        rate, info, _ = oracle_sample_rate(prob, args.cpu_seconds * 2, trees=min(args.steps, 3))
+        d = args.depth or P["max_depth"]
+        trees = max(1, min(args.steps, args.ref_trees))
+        rate, info = oracle_full_rows(prob, trees, d)
+        sample = (f"full rows ({prob.n} x {prob.m}, {prob.nnz} entries), first {trees} tree(s) at depth {d}, "
+                  f"presort {info['presort_s']:.1f} s excluded; 1 thread pinned to core {info['core']} of "
+                  f"{info['nproc']} ({info['cpu_model']})")
         line = {
             "impl": "reference", "metric": METRIC, "value": rate, "unit": UNIT, "n_gpus": args.gpus,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": rate * 1e3, "higher_is_better": False,
-            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": arm_config(args, prob, P, args.depth or P["max_depth"], world),
-            "cpu_baseline": {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": f"first {info['n_rows']} rows ({info['entries']} entries), "
-                                       f"{info['trees']} trees, presort excluded, scaled x{info['scale']:.1f} by entries"},
+            "steps": trees, "steps_requested": args.steps, "warmup": 0, "ms_per_step": rate * 1e3,
+            "higher_is_better": False, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": arm_config(args, prob, P, d, world),
+            "cpu_baseline": {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
+                             "tree_s": info["tree_s"], "presort_s": info["presort_s"]},
             "e2e": {"value": rate, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
         }
         print(json.dumps(line))
@@ -245,25 +262,45 @@ def main():
     nodes = model.nodes()
     ent = model.level_entries(d)                     # list entries per level, summed over the K trees
     peak, peak_kind = peaks()
-    b_split, b_sread, b_swrite = byte_model(args.rle != "off")
-    kern = {
-        "k_split": dict(bytes=float(ent.sum()) * b_split, launches=args.steps * d,
-                        ms=tim["k_split"], bytes_per_entry=b_split),
-        "k_scatter": dict(bytes=float(ent[:-1].sum()) * b_sread + float(ent[1:].sum()) * b_swrite,
-                          launches=args.steps * (d - 1), ms=tim["k_scatter"],
-                          bytes_per_entry=f"{b_sread} read + {b_swrite} per kept entry"),
-    }
-    for kname, kv in kern.items():
-        kv["avg_launch_ms"] = kv["ms"] / kv["launches"]
-        kv["achieved"] = (kv["bytes"] / kv["launches"] / 1e9) / (kv["avg_launch_ms"] / 1e3) if kv["ms"] > 0 else None
-        kv["frac"] = kv["achieved"] / peak if kv["achieved"] else None
-        kv["traffic"] = None
-        tp_path = os.path.join(ROOT, "profiles", f"ncu_{kname}_{args.config}.json")
-        if os.path.exists(tp_path):
-            with open(tp_path) as f:
-                kv["traffic"] = json.load(f).get("dram_bytes_per_launch")
-    dom = max(kern, key=lambda k: kern[k]["ms"])
+    rle = args.rle != "off"
+    sb, pb, nb, gb = s8d_bytes(P["loss"], rle)
+    T = args.steps
+    fused = os.environ.get("GBDT_FUSED", "0") not in ("", "0") and not rle
+    # entries per level summed over the K trees: split find scans every level, the partition
+    # levels 0 .. d-2; per-level (launch) averages divide by K
+    split_bytes = float(ent.sum()) * sb
+    part_bytes = float(ent[:-1].sum()) * pb
+    tree_bytes = split_bytes + part_bytes + T * (nb * prob.n * d + gb * prob.n)
+    traffic = None
+    tp_path = os.path.join(ROOT, "profiles", f"ncu_phases_{args.config}.json")
+    if os.path.exists(tp_path):
+        with open(tp_path) as f:
+            traffic = json.load(f)
 
+    def phase(name, nbytes, ms_total, launches, note):
+        per = nbytes / max(launches, 1)
+        avg = ms_total / max(launches, 1)
+        ach = (per / 1e9) / (avg / 1e3) if ms_total > 0 else None
+        tr = traffic.get(name, {}).get("dram_bytes_per_launch") if traffic else None
+        return {"achieved": ach, "frac": ach / peak if ach else None, "bytes_per_launch": per,
+                "avg_launch_ms": avg, "launches": launches, "traffic": tr, "bytes_model": note}
+
+    if fused:  # one pass per level: partition of level l + split find of level l+1 (fused.cu)
+        part_ph = phase("partition", part_bytes + float(ent[1:].sum()) * sb, tim["partition"], T * (d - 1),
+                        f"{pb} B/entry (partition, levels < d-1) + {sb} B/entry (split find of levels >= 1)")
+        split_ph = phase("split_find", float(ent[0]) * sb, tim["split_find"], T, f"{sb} B/entry, root level")
+    else:
+        part_ph = phase("partition", part_bytes, tim["partition"], T * (d - 1), f"{pb} B/entry, levels < d-1")
+        split_ph = phase("split_find", split_bytes, tim["split_find"], T * d, f"{sb} B/entry, every level")
+    tree_ph = phase("tree", tree_bytes, ms, T,
+                    f"§8(d): {sb} B/entry/level split + {pb} B/entry/level partition + {nb} B/instance/level "
+                    f"node map + {gb} B/instance gradient")
+    # the design's own streaming bytes (g travels with the entries) as a side field
+    d_split, d_sread, d_swrite = design_bytes(rle)
+    design = {"split_find_B_per_entry": d_split, "partition_B_per_entry": f"{d_sread} read + {d_swrite} per kept entry",
+              "split_find_GBps": (float(ent.sum()) * d_split / 1e9) / (tim["split_find"] / 1e3) if tim["split_find"] else None,
+              "partition_GBps": ((float(ent[:-1].sum()) * d_sread + float(ent[1:].sum()) * d_swrite) / 1e9) /
+                                (tim["partition"] / 1e3) if tim["partition"] and not fused else None}
     # e2e through the C ABI from pinned host buffers
     e2e = None
     if not args.no_e2e:
@@ -292,7 +329,8 @@ def main():
         d2h = margin2.nbytes + nodes.nbytes
         e2e = {"value": te / args.steps, "unit": UNIT, "h2d_bytes_per_step": int(h2d / args.steps),
                "d2h_bytes_per_step": int(d2h / args.steps),
-               "note": "one gbdt_load_csr (H2D + layout sort) + K-tree gbdt_train + margin D2H, amortised per tree"}
+               "note": "one gbdt_load_csr (H2D + layout sort) + K-tree gbdt_train + margin D2H, amortised per tree; "
+                       "library memory pool warm (the device-timed run's dataset was freed into it first)"}
         del ds2, model2
 
     # gbdt_predict on the training rows with the K trees: wall clock through the
@@ -310,10 +348,12 @@ def main():
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        rate, cinfo, _ = oracle_sample_rate(prob, args.cpu_seconds)
+        rate, cinfo = oracle_full_rows(prob, max(1, args.cpu_trees), d)
         cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"first {cinfo['n_rows']} rows ({cinfo['entries']} entries), {cinfo['trees']} trees, "
-                         f"presort excluded, scaled x{cinfo['scale']:.1f} by entries"}
+               "sample": f"full rows ({prob.n} x {prob.m}, {prob.nnz} entries), first {cinfo['trees']} tree(s) at "
+                         f"depth {d}, presort {cinfo['presort_s']:.1f} s excluded; 1 thread pinned to core "
+                         f"{cinfo['core']} of {cinfo['nproc']} ({cinfo['cpu_model']})",
+               "tree_s": cinfo["tree_s"], "presort_s": cinfo["presort_s"]}
 
     if rank == 0:
         value = ms / 1e3 / args.steps
@@ -322,11 +362,15 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": False,
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": arm_config(args, prob, P, d, world),
-            "roofline": {"bound": "hbm", "achieved": kern[dom]["achieved"], "peak": peak, "unit": "GB/s",
-                         "frac": kern[dom]["frac"], "traffic": kern[dom]["traffic"], "kernel": dom,
-                         "peak_kind": peak_kind, "bytes_per_launch": kern[dom]["bytes"] / kern[dom]["launches"],
-                         "launches": kern[dom]["launches"], "avg_launch_ms": kern[dom]["avg_launch_ms"],
-                         "kernels": {k: {kk: vv for kk, vv in v.items() if kk != "bytes"} for k, v in kern.items()}},
+            "roofline": {"bound": "hbm", "achieved": part_ph["achieved"], "peak": peak, "unit": "GB/s",
+                         "frac": part_ph["frac"], "traffic": part_ph["traffic"],
+                         "kernel": "partition phase (per level)" + (" = fused partition + next-level split find" if fused else
+                                   ": k_part_count* + count scans + plan + k_part_scatter"),
+                         "peak_kind": peak_kind, "bytes_per_launch": part_ph["bytes_per_launch"],
+                         "launches": part_ph["launches"], "avg_launch_ms": part_ph["avg_launch_ms"],
+                         "bytes_model": part_ph["bytes_model"],
+                         "phases": {"split_find": split_ph, "partition": part_ph, "tree": tree_ph},
+                         "design_bytes": design, "level_entries": [int(x) for x in ent]},
             "phases_ms_per_tree": {k: v / args.steps for k, v in tim.items()},
             "phases_note": "profiled re-run of the same K trees (event timers, eager launches)",
             "cpu_baseline": cpu,
