@@ -66,6 +66,10 @@ def parse():
     ap.add_argument("--config", default="C3")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--rle", default="off")
+    ap.add_argument("--rle-split", default="direct", choices=["direct", "decompress"],
+                    help="RLE node split: direct (P:250, Fig. 7) or the decompression ablation (P:248, Fig. 6)")
+    ap.add_argument("--dense", action="store_true",
+                    help="dense representation, absent values filled with 0 (P:116, P:405-413, SURVEY §8(f4))")
     ap.add_argument("--comm", default="nccl", choices=["nccl", "host"],
                     help="host: gloo + host-staged callbacks (several ranks may share one GPU; testing only)")
     ap.add_argument("--depth", type=int, default=0, help="override the config's max_depth (sweeps, SURVEY §8(f2))")
@@ -163,7 +167,8 @@ def arm_config(args, prob, P, d, world):
     """The `config` object of the JSON line; identical for both arms."""
     return {"workload": args.config, "n": prob.n, "m": prob.m, "nnz": prob.nnz, "loss": P["loss"],
             "max_depth": d, "trees_timed": args.steps, "lambda": P["lam"], "eta": P["eta"],
-            "rle": args.rle, "smartgd": args.smartgd, "parallelism": f"attr-shard{world}",
+            "rle": args.rle, "rle_split": args.rle_split, "dense": args.dense, "smartgd": args.smartgd,
+            "parallelism": f"attr-shard{world}",
             "l2": ("inputs larger than L2 (sorted lists %.2f GB)" % (prob.nnz * 8 / 1e9)) if prob.nnz * 8 > 126e6
                   else "inputs smaller than L2 (%.1f MB), not flushed between trees: latency-bound config"
                   % (prob.nnz * 8 / 1e6)}
@@ -228,11 +233,11 @@ def main():
         comm = gbdt.comm_from_callbacks(local) if host_comm else gbdt.comm_from_torch(local)
     stream = torch.cuda.current_stream()
     ds = gbdt.load_csr(prob.indptr, prob.indices, prob.values, prob.labels, prob.m, rle=args.rle,
-                       stream=stream.cuda_stream, comm=comm, keep_rows=args.smartgd == "off")
+                       stream=stream.cuda_stream, comm=comm, keep_rows=args.smartgd == "off", dense=args.dense)
     info = ds.info(0)
     m_local = info["attr_end"] - info["attr_begin"]
     tp = dict(max_depth=d, lam=P["lam"], gamma=P["gamma"], eta=P["eta"], base_margin=P["base_margin"],
-              loss=P["loss"], smartgd=args.smartgd == "on")
+              loss=P["loss"], smartgd=args.smartgd == "on", rle_split=args.rle_split)
 
     # warm-up (untimed)
     gbdt.train(ds, n_trees=max(args.warmup, 1), want_margin=False, **tp)
@@ -319,7 +324,7 @@ def main():
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         ds2 = gbdt.load_csr(hp, hi, hv, hl, prob.m, rle=args.rle, stream=stream.cuda_stream, comm=comm,
-                            keep_rows=args.smartgd == "off")
+                            keep_rows=args.smartgd == "off", dense=args.dense)
         model2, margin2 = gbdt.train(ds2, n_trees=args.steps, want_margin=True, **tp)
         torch.cuda.synchronize()
         te = time.perf_counter() - t0

@@ -77,6 +77,13 @@ typedef struct {
                              size w and owns attribute range r of w (nnz-balanced, contiguous);
                              n_shards must then be 0 or 1. */
   int32_t keep_rows;      /* 1: keep a device copy of the CSR rows (needed by smartgd_off) */
+  int32_t dense;          /* 1: dense representation (the paper's option "if the data set is
+                             small"): the n_rows x n_cols matrix with every absent or
+                             NaN value replaced by dense_fill ("in the dense presentation, missing
+                             values need to be filled (e.g., treated as 0)").  The trees then
+                             see no missing values; models trained this way fill absent values at
+                             predict time too.  Memory: n_rows * n_cols entries. */
+  float dense_fill;       /* the fill value (0 when zero-initialised) */
 } gbdt_load_opts;
 
 /* Training parameters, as the paper states them: d, T, gamma (Alg. 1 inputs),
@@ -95,7 +102,10 @@ typedef struct {
                              over its CSR row instead of adding its last leaf weight.  Same
                              arithmetic in the same order, so the trees are bit-identical.  Needs
                              a dataset loaded with keep_rows = 1 (else GBDT_E_STATE). */
-  int32_t reserved;       /* 0 */
+  int32_t rle_decompress; /* RLE shards only: 0 = split the runs directly (Fig. 7); 1 = the
+                             paper's baseline "splitting RLE with decompression" (Fig. 6):
+                             decompress, partition the plain lists, re-encode the children.  The
+                             trees are identical; this is the ablation of P:536. */
   gbdt_grad_fn grad_fn;   /* GBDT_LOSS_CUSTOM: the gradient callback (else ignored) */
   void* grad_user;        /* passed through to grad_fn */
 } gbdt_params;

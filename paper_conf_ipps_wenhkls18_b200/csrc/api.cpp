@@ -266,13 +266,27 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
         cudaStreamSynchronize(st);  // the copies still read the caller's buffers
         throw;
       }
+      int64_t nnz_l = nnz;
+      if (o.dense) {  // dense representation: the filled matrix replaces the CSR
+        if (!std::isfinite(o.dense_fill)) fail(GBDT_E_INVAL, "dense_fill must be finite");
+        if ((double)n_rows * (double)n_cols >= (double)kMax) fail(GBDT_E_RANGE, "dense matrix exceeds 2^31 - 1 entries");
+        DBuf fptr, fidx, fval;
+        densify(n_rows, n_cols, dptr.as<int64_t>(), didx.as<int32_t>(), dval.as<float>(), o.dense_fill, fptr, fidx,
+                fval, st);
+        dptr = std::move(fptr);
+        didx = std::move(fidx);
+        dval = std::move(fval);
+        nnz_l = n_rows * n_cols;
+      }
       // present entries per attribute, counted on the device
-      const std::vector<int64_t> col_counts = column_counts(nnz, n_cols, didx.as<int32_t>(), dval.as<float>(), st);
+      const std::vector<int64_t> col_counts = column_counts(nnz_l, n_cols, didx.as<int32_t>(), dval.as<float>(), st);
       bool missing = false;
       for (int64_t a = 0; a < n_cols; ++a) missing |= col_counts[a] != n_rows;
       ds.n = n_rows;
       ds.m = n_cols;
-      ds.nnz = nnz;
+      ds.nnz = nnz_l;
+      ds.dense = o.dense ? 1 : 0;
+      ds.fill = o.dense ? o.dense_fill : 0.f;
       ds.device = dev;
       ds.stream = st;
       ds.has_missing = missing;
@@ -281,10 +295,41 @@ gbdt_status gbdt_load_csr(int64_t n_rows, int64_t n_cols, const int64_t* indptr,
       ds.rle = o.rle;
       ds.h_labels_minmax = {lmin, lmax};
       const int world = comm ? comm->world : 1;
-      const int P = comm ? world : nsh;
-      ds.n_total_shards = P;
+      int P = comm ? world : nsh;
       // contiguous attribute ranges balanced by stored entries
-      const std::vector<int32_t> bnd = shard_ranges(n_cols, col_counts.data(), P);
+      std::vector<int32_t> bnd = shard_ranges(n_cols, col_counts.data(), P);
+      if (o.rle == GBDT_RLE_AUTO && !comm && nsh == 1) {
+        // AUTO per attribute (reading R21 of P:237, "dimensionality / cardinality > R"): attribute a
+        // is compressed iff entries_a / runs_a >= rle_min_ratio.  The runs are counted on an
+        // uncompressed layout; the attributes are then regrouped into shards of equal decision
+        // (maximal contiguous ranges; trees are identical for any attribute sharding), and each
+        // shard's aggregate ratio falls on the same side of the threshold as its attributes.
+        ds.rle = GBDT_RLE_OFF;
+        ds.n_total_shards = 1;
+        auto probe = std::make_unique<Shard>();
+        probe->index = 0; probe->a_begin = 0; probe->a_end = (int32_t)n_cols; probe->m = (int32_t)n_cols;
+        ds.shards.push_back(std::move(probe));
+        build_layout(ds, dptr.as<int64_t>(), didx.as<int32_t>(), dval.as<float>(), col_counts, o.rle_min_ratio);
+        int sms = 148;
+        GBDT_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+        const std::vector<uint32_t> runs = attribute_runs(*ds.shards[0], st, sms);
+        ds.shards.clear();
+        const double thr = o.rle_min_ratio > 0 ? o.rle_min_ratio : 2.0;
+        std::vector<int32_t> groups{0};
+        int prev = -1;
+        for (int64_t a = 0; a < n_cols; ++a) {
+          const int dcs = runs[a] > 0 && (double)col_counts[a] >= thr * (double)runs[a];
+          if (a > 0 && dcs != prev) groups.push_back((int32_t)a);
+          prev = dcs;
+        }
+        groups.push_back((int32_t)n_cols);
+        if (groups.size() - 1 <= 64) {  // else: many alternations, keep the entry-balanced single shard
+          bnd = groups;
+          P = (int)groups.size() - 1;
+        }
+        ds.rle = GBDT_RLE_AUTO;
+      }
+      ds.n_total_shards = P;
       for (int i = 0; i < P; ++i) {
         if (comm && i != comm->rank) continue;
         auto sh = std::make_unique<Shard>();

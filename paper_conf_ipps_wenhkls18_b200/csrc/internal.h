@@ -129,6 +129,8 @@ struct Dataset {
   int32_t n_total_shards = 1;    // across all ranks
   Comm* comm = nullptr;
   int rle = 0;
+  int dense = 0;                 // dense representation: absent values were filled
+  float fill = 0.f;
   DBuf rows_ptr, rows_idx, rows_val;  // CSR rows (gbdt_load_opts.keep_rows; SmartGD-off ablation)
 };
 
@@ -140,6 +142,8 @@ struct Model {
   double timings[GBDT_N_PHASES] = {0};
   std::vector<int64_t> level_entries;  // [max_depth] list entries scanned per level (profile = 1)
   int device = 0;
+  int dense = 0;                 // trained on the dense representation: predict fills absent values
+  float fill = 0.f;
   int64_t nh() const { return (int64_t(1) << (max_depth + 1)) - 1; }
 };
 
@@ -162,6 +166,9 @@ std::vector<int64_t> column_counts(int64_t nnz, int64_t m, const int32_t* d_indi
 void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices,
                   const float* d_values, const std::vector<int64_t>& col_counts,
                   double rle_min_ratio);
+std::vector<uint32_t> attribute_runs(const Shard& sh, cudaStream_t st, int sms);
+void densify(int64_t n, int64_t m, const int64_t* d_indptr, const int32_t* d_idx, const float* d_val, float fill,
+             DBuf& optr, DBuf& oidx, DBuf& oval, cudaStream_t st);
 // train.cu
 void train(Dataset& ds, const gbdt_params& p, Model& model, double* margin_out);
 // predict.cu

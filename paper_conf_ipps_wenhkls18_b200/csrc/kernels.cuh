@@ -219,6 +219,10 @@ struct LevelKernels {
   // a3: the level's chunk descriptors and scan flags when the previous scatter accumulated the
   // chunk aggregates, then the exact carry scan
   void chunk_desc(const SplitArgs& A, unsigned groups, cudaStream_t st);
+  // RLE split ablation (Fig. 6): decompress a level's runs into its value list; compress
+  // the next level's value list (per node segment) into its run tables
+  void rle_decompress(const Tables& tb, float* val, cudaStream_t st);
+  void rle_encode(const Tables& tn, int m, const int32_t* Knp, const float* val, uint32_t* cnt, cudaStream_t st);
 };
 
 }  // namespace gbdt

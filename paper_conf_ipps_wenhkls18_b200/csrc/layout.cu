@@ -260,6 +260,50 @@ __global__ void k_col_hist(int64_t nnz, int64_t m, const int32_t* __restrict__ i
 
 }  // namespace
 
+// Dense representation: the n x m matrix with every absent (or NaN)
+// value filled with `fill` (the paper: "in the dense presentation, missing values need to be
+// filled (e.g., treated as 0)"), as CSR rows of m entries each.  One thread per row.
+__global__ void k_densify(int64_t n, int64_t m, const int64_t* __restrict__ indptr, const int32_t* __restrict__ idx,
+                          const float* __restrict__ val, float fill, int64_t* __restrict__ dptr,
+                          int32_t* __restrict__ didx, float* __restrict__ dval) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    float* row = dval + i * m;
+    int32_t* ri = didx + i * m;
+    for (int64_t a = 0; a < m; ++a) { row[a] = fill; ri[a] = (int32_t)a; }
+    for (int64_t p = indptr[i]; p < indptr[i + 1]; ++p) {
+      const int32_t a = idx[p];
+      const float v = val[p];
+      if (a < m && !isnan(v)) row[a] = v == 0.0f ? 0.0f : v;
+    }
+    dptr[i] = i * m;
+    if (i == n - 1) dptr[n] = n * m;
+  }
+}
+
+void densify(int64_t n, int64_t m, const int64_t* d_indptr, const int32_t* d_idx, const float* d_val, float fill,
+             DBuf& optr, DBuf& oidx, DBuf& oval, cudaStream_t st) {
+  optr.alloc((size_t)(n + 1) * 8, st);
+  oidx.alloc((size_t)std::max<int64_t>(n * m, 1) * 4, st);
+  oval.alloc((size_t)std::max<int64_t>(n * m, 1) * 4, st);
+  const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 8));
+  k_densify<<<grid, 256, 0, st>>>(n, m, d_indptr, d_idx, d_val, fill, optr.as<int64_t>(), oidx.as<int32_t>(),
+                                  oval.as<float>());
+  GBDT_LAUNCH_CHECK();
+}
+
+// Runs (distinct values) of every attribute list of a built, uncompressed shard (AUTO RLE).
+std::vector<uint32_t> attribute_runs(const Shard& sh, cudaStream_t st, int sms) {
+  std::vector<uint32_t> hc((size_t)std::max(sh.m, 0), 0u);
+  if (sh.m == 0 || sh.nnz == 0) return hc;
+  DBuf cnt((size_t)sh.m * 4, st);
+  k_run_heads<<<(unsigned)std::min(sh.m, sms * 8), 256, 0, st>>>(sh.m, sh.root.col_start, sh.root.col_len,
+                                                               sh.val0.as<float>(), cnt.as<uint32_t>());
+  GBDT_LAUNCH_CHECK();
+  GBDT_CUDA(cudaMemcpyAsync(hc.data(), cnt.p, (size_t)sh.m * 4, cudaMemcpyDeviceToHost, st));
+  GBDT_CUDA(cudaStreamSynchronize(st));
+  return hc;
+}
+
 std::vector<int64_t> column_counts(int64_t nnz, int64_t m, const int32_t* d_indices, const float* d_values,
                                    cudaStream_t st) {
   int dev = 0, sms = 148;

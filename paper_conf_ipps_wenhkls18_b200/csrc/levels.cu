@@ -2302,6 +2302,115 @@ __global__ void __launch_bounds__(kThreads) k_run_scatter(RunArgs A) {
   }
 }
 
+// ---------------------------------------------------------------------------- RLE split ablation
+// "Splitting RLE with decompression" (Fig. 6), the baseline the paper's direct RLE split
+// (Fig. 7) is measured against: the level's runs are decompressed into the value
+// list, the entries are partitioned as plain lists (values moving with them), and the children
+// are compressed again -- one run per maximal group of equal values inside each (node, attribute)
+// segment.  Produces exactly the tables of the direct split (RLE(filter(root column))).
+__global__ void __launch_bounds__(kThreads) k_rle_decompress(Tables tb, float* __restrict__ val) {
+  const int R = *tb.R;
+  const int lane = threadIdx.x & 31;
+  for (int r = blockIdx.x * kWarps + (threadIdx.x >> 5); r < R; r += gridDim.x * kWarps) {
+    const long long P = tb.run_pos[r];
+    const int L = tb.run_len[r];
+    const float v = tb.run_val[r];
+    for (int q = lane; q < L; q += 32) val[P + q] = v;
+  }
+}
+
+// runs per next-level segment (one warp per segment)
+__global__ void __launch_bounds__(kThreads) k_enc_count(Tables tn, int m, const int32_t* __restrict__ Knp,
+                                                        const float* __restrict__ val, uint32_t* __restrict__ cnt) {
+  const long long S = (long long)m * *Knp;
+  const int lane = threadIdx.x & 31;
+  for (long long s = (long long)blockIdx.x * kWarps + (threadIdx.x >> 5); s <= S; s += (long long)gridDim.x * kWarps) {
+    uint32_t c = 0;
+    if (s < S) {
+      const long long b = tn.seg_start[s], L = tn.seg_cnt[s];
+      for (long long q = lane; q < L; q += 32) c += (q == 0 || val[b + q] != val[b + q - 1]) ? 1u : 0u;
+      for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+    }
+    if (lane == 0) cnt[s] = c;
+  }
+}
+
+// exclusive scan of the S + 1 counts -> the segment -> first run table, R
+__global__ void k_enc_scan(Tables tn, int m, const int32_t* __restrict__ Knp, const uint32_t* __restrict__ cnt) {
+  __shared__ uint32_t ws[32];
+  __shared__ uint32_t carry;
+  const long long n = (long long)m * *Knp + 1;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  for (long long base = 0; base < n; base += blockDim.x) {
+    const long long i = base + threadIdx.x;
+    const uint32_t x = i < n ? cnt[i] : 0u;
+    uint32_t incl = x;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += y;
+    }
+    if (lane == 31) ws[w] = incl;
+    __syncthreads();
+    if (w == 0) {
+      const uint32_t s0 = lane < nw ? ws[lane] : 0u;
+      uint32_t si = s0;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, si, o);
+        if (lane >= o) si += y;
+      }
+      if (lane < nw) ws[lane] = si - s0;
+    }
+    __syncthreads();
+    const uint32_t c = carry;
+    if (i < n) {
+      tn.seg_run[i] = (int32_t)(c + ws[w] + incl - x);
+      if (i == n - 1) *tn.R = (int32_t)(c + ws[w] + incl - x);
+    }
+    __syncthreads();
+    if (threadIdx.x == blockDim.x - 1) carry = c + ws[w] + incl;
+    __syncthreads();
+  }
+}
+
+// the runs themselves (one warp per segment, heads by ballots), their positions and run_chunk
+__global__ void __launch_bounds__(kThreads) k_enc_fill(Tables tn, int m, const int32_t* __restrict__ Knp,
+                                                       const float* __restrict__ val) {
+  const int Kn = *Knp;
+  const long long S = (long long)m * Kn;
+  const int lane = threadIdx.x & 31;
+  for (long long s = (long long)blockIdx.x * kWarps + (threadIdx.x >> 5); s < S; s += (long long)gridDim.x * kWarps) {
+    const long long b = tn.seg_start[s], L = tn.seg_cnt[s];
+    if (L == 0) continue;
+    const int a = (int)(s / Kn);
+    int r = tn.seg_run[s] - 1;
+    long long begin = 0;
+    for (long long base = 0; base < L; base += 32) {
+      const long long q = base + lane;
+      const bool head = q < L && (q == 0 || val[b + q] != val[b + q - 1]);
+      unsigned hm = __ballot_sync(0xffffffffu, head);
+      while (hm) {
+        const long long qh = base + (__ffs(hm) - 1);
+        hm &= hm - 1;
+        if (r >= tn.seg_run[s] && lane == 0) {  // close the previous run [begin, qh)
+          tn.run_len[r] = (int32_t)(qh - begin);
+          tn.run_pos[r] = b + begin;
+          fill_run_chunks(tn.run_chunk, tn, a, b + begin, qh - begin, r);
+        }
+        ++r;
+        begin = qh;
+        if (lane == 0) tn.run_val[r] = val[b + qh];
+      }
+    }
+    if (lane == 0) {
+      tn.run_len[r] = (int32_t)(L - begin);
+      tn.run_pos[r] = b + begin;
+      fill_run_chunks(tn.run_chunk, tn, a, b + begin, L - begin, r);
+    }
+  }
+}
+
 template <class KernelT>
 unsigned grid_for(KernelT kern, size_t smem, int sms) {
   if (smem) GBDT_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -2488,6 +2597,21 @@ void LevelKernels::partition_scatter(const PartArgs& A, int hmode, const RunArgs
   }
   GBDT_LAUNCH_CHECK();
   count_launch();
+}
+
+void LevelKernels::rle_decompress(const Tables& tb, float* val, cudaStream_t st) {
+  k_rle_decompress<<<(unsigned)(sms * 8), kThreads, 0, st>>>(tb, val);
+  GBDT_LAUNCH_CHECK();
+  count_launch();
+}
+
+void LevelKernels::rle_encode(const Tables& tn, int m, const int32_t* Knp, const float* val, uint32_t* cnt,
+                              cudaStream_t st) {
+  k_enc_count<<<(unsigned)(sms * 8), kThreads, 0, st>>>(tn, m, Knp, val, cnt);
+  k_enc_scan<<<1, 1024, 0, st>>>(tn, m, Knp, cnt);
+  k_enc_fill<<<(unsigned)(sms * 8), kThreads, 0, st>>>(tn, m, Knp, val);
+  GBDT_LAUNCH_CHECK();
+  count_launch(3);
 }
 
 void LevelKernels::chunk_desc(const SplitArgs& A, unsigned groups, cudaStream_t st) {

@@ -93,6 +93,13 @@ void predict(const Model& m, int64_t n_rows, int64_t n_cols, const int64_t* indp
     GBDT_CUDA(cudaMemcpyAsync(didx.p, indices, (size_t)nnz * 4, cudaMemcpyHostToDevice, st));
     GBDT_CUDA(cudaMemcpyAsync(dval.p, values, (size_t)nnz * 4, cudaMemcpyHostToDevice, st));
   }
+  if (m.dense) {  // trained on the dense representation: absent values are filled here too
+    DBuf fptr, fidx, fval;
+    densify(n_rows, m.n_cols, dptr.as<int64_t>(), didx.as<int32_t>(), dval.as<float>(), m.fill, fptr, fidx, fval, st);
+    dptr = std::move(fptr);
+    didx = std::move(fidx);
+    dval = std::move(fval);
+  }
   GBDT_CUDA(cudaMemcpyAsync(dnodes.p, m.nodes.data(), m.nodes.size() * sizeof(gbdt_node), cudaMemcpyHostToDevice, st));
   const int sig = (!output_margin && m.loss == GBDT_LOSS_LOGISTIC) ? 1 : 0;
   if (m.n_cols <= kDenseCols) {  // split attributes are < the training n_cols; other columns are ignored

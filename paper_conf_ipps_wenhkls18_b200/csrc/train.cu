@@ -429,6 +429,7 @@ struct ShardWork {
   unsigned long long *run_hl = nullptr, *rcnt = nullptr, *rfl = nullptr, *rsgrp = nullptr;
   int32_t* Rp1 = nullptr;
   unsigned rgroups = 1;
+  uint32_t* enc_cnt = nullptr;  // RLE split ablation: runs per next-level segment
   // fused dense levels: plans of two levels, per-tile records / carries / side bits
   DBuf fz;
   FusedPlan* fplan[2] = {nullptr, nullptr};
@@ -672,6 +673,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         q.take<int32_t>(Rcap); q.take<unsigned long long>(Rcap); q.take<unsigned long long>(2 * Rcap);
         q.take<unsigned long long>(2 * (Rcap + 1)); q.take<int32_t>(1);
         q.take<unsigned long long>(2 * (size_t)w.rgroups + 8);
+        q.take<uint32_t>((size_t)S + 1);
       };
       Carve rp{nullptr};
       rz(rp);
@@ -687,6 +689,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       w.run_seg = r.take<int32_t>(Rcap); w.run_hl = r.take<unsigned long long>(Rcap);
       w.rcnt = r.take<unsigned long long>(2 * Rcap); w.rfl = r.take<unsigned long long>(2 * (Rcap + 1));
       w.Rp1 = r.take<int32_t>(1); w.rsgrp = r.take<unsigned long long>(2 * (size_t)w.rgroups + 8);
+      w.enc_cnt = r.take<uint32_t>((size_t)S + 1);
     }
     if (fused && m > 0) {
       w.tiles = fused_tiles(n, m);
@@ -918,13 +921,21 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
           RA.slist = w.slist; RA.cpre = w.cpre; RA.run_seg = w.run_seg; RA.run_hl = w.run_hl; RA.cnt = w.rcnt; RA.fl = w.rfl;
           RA.Rp1 = w.Rp1; RA.sgrp = w.rsgrp; RA.groups = w.rgroups;
         }
+        // RLE split ablation (gbdt_params.rle_decompress, Fig. 6): the runs are decompressed
+        // into the level's value list, the lists partitioned as plain ones, the children re-encoded
+        const bool dec = sh.rle && P.rle_decompress;
+        if (dec && lvl > 0) {
+          LK.rle_decompress(tb, sh.valw[lvl & 1].as<float>(), st);
+          PA.t.val = sh.valw[lvl & 1].as<float>();
+        }
         kt.begin(GBDT_PHASE_K_COUNT);
         LK.partition_count(PA, PL, ds.has_missing, w.groups, st);
         kt.end();
         kt.begin(GBDT_PHASE_K_SCATTER);
         if (PA.cagg_next)
           GBDT_CUDA(cudaMemsetAsync(w.cagg, 0, sizeof(unsigned long long) * 5 * (size_t)std::max<int64_t>(sh.C0, 1), st));
-        LK.partition_scatter(PA, hmode, sh.rle ? &RA : nullptr, st);
+        LK.partition_scatter(PA, hmode, (sh.rle && !dec) ? &RA : nullptr, st);
+        if (dec) LK.rle_encode(tn, sh.m, nxt.K, sh.valw[(lvl + 1) & 1].as<float>(), w.enc_cnt, st);
         kt.end();
       }
       tm.end();
@@ -997,6 +1008,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   model.n_cols = ds.m;
   model.eta = P.eta;
   model.base_margin = P.base_margin;
+  model.dense = ds.dense;
+  model.fill = ds.fill;
   model.lambda = P.lambda;
   model.device = ds.device;
   model.nodes.resize((size_t)P.n_trees * NH);

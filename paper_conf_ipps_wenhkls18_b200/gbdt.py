@@ -41,7 +41,8 @@ class GbdtError(RuntimeError):
 
 class _LoadOpts(C.Structure):
     _fields_ = [("rle", C.c_int32), ("rle_min_ratio", C.c_double), ("n_shards", C.c_int32),
-                ("device", C.c_int32), ("stream", C.c_void_p), ("comm", C.c_void_p), ("keep_rows", C.c_int32)]
+                ("device", C.c_int32), ("stream", C.c_void_p), ("comm", C.c_void_p), ("keep_rows", C.c_int32),
+                ("dense", C.c_int32), ("dense_fill", C.c_float)]
 
 
 # gbdt_grad_fn(n, yhat, labels, g, h, stream, user): device pointers (GBDT_LOSS_CUSTOM)
@@ -52,7 +53,7 @@ class _Params(C.Structure):
     _fields_ = [("max_depth", C.c_int32), ("n_trees", C.c_int32), ("lam", C.c_double),
                 ("gamma", C.c_double), ("eta", C.c_double), ("base_margin", C.c_double),
                 ("loss", C.c_int32), ("profile", C.c_int32), ("smartgd_off", C.c_int32),
-                ("reserved", C.c_int32), ("grad_fn", GRAD_FN), ("grad_user", C.c_void_p)]
+                ("rle_decompress", C.c_int32), ("grad_fn", GRAD_FN), ("grad_user", C.c_void_p)]
 
 
 _lib = None
@@ -293,7 +294,8 @@ class Model:
 
 
 def load_csr(indptr, indices, values, labels, n_cols, rle="off", rle_min_ratio=0.0, n_shards=1,
-             device=-1, stream="current", comm: Comm | None = None, keep_rows=False) -> Dataset:
+             device=-1, stream="current", comm: Comm | None = None, keep_rows=False, dense=False,
+             dense_fill=0.0) -> Dataset:
     indptr = np.ascontiguousarray(indptr, np.int64)
     indices = np.ascontiguousarray(indices, np.int32)
     values = np.ascontiguousarray(values, np.float32)
@@ -302,7 +304,7 @@ def load_csr(indptr, indices, values, labels, n_cols, rle="off", rle_min_ratio=0
     if stream == "current":
         stream = _current_stream()
     o = _LoadOpts(RLE[rle], float(rle_min_ratio), int(n_shards), int(device), stream,
-                  comm._h if comm is not None else None, int(bool(keep_rows)))
+                  comm._h if comm is not None else None, int(bool(keep_rows)), int(bool(dense)), float(dense_fill))
     h = C.c_void_p()
     _check(lib().gbdt_load_csr(n, int(n_cols), _p(indptr), _p(indices), _p(values), _p(labels), C.byref(o),
                                C.byref(h)))
@@ -310,9 +312,10 @@ def load_csr(indptr, indices, values, labels, n_cols, rle="off", rle_min_ratio=0
 
 
 def train(ds: Dataset, max_depth=6, n_trees=40, lam=1.0, gamma=0.0, eta=0.3, base_margin=0.0,
-          loss="squared", profile=False, want_margin=True, smartgd=True, grad_fn=None):
+          loss="squared", profile=False, want_margin=True, smartgd=True, grad_fn=None, rle_split="direct"):
     """grad_fn (loss="custom"): python callable (n, yhat, labels, g, h, stream) -> None over
-    DEVICE addresses, run on the library's stream (see gbdt_grad_fn in include/gbdt.h)."""
+    DEVICE addresses, run on the library's stream (see gbdt_grad_fn in include/gbdt.h).
+    rle_split: "direct" (Fig. 7) or "decompress" (the P:248 / Fig. 6 ablation)."""
     cb = GRAD_FN()
     if grad_fn is not None:
         def _tramp(n, yh, y, g, h, st, user):
@@ -325,7 +328,7 @@ def train(ds: Dataset, max_depth=6, n_trees=40, lam=1.0, gamma=0.0, eta=0.3, bas
                 return 1
         cb = GRAD_FN(_tramp)
     prm = _Params(int(max_depth), int(n_trees), float(lam), float(gamma), float(eta), float(base_margin),
-                  LOSS[loss], int(bool(profile)), int(not smartgd), 0, cb, None)
+                  LOSS[loss], int(bool(profile)), int(not smartgd), {"direct": 0, "decompress": 1}[rle_split], cb, None)
     h = C.c_void_p()
     margin = np.zeros(ds.n, np.float64) if want_margin else None
     _check(lib().gbdt_train(ds._h, C.byref(prm), C.byref(h), _p(margin)))
@@ -351,7 +354,9 @@ def train_problem(prob, **overrides):
     P.update(overrides)
     rle = P.pop("rle", "off")
     n_shards = P.pop("n_shards", 1)
+    dense = P.pop("dense", False)
+    dense_fill = P.pop("dense_fill", 0.0)
     keep_rows = not P.get("smartgd", True)  # the SmartGD-off ablation traverses the CSR rows
     ds = load_csr(prob.indptr, prob.indices, prob.values, prob.labels, prob.m, rle=rle, n_shards=n_shards,
-                  keep_rows=keep_rows)
+                  keep_rows=keep_rows, dense=dense, dense_fill=dense_fill)
     return train(ds, **P)
