@@ -195,6 +195,13 @@ def c4b(seed=42, n=72_201, m=20_938, T=40) -> Problem:
     return c4(seed=seed, n=n, m=m, T=T, name="C4b")
 
 
+def c4s(seed=43, n=20_000, m=400, T=40) -> Problem:
+    """A SMALL sparse dataset (news20-shaped, 2 % density; 20k x 400 = 8M cells) for the dense-
+    representation ablation of SURVEY §8(f4) (dense "if the data set is small").  Not a
+    BASELINE.json config."""
+    return c4(seed=seed, n=n, m=m, density=0.02, T=T, name="C4s")
+
+
 def c5(seed=5, n=5_000_000, T=40, bins=64) -> Problem:
     """susy-shaped, low cardinality: continuous draws quantised into <=64 quantile bins per
     attribute, value = bin centre (fp32), so each root column has <=64 runs (RLE-heavy)."""
@@ -240,6 +247,7 @@ CONFIGS = {
     "C3": c3,
     "C4a": c4,
     "C4b": c4b,
+    "C4s": c4s,
     "C5": c5,
 }
 

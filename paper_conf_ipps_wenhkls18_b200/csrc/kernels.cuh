@@ -222,7 +222,8 @@ struct LevelKernels {
   // RLE split ablation (Fig. 6): decompress a level's runs into its value list; compress
   // the next level's value list (per node segment) into its run tables
   void rle_decompress(const Tables& tb, float* val, cudaStream_t st);
-  void rle_encode(const Tables& tn, int m, const int32_t* Knp, const float* val, uint32_t* cnt, cudaStream_t st);
+  void rle_encode(const Tables& tn, int m, const int32_t* Knp, const float* val, uint32_t* cnt, uint32_t* sbits,
+                  size_t sbits_bytes, cudaStream_t st);
 };
 
 }  // namespace gbdt

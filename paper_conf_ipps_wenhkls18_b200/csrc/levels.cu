@@ -2319,33 +2319,57 @@ __global__ void __launch_bounds__(kThreads) k_rle_decompress(Tables tb, float* _
   }
 }
 
-// runs per next-level segment (one warp per segment)
-__global__ void __launch_bounds__(kThreads) k_enc_count(Tables tn, int m, const int32_t* __restrict__ Knp,
-                                                        const float* __restrict__ val, uint32_t* __restrict__ cnt) {
+// Encoding the next level's lists, entry-parallel (one warp per 256-entry chunk of the next
+// level's tables): an entry starts a run iff it starts its (node, attribute) segment or its value
+// differs from the previous entry's.  Segment starts are marked in a bitmap first.
+__device__ __forceinline__ bool enc_head(const Tables& tn, const float* val, const uint32_t* sbits, long long p) {
+  return ((sbits[p >> 5] >> (p & 31)) & 1u) || val[p] != val[p - 1];
+}
+
+__global__ void k_enc_mark(Tables tn, int m, const int32_t* __restrict__ Knp, uint32_t* __restrict__ sbits) {
   const long long S = (long long)m * *Knp;
-  const int lane = threadIdx.x & 31;
-  for (long long s = (long long)blockIdx.x * kWarps + (threadIdx.x >> 5); s <= S; s += (long long)gridDim.x * kWarps) {
-    uint32_t c = 0;
-    if (s < S) {
-      const long long b = tn.seg_start[s], L = tn.seg_cnt[s];
-      for (long long q = lane; q < L; q += 32) c += (q == 0 || val[b + q] != val[b + q - 1]) ? 1u : 0u;
-      for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+  for (long long s = (long long)blockIdx.x * blockDim.x + threadIdx.x; s < S; s += (long long)gridDim.x * blockDim.x)
+    if (tn.seg_cnt[s] > 0) {
+      const long long p = tn.seg_start[s];
+      atomicOr(sbits + (p >> 5), 1u << (p & 31));
     }
-    if (lane == 0) cnt[s] = c;
+}
+
+__device__ __forceinline__ void enc_chunk_range(const Tables& tn, int c, long long& p0, long long& p1, int& a) {
+  a = tn.chunk_attr[c];
+  const long long cs = tn.col_start[a];
+  p0 = cs + (long long)(c - tn.chunk_start[a]) * kChunk;
+  p1 = min(p0 + (long long)kChunk, cs + tn.col_len[a]);
+}
+
+__global__ void __launch_bounds__(kThreads) k_enc_count(Tables tn, const float* __restrict__ val,
+                                                        const uint32_t* __restrict__ sbits, uint32_t* __restrict__ cnt) {
+  const int C = *tn.C;
+  const int lane = threadIdx.x & 31;
+  for (int c = blockIdx.x * kWarps + (threadIdx.x >> 5); c <= C; c += gridDim.x * kWarps) {
+    uint32_t k = 0;
+    if (c < C) {
+      long long p0, p1;
+      int a;
+      enc_chunk_range(tn, c, p0, p1, a);
+      for (long long p = p0 + lane; p < p1; p += 32) k += enc_head(tn, val, sbits, p) ? 1u : 0u;
+      for (int o = 16; o; o >>= 1) k += __shfl_xor_sync(0xffffffffu, k, o);
+    }
+    if (lane == 0) cnt[c] = k;
   }
 }
 
-// exclusive scan of the S + 1 counts -> the segment -> first run table, R
-__global__ void k_enc_scan(Tables tn, int m, const int32_t* __restrict__ Knp, const uint32_t* __restrict__ cnt) {
+// single-CTA exclusive scan of n counts in place; *total = the sum
+__global__ void k_enc_scan(uint32_t* __restrict__ a, const int32_t* __restrict__ np, int32_t* __restrict__ total) {
   __shared__ uint32_t ws[32];
   __shared__ uint32_t carry;
-  const long long n = (long long)m * *Knp + 1;
+  const long long n = (long long)*np + 1;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
   if (threadIdx.x == 0) carry = 0;
   __syncthreads();
   for (long long base = 0; base < n; base += blockDim.x) {
     const long long i = base + threadIdx.x;
-    const uint32_t x = i < n ? cnt[i] : 0u;
+    const uint32_t x = i < n ? a[i] : 0u;
     uint32_t incl = x;
     for (int o = 1; o < 32; o <<= 1) {
       const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
@@ -2365,8 +2389,8 @@ __global__ void k_enc_scan(Tables tn, int m, const int32_t* __restrict__ Knp, co
     __syncthreads();
     const uint32_t c = carry;
     if (i < n) {
-      tn.seg_run[i] = (int32_t)(c + ws[w] + incl - x);
-      if (i == n - 1) *tn.R = (int32_t)(c + ws[w] + incl - x);
+      a[i] = c + ws[w] + incl - x;
+      if (i == n - 1) *total = (int32_t)(c + ws[w] + incl - x);
     }
     __syncthreads();
     if (threadIdx.x == blockDim.x - 1) carry = c + ws[w] + incl;
@@ -2374,40 +2398,74 @@ __global__ void k_enc_scan(Tables tn, int m, const int32_t* __restrict__ Knp, co
   }
 }
 
-// the runs themselves (one warp per segment, heads by ballots), their positions and run_chunk
-__global__ void __launch_bounds__(kThreads) k_enc_fill(Tables tn, int m, const int32_t* __restrict__ Knp,
-                                                       const float* __restrict__ val) {
-  const int Kn = *Knp;
-  const long long S = (long long)m * Kn;
+// run values / positions (heads ranked by ballots); a segment's first run recorded in seg_run
+__global__ void __launch_bounds__(kThreads) k_enc_heads(Tables tn, int m, const int32_t* __restrict__ Knp,
+                                                        const float* __restrict__ val, const uint32_t* __restrict__ sbits,
+                                                        const uint32_t* __restrict__ base) {
+  const int C = *tn.C, Kn = *Knp;
   const int lane = threadIdx.x & 31;
-  for (long long s = (long long)blockIdx.x * kWarps + (threadIdx.x >> 5); s < S; s += (long long)gridDim.x * kWarps) {
-    const long long b = tn.seg_start[s], L = tn.seg_cnt[s];
-    if (L == 0) continue;
-    const int a = (int)(s / Kn);
-    int r = tn.seg_run[s] - 1;
-    long long begin = 0;
-    for (long long base = 0; base < L; base += 32) {
-      const long long q = base + lane;
-      const bool head = q < L && (q == 0 || val[b + q] != val[b + q - 1]);
-      unsigned hm = __ballot_sync(0xffffffffu, head);
-      while (hm) {
-        const long long qh = base + (__ffs(hm) - 1);
-        hm &= hm - 1;
-        if (r >= tn.seg_run[s] && lane == 0) {  // close the previous run [begin, qh)
-          tn.run_len[r] = (int32_t)(qh - begin);
-          tn.run_pos[r] = b + begin;
-          fill_run_chunks(tn.run_chunk, tn, a, b + begin, qh - begin, r);
+  for (int c = blockIdx.x * kWarps + (threadIdx.x >> 5); c < C; c += gridDim.x * kWarps) {
+    long long p0, p1;
+    int a;
+    enc_chunk_range(tn, c, p0, p1, a);
+    uint32_t r = base[c];
+    for (long long q = p0; q < p1; q += 32) {
+      const long long p = q + lane;
+      const bool h = p < p1 && enc_head(tn, val, sbits, p);
+      const unsigned hm = __ballot_sync(0xffffffffu, h);
+      if (h) {
+        const uint32_t rr = r + __popc(hm & ((1u << lane) - 1u));
+        tn.run_val[rr] = val[p];
+        tn.run_pos[rr] = p;
+        if ((sbits[p >> 5] >> (p & 31)) & 1u) {  // a segment start: which segment of attribute a
+          const int64_t* ss = tn.seg_start + (long long)a * Kn;
+          int lo = 0, hi = Kn - 1;  // the non-empty segment starting at p: the last with start <= p
+          while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (ss[mid] <= p) lo = mid; else hi = mid - 1;
+          }
+          tn.seg_run[(long long)a * Kn + lo] = (int32_t)rr;
         }
-        ++r;
-        begin = qh;
-        if (lane == 0) tn.run_val[r] = val[b + qh];
       }
+      r += __popc(hm);
     }
-    if (lane == 0) {
-      tn.run_len[r] = (int32_t)(L - begin);
-      tn.run_pos[r] = b + begin;
-      fill_run_chunks(tn.run_chunk, tn, a, b + begin, L - begin, r);
+  }
+}
+
+// run lengths (up to the next run or the segment's end) and the run -> chunk index
+__global__ void __launch_bounds__(kThreads) k_enc_len(Tables tn, int m, const int32_t* __restrict__ Knp) {
+  const int R = *tn.R, Kn = *Knp;
+  for (int r = blockIdx.x * blockDim.x + threadIdx.x; r < R; r += gridDim.x * blockDim.x) {
+    const long long p = tn.run_pos[r];
+    int lo = 0, hi = m - 1;  // attribute of p
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (tn.col_start[mid] <= p) lo = mid; else hi = mid - 1;
     }
+    const int a = lo;
+    const int64_t* ss = tn.seg_start + (long long)a * Kn;
+    const int64_t* sc = tn.seg_cnt + (long long)a * Kn;
+    int j0 = 0, j1 = Kn - 1;  // segment of p: the last with start <= p (segments tile the list)
+    while (j0 < j1) {
+      const int mid = (j0 + j1 + 1) >> 1;
+      if (ss[mid] <= p) j0 = mid; else j1 = mid - 1;
+    }
+    const long long se = ss[j0] + sc[j0];
+    const long long nx = r + 1 < R ? tn.run_pos[r + 1] : se;
+    const long long L = min(nx, se) - p;
+    tn.run_len[r] = (int32_t)L;
+    fill_run_chunks(tn.run_chunk, tn, a, p, L, r);
+  }
+}
+
+// empty segments point at the next segment's first run; seg_run[S] = R (one thread, backwards)
+__global__ void k_enc_segfix(Tables tn, int m, const int32_t* __restrict__ Knp) {
+  const long long S = (long long)m * *Knp;
+  int next = *tn.R;
+  tn.seg_run[S] = next;
+  for (long long s = S - 1; s >= 0; --s) {
+    if (tn.seg_cnt[s] == 0) tn.seg_run[s] = next;
+    next = tn.seg_run[s];
   }
 }
 
@@ -2606,12 +2664,16 @@ void LevelKernels::rle_decompress(const Tables& tb, float* val, cudaStream_t st)
 }
 
 void LevelKernels::rle_encode(const Tables& tn, int m, const int32_t* Knp, const float* val, uint32_t* cnt,
-                              cudaStream_t st) {
-  k_enc_count<<<(unsigned)(sms * 8), kThreads, 0, st>>>(tn, m, Knp, val, cnt);
-  k_enc_scan<<<1, 1024, 0, st>>>(tn, m, Knp, cnt);
-  k_enc_fill<<<(unsigned)(sms * 8), kThreads, 0, st>>>(tn, m, Knp, val);
+                              uint32_t* sbits, size_t sbits_bytes, cudaStream_t st) {
+  GBDT_CUDA(cudaMemsetAsync(sbits, 0, sbits_bytes, st));
+  k_enc_mark<<<(unsigned)(sms * 4), kThreads, 0, st>>>(tn, m, Knp, sbits);
+  k_enc_count<<<(unsigned)(sms * 8), kThreads, 0, st>>>(tn, val, sbits, cnt);
+  k_enc_scan<<<1, 1024, 0, st>>>(cnt, tn.C, tn.R);
+  k_enc_heads<<<(unsigned)(sms * 8), kThreads, 0, st>>>(tn, m, Knp, val, sbits, cnt);
+  k_enc_len<<<(unsigned)(sms * 8), kThreads, 0, st>>>(tn, m, Knp);
+  k_enc_segfix<<<1, 1, 0, st>>>(tn, m, Knp);
   GBDT_LAUNCH_CHECK();
-  count_launch(3);
+  count_launch(6);
 }
 
 void LevelKernels::chunk_desc(const SplitArgs& A, unsigned groups, cudaStream_t st) {

@@ -429,7 +429,8 @@ struct ShardWork {
   unsigned long long *run_hl = nullptr, *rcnt = nullptr, *rfl = nullptr, *rsgrp = nullptr;
   int32_t* Rp1 = nullptr;
   unsigned rgroups = 1;
-  uint32_t* enc_cnt = nullptr;  // RLE split ablation: runs per next-level segment
+  uint32_t* enc_cnt = nullptr;   // RLE split ablation: runs per next-level chunk
+  uint32_t* enc_bits = nullptr;  //   and the next level's segment-start bitmap
   // fused dense levels: plans of two levels, per-tile records / carries / side bits
   DBuf fz;
   FusedPlan* fplan[2] = {nullptr, nullptr};
@@ -673,7 +674,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         q.take<int32_t>(Rcap); q.take<unsigned long long>(Rcap); q.take<unsigned long long>(2 * Rcap);
         q.take<unsigned long long>(2 * (Rcap + 1)); q.take<int32_t>(1);
         q.take<unsigned long long>(2 * (size_t)w.rgroups + 8);
-        q.take<uint32_t>((size_t)S + 1);
+        q.take<uint32_t>((size_t)C0 + 2);
+        q.take<uint32_t>((size_t)sh.cap / 32 + 2);
       };
       Carve rp{nullptr};
       rz(rp);
@@ -689,7 +691,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       w.run_seg = r.take<int32_t>(Rcap); w.run_hl = r.take<unsigned long long>(Rcap);
       w.rcnt = r.take<unsigned long long>(2 * Rcap); w.rfl = r.take<unsigned long long>(2 * (Rcap + 1));
       w.Rp1 = r.take<int32_t>(1); w.rsgrp = r.take<unsigned long long>(2 * (size_t)w.rgroups + 8);
-      w.enc_cnt = r.take<uint32_t>((size_t)S + 1);
+      w.enc_cnt = r.take<uint32_t>((size_t)C0 + 2);
+      w.enc_bits = r.take<uint32_t>((size_t)sh.cap / 32 + 2);
     }
     if (fused && m > 0) {
       w.tiles = fused_tiles(n, m);
@@ -935,7 +938,9 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         if (PA.cagg_next)
           GBDT_CUDA(cudaMemsetAsync(w.cagg, 0, sizeof(unsigned long long) * 5 * (size_t)std::max<int64_t>(sh.C0, 1), st));
         LK.partition_scatter(PA, hmode, (sh.rle && !dec) ? &RA : nullptr, st);
-        if (dec) LK.rle_encode(tn, sh.m, nxt.K, sh.valw[(lvl + 1) & 1].as<float>(), w.enc_cnt, st);
+        if (dec)
+          LK.rle_encode(tn, sh.m, nxt.K, sh.valw[(lvl + 1) & 1].as<float>(), w.enc_cnt, w.enc_bits,
+                        ((size_t)sh.cap / 32 + 2) * 4, st);
         kt.end();
       }
       tm.end();
