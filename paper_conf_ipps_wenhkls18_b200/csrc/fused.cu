@@ -135,6 +135,16 @@ __device__ __forceinline__ int block_exscan_int(int x, int& total, int* wsum, in
   return wex + incl - x;
 }
 
+// 1/x for x > 0: hardware seed + two Newton steps (~1 ulp); ranks only (the exact Eq. 2 decides)
+__device__ __forceinline__ double rcp_nr(double x) {
+  double r;
+  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
+  double e = __fma_rn(-x, r, 1.0);
+  r = __fma_rn(r, e, r);
+  e = __fma_rn(-x, r, 1.0);
+  return __fma_rn(r, e, r);
+}
+
 __device__ __forceinline__ bool rec_better_f(unsigned long long gk, const Rec& r, unsigned long long gk0, const Rec& r0) {
   return gk > gk0 || (gk == gk0 && tie_key(r.attr, r.value, r.dir) < tie_key(r0.attr, r0.value, r0.dir));
 }
@@ -169,6 +179,7 @@ __global__ void __launch_bounds__(kFT) k_tile_agg(FusedArgs A) {
     const long long tbase = (long long)a * stride + q0;
     const int jf = seg_of(S.off, K, q0);              // the tile's first piece
     const int jl = seg_of(S.off, K, q0 + len - 1);    // its last piece
+    if ((jf != jl || !A.warp_tiles) && tid == 0) A.mlist[atomicAdd(A.mcount, 1)] = t;  // k_fused's (CTA) tiles
     const bool live_l = S.cidx[jl] >= 0;
     const int ql = S.off[jl] - q0;                    // the last piece's start, tile-relative
     int id[kFI];
@@ -424,6 +435,8 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
   const FusedPlan* P = A.plan;
   const int T = P->T;
   if (T == 0) return;
+  const int Tm = *A.mcount;  // the tiles holding several segment pieces (k_tile_agg's list)
+  if (Tm == 0) return;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int K = P->K, Kn = P->Kn, tpa = P->tpa;
   const int n_act = (int)P->n_act;
@@ -454,16 +467,17 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
     for (int st = 0; st < kFS; ++st) mbar_init(&S.bar[st], 1);
     fence_mbar_init();
     for (int st = 0; st < kFS; ++st) {
-      const int t = blockIdx.x + st * gridDim.x;
-      if (t < T) issue(st, t);
+      const int i = blockIdx.x + st * gridDim.x;
+      if (i < Tm) issue(st, A.mlist[i]);
     }
   }
   __syncthreads();
   uint32_t phase = 0;
   const int qi = tid * kFI;
   for (int it = 0;; ++it) {
-    const int t = blockIdx.x + it * gridDim.x;
-    if (t >= T) break;
+    const int ti = blockIdx.x + it * gridDim.x;
+    if (ti >= Tm) break;
+    const int t = A.mlist[ti];
     const int st = it % kFS;
     const int a = t / tpa;
     const int q0 = (t - a * tpa) * kFTile;
@@ -557,10 +571,10 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
         }
         __syncthreads();
         if (tid == 0) {  // the stage is drained: start the next tile's copy now
-          const int t2 = t + kFS * gridDim.x;
-          if (t2 < T) {
+          const int i2 = ti + kFS * gridDim.x;
+          if (i2 < Tm) {
             fence_proxy_async();
-            issue(st, t2);
+            issue(st, A.mlist[i2]);
           }
           issued = true;
         }
@@ -986,10 +1000,10 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
     }  // general path
     __syncthreads();  // stage st and the tile scratch are free
     if (tid == 0 && !issued) {
-      const int t2 = t + kFS * gridDim.x;
-      if (t2 < T) {
+      const int i2 = ti + kFS * gridDim.x;
+      if (i2 < Tm) {
         fence_proxy_async();
-        issue(st, t2);
+        issue(st, A.mlist[i2]);
       }
     }
   }
@@ -1004,11 +1018,325 @@ __global__ void __launch_bounds__(kFT, GBDT_FUSED_CTAS) k_fused(FusedArgs A) {
   }
 }
 
+// ============================================================================ k_fusedw
+// Warp-granular pass over the single-piece tiles (the common case: one parent segment per tile).
+// One warp owns a 2048-entry tile end to end and streams it as eight 256-entry chunks through a
+// per-warp 2-stage TMA ring; no CTA barrier anywhere.  Per chunk:
+//   blocked  (lane l: entries 8 l .. 8 l + 7): sides from k_tile_agg's byte, the per-side sums of
+//            the lane, one warp scan of (g_hi, h_hi, g_lo, h_lo), the lane's run ends of each
+//            child run, ranked by cross-multiplied scores; the chunk's best per side by integer
+//            reductions on the score bits, its exact Eq. 2 gain against the tile's best
+//   striped  (row r, lane l: entry 32 r + l): coalesced stores of the child runs, ranks by popc of
+//            the row's side word
+// The carry between chunks stays in registers; the tile's first carry is the tile scan's record.
+#ifndef GBDT_FUSEDW_CTAS
+#define GBDT_FUSEDW_CTAS 2
+#endif
+constexpr int kWCh = 256;   // entries per chunk
+constexpr int kWW = 8;      // warps per CTA
+struct __align__(16) WStage {
+  float val[kWCh];
+  int32_t ins[kWCh];
+  double g[kWCh];
+};
+struct __align__(16) WWarp {
+  WStage st[2];
+  unsigned long long bar[2];
+};
+struct WSmem {
+  WWarp w[kWW];
+  int off[kFusedMaxK + 1];
+  int cidx[kFusedMaxK];
+  int offn[2 * kFusedMaxK + 1];
+  double cG[2 * kFusedMaxK], cH[2 * kFusedMaxK], cP[2 * kFusedMaxK];
+};
+
+// order-preserving u64 of a score >= 0 or -inf (no NaN)
+__device__ __forceinline__ unsigned long long score_key(double x) {
+  unsigned long long b = (unsigned long long)__double_as_longlong(x);
+  return (b >> 63) ? ~b : (b | 0x8000000000000000ull);
+}
+__device__ __forceinline__ unsigned long long warp_max_u64(unsigned long long k) {
+  const unsigned hi = __reduce_max_sync(0xffffffffu, (unsigned)(k >> 32));
+  const unsigned lo = __reduce_max_sync(0xffffffffu, (unsigned)(k >> 32) == hi ? (unsigned)k : 0u);
+  return ((unsigned long long)hi << 32) | lo;
+}
+
+template <int HMODE, bool kWrite>
+__global__ void __launch_bounds__(kWW * 32, GBDT_FUSEDW_CTAS) k_fusedw(FusedArgs A) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  WSmem& S = *reinterpret_cast<WSmem*>(smem_raw);
+  const FusedPlan* P = A.plan;
+  const int T = P->T;
+  if (T == 0) return;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int K = P->K, Kn = P->Kn, tpa = P->tpa;
+  const int n_act = (int)P->n_act;
+  const long long stride = P->stride, stride_n = P->stride_next;
+  const unsigned ep = (unsigned)P->epoch;
+  const int Fg = A.fx[0], Fh = A.fx[1];
+  const double lam = A.lam;
+  for (int i = threadIdx.x; i <= K; i += blockDim.x) S.off[i] = P->off[i];
+  for (int i = threadIdx.x; i < K; i += blockDim.x) S.cidx[i] = P->cidx[i];
+  for (int i = threadIdx.x; i <= Kn; i += blockDim.x) S.offn[i] = P->offn[i];
+  for (int c = threadIdx.x; c < Kn; c += blockDim.x) { S.cG[c] = A.nxt.G[c]; S.cH[c] = A.nxt.H[c]; S.cP[c] = A.nxt.pterm[c]; }
+  WWarp& W = S.w[wid];
+  if (lane == 0) {
+    mbar_init(&W.bar[0], 1);
+    mbar_init(&W.bar[1], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();  // the only CTA barrier: tables and barriers are ready
+  const unsigned long long pol = policy_evict_first();
+  const unsigned ltm = (1u << lane) - 1u;
+  uint32_t ph = 0;
+  for (int t = blockIdx.x * kWW + wid; t < T; t += gridDim.x * kWW) {
+    const int a = t / tpa;
+    const int q0 = (t - a * tpa) * kFTile;
+    const int len = min(kFTile, n_act - q0);
+    const int j0 = seg_of(S.off, K, q0);
+    if (S.off[j0 + 1] < q0 + len) continue;  // several pieces: k_fused's
+    const int c0 = S.cidx[j0];
+    if (c0 < 0) continue;                    // the node became a leaf: entries dropped
+    const bool cont = S.off[j0] < q0;
+    const long long tbase = (long long)a * stride + q0;
+    const int nch = (len + kWCh - 1) / kWCh;
+    auto issue = [&](int ch) {
+      if (lane == 0 && ch < nch) {
+        const int st = ch & 1;
+        const long long p0 = tbase + (long long)ch * kWCh;
+        const uint32_t n = (uint32_t)((min(kWCh, len - ch * kWCh) + 3) & ~3);
+        fence_proxy_async();
+        mbar_arrive_expect_tx(&W.bar[st], 16u * n);
+        tma_load_1d(W.st[st].val, A.val + p0, 4u * n, &W.bar[st], pol);
+        tma_load_1d(W.st[st].ins, A.ins + p0, 4u * n, &W.bar[st], pol);
+        tma_load_1d(W.st[st].g, A.gl + p0, 8u * n, &W.bar[st], pol);
+      }
+    };
+    issue(0);
+    issue(1);
+    // carry per side (0 high, 1 low): entries, sums, last value / position (warp-uniform)
+    int ccnt[2] = {0, 0};
+    double cg[2] = {0.0, 0.0}, chh[2] = {0.0, 0.0};
+    float cv[2] = {0.f, 0.f};
+    long long cpos[2] = {0, 0};
+    if (cont) {
+      const TRec* pr = A.tinc + (t - 1);
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {
+        const TSide x = pr->s[q];
+        ccnt[q] = x.cnt;
+        cg[q] = from_fx((__int128)u128(x.g_lo, x.g_hi), Fg);
+        chh[q] = from_fx((__int128)u128(x.h_lo, x.h_hi), Fh);
+        cv[q] = x.val;
+        cpos[q] = x.pos;
+      }
+    }
+    double Gc[2], Hc[2], Hl[2], Pc[2];
+#pragma unroll
+    for (int q = 0; q < 2; ++q) { Gc[q] = S.cG[c0 + q]; Hc[q] = S.cH[c0 + q]; Hl[q] = Hc[q] + lam; Pc[q] = S.cP[c0 + q]; }
+    // the tile's best per side (warp-uniform): exact gain key, then the R12 tie (larger value)
+    unsigned long long bkey[2] = {0ull, 0ull};
+    double bGL[2] = {0, 0}, bHL[2] = {0, 0};
+    long long bcnt[2] = {0, 0}, bpos[2] = {0, 0};
+    float bval[2] = {0.f, 0.f};
+    const long long dbase0 = (long long)a * stride_n + S.offn[c0];
+    const long long dbase1 = (long long)a * stride_n + S.offn[c0 + 1];
+    const unsigned char* tb = A.tbits + (size_t)t * kFT;
+    for (int ch = 0; ch < nch; ++ch) {
+      const int st = ch & 1;
+      const int clen = min(kWCh, len - ch * kWCh);
+      const unsigned hb_raw = tb[ch * 32 + lane];
+      mbar_wait(&W.bar[st], (ph >> st) & 1);
+      ph ^= 1u << st;
+      const WStage& SG = W.st[st];
+      const int k0 = lane * 8;
+      const unsigned vm = k0 >= clen ? 0u : (k0 + 8 <= clen ? 0xffu : ((1u << (clen - k0)) - 1u));
+      const unsigned hm = hb_raw & vm, lm = ~hb_raw & vm;
+      double g[8];
+      float v[8];
+      {
+        const double2* pg = reinterpret_cast<const double2*>(SG.g + k0);
+        const float4* pv = reinterpret_cast<const float4*>(SG.val + k0);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) { const double2 z = pg[k]; g[2 * k] = z.x; g[2 * k + 1] = z.y; }
+        const float4 a0 = pv[0], a1 = pv[1];
+        v[0] = a0.x; v[1] = a0.y; v[2] = a0.z; v[3] = a0.w; v[4] = a1.x; v[5] = a1.y; v[6] = a1.z; v[7] = a1.w;
+      }
+      // lane sums per side, in item order
+      double lg[2] = {0.0, 0.0}, lh[2] = {0.0, 0.0};
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        if ((vm >> k) & 1u) {
+          const double h = hess_of<HMODE>(g[k]);
+          if ((hm >> k) & 1u) { lg[0] = lg[0] + g[k]; lh[0] = lh[0] + h; }
+          else { lg[1] = lg[1] + g[k]; lh[1] = lh[1] + h; }
+        }
+      }
+      // warp scans: inclusive (g, h) per side and the packed counts
+      double ig[2] = {lg[0], lg[1]}, ih[2] = {lh[0], lh[1]};
+      int icnt = __popc(hm) | (__popc(lm) << 16);
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          const double yg = __shfl_up_sync(0xffffffffu, ig[q], o), yh = __shfl_up_sync(0xffffffffu, ih[q], o);
+          if (lane >= o) { ig[q] = yg + ig[q]; ih[q] = yh + ih[q]; }
+        }
+        const int yc = __shfl_up_sync(0xffffffffu, icnt, o);
+        if (lane >= o) icnt += yc;
+      }
+      const int excnt = icnt - (__popc(hm) | (__popc(lm) << 16));
+      const int totc = __shfl_sync(0xffffffffu, icnt, 31);
+      // the lane's exclusive prefix per side: carry + (exclusive in-chunk) -- (carry + eg) + items
+      double rg[2], rh[2];
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {
+        double eg = __shfl_up_sync(0xffffffffu, ig[q], 1), eh = __shfl_up_sync(0xffffffffu, ih[q], 1);
+        if (lane == 0) { eg = 0.0; eh = 0.0; }
+        rg[q] = cg[q] + eg;
+        rh[q] = chh[q] + eh;
+      }
+      // the last same-side value before the lane's first item of that side
+      float pv[2];
+      bool prev[2];
+      int pidx[2];  // chunk index of that entry (or -1: the carry's)
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {
+        const unsigned m = q ? lm : hm;
+        const unsigned has = __ballot_sync(0xffffffffu, m != 0u);
+        const int lastk = m ? 31 - __clz(m) : 0;
+        const float lastv = v[lastk];
+        const unsigned below = has & ltm;
+        const int src = below ? 31 - __clz(below) : 0;
+        const float sv = __shfl_sync(0xffffffffu, lastv, src);
+        const int sk = __shfl_sync(0xffffffffu, k0 + lastk, src);  // the source lane's own index
+        prev[q] = below ? true : ccnt[q] > 0;
+        pv[q] = below ? sv : cv[q];
+        pidx[q] = below ? sk : -1;
+      }
+      // candidates: the boundary before each item whose predecessor on its side has another value
+      double bnum[2] = {-1.0, -1.0}, bden[2] = {1.0, 1.0};
+      int bk[2] = {-1, -1}, bpk[2] = {-1, -1};  // winning item, its predecessor's chunk index
+      double wGL[2] = {0, 0}, wHL[2] = {0, 0};
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        if ((vm >> k) & 1u) {
+          const int q = ((hm >> k) & 1u) ? 0 : 1;
+          const double GL = q ? rg[1] : rg[0], HL = q ? rh[1] : rh[0];
+          const bool pq = q ? prev[1] : prev[0];
+          const float pvq = q ? pv[1] : pv[0];
+          if (pq && pvq != v[k]) {
+            const double H_l = q ? Hl[1] : Hl[0], G_c = q ? Gc[1] : Gc[0];
+            const double dl = HL + lam, dr = H_l - HL, GR = G_c - GL;
+            const double num = __fma_rn(GL * GL, dr, (GR * GR) * dl), den = dl * dr;
+            const double on = q ? bnum[1] : bnum[0], od = q ? bden[1] : bden[0];
+            if (num * od > on * den) {
+              if (q) { bnum[1] = num; bden[1] = den; bk[1] = k; wGL[1] = GL; wHL[1] = HL; bpk[1] = q ? pidx[1] : pidx[0]; }
+              else { bnum[0] = num; bden[0] = den; bk[0] = k; wGL[0] = GL; wHL[0] = HL; bpk[0] = pidx[0]; }
+            }
+          }
+          const double h = hess_of<HMODE>(g[k]);
+          if (q) { rg[1] = rg[1] + g[k]; rh[1] = rh[1] + h; pv[1] = v[k]; prev[1] = true; pidx[1] = k0 + k; }
+          else { rg[0] = rg[0] + g[k]; rh[0] = rh[0] + h; pv[0] = v[k]; prev[0] = true; pidx[0] = k0 + k; }
+        }
+      }
+      // the chunk's best per side: approximate score max, then the smallest item (larger value)
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {
+        const double sc = bk[q] >= 0 ? bnum[q] * rcp_nr(bden[q]) : -INFINITY;
+        const unsigned long long key = warp_max_u64(score_key(sc));
+        if (key == score_key(-INFINITY)) continue;  // no candidate on this side in the chunk
+        const unsigned idx = __reduce_min_sync(0xffffffffu, (score_key(sc) == key && bk[q] >= 0) ? (unsigned)(k0 + bk[q]) : 0xffffffffu);
+        const int wl = (int)(idx >> 3);
+        double GL = __shfl_sync(0xffffffffu, wGL[q], wl), HL = __shfl_sync(0xffffffffu, wHL[q], wl);
+        const int pk = __shfl_sync(0xffffffffu, bpk[q], wl);
+        const unsigned long long gk = gain_key(eq2_gain(GL, HL, Gc[q], Hc[q], lam, Pc[q]));
+        // side counts before the winner: carry + same-side entries of the chunk before it
+        const int before_lane = q ? (__shfl_sync(0xffffffffu, excnt, wl) >> 16) : (__shfl_sync(0xffffffffu, excnt, wl) & 0xffff);
+        const unsigned wm = __shfl_sync(0xffffffffu, q ? lm : hm, wl);
+        const long long cntL = ccnt[q] + before_lane + __popc(wm & ((1u << (idx & 7)) - 1u));
+        const float pval = pk >= 0 ? SG.val[pk] : cv[q];
+        const long long ppos = pk >= 0 ? tbase + (long long)ch * kWCh + pk : cpos[q];
+        // R12 inside the tile: larger gain, then the larger value (the earlier candidate)
+        if (gk > bkey[q]) {
+          bkey[q] = gk; bGL[q] = GL; bHL[q] = HL; bcnt[q] = cntL; bval[q] = pval; bpos[q] = ppos;
+        }
+      }
+      // carry update per side (warp-uniform)
+      const int th = totc & 0xffff, tl = totc >> 16;
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {
+        const double tg = __shfl_sync(0xffffffffu, ig[q], 31), thh = __shfl_sync(0xffffffffu, ih[q], 31);
+        cg[q] = cg[q] + tg;
+        chh[q] = chh[q] + thh;
+        const unsigned m = q ? lm : hm;
+        const unsigned has = __ballot_sync(0xffffffffu, m != 0u);
+        if (has) {
+          const int src = 31 - __clz(has);
+          const int lastk = m ? 31 - __clz(m) : 0;
+          cv[q] = __shfl_sync(0xffffffffu, v[lastk], src);
+          cpos[q] = tbase + (long long)ch * kWCh + __shfl_sync(0xffffffffu, k0 + lastk, src);
+        }
+      }
+      if (kWrite) {  // striped stores: row r = entries 32 r .. 32 r + 31 of the chunk
+        const unsigned* words = reinterpret_cast<const unsigned*>(tb + ch * 32);
+        int rb0 = 0, rb1 = 0;  // same-side entries in the chunk's earlier rows
+#pragma unroll
+        for (int r = 0; r < 8; ++r) {
+          const int e = r * 32 + lane;
+          const int rowlen = min(32, clen - r * 32);
+          if (rowlen <= 0) break;
+          const unsigned rvm = rowlen >= 32 ? 0xffffffffu : ((1u << rowlen) - 1u);
+          const unsigned w = __ldg(words + r) & rvm;
+          if (e < clen) {
+            const bool hi = (w >> lane) & 1u;
+            const int rank = hi ? rb0 + __popc(w & ltm) : rb1 + __popc(~w & rvm & ltm);
+            const long long d = hi ? dbase0 + ccnt[0] + rank : dbase1 + ccnt[1] + rank;
+#ifdef GBDT_FUSEDW_DEBUG
+            {
+              const int cc = c0 + (hi ? 0 : 1);
+              const long long lo_ = (long long)a * stride_n + S.offn[cc], hi_ = lo_ + (S.offn[cc + 1] - S.offn[cc]);
+              if (d < lo_ || d >= hi_)
+                printf("BAD t=%d ch=%d r=%d lane=%d hi=%d rank=%d ccnt=%d,%d rb=%d,%d w=%08x clen=%d cont=%d j0=%d off=%d q0=%d len=%d\n",
+                       t, ch, r, lane, (int)hi, rank, ccnt[0], ccnt[1], rb0, rb1, w, clen, (int)cont, j0, S.off[j0], q0, len);
+            }
+#endif
+            __stcs(A.val_out + d, SG.val[e]);
+            __stcs(A.ins_out + d, SG.ins[e]);
+            __stcs(A.g_out + d, SG.g[e]);
+          }
+          rb0 += __popc(w);
+          rb1 += __popc(~w & rvm);
+        }
+      }
+      ccnt[0] += th;
+      ccnt[1] += tl;
+      __syncwarp();
+      issue(ch + 2);  // stage st is drained
+    }
+    // the tile's bests -> the global records (only if they can still win)
+    if (lane < 2) {
+      const int q = lane;
+      if (bkey[q] && bkey[q] >= __ldcg(A.gkey + c0 + q)) {
+        Rec rc;
+        rc.gain = eq2_gain(bGL[q], bHL[q], Gc[q], Hc[q], lam, Pc[q]);
+        rc.GL = bGL[q]; rc.HL = bHL[q]; rc.cntL = bcnt[q]; rc.pos = bpos[q]; rc.value = bval[q];
+        rc.attr = A.a_base + a; rc.dir = 0; rc.node = c0 + q; rc.epoch = (int)ep; rc.shard = A.shard;
+        A.rec[atomicAdd(A.nrec, 1)] = rc;
+        atomicMax(A.gkey + c0 + q, bkey[q]);
+      }
+    }
+  }
+}
+
 // ============================================================================ plan + mark
 // One thread: the level's segment offsets, child offsets / parents, tile count.
 __global__ void k_fused_plan(FusedPlan* P, NodeTab cur, NodeTab nxt, const int32_t* __restrict__ cidx,
-                             const int* __restrict__ epoch, int m, unsigned long long* lent, int lvl) {
+                             const int* __restrict__ epoch, int m, unsigned long long* lent, int lvl,
+                             int* __restrict__ mcount) {
   if (threadIdx.x != 0) return;
+  *mcount = 0;
   const int K = *cur.K, Kn = *nxt.K;
   P->K = K;
   P->Kn = Kn;
@@ -1062,6 +1390,18 @@ __global__ void k_mark_fused(const FusedPlan* __restrict__ P, const int32_t* __r
 
 unsigned g_fused_grid[2][2] = {{0, 0}, {0, 0}};
 unsigned g_agg_grid = 0;
+unsigned g_fusedw_grid = 0;
+
+template <int HM, bool W>
+void set_fusedw(int sms) {
+  const size_t smem = sizeof(WSmem);
+  GBDT_CUDA(cudaFuncSetAttribute(k_fusedw<HM, W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int occ = 0;
+  GBDT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fusedw<HM, W>, kWW * 32, smem));
+  if (occ < 1) fail(GBDT_E_CUDA, "k_fusedw does not fit on an SM");
+  const unsigned g = (unsigned)(occ * sms);
+  g_fusedw_grid = g_fusedw_grid ? std::min(g_fusedw_grid, g) : g;
+}
 
 template <int HM, bool W>
 void set_fused(int sms) {
@@ -1077,7 +1417,7 @@ void set_fused(int sms) {
 
 size_t fused_tile_bytes(int64_t max_tiles) {
   const int64_t groups = (max_tiles + kTSGroup - 1) / kTSGroup + 1;
-  return (size_t)max_tiles * (2 * sizeof(TRec) + 2 + kFT) + (size_t)groups * (2 * sizeof(TRec) + 1) + 8192 +
+  return (size_t)max_tiles * (2 * sizeof(TRec) + 2 + kFT + 4) + (size_t)groups * (2 * sizeof(TRec) + 1) + 8192 +
          sizeof(Rec) * 2 * kFusedMaxK * (size_t)kFusedMaxCTAs;
 }
 int64_t fused_tiles(int64_t n, int m) { return (int64_t)m * ((n + kFTile - 1) / kFTile); }
@@ -1087,6 +1427,8 @@ void fused_carve(FusedArgs& A, void* base, int64_t max_tiles) {
   char* p = static_cast<char*>(base);
   auto take = [&](size_t b) { char* r = p; p += (b + 255) & ~size_t(255); return r; };
   A.cta_rec = reinterpret_cast<Rec*>(take(sizeof(Rec) * 2 * kFusedMaxK * (size_t)kFusedMaxCTAs));
+  A.mcount = reinterpret_cast<int*>(take(16));
+  A.mlist = reinterpret_cast<int*>(take(4 * (size_t)max_tiles));
   A.tagg = reinterpret_cast<TRec*>(take(sizeof(TRec) * max_tiles));
   A.tinc = reinterpret_cast<TRec*>(take(sizeof(TRec) * max_tiles));
   A.tgagg = reinterpret_cast<TRec*>(take(sizeof(TRec) * groups));
@@ -1102,6 +1444,10 @@ void fused_init(int sms) {
   set_fused<kHConst2, false>(sms);
   set_fused<kHFromG, true>(sms);
   set_fused<kHFromG, false>(sms);
+  set_fusedw<kHConst2, true>(sms);
+  set_fusedw<kHConst2, false>(sms);
+  set_fusedw<kHFromG, true>(sms);
+  set_fusedw<kHFromG, false>(sms);
   int occ = 0;
   GBDT_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_tile_agg<kHFromG>, kFT, 0));
   g_agg_grid = (unsigned)(std::max(occ, 1) * sms);
@@ -1110,8 +1456,8 @@ void fused_init(int sms) {
 unsigned fused_grid(int hmode) { return std::max(g_fused_grid[hmode][0], g_fused_grid[hmode][1]); }
 
 void fused_plan(FusedPlan* P, const NodeTab& cur, const NodeTab& nxt, const int32_t* cidx, const int* epoch, int m,
-                unsigned long long* lent, int lvl, cudaStream_t st) {
-  k_fused_plan<<<1, 32, 0, st>>>(P, cur, nxt, cidx, epoch, m, lent, lvl);
+                unsigned long long* lent, int lvl, int* mcount, cudaStream_t st) {
+  k_fused_plan<<<1, 32, 0, st>>>(P, cur, nxt, cidx, epoch, m, lent, lvl, mcount);
   GBDT_LAUNCH_CHECK();
   count_launch();
 }
@@ -1125,6 +1471,16 @@ void fused_pass(const FusedArgs& A, int hmode, bool write, int64_t max_tiles, cu
   k_tscan1<<<gs, kTSGroup, 0, st>>>(A);
   k_tscan2<<<1, kTSGroup, 0, st>>>(A);
   k_tscan3<<<gs, kTSGroup, 0, st>>>(A);
+  const size_t smemw = sizeof(WSmem);
+  const unsigned gw = g_fusedw_grid;
+  if (!A.warp_tiles) {
+  } else if (hmode == kHConst2) {
+    if (write) k_fusedw<kHConst2, true><<<gw, kWW * 32, smemw, st>>>(A);
+    else k_fusedw<kHConst2, false><<<gw, kWW * 32, smemw, st>>>(A);
+  } else {
+    if (write) k_fusedw<kHFromG, true><<<gw, kWW * 32, smemw, st>>>(A);
+    else k_fusedw<kHFromG, false><<<gw, kWW * 32, smemw, st>>>(A);
+  }
   const size_t smem = sizeof(FusedSmem);
   const unsigned grid = g_fused_grid[hmode][write ? 1 : 0];
   if (hmode == kHConst2) {
@@ -1135,7 +1491,7 @@ void fused_pass(const FusedArgs& A, int hmode, bool write, int64_t max_tiles, cu
     else k_fused<kHFromG, false><<<grid, kFT, smem, st>>>(A);
   }
   GBDT_LAUNCH_CHECK();
-  count_launch(5);
+  count_launch(6);
 }
 
 void fused_mark(const FusedPlan* P, const int32_t* Kp, const int32_t* cidx, const Rec* winner, int shard, int a_base,

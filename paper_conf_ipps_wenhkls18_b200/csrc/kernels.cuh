@@ -180,6 +180,9 @@ struct FusedArgs {
   unsigned char* tgf;
   unsigned char* tbits;       // [tiles][256]: bit k of byte i = entry 8 i + k goes high
   Rec* cta_rec;               // [CTAs][2 kFusedMaxK] node-best records of each k_fused CTA
+  int warp_tiles;             // 1: single-piece tiles go to k_fusedw (0: every tile to k_fused; A/B)
+  int* mcount;                // tiles holding several segment pieces (k_tile_agg appends them)
+  int* mlist;
   const int32_t* fx;          // [2] fixed-point scales of this tree
   double lam;
   int m, a_base, shard;
@@ -193,7 +196,7 @@ void fused_carve(FusedArgs& A, void* base, int64_t max_tiles);
 void fused_init(int sms);
 unsigned fused_grid(int hmode);
 void fused_plan(FusedPlan* P, const NodeTab& cur, const NodeTab& nxt, const int32_t* cidx, const int* epoch, int m,
-                unsigned long long* lent, int lvl, cudaStream_t st);
+                unsigned long long* lent, int lvl, int* mcount, cudaStream_t st);
 void fused_pass(const FusedArgs& A, int hmode, bool write, int64_t max_tiles, cudaStream_t st);
 void fused_mark(const FusedPlan* P, const int32_t* Kp, const int32_t* cidx, const Rec* winner, int shard, int a_base,
                 const int32_t* ins, const uint32_t* hbit, uint32_t* bits, int64_t n, int Kl, int sms, cudaStream_t st);

@@ -865,8 +865,9 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
           Shard& sh = *ds.shards[li];
           ShardWork& w = sw[li];
           if (sh.m == 0) continue;
-          fused_plan(w.fplan[lvl & 1], cur, nxt, cidx, epoch, sh.m, P.profile ? lent : nullptr, lvl, st);
           FusedArgs FA;
+          fused_carve(FA, w.tilemem, w.tiles);
+          fused_plan(w.fplan[lvl & 1], cur, nxt, cidx, epoch, sh.m, P.profile ? lent : nullptr, lvl, FA.mcount, st);
           FA.val = lvl == 0 ? sh.val0.as<float>() : sh.valw[lvl & 1].as<float>();
           FA.ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
           FA.gl = w.glist[lvl & 1];
@@ -876,7 +877,10 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
           FA.hbit = hbitF[lvl & 1];
           FA.plan = w.fplan[lvl & 1];
           FA.nxt = nxt;
-          fused_carve(FA, w.tilemem, w.tiles);
+          {
+            const char* fw = getenv("GBDT_FUSEDW");
+            FA.warp_tiles = fw ? fw[0] != '0' : 1;
+          }
           FA.fx = fxs; FA.lam = P.lambda; FA.m = sh.m; FA.a_base = sh.a_begin; FA.shard = sh.index;
           FA.rec = w.rec; FA.nrec = w.nrec; FA.gkey = w.gkey;
           kt.begin(GBDT_PHASE_K_FUSED);
