@@ -181,6 +181,11 @@ gbdt_status gbdt_model_num_trees(const gbdt_model* m, int32_t* out);
 gbdt_status gbdt_model_num_nodes(const gbdt_model* m, int32_t tree, int32_t* out);
 gbdt_status gbdt_model_export(const gbdt_model* m, int32_t tree, gbdt_node* nodes);
 
+/* Mean training loss of the model after 0, 1, ..., n_trees trees (out: n_trees + 1 doubles,
+ * caller-owned): squared (y - yhat)^2, logistic the cross-entropy of P:120; the paper's RMSE
+ * (Table II) is the square root of the squared-loss entries.  NaN for a custom loss. */
+gbdt_status gbdt_model_train_loss(const gbdt_model* m, double* out);
+
 /* Per-phase device milliseconds of the gbdt_train that produced m (profile = 1), else zeros.
  * ms_by_phase: caller-owned, n_phases entries (<= GBDT_N_PHASES filled). */
 gbdt_status gbdt_get_timings(const gbdt_model* m, double* ms_by_phase, int32_t n_phases);

@@ -410,6 +410,13 @@ gbdt_status gbdt_predict_on_stream(const gbdt_model* mh, int64_t n_rows, int64_t
   });
 }
 
+gbdt_status gbdt_model_train_loss(const gbdt_model* m, double* out) {
+  return guarded([&] {
+    if (!m || !out) fail(GBDT_E_INVAL, "NULL argument");
+    for (size_t i = 0; i < m->m.train_loss.size(); ++i) out[i] = m->m.train_loss[i];
+  });
+}
+
 gbdt_status gbdt_model_num_trees(const gbdt_model* m, int32_t* out) {
   return guarded([&] {
     if (!m || !out) fail(GBDT_E_INVAL, "NULL argument");

@@ -141,6 +141,7 @@ struct Model {
   std::vector<gbdt_node> nodes;  // n_trees * NH
   double timings[GBDT_N_PHASES] = {0};
   std::vector<int64_t> level_entries;  // [max_depth] list entries scanned per level (profile = 1)
+  std::vector<double> train_loss;      // [n_trees + 1] mean training loss after 0 .. T trees
   int device = 0;
   int dense = 0;                 // trained on the dense representation: predict fills absent values
   float fill = 0.f;

@@ -65,7 +65,7 @@ __global__ void k_grad(int64_t n, int loss, const int32_t* __restrict__ tidx, do
   const int first = t == 0;
   const double* wprev = hweight + (size_t)((t + 1) & 1) * NH;
   R.t = t;
-  double sg = 0.0, sh = 0.0, mg = 0.0, mh = 0.0;
+  double sg = 0.0, sh = 0.0, mg = 0.0, mh = 0.0, sl = 0.0;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
     double g, h;
@@ -81,6 +81,10 @@ __global__ void k_grad(int64_t n, int loss, const int32_t* __restrict__ tidx, do
       pos[i] = 0;
       if (mode == 1) continue;
       const double yi = (double)y[i];
+      // training loss at this margin (the model of the t trees before this one): (y - yhat)^2, or
+      // the cross-entropy max(yhat, 0) - y yhat + log(1 + exp(-|yhat|)) (reported per tree)
+      sl += loss == GBDT_LOSS_SQUARED ? (yi - yh) * (yi - yh)
+                                      : fmax(yh, 0.0) - yi * yh + log1p(exp(-fabs(yh)));
     if (loss == GBDT_LOSS_SQUARED) {  // l = (y - yhat)^2: g = 2(yhat - y), h = 2 (R6)
       g = __dmul_rn(2.0, __dsub_rn(yh, yi));
       h = 2.0;
@@ -107,21 +111,25 @@ __global__ void k_grad(int64_t n, int loss, const int32_t* __restrict__ tidx, do
     sh += __shfl_xor_sync(0xffffffffu, sh, o);
     mg = fmax(mg, __shfl_xor_sync(0xffffffffu, mg, o));
     mh = fmax(mh, __shfl_xor_sync(0xffffffffu, mh, o));
+    sl += __shfl_xor_sync(0xffffffffu, sl, o);
   }
   if (mode == 1) return;
-  __shared__ double wg[32], wh[32], wmg[32], wmh[32];
+  __shared__ double wg[32], wh[32], wmg[32], wmh[32], wl[32];
   if ((threadIdx.x & 31) == 0) {
     wg[threadIdx.x >> 5] = sg; wh[threadIdx.x >> 5] = sh;
-    wmg[threadIdx.x >> 5] = mg; wmh[threadIdx.x >> 5] = mh;
+    wmg[threadIdx.x >> 5] = mg; wmh[threadIdx.x >> 5] = mh; wl[threadIdx.x >> 5] = sl;
   }
   __syncthreads();
   if (threadIdx.x == 0) {
-    double a = 0.0, b = 0.0, c = 0.0, e = 0.0;
-    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) { a += wg[w]; b += wh[w]; c = fmax(c, wmg[w]); e = fmax(e, wmh[w]); }
-    partial[4 * blockIdx.x] = a;
-    partial[4 * blockIdx.x + 1] = b;
-    partial[4 * blockIdx.x + 2] = c;
-    partial[4 * blockIdx.x + 3] = e;
+    double a = 0.0, b = 0.0, c = 0.0, e = 0.0, f = 0.0;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) {
+      a += wg[w]; b += wh[w]; c = fmax(c, wmg[w]); e = fmax(e, wmh[w]); f += wl[w];
+    }
+    partial[5 * blockIdx.x] = a;
+    partial[5 * blockIdx.x + 1] = b;
+    partial[5 * blockIdx.x + 2] = c;
+    partial[5 * blockIdx.x + 3] = e;
+    partial[5 * blockIdx.x + 4] = mode == 0 ? f : __longlong_as_double(0x7ff8000000000000ll);  // custom: unknown
   }
 }
 
@@ -139,7 +147,7 @@ __device__ int fx_scale(double n, double mx) {
 __global__ void k_tree_begin(int nblk, const double* __restrict__ partial, int64_t n, double lam,
                              NodeTab root, int64_t NH, double* __restrict__ hweight,
                              uint8_t* __restrict__ hstate, gbdt_node* __restrict__ trees, int32_t* __restrict__ fx,
-                             const int32_t* __restrict__ tidx) {
+                             const int32_t* __restrict__ tidx, double* __restrict__ tloss) {
   const int t = *tidx;
   double* wcur = hweight + (size_t)(t & 1) * NH;
   gbdt_node* tree = trees + (size_t)t * NH;
@@ -152,11 +160,13 @@ __global__ void k_tree_begin(int nblk, const double* __restrict__ partial, int64
     tree[k] = z;
   }
   if (threadIdx.x == 0) {
-    double G = 0.0, H = 0.0, mg = 0.0, mh = 0.0;
+    double G = 0.0, H = 0.0, mg = 0.0, mh = 0.0, L = 0.0;
     for (int b = 0; b < nblk; ++b) {
-      G += partial[4 * b]; H += partial[4 * b + 1];
-      mg = fmax(mg, partial[4 * b + 2]); mh = fmax(mh, partial[4 * b + 3]);
+      G += partial[5 * b]; H += partial[5 * b + 1];
+      mg = fmax(mg, partial[5 * b + 2]); mh = fmax(mh, partial[5 * b + 3]);
+      L += partial[5 * b + 4];
     }
+    tloss[t] = L / (double)n;  // mean training loss of the model of trees 0 .. t-1
     fx[0] = fx_scale((double)n, mg);
     fx[1] = fx_scale((double)n, mh);
     *root.K = 1;
@@ -376,6 +386,32 @@ __global__ void k_nodemap(int64_t n, const uint32_t* __restrict__ bits, const ui
   }
 }
 
+// Mean training loss of the final model (after the last tree's SmartGD update), same terms and
+// block-then-ordered association as k_grad's
+__global__ void k_loss_partial(int64_t n, int loss, const double* __restrict__ yhat, const float* __restrict__ y,
+                               double* __restrict__ partial) {
+  double sl = 0.0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const double yh = yhat[i], yi = (double)y[i];
+    sl += loss == GBDT_LOSS_SQUARED ? (yi - yh) * (yi - yh) : fmax(yh, 0.0) - yi * yh + log1p(exp(-fabs(yh)));
+  }
+  for (int o = 16; o; o >>= 1) sl += __shfl_xor_sync(0xffffffffu, sl, o);
+  __shared__ double wl[32];
+  if ((threadIdx.x & 31) == 0) wl[threadIdx.x >> 5] = sl;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double f = 0.0;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) f += wl[w];
+    partial[5 * blockIdx.x + 4] = f;
+  }
+}
+__global__ void k_loss_final(int nblk, const double* __restrict__ partial, int64_t n, int custom,
+                             double* __restrict__ out) {
+  double L = 0.0;
+  for (int b = 0; b < nblk; ++b) L += partial[5 * b + 4];
+  *out = custom ? __longlong_as_double(0x7ff8000000000000ll) : L / (double)n;
+}
+
 __global__ void k_apply(int64_t n, double eta, const double* __restrict__ w, const int32_t* __restrict__ pos,
                         double* __restrict__ yhat) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
@@ -536,7 +572,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     c.take<double>(n); c.take<double>(hmode == kHGather ? n : 1); c.take<double>(n); c.take<int32_t>(n);
     c.take<uint8_t>(npad); c.take<uint32_t>((size_t)(n + 31) / 32 + 1);
     c.take<double>(2 * NH); c.take<uint8_t>(NH); c.take<uint8_t>(NH);
-    c.take<gbdt_node>((size_t)P.n_trees * NH); c.take<double>(4 * grad_blocks); c.take<int32_t>(2);
+    c.take<gbdt_node>((size_t)P.n_trees * NH); c.take<double>(5 * grad_blocks); c.take<int32_t>(2);
+    c.take<double>((size_t)P.n_trees + 1);
     for (int b = 0; b < 2; ++b) { c.take<int32_t>(1); c.take<int32_t>(Kcap); c.take<double>(Kcap); c.take<double>(Kcap); c.take<int32_t>(Kcap); c.take<double>(Kcap); }
     c.take<int32_t>(Kcap); c.take<Rec>(Kcap); c.take<Rec>((size_t)nsh * Kcap); c.take<int>(1);
     c.take<unsigned long long>((size_t)nloc * Kcap); c.take<unsigned long long>((size_t)nloc * Kcap);
@@ -561,8 +598,9 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   uint8_t* hstate = c.take<uint8_t>(NH);
   uint8_t* hdef = c.take<uint8_t>(NH);
   gbdt_node* trees = c.take<gbdt_node>((size_t)P.n_trees * NH);
-  double* partial = c.take<double>(4 * grad_blocks);
+  double* partial = c.take<double>(5 * grad_blocks);
   int32_t* fxs = c.take<int32_t>(2);
+  double* tloss = c.take<double>((size_t)P.n_trees + 1);  // mean training loss after 0 .. T trees
   NodeTab nt[2];
   for (int b = 0; b < 2; ++b) {
     nt[b].K = c.take<int32_t>(1); nt[b].heap = c.take<int32_t>(Kcap); nt[b].G = c.take<double>(Kcap);
@@ -743,7 +781,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       GBDT_CUDA(cudaStreamSynchronize(st));
       if (bad) fail(GBDT_E_INVAL, "grad_fn returned a non-finite g or h, or h < 0, at tree " + std::to_string(t));
     }
-    k_tree_begin<<<1, 1024, 0, st>>>(grad_blocks, partial, n, P.lambda, nt[0], NH, hweight, hstate, trees, fxs, tidx);
+    k_tree_begin<<<1, 1024, 0, st>>>(grad_blocks, partial, n, P.lambda, nt[0], NH, hweight, hstate, trees, fxs, tidx,
+                                     tloss);
     GBDT_LAUNCH_CHECK();
     count_launch(2);
     tm.end();
@@ -1009,6 +1048,10 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     }
     GBDT_LAUNCH_CHECK();
     count_launch();
+    k_loss_partial<<<grad_blocks, 256, 0, st>>>(n, P.loss, yhat, ds.y.as<float>(), partial);
+    k_loss_final<<<1, 1, 0, st>>>(grad_blocks, partial, n, custom ? 1 : 0, tloss + P.n_trees);
+    GBDT_LAUNCH_CHECK();
+    count_launch(2);
   }
   if (tm.on) GBDT_CUDA(cudaEventRecord(tot1, st));
   model.n_trees = P.n_trees;
@@ -1031,6 +1074,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   }
   GBDT_CUDA(cudaMemcpyAsync(model.nodes.data(), trees, sizeof(gbdt_node) * model.nodes.size(),
                             cudaMemcpyDeviceToHost, st));
+  model.train_loss.assign((size_t)P.n_trees + 1, 0.0);
+  GBDT_CUDA(cudaMemcpyAsync(model.train_loss.data(), tloss, sizeof(double) * (P.n_trees + 1), cudaMemcpyDeviceToHost, st));
   if (margin_out)
     GBDT_CUDA(cudaMemcpyAsync(margin_out, yhat, sizeof(double) * (size_t)n, cudaMemcpyDeviceToHost, st));
   GBDT_CUDA(cudaStreamSynchronize(st));

@@ -74,6 +74,7 @@ def lib():
     L.gbdt_train.argtypes = [p, C.POINTER(_Params), C.POINTER(p), p]
     L.gbdt_predict.argtypes = [p, i64, i64, p, p, p, i32, p]
     L.gbdt_predict_on_stream.argtypes = [p, i64, i64, p, p, p, i32, p, p]
+    L.gbdt_model_train_loss.argtypes = [p, p]
     L.gbdt_model_num_trees.argtypes = [p, C.POINTER(i32)]
     L.gbdt_model_num_nodes.argtypes = [p, i32, C.POINTER(i32)]
     L.gbdt_model_export.argtypes = [p, i32, p]
@@ -89,7 +90,8 @@ def lib():
     L.gbdt_shard_ranges.argtypes = [i64, p, i32, p]
     L.gbdt_dataset_free.argtypes = [p]
     L.gbdt_model_free.argtypes = [p]
-    for f in ("gbdt_load_csr", "gbdt_train", "gbdt_predict", "gbdt_predict_on_stream", "gbdt_model_num_trees", "gbdt_model_num_nodes",
+    for f in ("gbdt_load_csr", "gbdt_train", "gbdt_predict", "gbdt_predict_on_stream", "gbdt_model_train_loss",
+              "gbdt_model_num_trees", "gbdt_model_num_nodes",
               "gbdt_model_export", "gbdt_get_timings", "gbdt_get_level_entries", "gbdt_dataset_info", "gbdt_dataset_export_layout",
               "gbdt_dataset_export_rle", "gbdt_comm_unique_id", "gbdt_comm_init", "gbdt_comm_init_callbacks",
               "gbdt_shard_ranges"):
@@ -277,6 +279,12 @@ class Model:
             _check(lib().gbdt_model_export(self._h, t, _p(row)))
             out[t] = row
         return out
+
+    def train_loss(self) -> np.ndarray:
+        """Mean training loss after 0 .. T trees (squared: (y-yhat)^2, RMSE = sqrt; logistic: log loss)."""
+        a = np.zeros(self.n_trees() + 1, np.float64)
+        _check(lib().gbdt_model_train_loss(self._h, _p(a)))
+        return a
 
     def timings(self) -> dict:
         a = np.zeros(len(PHASES), np.float64)

@@ -184,3 +184,25 @@ def test_predict_kernels_match_host_traversal(m_train):
     assert got.tobytes() == want.tobytes()
     # and the training rows reproduce the training margin
     assert np.array_equal(model.predict(p.indptr, p.indices, p.values, p.m), margin)
+
+
+@pytest.mark.parametrize("maker", [lambda: synth.c1(n=2000), lambda: synth.c2(n=5000, T=4)])
+def test_train_loss_per_tree(maker):
+    """gbdt_model_train_loss: the mean training loss after 0 .. T trees (P:415-431 reports RMSE),
+    against the loss of the oracle's prediction with the first k trees on the training rows."""
+    from oracle import oracle
+    p = maker()
+    model, margin = gbdt.train_problem(p)
+    L = model.train_loss()
+    nodes = model.nodes()
+    T = nodes.shape[0]
+    assert L.shape == (T + 1,)
+    y = p.labels.astype(np.float64)
+    for k in range(T + 1):
+        m = oracle.predict(nodes[:k], p.indptr, p.indices, p.values, eta=p.params["eta"]) if k else np.zeros(p.n)
+        if p.params["loss"] == "squared":
+            ref = np.mean((y - m) ** 2)
+        else:
+            ref = np.mean(np.maximum(m, 0) - y * m + np.log1p(np.exp(-np.abs(m))))
+        assert L[k] == pytest.approx(ref, rel=1e-9), (k, L[k], ref)
+    assert L[-1] < L[0]
