@@ -186,6 +186,20 @@ gbdt_status gbdt_model_export(const gbdt_model* m, int32_t tree, gbdt_node* node
  * (Table II) is the square root of the squared-loss entries.  NaN for a custom loss. */
 gbdt_status gbdt_model_train_loss(const gbdt_model* m, double* out);
 
+/* Test hook for the kernel-level invariants (every child segment equals the root
+ * column filtered by node membership, Fig. 2; with RLE its runs equal RLE of that,
+ * P:250 Fig. 7).  When the environment variable GBDT_CAPTURE_LEVEL=l is set at gbdt_train time
+ * (level-by-level path, eager launches), the lists of level l of tree 0 are copied into the model,
+ * one capture per local shard i.  info[5] = {shard, m_shard, K (nodes), list length (padded),
+ * runs}; call with NULL arrays first to size them.  Arrays: col_start[m+1] (padded list starts),
+ * col_len[m], seg_start[m*K], seg_cnt[m*K] (segment a*K+j = node j's part of attribute a),
+ * val/ins[list length], RLE: run_val/run_len/run_pos[runs], seg_run[m*K+1].  Any may be NULL.
+ * GBDT_E_STATE if nothing was captured. */
+gbdt_status gbdt_model_export_level(const gbdt_model* m, int32_t shard, int64_t info[5], int64_t* col_start,
+                                    int64_t* col_len, int64_t* seg_start, int64_t* seg_cnt, float* val,
+                                    int32_t* ins, float* run_val, int32_t* run_len, int64_t* run_pos,
+                                    int32_t* seg_run);
+
 /* Per-phase device milliseconds of the gbdt_train that produced m (profile = 1), else zeros.
  * ms_by_phase: caller-owned, n_phases entries (<= GBDT_N_PHASES filled). */
 gbdt_status gbdt_get_timings(const gbdt_model* m, double* ms_by_phase, int32_t n_phases);

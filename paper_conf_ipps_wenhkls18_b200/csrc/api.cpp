@@ -410,6 +410,26 @@ gbdt_status gbdt_predict_on_stream(const gbdt_model* mh, int64_t n_rows, int64_t
   });
 }
 
+gbdt_status gbdt_model_export_level(const gbdt_model* mh, int32_t i, int64_t info[5], int64_t* col_start,
+                                    int64_t* col_len, int64_t* seg_start, int64_t* seg_cnt, float* val, int32_t* ins,
+                                    float* run_val, int32_t* run_len, int64_t* run_pos, int32_t* seg_run) {
+  return guarded([&] {
+    if (!mh || !info) fail(GBDT_E_INVAL, "NULL argument");
+    const auto& caps = mh->m.captures;
+    if (i < 0 || i >= (int32_t)caps.size()) fail(GBDT_E_STATE, "no captured level (set GBDT_CAPTURE_LEVEL before gbdt_train)");
+    const LevelCapture& L = caps[i];
+    info[0] = L.shard;
+    info[1] = (int64_t)L.col_len.size();
+    info[2] = L.K;
+    info[3] = (int64_t)L.val.size();
+    info[4] = (int64_t)L.run_val.size();
+    auto cp = [](auto* dst, const auto& v) { if (dst) std::copy(v.begin(), v.end(), dst); };
+    cp(col_start, L.col_start); cp(col_len, L.col_len); cp(seg_start, L.seg_start); cp(seg_cnt, L.seg_cnt);
+    cp(val, L.val); cp(ins, L.ins); cp(run_val, L.run_val); cp(run_len, L.run_len); cp(run_pos, L.run_pos);
+    cp(seg_run, L.seg_run);
+  });
+}
+
 gbdt_status gbdt_model_train_loss(const gbdt_model* m, double* out) {
   return guarded([&] {
     if (!m || !out) fail(GBDT_E_INVAL, "NULL argument");

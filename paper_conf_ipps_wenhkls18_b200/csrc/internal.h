@@ -134,6 +134,14 @@ struct Dataset {
   DBuf rows_ptr, rows_idx, rows_val;  // CSR rows (gbdt_load_opts.keep_rows; SmartGD-off ablation)
 };
 
+// One shard's level lists and tables (test hook GBDT_CAPTURE_LEVEL; gbdt_model_export_level)
+struct LevelCapture {
+  int shard = 0, K = 0;
+  std::vector<int64_t> col_start, col_len, seg_start, seg_cnt, run_pos;
+  std::vector<float> val, run_val;
+  std::vector<int32_t> ins, run_len, seg_run;
+};
+
 struct Model {
   int32_t n_trees = 0, max_depth = 0, loss = 0;
   int64_t n_cols = 0;
@@ -142,6 +150,7 @@ struct Model {
   double timings[GBDT_N_PHASES] = {0};
   std::vector<int64_t> level_entries;  // [max_depth] list entries scanned per level (profile = 1)
   std::vector<double> train_loss;      // [n_trees + 1] mean training loss after 0 .. T trees
+  std::vector<LevelCapture> captures;  // per local shard (GBDT_CAPTURE_LEVEL)
   int device = 0;
   int dense = 0;                 // trained on the dense representation: predict fills absent values
   float fill = 0.f;

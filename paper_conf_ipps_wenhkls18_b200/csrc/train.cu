@@ -18,6 +18,8 @@
 // shards, other runs).  The per-node argmax is over a strict
 // total order (gain desc, attr asc, value desc, dir), so its result does not depend on the order
 // in which pieces are reduced.
+#include <nvtx3/nvToolsExt.h>
+
 #include <algorithm>
 #include <cstring>
 #include <mutex>
@@ -478,13 +480,20 @@ struct ShardWork {
   unsigned pgroups = 1;
 };
 
+// NVTX names of the phases (host-side ranges for nsys / ncu --nvtx; no-ops without a tool)
+const char* const kPhaseName[GBDT_N_PHASES] = {"grad", "split_find", "decide", "nodemap", "partition", "comm",
+                                               "total", "k_chunk_agg", "k_split", "k_count", "k_scatter",
+                                               "k_fused"};
+
 struct PhaseTimer {
   bool on = false;
+  bool nvtx = false;  // phase ranges (the outer timer only, so the ranges nest)
   cudaStream_t st = nullptr;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> ev;
   int cur = -1;
   cudaEvent_t e0 = nullptr;
   void begin(int phase) {
+    if (nvtx) nvtxRangePushA(kPhaseName[phase]);
     if (!on) return;
     cudaEvent_t a;
     GBDT_CUDA(cudaEventCreate(&a));
@@ -493,6 +502,7 @@ struct PhaseTimer {
     e0 = a;
   }
   void end() {
+    if (nvtx) nvtxRangePop();
     if (!on) return;
     cudaEvent_t b;
     GBDT_CUDA(cudaEventCreate(&b));
@@ -628,6 +638,11 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     for (int a = 0; a < sh.m && fused; ++a)
       if (sh.h_col_len[a] != n || sh.h_col_start[a] != (int64_t)a * pad4(n)) fused = false;
   }
+  // Test hook (kernel-level invariants): GBDT_CAPTURE_LEVEL=l copies level l's lists,
+  // segment tables and runs of tree 0 to the model (gbdt_model_export_level); eager launches only
+  int cap_level = -1;
+  if (const char* cl = getenv("GBDT_CAPTURE_LEVEL")) cap_level = atoi(cl);
+  if (cap_level >= 0) fused = false;
   {  // opt-in while the fused pass is being tuned (GBDT_FUSED=1)
     const char* fe = getenv("GBDT_FUSED");
     fused = fused && fe && fe[0] != '0';
@@ -749,6 +764,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
 
   PhaseTimer tm, kt;  // phases; kernel-level timers nested inside them
   tm.on = kt.on = P.profile != 0;
+  tm.nvtx = true;
   tm.st = kt.st = st;
   cudaEvent_t tot0 = nullptr, tot1 = nullptr;
   if (tm.on) {
@@ -763,6 +779,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   // when nothing in it needs the host (no profiling events, no user-loss callback, no
   // host-staged collectives); launched directly otherwise.
   auto tree_body = [&](int t) {
+    nvtxRangePushA("tree");
     tm.begin(GBDT_PHASE_GRAD);
     if (rows.indptr) rows.trees = trees;
     k_grad<<<grad_blocks, 256, 0, st>>>(n, P.loss, tidx, P.eta, P.base_margin, ds.y.as<float>(), hweight, NH,
@@ -792,6 +809,53 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       NodeTab& nxt = nt[(lvl + 1) & 1];
       const bool last = (lvl == d - 1);
       const int Kl = 1 << lvl;  // upper bound of active nodes at this level
+      if (cap_level == lvl && t == 0) {  // test hook: this level's lists and tables, tree 0
+        GBDT_CUDA(cudaStreamSynchronize(st));
+        int32_t Kh = 0;
+        GBDT_CUDA(cudaMemcpy(&Kh, cur.K, 4, cudaMemcpyDeviceToHost));
+        model.captures.clear();
+        for (int li = 0; li < nloc; ++li) {
+          Shard& sh = *ds.shards[li];
+          const Tables tb = lvl == 0 ? sh.root : sw[li].tab[lvl & 1];
+          LevelCapture L;
+          L.shard = sh.index;
+          L.K = Kh;
+          L.col_start.resize((size_t)sh.m + 1);
+          L.col_len.resize((size_t)sh.m);
+          L.seg_start.resize((size_t)sh.m * Kh);
+          L.seg_cnt.resize((size_t)sh.m * Kh);
+          if (sh.m) {
+            GBDT_CUDA(cudaMemcpy(L.col_start.data(), tb.col_start, 8 * ((size_t)sh.m + 1), cudaMemcpyDeviceToHost));
+            GBDT_CUDA(cudaMemcpy(L.col_len.data(), tb.col_len, 8 * (size_t)sh.m, cudaMemcpyDeviceToHost));
+            GBDT_CUDA(cudaMemcpy(L.seg_start.data(), tb.seg_start, 8 * L.seg_start.size(), cudaMemcpyDeviceToHost));
+            GBDT_CUDA(cudaMemcpy(L.seg_cnt.data(), tb.seg_cnt, 8 * L.seg_cnt.size(), cudaMemcpyDeviceToHost));
+          }
+          const size_t len = (size_t)L.col_start[sh.m];
+          L.val.resize(len);
+          L.ins.resize(len);
+          const float* val = lvl == 0 ? sh.val0.as<float>() : sh.valw[lvl & 1].as<float>();
+          const int32_t* ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
+          if (len) {
+            GBDT_CUDA(cudaMemcpy(L.val.data(), val, 4 * len, cudaMemcpyDeviceToHost));
+            GBDT_CUDA(cudaMemcpy(L.ins.data(), ins, 4 * len, cudaMemcpyDeviceToHost));
+          }
+          if (sh.rle) {
+            int32_t R = 0;
+            GBDT_CUDA(cudaMemcpy(&R, tb.R, 4, cudaMemcpyDeviceToHost));
+            L.seg_run.resize((size_t)sh.m * Kh + 1);
+            L.run_val.resize((size_t)R);
+            L.run_len.resize((size_t)R);
+            L.run_pos.resize((size_t)R);
+            GBDT_CUDA(cudaMemcpy(L.seg_run.data(), tb.seg_run, 4 * L.seg_run.size(), cudaMemcpyDeviceToHost));
+            if (R) {
+              GBDT_CUDA(cudaMemcpy(L.run_val.data(), tb.run_val, 4 * (size_t)R, cudaMemcpyDeviceToHost));
+              GBDT_CUDA(cudaMemcpy(L.run_len.data(), tb.run_len, 4 * (size_t)R, cudaMemcpyDeviceToHost));
+              GBDT_CUDA(cudaMemcpy(L.run_pos.data(), tb.run_pos, 8 * (size_t)R, cudaMemcpyDeviceToHost));
+            }
+          }
+          model.captures.push_back(std::move(L));
+        }
+      }
       // fz: this level's node bests were found by the previous level's fused pass
       const bool fz = fused && lvl >= 1;
       if (!fz) {
@@ -991,6 +1055,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     k_tree_end<<<1, 1, 0, st>>>(tidx);
     GBDT_LAUNCH_CHECK();
     count_launch();
+    nvtxRangePop();
   };
 
   // One CUDA graph per tree, NCCL collectives included (captured on the library's stream; a world
@@ -999,7 +1064,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   const bool host_comm = ds.comm && !ds.comm->nccl;
   const char* ge = getenv("GBDT_GRAPH");
   const bool graph_ok = ge ? ge[0] != '0' : true;
-  const bool graph = !tm.on && !custom && !host_comm && P.n_trees > 1 && graph_ok;
+  const bool graph = !tm.on && !custom && !host_comm && P.n_trees > 1 && graph_ok && cap_level < 0;
   if (!graph) {
     for (int t = 0; t < P.n_trees; ++t) tree_body(t);
   } else {

@@ -75,6 +75,7 @@ def lib():
     L.gbdt_predict.argtypes = [p, i64, i64, p, p, p, i32, p]
     L.gbdt_predict_on_stream.argtypes = [p, i64, i64, p, p, p, i32, p, p]
     L.gbdt_model_train_loss.argtypes = [p, p]
+    L.gbdt_model_export_level.argtypes = [p, i32] + [p] * 11
     L.gbdt_model_num_trees.argtypes = [p, C.POINTER(i32)]
     L.gbdt_model_num_nodes.argtypes = [p, i32, C.POINTER(i32)]
     L.gbdt_model_export.argtypes = [p, i32, p]
@@ -91,6 +92,7 @@ def lib():
     L.gbdt_dataset_free.argtypes = [p]
     L.gbdt_model_free.argtypes = [p]
     for f in ("gbdt_load_csr", "gbdt_train", "gbdt_predict", "gbdt_predict_on_stream", "gbdt_model_train_loss",
+              "gbdt_model_export_level",
               "gbdt_model_num_trees", "gbdt_model_num_nodes",
               "gbdt_model_export", "gbdt_get_timings", "gbdt_get_level_entries", "gbdt_dataset_info", "gbdt_dataset_export_layout",
               "gbdt_dataset_export_rle", "gbdt_comm_unique_id", "gbdt_comm_init", "gbdt_comm_init_callbacks",
@@ -280,9 +282,25 @@ class Model:
             out[t] = row
         return out
 
+    def export_level(self, shard=0) -> dict:
+        """The level captured with GBDT_CAPTURE_LEVEL (test hook; see gbdt_model_export_level)."""
+        info = np.zeros(5, np.int64)
+        L = lib()
+        N = None
+        _check(L.gbdt_model_export_level(self._h, shard, _p(info), N, N, N, N, N, N, N, N, N, N))
+        m, K, n, R = int(info[1]), int(info[2]), int(info[3]), int(info[4])
+        out = dict(shard=int(info[0]), m=m, K=K, col_start=np.zeros(m + 1, np.int64), col_len=np.zeros(m, np.int64),
+                   seg_start=np.zeros(m * K, np.int64), seg_cnt=np.zeros(m * K, np.int64),
+                   val=np.zeros(n, np.float32), ins=np.zeros(n, np.int32), run_val=np.zeros(R, np.float32),
+                   run_len=np.zeros(R, np.int32), run_pos=np.zeros(R, np.int64),
+                   seg_run=np.zeros(m * K + 1 if R else 0, np.int32))
+        _check(L.gbdt_model_export_level(self._h, shard, _p(info), *[_p(out[k]) for k in (
+            "col_start", "col_len", "seg_start", "seg_cnt", "val", "ins", "run_val", "run_len", "run_pos", "seg_run")]))
+        return out
+
     def train_loss(self) -> np.ndarray:
         """Mean training loss after 0 .. T trees (squared: (y-yhat)^2, RMSE = sqrt; logistic: log loss)."""
-        a = np.zeros(self.n_trees() + 1, np.float64)
+        a = np.zeros(self.n_trees + 1, np.float64)
         _check(lib().gbdt_model_train_loss(self._h, _p(a)))
         return a
 

@@ -446,3 +446,38 @@ def test_lambda0_squared_is_cart_on_gpu():
     groups_gpu = {frozenset(np.where(margin == v)[0]) for v in np.unique(margin)}
     assert groups_sk == groups_gpu
     np.testing.assert_allclose(margin, sk.predict(X.astype(np.float32)), rtol=0, atol=1e-9)
+
+
+# ------------------------------------------------------------------ near-ties decided exactly (no follow mode)
+# Two candidates of one chunk whose Eq. 2 gains differ by ~1e-9 relative (far below the 1e-6 band
+# follow mode would forgive, far above the ~1e-15 ranking error of the in-chunk scores, DESIGN.md
+# I3): the CUDA path must pick the exact maximiser the oracle picks, with no follow mode.
+@pytest.mark.parametrize("delta", [3e-7, -3e-7])
+@pytest.mark.parametrize("fused", ["0", "1"])
+def test_close_candidates_in_one_chunk_pick_the_exact_best(delta, fused, monkeypatch):
+    monkeypatch.setenv("GBDT_FUSED", fused)
+    n = 200
+    x = np.arange(n, dtype=np.float64)
+    y = np.where((x < 60) | (x >= 140), 1.0, -1.0)
+    y[0] += delta                      # breaks the symmetry of the splits at 60 and at 140
+    X = np.stack([x, np.zeros(n)], axis=1)  # a second constant column (no candidate)
+    for depth in (1, 2):
+        p = synth.from_dense("near", X, y, dict(loss="squared", max_depth=depth, n_trees=1, lam=1.0, gamma=0.0,
+                                                eta=1.0, base_margin=0.0))
+        on, om, _ = oracle.train(p)
+        model, margin = _train(p)
+        nodes = model.nodes()
+        g0, g1 = oracle.gain(*_two(p, 60)), oracle.gain(*_two(p, 140))
+        rel = abs(g0 - g1) / max(g0, g1)
+        assert 1e-12 < rel < 1e-7, rel
+        for f in ("heap_id", "is_leaf", "attr", "split_value", "default_left", "count"):
+            assert np.array_equal(nodes[f], on[f]), (f, nodes[f][0], on[f][0])
+        np.testing.assert_allclose(margin, om, rtol=1e-12, atol=1e-12)
+
+
+def _two(p, cut):
+    """(GL, HL, G, H, lambda) of the split 'x >= cut' at the root, squared loss at yhat = 0."""
+    g = -2.0 * p.labels.astype(np.float64)
+    X = p.dense()
+    hi = X[:, 0] >= cut
+    return float(g[hi].sum()), 2.0 * float(hi.sum()), float(g.sum()), 2.0 * p.n, 1.0
