@@ -1,4 +1,6 @@
-# GPU: compute-sanitizer memcheck (all cases) and racecheck / synccheck (dense + sparse cases)
-compute-sanitizer --tool memcheck --leak-check no --error-exitcode 9 python tools/sanitize_cases.py > gpurun_out/sanitize_memcheck.log 2>&1; echo "rc=$?" >> gpurun_out/sanitize_memcheck.log
-compute-sanitizer --tool racecheck --error-exitcode 9 python tools/sanitize_cases.py > gpurun_out/sanitize_racecheck.log 2>&1; echo "rc=$?" >> gpurun_out/sanitize_racecheck.log
-compute-sanitizer --tool synccheck --error-exitcode 9 python tools/sanitize_cases.py > gpurun_out/sanitize_synccheck.log 2>&1; echo "rc=$?" >> gpurun_out/sanitize_synccheck.log
+# GPU: compute-sanitizer memcheck, racecheck and synccheck over tools/sanitize_cases.py
+make -s -j8 -C paper_conf_ipps_wenhkls18_b200/csrc >/dev/null 2>&1
+for T in memcheck racecheck synccheck; do
+  X=""; [ $T = memcheck ] && X="--leak-check no"
+  timeout 1500 compute-sanitizer --tool $T $X --error-exitcode 9 python tools/sanitize_cases.py > gpurun_out/sanitize_$T.log 2>&1; echo "rc=$?" >> gpurun_out/sanitize_$T.log
+done

@@ -1,5 +1,7 @@
-"""Small trainings covering every kernel family (dense, missing values, sparse short lists, RLE,
-loopback shards, deep trees, SmartGD-off, prediction), for compute-sanitizer runs."""
+"""Small trainings covering every kernel family (dense, missing values, sparse short lists, RLE and
+its decompression ablation, AUTO RLE, dense representation, loopback shards, deep trees,
+SmartGD-off, the fused dense pass, prediction), for compute-sanitizer runs."""
+import os
 import sys
 
 sys.path.insert(0, ".")
@@ -14,8 +16,17 @@ cases = [
     ("shards", synth.c1(n=2000), {"n_shards": 4}),
     ("deep", synth.random_small(77, n=6000, m=6, nan_frac=0.0, n_distinct=400, loss="logistic", d=8, T=2), {}),
     ("smartgd_off", synth.c1(n=1000), {"smartgd": False}),
+    ("rle_decompress", synth.c5(n=20000, T=2), {"rle": "on", "rle_split": "decompress"}),
+    ("rle_auto", synth.c2(n=6000, T=2), {"rle": "auto"}),
+    ("dense_repr", synth.c4(seed=12, n=800, m=200, density=0.05, T=2), {"dense": True}),
+    ("fused", synth.c3(n=20000, T=2), {"_env": "GBDT_FUSED"}),
 ]
 for name, p, kw in cases:
+    env = kw.pop("_env", None)
+    if env:
+        os.environ[env] = "1"
     model, margin = gbdt.train_problem(p, **kw)
+    if env:
+        del os.environ[env]
     model.predict(p.indptr, p.indices, p.values, p.m)
     print(name, "ok", flush=True)
