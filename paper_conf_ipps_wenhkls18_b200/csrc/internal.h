@@ -79,6 +79,10 @@ struct Tables {
   int64_t* run_pos = nullptr;
   int32_t* R = nullptr;           // [1] runs at this level
   int32_t* run_chunk = nullptr;   // [C] the run holding each chunk's first entry
+  // short-attribute path (levels.cu k_short_*): the chunks the chunk kernels take, i.e. those of
+  // the attributes not on the short path (all chunks when nullptr, or when K > 32)
+  int32_t* lc = nullptr;          // [C]
+  int32_t* nlc = nullptr;         // [1]
 };
 
 // Best split of one node found in one shard ("piece" records are reduced to this).

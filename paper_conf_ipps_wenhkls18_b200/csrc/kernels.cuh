@@ -23,6 +23,15 @@ struct TileArgs {
   int a_base;          // global id of local attribute 0
   const int32_t* Kp;   // active nodes at this level
   int* counter;        // dynamic tile claim counter (reset per level)
+  const uint8_t* sflag = nullptr;  // [m] 1: attribute on the short path (k_short_*); nullptr: none
+};
+
+// Attributes whose whole root list has at most a few dozen entries (the typical sparse attribute,
+// P:214-216) take the short path at every level with K <= 32: one LANE per (attribute, node)
+// segment walks the segment's entries in list order (levels.cu k_short_split / _count / _scatter).
+struct ShortList {
+  const int32_t* attrs = nullptr;  // shard-local ids, longest root list first (load balance)
+  int n = 0;
 };
 
 
@@ -114,6 +123,7 @@ struct PlanArgs {
   unsigned egroups;
   const int32_t* mp1;     // m + 1 (device)
   Tables nxt;
+  const uint8_t* sflag = nullptr;  // short-path attributes: left out of nxt.lc when K' <= 32
 };
 
 struct RunArgs {
@@ -207,6 +217,7 @@ struct LevelKernels {
   unsigned grid_fast[3][2] = {{0}};  // [hmode][rle]
   unsigned grid_gen = 0;
   unsigned grid_short = 0;
+  unsigned grid_sl = 0;  // k_short_split
   unsigned grid_agg[3] = {0};
   unsigned grid_fused = 0;
   unsigned grid_scatter[3][2] = {{0}}, grid_count = 0, grid_count_dense = 0, grid_agg_list[3] = {0};  // scatter: [hmode][agg]
@@ -217,8 +228,12 @@ struct LevelKernels {
   void split_find(const SplitArgs& A, int hmode, bool missing, bool rle, cudaStream_t st);
   void seg_totals(const SplitArgs& A, int hmode, cudaStream_t st);
   // a8: count -> exact scan -> plan (next level's tables), then the stable scatter
-  void partition_count(const PartArgs& A, const PlanArgs& P, bool counted, unsigned groups, cudaStream_t st);
-  void partition_scatter(const PartArgs& A, int hmode, const RunArgs* rle, cudaStream_t st);
+  void partition_count(const PartArgs& A, const PlanArgs& P, bool counted, unsigned groups, cudaStream_t st,
+                       const ShortList* sl = nullptr);
+  void partition_scatter(const PartArgs& A, int hmode, const RunArgs* rle, cudaStream_t st,
+                         const ShortList* sl = nullptr);
+  // split find of the short-path attributes (root: gathers their g-lists too)
+  void short_split(const SplitArgs& A, const ShortList& S, int hmode, bool gather, cudaStream_t st);
   // a3: the level's chunk descriptors and scan flags when the previous scatter accumulated the
   // chunk aggregates, then the exact carry scan
   void chunk_desc(const SplitArgs& A, unsigned groups, cudaStream_t st);

@@ -152,6 +152,11 @@ __device__ __forceinline__ int find_attr(const int* start, int m, int x) {
   return lo;
 }
 
+// The chunk set of the chunk kernels: every chunk, or (short path, levels.cu k_short_*) the list of
+// the chunks of the other attributes
+__device__ __forceinline__ int nchunks(const Tables& tb) { return tb.lc ? *tb.nlc : *tb.C; }
+__device__ __forceinline__ int chunk_at(const Tables& tb, int i) { return tb.lc ? tb.lc[i] : i; }
+
 // Range of one chunk (all lanes compute it; the tables are in smem when m is small).
 struct ChunkMeta {
   long long p0, p1, sb;
@@ -373,12 +378,14 @@ __global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
   tab_load(tc, A.t);
   __syncthreads();
   const int nw = (gridDim.x * blockDim.x) >> 5;
-  for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nw) {
+  const int NC = nchunks(A.t.tb);
+  for (int i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < NC; i += nw) {
+    const int c = chunk_at(A.t.tb, i);
     const ChunkMeta M = chunk_meta(tc, A.t, K, c);
     const long long p1 = M.p1;
     const long long base = M.p0 + (long long)lane * kItems;
-    if (!kGather && c + nw < C) {  // the warp's next chunk streams into L2 meanwhile
-      const ChunkMeta Mn = chunk_meta(tc, A.t, K, c + nw);
+    if (!kGather && i + nw < NC) {  // the warp's next chunk streams into L2 meanwhile
+      const ChunkMeta Mn = chunk_meta(tc, A.t, K, chunk_at(A.t.tb, i + nw));
       prefetch_chunk(A.glist, Mn.p0, 8, lane);
       if (HMODE == kHGather) prefetch_chunk(A.hlist, Mn.p0, 8, lane);
     }
@@ -1252,7 +1259,7 @@ __global__ void __launch_bounds__(kThreads) k_sf_short(SplitArgs A) {
   for (int j = threadIdx.x; j < kWarps * kWarpK; j += blockDim.x) wgk[j / kWarpK][j % kWarpK] = 0ull;
   __syncthreads();
   const int nw = (gridDim.x * blockDim.x) >> 5;
-  const int n = kMissing ? C : *A.ngen;  // k_sf_gen's chunk set
+  const int n = kMissing ? nchunks(A.t.tb) : *A.ngen;  // k_sf_gen's chunk set
   // 32 chunks per warp step, lane l testing chunk bt + l * nbat (strided, so the chunks of one long
   // list spread over the warps); the warp then runs the short ones
   // (only when the chunks outnumber the warps 32 to 1: a short list of heavy chunks, e.g. the
@@ -1264,7 +1271,7 @@ __global__ void __launch_bounds__(kThreads) k_sf_short(SplitArgs A) {
     int cc = 0;
     bool take = false;
     if (lane < bw && ii < n) {
-      cc = kMissing ? ii : A.genlist[ii];
+      cc = kMissing ? chunk_at(A.t.tb, ii) : A.genlist[ii];
       take = A.desc[cc].len <= 32;
     }
     unsigned todo = __ballot_sync(0xffffffffu, take);
@@ -1284,6 +1291,223 @@ __global__ void __launch_bounds__(kThreads) k_sf_short(SplitArgs A) {
       const int gs = atomicAdd(A.nrec, 1);
       A.rec[gs] = wrec[bw][j];
       atomicMax(A.gkey + j, wgk[bw][j]);
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------- short attributes
+// The typical attribute of a sparse data set has a handful of entries ("many small
+// segments"; C4a: 1.08 M of its 1.13 M non-empty lists hold <= 32), so a warp per 256-entry chunk
+// spends ~500 instructions per list on shuffles and table walks whatever its length.  These
+// attributes (ShortList, fixed at the root: lists only shrink) take a path of their own at every
+// level with K <= 32: a group of Kp lanes per attribute (Kp = K rounded up to a power of two; 32/Kp
+// attributes per warp), lane j of the group on segment (a, j), walking the segment's entries in list
+// order.  Segments are contiguous and node-ordered, so the segment's present totals, its
+// prefix sums and run ends need no cross-lane step at all; the chunk kernels skip these
+// attributes (Tables::lc) and the exact chunk scans are not involved (a whole list is one piece).
+// Candidates, their order and the record semantics are k_sf_short's: a run end (the next value
+// differs, or the segment's last entry), missing -> right before missing -> left, earliest entry
+// on equal scores; the segment's winner gets its Eq. 2 gain with IEEE divisions.
+__device__ __forceinline__ int short_group(int K) {  // K <= 32
+  int G = 1;
+  while (G < K) G <<= 1;
+  return G;
+}
+
+template <int HMODE, bool kGather>
+__global__ void __launch_bounds__(kThreads) k_short_split(SplitArgs A, ShortList S) {
+  constexpr bool kH = HMODE == kHGather;
+  __shared__ NodeBest B;
+  __shared__ unsigned long long wgk[kWarps][kWarpK];
+  __shared__ Rec wrec[kWarps][kWarpK];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int K = *A.t.Kp;
+  if (K == 0 || K > kWarpK || S.n == 0) return;
+  const int epoch = *A.epochp;
+  const double lam = A.lam;
+  nb_init(B, A, K);
+  for (int j = threadIdx.x; j < kWarps * kWarpK; j += blockDim.x) wgk[j / kWarpK][j % kWarpK] = 0ull;
+  __syncthreads();
+  const unsigned long long pol_keep = policy_evict_last();
+  const int Kp = short_group(K), G = 32 / Kp, sub = lane / Kp, j = lane % Kp;
+  const NodeV nv = j < K ? node_v(B, A, K, j) : NodeV{0.0, 0.0, 0.0, 0};
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int i0 = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * G; i0 < S.n; i0 += nw * G) {
+    const int i = i0 + sub;
+    const int a = (i < S.n && j < K) ? S.attrs[i] : -1;
+    long long s0 = 0;
+    int cnt = 0;
+    if (a >= 0) {
+      const long long sI = (long long)a * K + j;
+      s0 = A.t.tb.seg_start[sI];
+      cnt = (int)A.t.tb.seg_cnt[sI];
+    }
+    bool ok = false;
+    double best = 0.0, bg = 0.0, bh = 0.0, PG = 0.0, PH = 0.0;
+    int be = 0, bd = 0, bc = 0;
+    float bv = 0.f;
+    const int cM = nv.C - cnt;  // the node's instances missing from this attribute
+    if (cnt > 0) {
+      // pass 1: present totals of the segment (root: the g-list gathered on the way)
+      if (kGather || cM > 0) {
+        for (int e = 0; e < cnt; ++e) {
+          const long long p = s0 + e;
+          double g, h;
+          if (kGather) {
+            const int id = __ldg(A.t.ins + p);
+            g = ld_keep(A.g + id, pol_keep);
+            h = kH ? ld_keep(A.h + id, pol_keep) : hess_of<HMODE>(g);
+            A.glist[p] = g;
+            if (kH) A.hlist[p] = h;
+          } else {
+            g = A.glist[p];
+            h = kH ? A.hlist[p] : hess_of<HMODE>(g);
+          }
+          PG = PG + g;
+          PH = PH + h;
+        }
+      }
+      // pass 2: prefix sums in list order, candidates at run ends
+      double ig = 0.0, ih = 0.0;
+      float v = A.t.val[s0];
+#pragma unroll 2
+      for (int e = 0; e < cnt; ++e) {
+        const long long p = s0 + e;
+        const bool last = e + 1 == cnt;
+        const float vn = last ? v : A.t.val[p + 1];
+        const double g = A.glist[p];
+        const double h = kH ? A.hlist[p] : hess_of<HMODE>(g);
+        ig = ig + g;
+        ih = ih + h;
+        const int icn = e + 1;
+        if (last || vn != v) {
+          if (nv.C - icn >= 1) {
+            const double sc = split_score(ig, ih, nv.G, nv.H, lam);
+            if (!ok || sc > best) { best = sc; ok = true; bd = 0; be = e; bg = ig; bh = ih; bc = icn; bv = v; }
+          }
+          if (cM > 0 && nv.C - (icn + cM) >= 1) {
+            const double s1 = split_score(ig + (nv.G - PG), ih + (nv.H - PH), nv.G, nv.H, lam);
+            if (!ok || s1 > best) { best = s1; ok = true; bd = 1; be = e; bg = ig; bh = ih; bc = icn; bv = v; }
+          }
+        }
+        v = vn;
+      }
+    }
+    // the segment's record; then the best per node over the warp's attributes (lanes j, j + Kp, ...)
+    Rec r;
+    unsigned long long gk = 0ull, tk = ~0ull;
+    if (ok) {
+      r.value = bv;
+      r.attr = A.t.a_base + a;
+      r.dir = bd;
+      r.node = j;
+      r.epoch = epoch;
+      r.shard = A.shard;
+      r.pos = s0 + be;
+      if (bd) {
+        r.GL = bg + (nv.G - PG);
+        r.HL = bh + (nv.H - PH);
+        r.cntL = bc + cM;
+      } else {
+        r.GL = bg; r.HL = bh; r.cntL = bc;
+      }
+      r.gain = eq2_gain(r.GL, r.HL, nv.G, nv.H, lam, nv.P);
+      gk = gain_key(r.gain);
+      tk = tie_key(r.attr, r.value, r.dir);
+    }
+    int src = lane;
+    for (int o = Kp; o < 32; o <<= 1) {
+      const unsigned long long og = __shfl_xor_sync(0xffffffffu, gk, o), ot = __shfl_xor_sync(0xffffffffu, tk, o);
+      const int os = __shfl_xor_sync(0xffffffffu, src, o);
+      if (og > gk || (og == gk && ot < tk)) { gk = og; tk = ot; src = os; }
+    }
+    if (!__any_sync(0xffffffffu, gk != 0ull)) continue;
+    Rec w;
+    w.gain = __shfl_sync(0xffffffffu, r.gain, src);
+    w.GL = __shfl_sync(0xffffffffu, r.GL, src);
+    w.HL = __shfl_sync(0xffffffffu, r.HL, src);
+    w.cntL = __shfl_sync(0xffffffffu, r.cntL, src);
+    w.pos = __shfl_sync(0xffffffffu, r.pos, src);
+    w.value = __shfl_sync(0xffffffffu, r.value, src);
+    w.attr = __shfl_sync(0xffffffffu, r.attr, src);
+    w.dir = __shfl_sync(0xffffffffu, r.dir, src);
+    w.node = j;
+    w.epoch = epoch;
+    w.shard = A.shard;
+    if (sub == 0 && gk != 0ull && j < K && rec_better(gk, w, wgk[wid][j], wrec[wid][j])) {
+      wgk[wid][j] = gk;
+      wrec[wid][j] = w;
+    }
+  }
+  __syncthreads();  // merge the warp tables, one record per node and CTA
+  for (int jj = threadIdx.x; jj < K; jj += blockDim.x) {
+    int bw = -1;
+    for (int w = 0; w < kWarps; ++w)
+      if (wgk[w][jj] && (bw < 0 || rec_better(wgk[w][jj], wrec[w][jj], wgk[bw][jj], wrec[bw][jj]))) bw = w;
+    if (bw >= 0) {
+      const int gs = atomicAdd(A.nrec, 1);
+      A.rec[gs] = wrec[bw][jj];
+      atomicMax(A.gkey + jj, wgk[bw][jj]);
+    }
+  }
+}
+
+// Partition count of the short-path segments: a lane per segment counts its entries per side
+// (segH / segL of the plan; the chunk kernels' slist is not needed, the scatter gathers again)
+__global__ void __launch_bounds__(kThreads) k_short_count(PartArgs A, ShortList S) {
+  const int K = *A.t.Kp;
+  if (K == 0 || K > kWarpK || S.n == 0) return;
+  const int lane = threadIdx.x & 31;
+  const int Kp = short_group(K), G = 32 / Kp, sub = lane / Kp, j = lane % Kp;
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int i0 = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * G; i0 < S.n; i0 += nw * G) {
+    const int i = i0 + sub;
+    if (i >= S.n || j >= K) continue;
+    const long long sI = (long long)S.attrs[i] * K + j;
+    const int cnt = (int)A.t.tb.seg_cnt[sI];
+    if (cnt == 0 || A.cidx[j] < 0) continue;  // a new leaf drops its entries
+    const long long s0 = A.t.tb.seg_start[sI];
+    int hi = 0, lo = 0;
+#pragma unroll 4
+    for (int e = 0; e < cnt; ++e) {
+      const uint8_t sd = __ldg(A.side + __ldg(A.t.ins + s0 + e));
+      hi += sd == 1;
+      lo += sd == 2;
+    }
+    A.segH[sI] = hi;
+    A.segL[sI] = lo;
+  }
+}
+
+// Stable scatter of the short-path segments: the lane walks its segment in list order,
+// so each child's entries keep their order; destinations from the plan (out_hi / out_lo)
+template <int HMODE>
+__global__ void __launch_bounds__(kThreads) k_short_scatter(PartArgs A, ShortList S) {
+  constexpr bool kH = HMODE == kHGather;
+  const int K = *A.t.Kp;
+  if (K == 0 || K > kWarpK || S.n == 0) return;
+  const int lane = threadIdx.x & 31;
+  const int Kp = short_group(K), G = 32 / Kp, sub = lane / Kp, j = lane % Kp;
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int i0 = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * G; i0 < S.n; i0 += nw * G) {
+    const int i = i0 + sub;
+    if (i >= S.n || j >= K) continue;
+    const long long sI = (long long)S.attrs[i] * K + j;
+    const int cnt = (int)A.t.tb.seg_cnt[sI];
+    if (cnt == 0 || A.cidx[j] < 0) continue;
+    const long long s0 = A.t.tb.seg_start[sI];
+    long long dh = A.out_hi[sI], dl = A.out_lo[sI];
+#pragma unroll 4
+    for (int e = 0; e < cnt; ++e) {
+      const long long p = s0 + e;
+      const int id = __ldg(A.t.ins + p);
+      const uint8_t sd = __ldg(A.side + id);
+      if (!sd) continue;
+      const long long d = sd == 1 ? dh++ : dl++;
+      A.val_out[d] = A.t.val[p];
+      A.ins_out[d] = id;
+      A.g_out[d] = A.g_in[p];
+      if (kH) A.h_out[d] = A.h_in[p];
     }
   }
 }
@@ -1312,7 +1536,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
   const int nw = (gridDim.x * blockDim.x) >> 5;
   // with missing values every chunk; else the chunks k_chunk_agg listed (they cross segments)
   constexpr bool kAll = kMissing || kTotals;
-  const int n = kAll ? C : *A.ngen;
+  const int n = kAll ? nchunks(A.t.tb) : *A.ngen;
   // 32 chunks per warp step (lane l tests chunk bt + l * nbat); the short ones are k_sf_short's,
   // so they cost one descriptor word here instead of a dependent descriptor load each
   // (only when the chunks outnumber the warps 32 to 1: a short list of heavy chunks, e.g. the
@@ -1324,7 +1548,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
     int cc = 0;
     bool take = false;
     if (lane < bw && ii < n) {
-      cc = kAll ? ii : A.genlist[ii];
+      cc = kAll ? chunk_at(A.t.tb, ii) : A.genlist[ii];
       take = kTotals || !GBDT_SF_SHORT_KERNEL || !kMissing || !(A.desc[cc].len <= 32 && K <= kWarpK);
     }
     unsigned todo = __ballot_sync(0xffffffffu, take);
@@ -1600,7 +1824,8 @@ __global__ void __launch_bounds__(kThreads) k_part_count(PartArgs A, int counted
   const int nw = (gridDim.x * blockDim.x) >> 5;
   // software pipeline: the instance ids of the warp's next chunk are loaded before the side
   // gathers of the current one, so the list stream and the (L2) gathers overlap
-  int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int NC = nchunks(A.t.tb);
+  int i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   int4 n0 = make_int4(0, 0, 0, 0), n1 = n0;
   auto load_ids = [&](int cc, int4& a0, int4& a1) {
     const ChunkMeta Mx = chunk_meta(tc, A.t, K, cc);
@@ -1610,12 +1835,13 @@ __global__ void __launch_bounds__(kThreads) k_part_count(PartArgs A, int counted
       if (b + 4 < Mx.p1) a1 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + b + 4));
     }
   };
-  if (c < C) load_ids(c, n0, n1);
-  for (; c < C; c += nw) {
+  if (i < NC) load_ids(chunk_at(A.t.tb, i), n0, n1);
+  for (; i < NC; i += nw) {
+    const int c = chunk_at(A.t.tb, i);
     const ChunkMeta M = chunk_meta(tc, A.t, K, c);
     const long long base = M.p0 + (long long)lane * kItems;
     const int4 i0 = n0, i1 = n1;
-    if (c + nw < C) load_ids(c + nw, n0, n1);
+    if (i + nw < NC) load_ids(chunk_at(A.t.tb, i + nw), n0, n1);
 #if GBDT_COUNT_SHORT
     if (counted && M.p1 - M.p0 <= 32 && K <= 32) {
       count_short(A, M, c, K, lane);
@@ -1868,6 +2094,7 @@ __global__ void __launch_bounds__(kThreads) k_plan_seg(PlanArgs A) {
         if (a == m) {
           *A.nxt.C = ch;
           *A.nxt.T = (ch + kChunksPerTile - 1) / kChunksPerTile;
+          if (A.nxt.nlc) *A.nxt.nlc = 0;  // k_chunk_attr lists the chunk kernels' chunks
         }
       }
     }
@@ -1900,10 +2127,28 @@ __global__ void __launch_bounds__(kThreads) k_plan_seg(PlanArgs A) {
 }
 
 // attribute of every chunk of the next level (the largest a with chunk_start[a] <= c)
+// and, on the short path, the list of the chunk kernels' chunks: those of the other attributes
+// (every chunk when K' > 32, where the short kernels stand down)
 __global__ void __launch_bounds__(kThreads) k_chunk_attr(PlanArgs A) {
   const int C = *A.nxt.C, m = A.m;
-  for (int c = blockIdx.x * blockDim.x + threadIdx.x; c < C; c += gridDim.x * blockDim.x)
-    A.nxt.chunk_attr[c] = find_attr(A.nxt.chunk_start, m, c);
+  const int lane = threadIdx.x & 31;
+  const bool sp = A.nxt.lc && A.sflag && *A.Knp <= 32;
+  for (int c0 = (blockIdx.x * blockDim.x + threadIdx.x) - lane; c0 < C; c0 += gridDim.x * blockDim.x) {
+    const int c = c0 + lane;
+    int a = 0;
+    if (c < C) {
+      a = find_attr(A.nxt.chunk_start, m, c);
+      A.nxt.chunk_attr[c] = a;
+    }
+    if (A.nxt.lc) {  // warp-aggregated append, chunk order kept inside the warp
+      const bool keep = c < C && !(sp && A.sflag[a]);
+      const unsigned b = __ballot_sync(0xffffffffu, keep);
+      int base = 0;
+      if (lane == 0 && b) base = atomicAdd(A.nxt.nlc, __popc(b));
+      base = __shfl_sync(0xffffffffu, base, 0);
+      if (keep) A.nxt.lc[base + __popc(b & ((1u << lane) - 1u))] = c;
+    }
+  }
 }
 
 // Stable scatter ("Scatter"), one warp per chunk: out(e) = out_base(seg, side) + rank of
@@ -1974,12 +2219,14 @@ __global__ void __launch_bounds__(kThreads, GBDT_SCATTER_CTAS) k_part_scatter(Pa
   __syncthreads();
   const unsigned lt = (1u << lane) - 1u;
   const int nw = (gridDim.x * blockDim.x) >> 5;
-  for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nw) {
+  const int NC = nchunks(A.t.tb);
+  for (int i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < NC; i += nw) {
+    const int c = chunk_at(A.t.tb, i);
     const ChunkMeta M = chunk_meta(tc, A.t, K, c);
     const long long p0 = M.p0;
     const int len = (int)(M.p1 - p0);
-    if (c + nw < C) {  // the warp's next chunk streams into L2 meanwhile
-      const long long pn = chunk_meta(tc, A.t, K, c + nw).p0;
+    if (i + nw < NC) {  // the warp's next chunk streams into L2 meanwhile
+      const long long pn = chunk_meta(tc, A.t, K, chunk_at(A.t.tb, i + nw)).p0;
       prefetch_chunk(A.t.ins, pn, 4, lane);
       prefetch_chunk(A.g_in, pn, 8, lane);
       if (!kRLE) prefetch_chunk(A.t.val, pn, 4, lane);
@@ -2509,9 +2756,12 @@ void launch_scan(const int32_t* Cp, unsigned long long* in, unsigned long long* 
 // Present totals of every segment (missing values): the partial written by k_chunk_agg at the
 // segment's last entry, plus the exact carry of that chunk when the segment began before it.
 __global__ void __launch_bounds__(kThreads) k_seg_totals(SplitArgs A) {
-  const long long S = (long long)A.t.m * *A.t.Kp;
+  const int K = *A.t.Kp;
+  const long long S = (long long)A.t.m * K;
+  const bool sp = A.t.sflag && K <= 32;  // the short path's segments sum their own totals
   for (long long s = blockIdx.x * (long long)blockDim.x + threadIdx.x; s < S; s += (long long)gridDim.x * blockDim.x) {
     if (A.t.tb.seg_cnt[s] == 0) continue;
+    if (sp && A.t.sflag[s / K]) continue;
     const int ce = A.segEnd[s];
     if (ce < 0) continue;
     const CarryD cx = carry_load(A.carry + 5ll * ce);
@@ -2532,6 +2782,7 @@ void LevelKernels::init(int device) {
   grid_fast[2][1] = grid_for(k_sf_fast<2, true>, fast_smem(2), sms);
   grid_gen = grid_for(k_sf_gen<2, true, false, true>, 0, sms);  // the largest variant
   grid_short = grid_for(k_sf_short<2, true, true>, 0, sms);
+  grid_sl = grid_for(k_short_split<2, true>, 0, sms);
   grid_agg[0] = grid_for(k_chunk_agg<0, true>, 0, sms);
   grid_agg[1] = grid_for(k_chunk_agg<1, true>, 0, sms);
   grid_agg[2] = grid_for(k_chunk_agg<2, true>, 0, sms);
@@ -2614,11 +2865,16 @@ void LevelKernels::seg_totals(const SplitArgs& A, int hmode, cudaStream_t st) {
 }
 
 void LevelKernels::partition_count(const PartArgs& A, const PlanArgs& P, bool counted, unsigned groups,
-                                   cudaStream_t st) {
+                                   cudaStream_t st, const ShortList* sl) {
   if (counted) k_part_count<<<grid_count, kThreads, 0, st>>>(A, 1);
   else k_part_count_dense<<<grid_count_dense, kThreads, 0, st>>>(A);
   GBDT_LAUNCH_CHECK();
   count_launch();
+  if (sl && sl->n) {
+    k_short_count<<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);
+    GBDT_LAUNCH_CHECK();
+    count_launch();
+  }
   launch_scan<false>(A.t.tb.C, A.ccnt, A.sgrp, A.cpre, groups, st);
   const unsigned pg = (unsigned)std::max(1, std::min((P.m + kWarps) / kWarps, sms * 8));  // a warp per attribute
   k_plan_attr<<<pg, kThreads, 0, st>>>(P);
@@ -2635,7 +2891,15 @@ void launch_scatter(const LevelKernels& L, const PartArgs& A, cudaStream_t st) {
   else k_part_scatter<HM, kR, false><<<L.grid_scatter[HM][0], kThreads, 0, st>>>(A);
 }
 
-void LevelKernels::partition_scatter(const PartArgs& A, int hmode, const RunArgs* rle, cudaStream_t st) {
+void LevelKernels::partition_scatter(const PartArgs& A, int hmode, const RunArgs* rle, cudaStream_t st,
+                                     const ShortList* sl) {
+  if (sl && sl->n) {
+    if (hmode == 0) k_short_scatter<0><<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);
+    else if (hmode == 1) k_short_scatter<1><<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);
+    else k_short_scatter<2><<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);
+    GBDT_LAUNCH_CHECK();
+    count_launch();
+  }
   if (rle) {
     if (hmode == 0) launch_scatter<0, true>(*this, A, st);
     else if (hmode == 1) launch_scatter<1, true>(*this, A, st);
@@ -2652,6 +2916,22 @@ void LevelKernels::partition_scatter(const PartArgs& A, int hmode, const RunArgs
     if (hmode == 0) launch_scatter<0, false>(*this, A, st);
     else if (hmode == 1) launch_scatter<1, false>(*this, A, st);
     else launch_scatter<2, false>(*this, A, st);
+  }
+  GBDT_LAUNCH_CHECK();
+  count_launch();
+}
+
+void LevelKernels::short_split(const SplitArgs& A, const ShortList& S, int hmode, bool gather, cudaStream_t st) {
+  if (!S.n) return;
+  const unsigned g = grid_sl;
+  if (gather) {
+    if (hmode == 0) k_short_split<0, true><<<g, kThreads, 0, st>>>(A, S);
+    else if (hmode == 1) k_short_split<1, true><<<g, kThreads, 0, st>>>(A, S);
+    else k_short_split<2, true><<<g, kThreads, 0, st>>>(A, S);
+  } else {
+    if (hmode == 0) k_short_split<0, false><<<g, kThreads, 0, st>>>(A, S);
+    else if (hmode == 1) k_short_split<1, false><<<g, kThreads, 0, st>>>(A, S);
+    else k_short_split<2, false><<<g, kThreads, 0, st>>>(A, S);
   }
   GBDT_LAUNCH_CHECK();
   count_launch();

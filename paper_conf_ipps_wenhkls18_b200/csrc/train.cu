@@ -478,6 +478,12 @@ struct ShardWork {
   unsigned long long *pel = nullptr, *pgrp = nullptr;
   int32_t* mp1 = nullptr;
   unsigned pgroups = 1;
+  // short-attribute path (levels.cu k_short_*): the attributes, their flags, the chunk kernels'
+  // chunk lists of the root and of the two level tables
+  DBuf shortmem;
+  ShortList sl;
+  uint8_t* sflag = nullptr;
+  Tables root;  // the shard's root tables (+ the root chunk list on the short path)
 };
 
 // NVTX names of the phases (host-side ranges for nsys / ncu --nvtx; no-ops without a tool)
@@ -657,7 +663,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     const int64_t S = (int64_t)m * Kcap;
     const int64_t C0 = std::max(sh.C0, 1);
     // node-best records per level: one per CTA and node (K <= 32), else one per chunk and segment
-    const int64_t R = (int64_t)(LK.grid_fast[2][1] + LK.grid_fast[1][1] + LK.grid_fast[0][1] + LK.grid_gen + LK.grid_short) * 64 +
+    const int64_t R = (int64_t)(LK.grid_fast[2][1] + LK.grid_fast[1][1] + LK.grid_fast[0][1] + LK.grid_gen + LK.grid_short +
+                                LK.grid_sl) * 64 +
                       (int64_t)LK.grid_fused * 2 * kFusedMaxK + 2 * C0 + S + 64;
     auto sz = [&](Carve& q) {
       for (int b = 0; b < 2; ++b) {
@@ -757,6 +764,70 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       w.fplan[1] = f.take<FusedPlan>(1);
       w.tilemem = f.take<char>(tb);
     }
+    // Short path: sparse lists (missing values) kept as plain lists, attributes whose root list has
+    // at most short_max entries (GBDT_SHORT_MAX, default 32; GBDT_SHORT=0 turns the path off)
+    w.root = sh.root;
+    {
+      const char* se = getenv("GBDT_SHORT");
+      const char* sm = getenv("GBDT_SHORT_MAX");
+      const int64_t short_max = sm ? std::max(0, atoi(sm)) : 32;
+      const bool on = (se ? se[0] != '0' : true) && ds.has_missing && !sh.rle && !ds.dense && m > 0 && short_max > 0;
+      std::vector<int32_t> attrs;
+      if (on) {
+        // longest first (a counting sort by root length), so the warps' loads even out
+        std::vector<int64_t> bucket((size_t)short_max + 2, 0);
+        for (int a = 0; a < m; ++a) {
+          const int64_t L = sh.h_col_len[a];
+          if (L > 0 && L <= short_max) ++bucket[(size_t)(short_max - L)];
+        }
+        int64_t acc = 0;
+        for (auto& b : bucket) { const int64_t x = b; b = acc; acc += x; }
+        attrs.resize((size_t)acc);
+        for (int a = 0; a < m; ++a) {
+          const int64_t L = sh.h_col_len[a];
+          if (L > 0 && L <= short_max) attrs[(size_t)bucket[(size_t)(short_max - L)]++] = a;
+        }
+      }
+      if (!attrs.empty()) {
+        std::vector<uint8_t> flag((size_t)m, 0);
+        for (int32_t a : attrs) flag[(size_t)a] = 1;
+        std::vector<int32_t> lc;  // root chunks of the other attributes (chunk_start as build_layout)
+        lc.reserve((size_t)C0);
+        int32_t cs = 0;
+        for (int a = 0; a < m; ++a) {
+          const int32_t nc = (int32_t)ceil_div(sh.h_col_len[a], kChunk);
+          if (!flag[(size_t)a])
+            for (int32_t k = 0; k < nc; ++k) lc.push_back(cs + k);
+          cs += nc;
+        }
+        const int32_t nlc = (int32_t)lc.size();
+        Carve zp{nullptr};
+        auto zs = [&](Carve& z) {
+          z.take<int32_t>(attrs.size()); z.take<uint8_t>((size_t)m); z.take<int32_t>((size_t)C0); z.take<int32_t>(4);
+          z.take<int32_t>((size_t)C0); z.take<int32_t>((size_t)C0);
+        };
+        zs(zp);
+        w.shortmem.alloc(zp.off + 1024, st);
+        Carve z{w.shortmem.as<char>()};
+        int32_t* d_attrs = z.take<int32_t>(attrs.size());
+        w.sflag = z.take<uint8_t>((size_t)m);
+        int32_t* rlc = z.take<int32_t>((size_t)C0);
+        int32_t* nl = z.take<int32_t>(4);
+        w.tab[0].lc = z.take<int32_t>((size_t)C0);
+        w.tab[1].lc = z.take<int32_t>((size_t)C0);
+        w.root.lc = rlc;
+        w.root.nlc = nl;
+        w.tab[0].nlc = nl + 1;
+        w.tab[1].nlc = nl + 2;
+        GBDT_CUDA(cudaMemcpyAsync(d_attrs, attrs.data(), 4 * attrs.size(), cudaMemcpyHostToDevice, st));
+        GBDT_CUDA(cudaMemcpyAsync(w.sflag, flag.data(), (size_t)m, cudaMemcpyHostToDevice, st));
+        if (nlc) GBDT_CUDA(cudaMemcpyAsync(rlc, lc.data(), 4 * (size_t)nlc, cudaMemcpyHostToDevice, st));
+        GBDT_CUDA(cudaMemcpyAsync(nl, &nlc, 4, cudaMemcpyHostToDevice, st));
+        GBDT_CUDA(cudaStreamSynchronize(st));  // the host vectors must outlive the copies
+        w.sl.attrs = d_attrs;
+        w.sl.n = (int)attrs.size();
+      }
+    }
     w.nrec = nrec + li;
     w.gkey = gkey + (size_t)li * Kcap;
     w.tkey = tkey + (size_t)li * Kcap;
@@ -816,7 +887,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         model.captures.clear();
         for (int li = 0; li < nloc; ++li) {
           Shard& sh = *ds.shards[li];
-          const Tables tb = lvl == 0 ? sh.root : sw[li].tab[lvl & 1];
+          const Tables tb = lvl == 0 ? sw[li].root : sw[li].tab[lvl & 1];
           LevelCapture L;
           L.shard = sh.index;
           L.K = Kh;
@@ -871,11 +942,11 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         Shard& sh = *ds.shards[li];
         ShardWork& w = sw[li];
         if (sh.m == 0) continue;
-        const Tables tb = lvl == 0 ? sh.root : w.tab[lvl & 1];
+        const Tables tb = lvl == 0 ? w.root : w.tab[lvl & 1];
         const float* val = lvl == 0 ? sh.val0.as<float>() : sh.valw[lvl & 1].as<float>();
         const int32_t* ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
         SplitArgs A;
-        A.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters};
+        A.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters, w.sflag};
         A.desc = w.desc; A.rle = sh.rle ? 1 : 0; A.genlist = w.genlist; A.ngen = w.counters + 2;
         A.g = gv; A.h = hv; A.nodes = cur; A.segPG = w.segPG; A.segPH = w.segPH; A.lam = P.lambda;
         A.epochp = epoch; A.fx = fxs; A.rec = w.rec;
@@ -890,6 +961,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         kt.end();
 
         kt.begin(GBDT_PHASE_K_SPLIT);
+        LK.short_split(A, w.sl, hmode, /*gather=*/lvl == 0, st);
         LK.split_find(A, hmode, ds.has_missing, sh.rle, st);
         kt.end();
         if (P.profile) {  // the level's list entries (byte model of the bench), off the timed kernels
@@ -937,7 +1009,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
                      hbitF[(lvl - 1) & 1], bits, n, Kl, sms, st);
           continue;
         }
-        const Tables tb = lvl == 0 ? sh.root : sw[li].tab[lvl & 1];
+        const Tables tb = lvl == 0 ? sw[li].root : sw[li].tab[lvl & 1];
         const int32_t* ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
         dim3 grid((unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256 * (int64_t)Kl), (int64_t)sms * 4)), (unsigned)Kl);
         k_mark<<<grid, 256, 0, st>>>(cur.K, cidx, winner, sh.index, sh.a_begin, tb, ins, bits);
@@ -997,7 +1069,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         Shard& sh = *ds.shards[li];
         ShardWork& w = sw[li];
         if (sh.m == 0) continue;
-        const Tables tb = lvl == 0 ? sh.root : w.tab[lvl & 1];
+        const Tables tb = lvl == 0 ? w.root : w.tab[lvl & 1];
         const Tables tn = w.tab[(lvl + 1) & 1];
         const float* val = lvl == 0 ? sh.val0.as<float>() : sh.valw[lvl & 1].as<float>();
         const int32_t* ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
@@ -1007,7 +1079,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
           GBDT_CUDA(cudaMemsetAsync(w.segL, 0, Sl * 4, st));
         }
         PartArgs PA;
-        PA.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters + 1};
+        PA.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters + 1, w.sflag};
         PA.side = side; PA.hbit = hbit; PA.cidx = cidx; PA.slist = w.slist; PA.segH = w.segH; PA.segL = w.segL;
         PA.seg_pre = w.seg_pre; PA.out_hi = w.out_hi; PA.out_lo = w.out_lo;
         PA.val_out = sh.valw[(lvl + 1) & 1].as<float>();
@@ -1024,7 +1096,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         PL.m = sh.m; PL.counted = ds.has_missing; PL.Kp = cur.K; PL.Knp = nxt.K; PL.cidx = cidx; PL.ncnt = nxt.cnt;
         PL.segH = w.segH; PL.segL = w.segL; PL.seg_pre = w.seg_pre;
         PL.out_hi = w.out_hi; PL.out_lo = w.out_lo; PL.len_tmp = w.len_tmp; PL.nxt = tn;
-        PL.el = w.pel; PL.egrp = w.pgrp; PL.egroups = w.pgroups; PL.mp1 = w.mp1;
+        PL.el = w.pel; PL.egrp = w.pgrp; PL.egroups = w.pgroups; PL.mp1 = w.mp1; PL.sflag = w.sflag;
         RunArgs RA;
         if (sh.rle) {
           RA.m = sh.m; RA.Kp = cur.K; RA.Knp = nxt.K; RA.cidx = cidx; RA.cur = tb; RA.nxt = tn;
@@ -1039,12 +1111,12 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
           PA.t.val = sh.valw[lvl & 1].as<float>();
         }
         kt.begin(GBDT_PHASE_K_COUNT);
-        LK.partition_count(PA, PL, ds.has_missing, w.groups, st);
+        LK.partition_count(PA, PL, ds.has_missing, w.groups, st, &w.sl);
         kt.end();
         kt.begin(GBDT_PHASE_K_SCATTER);
         if (PA.cagg_next)
           GBDT_CUDA(cudaMemsetAsync(w.cagg, 0, sizeof(unsigned long long) * 5 * (size_t)std::max<int64_t>(sh.C0, 1), st));
-        LK.partition_scatter(PA, hmode, (sh.rle && !dec) ? &RA : nullptr, st);
+        LK.partition_scatter(PA, hmode, (sh.rle && !dec) ? &RA : nullptr, st, &w.sl);
         if (dec)
           LK.rle_encode(tn, sh.m, nxt.K, sh.valw[(lvl + 1) & 1].as<float>(), w.enc_cnt, w.enc_bits,
                         ((size_t)sh.cap / 32 + 2) * 4, st);

@@ -202,7 +202,8 @@ def test_deterministic_across_runs():
 # The RLE path reads values from the runs and splits the runs themselves (no decompression in HBM);
 # it sees the same entry streams, so its trees and margins must be bit-identical to the plain
 # level-by-level path (GBDT_FUSED=0: dense data otherwise takes the fused pass of fused.cu, whose
-# sums associate differently), and both match the oracle.
+# sums associate differently; GBDT_SHORT=0: the same for the short-list path), and both match the
+# oracle.
 @pytest.mark.parametrize("maker", [
     lambda: synth.c5(n=40000, T=3),
     lambda: synth.table1(),
@@ -214,6 +215,9 @@ def test_deterministic_across_runs():
 def test_rle_direct_split_bit_identical(maker, monkeypatch):
     p = maker()
     monkeypatch.setenv("GBDT_FUSED", "0")
+    # plain lists route short sparse attributes through the short path (levels.cu k_short_*), whose
+    # prefix sums associate in list order; the RLE path keeps the chunk kernels throughout
+    monkeypatch.setenv("GBDT_SHORT", "0")
     ref_model, ref_margin = _train(p)
     model, margin = _train(p, rle="on")
     assert np.array_equal(model.nodes().view(np.uint8), ref_model.nodes().view(np.uint8))
