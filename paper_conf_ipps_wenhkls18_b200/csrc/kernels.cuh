@@ -26,12 +26,16 @@ struct TileArgs {
   const uint8_t* sflag = nullptr;  // [m] 1: attribute on the short path (k_short_*); nullptr: none
 };
 
-// Attributes whose whole root list has at most a few dozen entries (the typical sparse attribute,
-// P:214-216) take the short path at every level with K <= 32: one LANE per (attribute, node)
-// segment walks the segment's entries in list order (levels.cu k_short_split / _count / _scatter).
+// Attributes whose whole root list has at most 32 entries (the typical sparse attribute)
+// take the short path at levels 0-5 (K <= 32): a lane per list entry, 32/W lists per warp
+// (levels.cu k_short_split / _count / _scatter).
 struct ShortList {
-  const int32_t* attrs = nullptr;  // shard-local ids, longest root list first (load balance)
+  const int32_t* attrs = nullptr;  // shard-local ids, longest root list first
   int n = 0;
+  const int2* batch = nullptr;     // warp batches: (first index into attrs, count | log2 W << 16)
+  int nb = 0;
+  const uint8_t* jl = nullptr;     // per list entry: its node j at this level (nullptr: root, j = 0)
+  uint8_t* jl_out = nullptr;       // the next level's, written by the scatter (nullptr: not needed)
 };
 
 

@@ -1297,21 +1297,48 @@ __global__ void __launch_bounds__(kThreads) k_sf_short(SplitArgs A) {
 
 // ---------------------------------------------------------------------------- short attributes
 // The typical attribute of a sparse data set has a handful of entries ("many small
-// segments"; C4a: 1.08 M of its 1.13 M non-empty lists hold <= 32), so a warp per 256-entry chunk
-// spends ~500 instructions per list on shuffles and table walks whatever its length.  These
-// attributes (ShortList, fixed at the root: lists only shrink) take a path of their own at every
-// level with K <= 32: a group of Kp lanes per attribute (Kp = K rounded up to a power of two; 32/Kp
-// attributes per warp), lane j of the group on segment (a, j), walking the segment's entries in list
-// order.  Segments are contiguous and node-ordered, so the segment's present totals, its
-// prefix sums and run ends need no cross-lane step at all; the chunk kernels skip these
-// attributes (Tables::lc) and the exact chunk scans are not involved (a whole list is one piece).
-// Candidates, their order and the record semantics are k_sf_short's: a run end (the next value
-// differs, or the segment's last entry), missing -> right before missing -> left, earliest entry
-// on equal scores; the segment's winner gets its Eq. 2 gain with IEEE divisions.
-__device__ __forceinline__ int short_group(int K) {  // K <= 32
-  int G = 1;
-  while (G < K) G <<= 1;
-  return G;
+// segments"; C4a: 1.08 M of its 1.13 M non-empty lists hold <= 32, 0.78 M of them <= 4), so a warp
+// per chunk spends ~500 instructions and several dependent table walks per list whatever its
+// length.  These attributes (ShortList, fixed at the root: lists only shrink) take a path of their
+// own at levels 0-5 (K <= 32): a warp takes a BATCH of 32/W attributes of similar root length (W =
+// the batch's longest root list rounded up to a power of two), a group of W lanes per attribute,
+// lane e on entry e of the list.  The entry's node j comes from a byte list carried with the
+// entries (ShortList::jl, written by the scatter), so segment heads and ends are lane compares and
+// no segment table is walked; the attribute's list start and length are the only table reads.
+// The arithmetic is k_sf_short's over a chunk that is the whole list (and agg_short's for the
+// present totals), in the same association, so trees are bit-identical to the chunk kernels'.
+struct SLane {
+  int a;        // attribute (-1: none)
+  long long p;  // list position of the lane's entry
+  bool valid;
+  int j;        // node of the entry
+  int hs, se;   // first / last lane of the entry's segment
+  int lw;       // log2 W
+  unsigned hm;  // segment heads of the warp
+  unsigned gm;  // the lane's group
+  long long p0; // list start of the lane's attribute
+};
+__device__ __forceinline__ SLane short_lane(const ShortList& S, const Tables& tb, int bi, int lane) {
+  const int2 b = S.batch[bi];
+  SLane L;
+  L.lw = b.y >> 16;
+  const int W = 1 << L.lw, sub = lane >> L.lw, e = lane & (W - 1);
+  L.gm = W == 32 ? 0xffffffffu : ((1u << W) - 1u) << (sub * W);
+  L.a = sub < (b.y & 0xffff) ? S.attrs[b.x + sub] : -1;
+  long long len = 0;
+  L.p0 = 0;
+  if (L.a >= 0) { L.p0 = tb.col_start[L.a]; len = tb.col_len[L.a]; }
+  L.valid = e < len;
+  L.p = L.p0 + e;
+  L.j = (L.valid && S.jl) ? (int)S.jl[L.p] : 0;
+  const int jp = __shfl_up_sync(0xffffffffu, L.j, 1);
+  L.hm = __ballot_sync(0xffffffffu, L.valid && (e == 0 || jp != L.j));
+  const unsigned vm = __ballot_sync(0xffffffffu, L.valid) & L.gm;
+  const unsigned le = lane == 31 ? 0xffffffffu : (2u << lane) - 1u;  // lanes <= lane
+  const unsigned hb = L.hm & le, nh = L.hm & ~le & L.gm;
+  L.hs = hb ? 31 - __clz(hb) : lane;
+  L.se = nh ? __ffs(nh) - 2 : (vm ? 31 - __clz(vm) : lane);
+  return L;
 }
 
 template <int HMODE, bool kGather>
@@ -1322,121 +1349,110 @@ __global__ void __launch_bounds__(kThreads) k_short_split(SplitArgs A, ShortList
   __shared__ Rec wrec[kWarps][kWarpK];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int K = *A.t.Kp;
-  if (K == 0 || K > kWarpK || S.n == 0) return;
+  if (K == 0 || K > kWarpK || S.nb == 0) return;
   const int epoch = *A.epochp;
   const double lam = A.lam;
   nb_init(B, A, K);
   for (int j = threadIdx.x; j < kWarps * kWarpK; j += blockDim.x) wgk[j / kWarpK][j % kWarpK] = 0ull;
   __syncthreads();
   const unsigned long long pol_keep = policy_evict_last();
-  const int Kp = short_group(K), G = 32 / Kp, sub = lane / Kp, j = lane % Kp;
-  const NodeV nv = j < K ? node_v(B, A, K, j) : NodeV{0.0, 0.0, 0.0, 0};
   const int nw = (gridDim.x * blockDim.x) >> 5;
-  for (int i0 = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * G; i0 < S.n; i0 += nw * G) {
-    const int i = i0 + sub;
-    const int a = (i < S.n && j < K) ? S.attrs[i] : -1;
-    long long s0 = 0;
-    int cnt = 0;
-    if (a >= 0) {
-      const long long sI = (long long)a * K + j;
-      s0 = A.t.tb.seg_start[sI];
-      cnt = (int)A.t.tb.seg_cnt[sI];
+  for (int bi = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; bi < S.nb; bi += nw) {
+    const SLane L = short_lane(S, A.t.tb, bi, lane);
+    const int W = 1 << L.lw;
+    float v = 0.f;
+    double g = 0.0, h = 0.0;
+    if (L.valid) {
+      v = __ldcs(A.t.val + L.p);
+      if (kGather) {
+        const int id = __ldcs(A.t.ins + L.p);
+        g = ld_keep(A.g + id, pol_keep);
+        h = kH ? ld_keep(A.h + id, pol_keep) : hess_of<HMODE>(g);
+        __stcs(A.glist + L.p, g);
+        if (kH) __stcs(A.hlist + L.p, h);
+      } else {
+        g = __ldcs(A.glist + L.p);
+        h = kH ? __ldcs(A.hlist + L.p) : hess_of<HMODE>(g);
+      }
     }
+    // segmented inclusive scan (k_sf_short's association)
+    double ig = g, ih = h;
+    for (int o = 1; o < W; o <<= 1) {
+      const double yg = __shfl_up_sync(0xffffffffu, ig, o), yh = __shfl_up_sync(0xffffffffu, ih, o);
+      if (lane - o >= L.hs) { ig = yg + ig; ih = yh + ih; }
+    }
+    const int icn = lane - L.hs + 1, cseg = L.se - L.hs + 1;
+    // present totals of the segment (agg_short's association: a butterfly when the list is one
+    // segment, else the scan at the segment's last entry)
+    const bool one = __popc(L.hm & L.gm) == 1;
+    double tg = g, th = h;
+    for (int o = W >> 1; o; o >>= 1) {
+      tg = tg + __shfl_xor_sync(0xffffffffu, tg, o);
+      th = th + __shfl_xor_sync(0xffffffffu, th, o);
+    }
+    const double sg = __shfl_sync(0xffffffffu, ig, L.se), sh = __shfl_sync(0xffffffffu, ih, L.se);
+    const double PG = one ? tg : sg, PH = one ? th : sh;
+    const float vn = __shfl_down_sync(0xffffffffu, v, 1);
+    const bool seg_last = L.valid && lane == L.se;
+    const bool cand = L.valid && (seg_last || vn != v);
+    const NodeV nv = node_v(B, A, K, L.j);
+    double best = -INFINITY;
+    int bd = 0;
     bool ok = false;
-    double best = 0.0, bg = 0.0, bh = 0.0, PG = 0.0, PH = 0.0;
-    int be = 0, bd = 0, bc = 0;
-    float bv = 0.f;
-    const int cM = nv.C - cnt;  // the node's instances missing from this attribute
-    if (cnt > 0) {
-      // pass 1: present totals of the segment (root: the g-list gathered on the way)
-      if (kGather || cM > 0) {
-        for (int e = 0; e < cnt; ++e) {
-          const long long p = s0 + e;
-          double g, h;
-          if (kGather) {
-            const int id = __ldg(A.t.ins + p);
-            g = ld_keep(A.g + id, pol_keep);
-            h = kH ? ld_keep(A.h + id, pol_keep) : hess_of<HMODE>(g);
-            A.glist[p] = g;
-            if (kH) A.hlist[p] = h;
-          } else {
-            g = A.glist[p];
-            h = kH ? A.hlist[p] : hess_of<HMODE>(g);
-          }
-          PG = PG + g;
-          PH = PH + h;
-        }
-      }
-      // pass 2: prefix sums in list order, candidates at run ends
-      double ig = 0.0, ih = 0.0;
-      float v = A.t.val[s0];
-#pragma unroll 2
-      for (int e = 0; e < cnt; ++e) {
-        const long long p = s0 + e;
-        const bool last = e + 1 == cnt;
-        const float vn = last ? v : A.t.val[p + 1];
-        const double g = A.glist[p];
-        const double h = kH ? A.hlist[p] : hess_of<HMODE>(g);
-        ig = ig + g;
-        ih = ih + h;
-        const int icn = e + 1;
-        if (last || vn != v) {
-          if (nv.C - icn >= 1) {
-            const double sc = split_score(ig, ih, nv.G, nv.H, lam);
-            if (!ok || sc > best) { best = sc; ok = true; bd = 0; be = e; bg = ig; bh = ih; bc = icn; bv = v; }
-          }
-          if (cM > 0 && nv.C - (icn + cM) >= 1) {
-            const double s1 = split_score(ig + (nv.G - PG), ih + (nv.H - PH), nv.G, nv.H, lam);
-            if (!ok || s1 > best) { best = s1; ok = true; bd = 1; be = e; bg = ig; bh = ih; bc = icn; bv = v; }
-          }
-        }
-        v = vn;
+    if (cand) {
+      if (icn >= 1 && nv.C - icn >= 1) { best = split_score(ig, ih, nv.G, nv.H, lam); ok = true; }
+      const int cM = nv.C - cseg;
+      const int cL1 = icn + cM;
+      if (cM > 0 && cL1 >= 1 && nv.C - cL1 >= 1) {
+        const double g1 = split_score(ig + (nv.G - PG), ih + (nv.H - PH), nv.G, nv.H, lam);
+        if (!ok || g1 > best) { best = g1; bd = 1; ok = true; }
       }
     }
-    // the segment's record; then the best per node over the warp's attributes (lanes j, j + Kp, ...)
+    // per-segment argmax, earlier lane (larger value, R12) on equal scores
+    double lg = ok ? best : -INFINITY;
+    int lq = ok ? lane : INT_MAX;
+    for (int o = 1; o < W; o <<= 1) {
+      const double yg = __shfl_up_sync(0xffffffffu, lg, o);
+      const int yq = __shfl_up_sync(0xffffffffu, lq, o);
+      if (lane - o >= L.hs && (yg > lg || (yg == lg && yq < lq))) { lg = yg; lq = yq; }
+    }
+    const bool post = seg_last && lq != INT_MAX;
+    const int q = post ? lq : lane;
+    const double wg = __shfl_sync(0xffffffffu, ig, q), wh = __shfl_sync(0xffffffffu, ih, q);
+    const int wd = __shfl_sync(0xffffffffu, bd, q);
+    const float wv = __shfl_sync(0xffffffffu, v, q);
     Rec r;
-    unsigned long long gk = 0ull, tk = ~0ull;
-    if (ok) {
-      r.value = bv;
-      r.attr = A.t.a_base + a;
-      r.dir = bd;
-      r.node = j;
+    unsigned long long gk = 0ull;
+    if (post) {
+      const int wc = q - L.hs + 1;
+      r.value = wv;
+      r.attr = A.t.a_base + L.a;
+      r.dir = wd;
+      r.node = L.j;
       r.epoch = epoch;
       r.shard = A.shard;
-      r.pos = s0 + be;
-      if (bd) {
-        r.GL = bg + (nv.G - PG);
-        r.HL = bh + (nv.H - PH);
-        r.cntL = bc + cM;
+      r.pos = L.p + (q - lane);
+      if (wd) {
+        r.GL = wg + (nv.G - PG);
+        r.HL = wh + (nv.H - PH);
+        r.cntL = wc + (nv.C - cseg);
       } else {
-        r.GL = bg; r.HL = bh; r.cntL = bc;
+        r.GL = wg; r.HL = wh; r.cntL = wc;
       }
       r.gain = eq2_gain(r.GL, r.HL, nv.G, nv.H, lam, nv.P);
       gk = gain_key(r.gain);
-      tk = tie_key(r.attr, r.value, r.dir);
     }
-    int src = lane;
-    for (int o = Kp; o < 32; o <<= 1) {
-      const unsigned long long og = __shfl_xor_sync(0xffffffffu, gk, o), ot = __shfl_xor_sync(0xffffffffu, tk, o);
-      const int os = __shfl_xor_sync(0xffffffffu, src, o);
-      if (og > gk || (og == gk && ot < tk)) { gk = og; tk = ot; src = os; }
-    }
-    if (!__any_sync(0xffffffffu, gk != 0ull)) continue;
-    Rec w;
-    w.gain = __shfl_sync(0xffffffffu, r.gain, src);
-    w.GL = __shfl_sync(0xffffffffu, r.GL, src);
-    w.HL = __shfl_sync(0xffffffffu, r.HL, src);
-    w.cntL = __shfl_sync(0xffffffffu, r.cntL, src);
-    w.pos = __shfl_sync(0xffffffffu, r.pos, src);
-    w.value = __shfl_sync(0xffffffffu, r.value, src);
-    w.attr = __shfl_sync(0xffffffffu, r.attr, src);
-    w.dir = __shfl_sync(0xffffffffu, r.dir, src);
-    w.node = j;
-    w.epoch = epoch;
-    w.shard = A.shard;
-    if (sub == 0 && gk != 0ull && j < K && rec_better(gk, w, wgk[wid][j], wrec[wid][j])) {
-      wgk[wid][j] = gk;
-      wrec[wid][j] = w;
+    // the warp's node table, one group at a time (the segments of one list are distinct nodes)
+    unsigned pm = __ballot_sync(0xffffffffu, post);
+    while (pm) {
+      const int g0 = (__ffs(pm) - 1) >> L.lw;
+      const unsigned gmask = W == 32 ? 0xffffffffu : ((1u << W) - 1u) << (g0 * W);
+      if (post && (lane >> L.lw) == g0 && rec_better(gk, r, wgk[wid][L.j], wrec[wid][L.j])) {
+        wgk[wid][L.j] = gk;
+        wrec[wid][L.j] = r;
+      }
+      pm &= ~gmask;
+      __syncwarp();
     }
   }
   __syncthreads();  // merge the warp tables, one record per node and CTA
@@ -1452,69 +1468,71 @@ __global__ void __launch_bounds__(kThreads) k_short_split(SplitArgs A, ShortList
   }
 }
 
-// Partition count of the short-path segments: a lane per segment counts its entries per side
-// (segH / segL of the plan; the chunk kernels' slist is not needed, the scatter gathers again)
+// Partition count of the short lists: per segment, its entries of each side (segH / segL of the
+// plan) by ballots over the segment's lanes
 __global__ void __launch_bounds__(kThreads) k_short_count(PartArgs A, ShortList S) {
   const int K = *A.t.Kp;
-  if (K == 0 || K > kWarpK || S.n == 0) return;
+  if (K == 0 || K > kWarpK || S.nb == 0) return;
   const int lane = threadIdx.x & 31;
-  const int Kp = short_group(K), G = 32 / Kp, sub = lane / Kp, j = lane % Kp;
   const int nw = (gridDim.x * blockDim.x) >> 5;
-  for (int i0 = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * G; i0 < S.n; i0 += nw * G) {
-    const int i = i0 + sub;
-    if (i >= S.n || j >= K) continue;
-    const long long sI = (long long)S.attrs[i] * K + j;
-    const int cnt = (int)A.t.tb.seg_cnt[sI];
-    if (cnt == 0 || A.cidx[j] < 0) continue;  // a new leaf drops its entries
-    const long long s0 = A.t.tb.seg_start[sI];
-    int hi = 0, lo = 0;
-#pragma unroll 4
-    for (int e = 0; e < cnt; ++e) {
-      const uint8_t sd = __ldg(A.side + __ldg(A.t.ins + s0 + e));
-      hi += sd == 1;
-      lo += sd == 2;
+  for (int bi = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; bi < S.nb; bi += nw) {
+    const SLane L = short_lane(S, A.t.tb, bi, lane);
+    const uint8_t sd = L.valid ? __ldg(A.side + __ldcs(A.t.ins + L.p)) : 0;
+    const unsigned bh = __ballot_sync(0xffffffffu, sd == 1), bl = __ballot_sync(0xffffffffu, sd == 2);
+    if (L.valid && lane == L.se) {
+      const unsigned m = (L.se == 31 ? 0xffffffffu : (2u << L.se) - 1u) & ~((1u << L.hs) - 1u);
+      const long long s = (long long)L.a * K + L.j;
+      A.segH[s] = __popc(bh & m);
+      A.segL[s] = __popc(bl & m);
     }
-    A.segH[sI] = hi;
-    A.segL[sI] = lo;
   }
 }
 
-// Stable scatter of the short-path segments: the lane walks its segment in list order,
-// so each child's entries keep their order; destinations from the plan (out_hi / out_lo)
+// Stable scatter of the short lists: rank among the segment's same-side entries by
+// ballot; the entries' next-level node index goes with them (ShortList::jl_out)
 template <int HMODE>
 __global__ void __launch_bounds__(kThreads) k_short_scatter(PartArgs A, ShortList S) {
   constexpr bool kH = HMODE == kHGather;
   const int K = *A.t.Kp;
-  if (K == 0 || K > kWarpK || S.n == 0) return;
+  if (K == 0 || K > kWarpK || S.nb == 0) return;
   const int lane = threadIdx.x & 31;
-  const int Kp = short_group(K), G = 32 / Kp, sub = lane / Kp, j = lane % Kp;
   const int nw = (gridDim.x * blockDim.x) >> 5;
-  for (int i0 = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * G; i0 < S.n; i0 += nw * G) {
-    const int i = i0 + sub;
-    if (i >= S.n || j >= K) continue;
-    const long long sI = (long long)S.attrs[i] * K + j;
-    const int cnt = (int)A.t.tb.seg_cnt[sI];
-    if (cnt == 0 || A.cidx[j] < 0) continue;
-    const long long s0 = A.t.tb.seg_start[sI];
-    long long dh = A.out_hi[sI], dl = A.out_lo[sI];
-#pragma unroll 4
-    for (int e = 0; e < cnt; ++e) {
-      const long long p = s0 + e;
-      const int id = __ldg(A.t.ins + p);
-      const uint8_t sd = __ldg(A.side + id);
-      if (!sd) continue;
-      const long long d = sd == 1 ? dh++ : dl++;
-      A.val_out[d] = A.t.val[p];
-      A.ins_out[d] = id;
-      A.g_out[d] = A.g_in[p];
-      if (kH) A.h_out[d] = A.h_in[p];
+  for (int bi = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; bi < S.nb; bi += nw) {
+    const SLane L = short_lane(S, A.t.tb, bi, lane);
+    int id = 0;
+    uint8_t sd = 0;
+    if (L.valid) {
+      id = __ldcs(A.t.ins + L.p);
+      sd = __ldg(A.side + id);
+    }
+    const unsigned bh = __ballot_sync(0xffffffffu, sd == 1), bl = __ballot_sync(0xffffffffu, sd == 2);
+    if (sd) {
+      const bool hi = sd == 1;
+      const unsigned below = ((1u << lane) - 1u) & ~((1u << L.hs) - 1u);
+      const int rk = __popc((hi ? bh : bl) & below);
+      const long long s = (long long)L.a * K + L.j;
+      const long long d = (hi ? A.out_hi[s] : A.out_lo[s]) + rk;
+      __stcs(A.val_out + d, __ldcs(A.t.val + L.p));
+      __stcs(A.ins_out + d, id);
+      __stcs(A.g_out + d, __ldcs(A.g_in + L.p));
+      if (kH) __stcs(A.h_out + d, __ldcs(A.h_in + L.p));
+      if (S.jl_out) {
+        const int c = A.cidx[L.j];
+        S.jl_out[d] = (uint8_t)(hi ? c : c + 1);
+      }
     }
   }
 }
 
 // ---------------------------------------------------------------------------- k_sf_gen
+#ifndef GBDT_GEN_CTAS
+#define GBDT_GEN_CTAS 2
+#endif
+#ifndef GBDT_GEN_DYN
+#define GBDT_GEN_DYN 0  // dynamic claim of the chunk steps (missing values)
+#endif
 template <int HMODE, bool kMissing, bool kTotals, bool kRLE>
-__global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
+__global__ void __launch_bounds__(kThreads, GBDT_GEN_CTAS) k_sf_gen(SplitArgs A) {
   constexpr bool kH = HMODE == kHGather;
   __shared__ NodeBest B;
   __shared__ unsigned char flg[kWarps][kChunk];
@@ -1543,7 +1561,13 @@ __global__ void __launch_bounds__(kThreads, 2) k_sf_gen(SplitArgs A) {
   // segment-crossing chunks of dense data, stays one chunk per warp)
   const int bw = n >= 32 * nw ? 32 : 1;
   const int nbat = (n + bw - 1) / bw;
-  for (int bt = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; bt < nbat; bt += nw) {
+  constexpr bool kDyn = GBDT_GEN_DYN && kMissing && !kTotals;
+  auto claim = [&]() {
+    int x = 0;
+    if (lane == 0) x = atomicAdd(A.t.counter, 1);
+    return __shfl_sync(0xffffffffu, x, 0);
+  };
+  for (int bt = kDyn ? claim() : (blockIdx.x * blockDim.x + threadIdx.x) >> 5; bt < nbat; bt = kDyn ? claim() : bt + nw) {
     const int ii = bt + lane * nbat;
     int cc = 0;
     bool take = false;
@@ -2870,7 +2894,7 @@ void LevelKernels::partition_count(const PartArgs& A, const PlanArgs& P, bool co
   else k_part_count_dense<<<grid_count_dense, kThreads, 0, st>>>(A);
   GBDT_LAUNCH_CHECK();
   count_launch();
-  if (sl && sl->n) {
+  if (sl && sl->nb) {
     k_short_count<<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);
     GBDT_LAUNCH_CHECK();
     count_launch();
@@ -2893,7 +2917,7 @@ void launch_scatter(const LevelKernels& L, const PartArgs& A, cudaStream_t st) {
 
 void LevelKernels::partition_scatter(const PartArgs& A, int hmode, const RunArgs* rle, cudaStream_t st,
                                      const ShortList* sl) {
-  if (sl && sl->n) {
+  if (sl && sl->nb) {
     if (hmode == 0) k_short_scatter<0><<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);
     else if (hmode == 1) k_short_scatter<1><<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);
     else k_short_scatter<2><<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);
@@ -2922,7 +2946,7 @@ void LevelKernels::partition_scatter(const PartArgs& A, int hmode, const RunArgs
 }
 
 void LevelKernels::short_split(const SplitArgs& A, const ShortList& S, int hmode, bool gather, cudaStream_t st) {
-  if (!S.n) return;
+  if (!S.nb) return;
   const unsigned g = grid_sl;
   if (gather) {
     if (hmode == 0) k_short_split<0, true><<<g, kThreads, 0, st>>>(A, S);

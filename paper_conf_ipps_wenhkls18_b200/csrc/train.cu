@@ -440,6 +440,8 @@ struct Carve {
   }
 };
 
+constexpr int kShortLevels = 6;  // levels with K <= 32 (2^5): the short path's node tables
+
 struct ShardWork {
   DBuf mem;
   Tables tab[2];
@@ -483,6 +485,16 @@ struct ShardWork {
   DBuf shortmem;
   ShortList sl;
   uint8_t* sflag = nullptr;
+  uint8_t* jl[2] = {nullptr, nullptr};  // node index of each short-list entry, two levels
+  // the level's short-path arguments (levels 0..kShortLevels-1, where K <= 32), else none
+  ShortList level_sl(int lvl) const {
+    ShortList r = sl;
+    if (lvl >= kShortLevels) { r.n = 0; r.nb = 0; return r; }
+    r.jl = lvl == 0 ? nullptr : jl[lvl & 1];
+    r.jl_out = lvl + 1 < kShortLevels ? jl[(lvl + 1) & 1] : nullptr;
+    return r;
+  }
+  const uint8_t* level_flag(int lvl) const { return (sl.nb && lvl < kShortLevels) ? sflag : nullptr; }
   Tables root;  // the shard's root tables (+ the root chunk list on the short path)
 };
 
@@ -764,14 +776,13 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       w.fplan[1] = f.take<FusedPlan>(1);
       w.tilemem = f.take<char>(tb);
     }
-    // Short path: sparse lists (missing values) kept as plain lists, attributes whose root list has
-    // at most short_max entries (GBDT_SHORT_MAX, default 32; GBDT_SHORT=0 turns the path off)
+    // Short path (levels.cu k_short_*): sparse lists (missing values) kept as plain lists, the
+    // attributes whose root list has at most 32 entries (GBDT_SHORT=0 turns the path off)
     w.root = sh.root;
     {
       const char* se = getenv("GBDT_SHORT");
-      const char* sm = getenv("GBDT_SHORT_MAX");
-      const int64_t short_max = sm ? std::max(0, atoi(sm)) : 32;
-      const bool on = (se ? se[0] != '0' : true) && ds.has_missing && !sh.rle && !ds.dense && m > 0 && short_max > 0;
+      const int64_t short_max = 32;
+      const bool on = (se ? se[0] != '0' : true) && ds.has_missing && !sh.rle && !ds.dense && m > 0;
       std::vector<int32_t> attrs;
       if (on) {
         // longest first (a counting sort by root length), so the warps' loads even out
@@ -801,10 +812,21 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
           cs += nc;
         }
         const int32_t nlc = (int32_t)lc.size();
+        // warp batches: 32/W lists of root length <= W (W a power of two), longest first
+        std::vector<int2> batch;
+        for (size_t i = 0; i < attrs.size();) {
+          const int64_t L = sh.h_col_len[(size_t)attrs[i]];
+          int lw = 0;
+          while ((1 << lw) < L) ++lw;
+          const int cnt = (int)std::min<size_t>((size_t)(32 >> lw), attrs.size() - i);
+          batch.push_back(make_int2((int)i, cnt | (lw << 16)));
+          i += (size_t)cnt;
+        }
         Carve zp{nullptr};
         auto zs = [&](Carve& z) {
           z.take<int32_t>(attrs.size()); z.take<uint8_t>((size_t)m); z.take<int32_t>((size_t)C0); z.take<int32_t>(4);
-          z.take<int32_t>((size_t)C0); z.take<int32_t>((size_t)C0);
+          z.take<int32_t>((size_t)C0); z.take<int32_t>((size_t)C0); z.take<int2>(batch.size());
+          z.take<uint8_t>((size_t)sh.cap); z.take<uint8_t>((size_t)sh.cap);
         };
         zs(zp);
         w.shortmem.alloc(zp.off + 1024, st);
@@ -815,6 +837,9 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         int32_t* nl = z.take<int32_t>(4);
         w.tab[0].lc = z.take<int32_t>((size_t)C0);
         w.tab[1].lc = z.take<int32_t>((size_t)C0);
+        int2* d_batch = z.take<int2>(batch.size());
+        w.jl[0] = z.take<uint8_t>((size_t)sh.cap);
+        w.jl[1] = z.take<uint8_t>((size_t)sh.cap);
         w.root.lc = rlc;
         w.root.nlc = nl;
         w.tab[0].nlc = nl + 1;
@@ -823,9 +848,12 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         GBDT_CUDA(cudaMemcpyAsync(w.sflag, flag.data(), (size_t)m, cudaMemcpyHostToDevice, st));
         if (nlc) GBDT_CUDA(cudaMemcpyAsync(rlc, lc.data(), 4 * (size_t)nlc, cudaMemcpyHostToDevice, st));
         GBDT_CUDA(cudaMemcpyAsync(nl, &nlc, 4, cudaMemcpyHostToDevice, st));
+        GBDT_CUDA(cudaMemcpyAsync(d_batch, batch.data(), sizeof(int2) * batch.size(), cudaMemcpyHostToDevice, st));
         GBDT_CUDA(cudaStreamSynchronize(st));  // the host vectors must outlive the copies
         w.sl.attrs = d_attrs;
         w.sl.n = (int)attrs.size();
+        w.sl.batch = d_batch;
+        w.sl.nb = (int)batch.size();
       }
     }
     w.nrec = nrec + li;
@@ -946,7 +974,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         const float* val = lvl == 0 ? sh.val0.as<float>() : sh.valw[lvl & 1].as<float>();
         const int32_t* ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
         SplitArgs A;
-        A.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters, w.sflag};
+        A.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters, w.level_flag(lvl)};
         A.desc = w.desc; A.rle = sh.rle ? 1 : 0; A.genlist = w.genlist; A.ngen = w.counters + 2;
         A.g = gv; A.h = hv; A.nodes = cur; A.segPG = w.segPG; A.segPH = w.segPH; A.lam = P.lambda;
         A.epochp = epoch; A.fx = fxs; A.rec = w.rec;
@@ -961,7 +989,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         kt.end();
 
         kt.begin(GBDT_PHASE_K_SPLIT);
-        LK.short_split(A, w.sl, hmode, /*gather=*/lvl == 0, st);
+        LK.short_split(A, w.level_sl(lvl), hmode, /*gather=*/lvl == 0, st);
         LK.split_find(A, hmode, ds.has_missing, sh.rle, st);
         kt.end();
         if (P.profile) {  // the level's list entries (byte model of the bench), off the timed kernels
@@ -1079,7 +1107,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
           GBDT_CUDA(cudaMemsetAsync(w.segL, 0, Sl * 4, st));
         }
         PartArgs PA;
-        PA.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters + 1, w.sflag};
+        PA.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters + 1, w.level_flag(lvl)};
+        const ShortList lsl = w.level_sl(lvl);
         PA.side = side; PA.hbit = hbit; PA.cidx = cidx; PA.slist = w.slist; PA.segH = w.segH; PA.segL = w.segL;
         PA.seg_pre = w.seg_pre; PA.out_hi = w.out_hi; PA.out_lo = w.out_lo;
         PA.val_out = sh.valw[(lvl + 1) & 1].as<float>();
@@ -1096,7 +1125,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         PL.m = sh.m; PL.counted = ds.has_missing; PL.Kp = cur.K; PL.Knp = nxt.K; PL.cidx = cidx; PL.ncnt = nxt.cnt;
         PL.segH = w.segH; PL.segL = w.segL; PL.seg_pre = w.seg_pre;
         PL.out_hi = w.out_hi; PL.out_lo = w.out_lo; PL.len_tmp = w.len_tmp; PL.nxt = tn;
-        PL.el = w.pel; PL.egrp = w.pgrp; PL.egroups = w.pgroups; PL.mp1 = w.mp1; PL.sflag = w.sflag;
+        PL.el = w.pel; PL.egrp = w.pgrp; PL.egroups = w.pgroups; PL.mp1 = w.mp1; PL.sflag = w.level_flag(lvl + 1);
         RunArgs RA;
         if (sh.rle) {
           RA.m = sh.m; RA.Kp = cur.K; RA.Knp = nxt.K; RA.cidx = cidx; RA.cur = tb; RA.nxt = tn;
@@ -1111,12 +1140,12 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
           PA.t.val = sh.valw[lvl & 1].as<float>();
         }
         kt.begin(GBDT_PHASE_K_COUNT);
-        LK.partition_count(PA, PL, ds.has_missing, w.groups, st, &w.sl);
+        LK.partition_count(PA, PL, ds.has_missing, w.groups, st, &lsl);
         kt.end();
         kt.begin(GBDT_PHASE_K_SCATTER);
         if (PA.cagg_next)
           GBDT_CUDA(cudaMemsetAsync(w.cagg, 0, sizeof(unsigned long long) * 5 * (size_t)std::max<int64_t>(sh.C0, 1), st));
-        LK.partition_scatter(PA, hmode, (sh.rle && !dec) ? &RA : nullptr, st, &w.sl);
+        LK.partition_scatter(PA, hmode, (sh.rle && !dec) ? &RA : nullptr, st, &lsl);
         if (dec)
           LK.rle_encode(tn, sh.m, nxt.K, sh.valw[(lvl + 1) & 1].as<float>(), w.enc_cnt, w.enc_bits,
                         ((size_t)sh.cap / 32 + 2) * 4, st);
