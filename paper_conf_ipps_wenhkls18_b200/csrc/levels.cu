@@ -1529,7 +1529,10 @@ __global__ void __launch_bounds__(kThreads) k_short_scatter(PartArgs A, ShortLis
 #define GBDT_GEN_CTAS 2
 #endif
 #ifndef GBDT_GEN_DYN
-#define GBDT_GEN_DYN 0  // dynamic claim of the chunk steps (missing values)
+#define GBDT_GEN_DYN 1  // dynamic claim of the chunk steps (missing values)
+#endif
+#ifndef GBDT_GEN_COMPACT
+#define GBDT_GEN_COMPACT 1
 #endif
 template <int HMODE, bool kMissing, bool kTotals, bool kRLE>
 __global__ void __launch_bounds__(kThreads, GBDT_GEN_CTAS) k_sf_gen(SplitArgs A) {
@@ -1745,6 +1748,41 @@ __global__ void __launch_bounds__(kThreads, GBDT_GEN_CTAS) k_sf_gen(SplitArgs A)
       if (((pem >> k) & 1) && cq != INT_MAX) sfl[cq] = 1;  // each segment marks one item
     }
     __syncwarp();
+#if GBDT_GEN_COMPACT
+    // the marked items (a few per warp) through one copy of the record code: the eight unrolled
+    // copies of the exact Eq. 2 (two IEEE divisions each) made the kernel overflow the
+    // instruction cache (35 % of stall samples on instruction fetch, C4a)
+    unsigned pmk = 0;
+#pragma unroll
+    for (int k = 0; k < kItems; ++k)
+      if (((vm >> k) & 1) && sfl[lane * kItems + k]) pmk |= 1u << k;
+    while (pmk) {
+      const int k = __ffs(pmk) - 1;
+      pmk &= pmk - 1;
+      double gq = g[0], hq = h[0];
+      int cq2 = cnt[0], j = sj[0];
+      float vq = v[0];
+#pragma unroll
+      for (int t = 1; t < kItems; ++t)
+        if (k == t) { gq = g[t]; hq = h[t]; cq2 = cnt[t]; j = sj[t]; vq = v[t]; }
+      const long long s = sb + j;
+      const NodeV nv = node_v(B, A, K, j);
+      Rec r;
+      r.value = vq;
+      r.attr = A.t.a_base + d.a;
+      r.dir = (dm >> k) & 1;
+      r.node = j;
+      r.epoch = epoch;
+      r.shard = A.shard;
+      r.pos = base + k;
+      if (r.dir) {
+        r.GL = gq + (nv.G - A.segPG[s]);
+        r.HL = hq + (nv.H - A.segPH[s]);
+        r.cntL = cq2 + (nv.C - (int)sc[j]);
+      } else {
+        r.GL = gq; r.HL = hq; r.cntL = cq2;
+      }
+#else
 #pragma unroll
     for (int k = 0; k < kItems; ++k) {
       if (!((vm >> k) & 1) || !sfl[lane * kItems + k]) continue;
@@ -1766,6 +1804,7 @@ __global__ void __launch_bounds__(kThreads, GBDT_GEN_CTAS) k_sf_gen(SplitArgs A)
       } else {
         r.GL = g[k]; r.HL = h[k]; r.cntL = cnt[k];
       }
+#endif
       r.gain = eq2_gain(r.GL, r.HL, nv.G, nv.H, lam, nv.P);
       if (K <= kWarpK) {
         const unsigned long long gk = gain_key(r.gain);
