@@ -2612,6 +2612,309 @@ __global__ void __launch_bounds__(kThreads) k_run_scatter(RunArgs A) {
   }
 }
 
+// ============================================================================ a4-a6 RLE: split on runs
+// "the RLE elements are the candidates": with the values in runs and no missing values,
+// split finding needs only each run's (G, H, count), a prefix over the runs of a segment and Eq. 2
+// at every run end -- O(runs) work instead of a scan over every entry.
+//   k_run_zero   clears the level's run records
+//   k_run_agg    one warp per 256-entry chunk of the g-list: for every run touching the chunk, the
+//                fp64 sums of g and h over the run's entries in the chunk (lane partials in item
+//                order, then a butterfly, so a fixed association), added to the run's record as
+//                exact 128-bit fixed point: every run total is exact and independent of the order
+//                of the adds and of the attribute sharding (chunks are attribute-aligned)
+//   k_run_split  one warp per (attribute, node) segment: exact prefix over its runs (32 runs per
+//                step), the exact Eq. 2 gain at every run end but the segment's last (non-empty
+//                low side), the segment's best (R12: largest gain, then the earlier run = the
+//                larger value) posted as a node-best record
+// segment of run r: the largest s with seg_run[s] <= r (runs are stored in segment order)
+__device__ __forceinline__ long long run_segment(const int32_t* __restrict__ seg_run, long long S, int r) {
+  long long lo = 0, hi = S - 1;
+  while (lo < hi) {
+    const long long mid = (lo + hi + 1) >> 1;
+    if (seg_run[mid] <= r) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+// racc: per run a 5-word scan record: fixed-point g (lo, hi), h (lo, hi) -- cleared here, summed
+// by k_run_agg -- and word 4 = run length | first run of its segment << 33 (the scan's reset flag)
+__global__ void __launch_bounds__(kThreads) k_run_init(SplitArgs A, unsigned long long* __restrict__ racc) {
+  const int K = *A.t.Kp;
+  const int R = *A.t.tb.R;
+  const long long S = (long long)A.t.m * K;
+  for (int r = blockIdx.x * blockDim.x + threadIdx.x; r < R; r += gridDim.x * blockDim.x) {
+    const long long s = run_segment(A.t.tb.seg_run, S, r);
+    unsigned long long* x = racc + 5ll * r;
+    x[0] = 0ull; x[1] = 0ull; x[2] = 0ull; x[3] = 0ull;
+    x[4] = (unsigned long long)(unsigned)A.t.tb.run_len[r] | ((unsigned long long)(A.t.tb.seg_run[s] == r) << 33);
+  }
+}
+
+// k_run_agg: one warp per 256-entry chunk lying inside one run (nearly all chunks of
+// low-cardinality lists), two chunks in flight per warp: lane sums in item order, a butterfly, one
+// exact add per total.  Chunks holding several runs are listed (A.genlist) for k_run_agg_multi.
+template <int HMODE>
+__global__ void __launch_bounds__(kThreads) k_run_agg(SplitArgs A, unsigned long long* __restrict__ racc) {
+  constexpr bool kH = HMODE == kHGather;
+  __shared__ TabCache tc;
+  const int lane = threadIdx.x & 31;
+  const int K = *A.t.Kp;
+  const int C = *A.t.tb.C;
+  if (K == 0) return;
+  tab_load(tc, A.t);
+  __syncthreads();
+  const Tables& tb = A.t.tb;
+  const int Fg = A.fx[0], Fh = A.fx[1];
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += 2 * nw) {
+    long long p0[2];
+    int len[2], rb[2];
+    bool one[2];
+    double g[2][kItems];
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      const int cu = c + u * nw;
+      len[u] = 0;
+      p0[u] = 0;
+      rb[u] = 0;
+      one[u] = false;
+      if (cu < C) {
+        const ChunkMeta M = chunk_meta(tc, A.t, K, cu);
+        p0[u] = M.p0;
+        len[u] = (int)(M.p1 - M.p0);
+        rb[u] = tb.run_chunk[cu];
+        one[u] = tb.run_pos[rb[u]] + tb.run_len[rb[u]] >= M.p1;
+      }
+      const double* gp = A.glist + p0[u] + lane;
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) g[u][k] = (one[u] && 32 * k + lane < len[u]) ? __ldcs(gp + 32 * k) : 0.0;
+    }
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      const int cu = c + u * nw;
+      if (cu >= C) break;
+      if (!one[u]) {
+        if (lane == 0) A.genlist[atomicAdd(A.ngen, 1)] = cu;
+        continue;
+      }
+      double sg = 0.0, sh = 0.0;
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) {
+        const bool in = 32 * k + lane < len[u];
+        const double hk = in ? (kH ? __ldcs(A.hlist + p0[u] + 32 * k + lane) : hess_of<HMODE>(g[u][k])) : 0.0;
+        sg = sg + g[u][k];
+        sh = sh + hk;
+      }
+#pragma unroll
+      for (int o = 16; o; o >>= 1) {
+        sg = sg + __shfl_xor_sync(0xffffffffu, sg, o);
+        sh = sh + __shfl_xor_sync(0xffffffffu, sh, o);
+      }
+      if (lane == 0) {
+        fx_atomic_add(racc + 5ll * rb[u], to_fx(sg, Fg));
+        fx_atomic_add(racc + 5ll * rb[u] + 2, to_fx(sh, Fh));
+      }
+    }
+  }
+}
+
+// k_run_agg_multi: the listed chunks holding several runs, lane l on entries 8l .. 8l+7 (blocked).
+// The runs starting inside the chunk mark a 256-bit head mask, a segmented scan (in-lane, then
+// across the lanes) forms every run piece's sum at its last entry, and that lane adds it --
+// O(entries) work whatever the number of runs.
+template <int HMODE>
+__global__ void __launch_bounds__(kThreads) k_run_agg_multi(SplitArgs A, unsigned long long* __restrict__ racc) {
+  constexpr bool kH = HMODE == kHGather;
+  __shared__ unsigned heads[kWarps][kChunk / 32];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int K = *A.t.Kp;
+  const int NL = *A.ngen;
+  if (K == 0) return;
+  const Tables& tb = A.t.tb;
+  const int Fg = A.fx[0], Fh = A.fx[1];
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  unsigned* hw = heads[wid];
+  for (int i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < NL; i += nw) {
+    const int c = A.genlist[i];
+    const int a = tb.chunk_attr[c];
+    const long long cs = tb.col_start[a], ce = cs + tb.col_len[a];
+    const long long p0 = cs + (long long)(c - tb.chunk_start[a]) * kChunk;
+    const int len = (int)(min(p0 + (long long)kChunk, ce) - p0);
+    const int rb = tb.run_chunk[c];
+    const int re = p0 + len < ce ? tb.run_chunk[c + 1] : tb.seg_run[(long long)a * K + K] - 1;
+    const int q0 = kItems * lane;
+    double g[kItems], h[kItems];
+    if (q0 + kItems <= len) {
+      const double2* gp = reinterpret_cast<const double2*>(A.glist + p0 + q0);
+#pragma unroll
+      for (int j = 0; j < kItems / 2; ++j) {
+        const double2 z = __ldcs(gp + j);
+        g[2 * j] = z.x;
+        g[2 * j + 1] = z.y;
+      }
+      if (kH) {
+        const double2* hp = reinterpret_cast<const double2*>(A.hlist + p0 + q0);
+#pragma unroll
+        for (int j = 0; j < kItems / 2; ++j) {
+          const double2 z = __ldcs(hp + j);
+          h[2 * j] = z.x;
+          h[2 * j + 1] = z.y;
+        }
+      }
+    } else {
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) {
+        g[k] = q0 + k < len ? __ldcs(A.glist + p0 + q0 + k) : 0.0;
+        if (kH) h[k] = q0 + k < len ? __ldcs(A.hlist + p0 + q0 + k) : 0.0;
+      }
+    }
+    if (!kH) {
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) h[k] = q0 + k < len ? hess_of<HMODE>(g[k]) : 0.0;
+    }
+    // heads: the first entries of the runs that start inside the chunk (after its first entry)
+    if (lane < kChunk / 32) hw[lane] = 0u;
+    __syncwarp();
+    for (int r = rb + 1 + lane; r <= re; r += 32) {
+      const long long q = tb.run_pos[r] - p0;
+      if (q > 0 && q < len) atomicOr(&hw[q >> 5], 1u << (q & 31));
+    }
+    __syncwarp();
+    const unsigned hword = hw[lane >> 2];
+    const unsigned hb = (hword >> ((lane & 3) * 8)) & 0xffu;  // heads among the lane's items
+    // heads before the lane's first item (positions 1 .. q0-1): the run of its first item
+    int before = 0;
+#pragma unroll
+    for (int wdx = 0; wdx < kChunk / 32; ++wdx)
+      if (wdx < (lane >> 2)) before += __popc(hw[wdx]);
+    before += __popc(hword & ((1u << ((lane & 3) * 8)) - 1u));
+    // the head bit of the entry after the lane's last item
+    const bool next_head = (q0 + kItems < kChunk) && ((hw[(q0 + kItems) >> 5] >> ((q0 + kItems) & 31)) & 1u);
+    __syncwarp();  // hw is rewritten by the warp's next chunk
+    double pg[kItems], ph[kItems];
+    double rg = 0.0, rh = 0.0;
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) {
+      if ((hb >> k) & 1u) { rg = 0.0; rh = 0.0; }
+      rg = rg + g[k];
+      rh = rh + h[k];
+      pg[k] = rg;
+      ph[k] = rh;
+    }
+    // segmented inclusive scan of the lane tails across the lanes (lane 0 starts the chunk)
+    double ig = rg, ih = rh;
+    int fl = (hb != 0u || lane == 0) ? 1 : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const double yg = __shfl_up_sync(0xffffffffu, ig, o), yh = __shfl_up_sync(0xffffffffu, ih, o);
+      const int yf = __shfl_up_sync(0xffffffffu, fl, o);
+      if (lane >= o) {
+        if (!fl) { ig = yg + ig; ih = yh + ih; }
+        fl |= yf;
+      }
+    }
+    double cg = __shfl_up_sync(0xffffffffu, ig, 1), ch = __shfl_up_sync(0xffffffffu, ih, 1);
+    if (lane == 0) { cg = 0.0; ch = 0.0; }
+    int run = rb + before;
+    bool open = true;  // the lane's current piece began in an earlier lane
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) {
+      const int q = q0 + k;
+      if ((hb >> k) & 1u) { ++run; open = false; }
+      const bool end = q < len && (q + 1 == len || (k + 1 < kItems ? ((hb >> (k + 1)) & 1u) != 0u : next_head));
+      if (end) {
+        const double tg = open ? cg + pg[k] : pg[k], th = open ? ch + ph[k] : ph[k];
+        fx_atomic_add(racc + 5ll * run, to_fx(tg, Fg));
+        fx_atomic_add(racc + 5ll * run + 2, to_fx(th, Fh));
+      }
+    }
+  }
+}
+
+// One warp per 256 consecutive runs (8 steps of 32): the candidate at the end of run r (not the
+// last run of its segment) has the high side = runs up to r, whose totals are the exact carry of
+// run r+1 (k_scan3, converted once to fp64).  Segmented argmax over the lanes (segments are
+// contiguous runs), the best of a segment piece carried across steps; a piece that ends its
+// segment or the warp's range posts one record (<= runs/256 + segments records per level).
+constexpr int kRunSteps = 8;
+__global__ void __launch_bounds__(kThreads) k_run_split(SplitArgs A, const unsigned long long* __restrict__ rcar) {
+  const int lane = threadIdx.x & 31;
+  const int K = *A.t.Kp;
+  if (K == 0) return;
+  const Tables& tb = A.t.tb;
+  const int R = *tb.R;
+  const long long S = (long long)A.t.m * K;
+  const int epoch = *A.epochp;
+  const double lam = A.lam;
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int base = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 * kRunSteps); base < R;
+       base += nw * 32 * kRunSteps) {
+    long long cs_ = -1;  // segment of the carried best (-1: none)
+    unsigned long long ckey = 0ull;
+    int cr = -1;
+    for (int step = 0; step < kRunSteps; ++step) {
+      const int rb = base + 32 * step;
+      if (rb >= R) break;
+      const int r = rb + lane;
+      const bool act = r < R;
+      long long s = act ? run_segment(tb.seg_run, S, r) : LLONG_MAX;
+      const bool seg_last = act && r + 1 >= tb.seg_run[s + 1];
+      const bool cand = act && !seg_last;
+      unsigned long long key = 0ull;
+      double GL = 0.0, HL = 0.0;
+      int j = 0;
+      if (act) j = (int)(s % K);
+      if (cand) {
+        const CarryD cx = carry_load(rcar + 5ll * (r + 1));
+        GL = cx.g;
+        HL = cx.h;
+        key = gain_key(eq2_gain(GL, HL, A.nodes.G[j], A.nodes.H[j], lam, A.nodes.pterm[j]));
+      }
+      // segmented argmax over the lanes: larger key, then the earlier run (R12)
+      unsigned long long bk = key;
+      int bl = lane;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long yk = __shfl_up_sync(0xffffffffu, bk, o);
+        const int yl = __shfl_up_sync(0xffffffffu, bl, o);
+        const long long ys = __shfl_up_sync(0xffffffffu, s, o);
+        if (lane >= o && ys == s && yk >= bk) { bk = yk; bl = yl; }
+      }
+      // the first piece of the step continues the carried segment
+      if (s == cs_ && ckey >= bk && ckey) { bk = ckey; bl = -1 - cr; }  // encode a carried run as < 0
+      const long long sn = __shfl_down_sync(0xffffffffu, s, 1);
+      const bool piece_end = act && (lane == 31 || sn != s);
+      const bool range_end = act && (lane == 31 ? step == kRunSteps - 1 : false) || (act && r == R - 1);
+      // carry: the last lane's piece when it does not end its segment
+      const unsigned long long lk = __shfl_sync(0xffffffffu, bk, 31);
+      const int ll = __shfl_sync(0xffffffffu, bl, 31);
+      const long long ls = __shfl_sync(0xffffffffu, s, 31);
+      const bool lend = __shfl_sync(0xffffffffu, seg_last, 31);
+      const int lr = ll < 0 ? -1 - ll : rb + ll;
+      if (piece_end && (seg_last || range_end) && bk) {
+        const int wr = bl < 0 ? -1 - bl : rb + bl;
+        const CarryD cx = carry_load(rcar + 5ll * (wr + 1));
+        const long long ws = bl < 0 ? cs_ : s;
+        const int wj = (int)(ws % K);
+        Rec rc;
+        rc.GL = cx.g;
+        rc.HL = cx.h;
+        rc.cntL = cx.c;
+        rc.gain = eq2_gain(cx.g, cx.h, A.nodes.G[wj], A.nodes.H[wj], lam, A.nodes.pterm[wj]);
+        rc.value = tb.run_val[wr];
+        rc.attr = A.t.a_base + (int)(ws / K);
+        rc.dir = 0;
+        rc.node = wj;
+        rc.epoch = epoch;
+        rc.shard = A.shard;
+        rc.pos = tb.run_pos[wr] + tb.run_len[wr] - 1;
+        post_global(A, rc);
+      }
+      if (ls != LLONG_MAX && !lend) { cs_ = ls; ckey = lk; cr = lr; } else { cs_ = -1; ckey = 0ull; cr = -1; }
+    }
+  }
+}
+
 // ---------------------------------------------------------------------------- RLE split ablation
 // "Splitting RLE with decompression" (Fig. 6), the baseline the paper's direct RLE split
 // (Fig. 7) is measured against: the level's runs are decompressed into the value
@@ -3017,6 +3320,21 @@ void LevelKernels::rle_encode(const Tables& tn, int m, const int32_t* Knp, const
   k_enc_segfix<<<1, 1, 0, st>>>(tn, m, Knp);
   GBDT_LAUNCH_CHECK();
   count_launch(6);
+}
+
+void LevelKernels::run_split(const SplitArgs& A, int hmode, unsigned long long* racc, unsigned long long* rcar,
+                             unsigned long long* rsg, unsigned groups, cudaStream_t st) {
+  k_run_init<<<(unsigned)(sms * 4), kThreads, 0, st>>>(A, racc);
+  const unsigned ga = (unsigned)(sms * 8);
+  if (hmode == 0) { k_run_agg<0><<<ga, kThreads, 0, st>>>(A, racc); k_run_agg_multi<0><<<ga, kThreads, 0, st>>>(A, racc); }
+  else if (hmode == 1) { k_run_agg<1><<<ga, kThreads, 0, st>>>(A, racc); k_run_agg_multi<1><<<ga, kThreads, 0, st>>>(A, racc); }
+  else { k_run_agg<2><<<ga, kThreads, 0, st>>>(A, racc); k_run_agg_multi<2><<<ga, kThreads, 0, st>>>(A, racc); }
+  GBDT_LAUNCH_CHECK();
+  count_launch(3);
+  launch_scan<true>(A.t.tb.R, racc, rsg, rcar, groups, st, A.fx);
+  k_run_split<<<(unsigned)(sms * 4), kThreads, 0, st>>>(A, rcar);
+  GBDT_LAUNCH_CHECK();
+  count_launch();
 }
 
 void LevelKernels::chunk_desc(const SplitArgs& A, unsigned groups, cudaStream_t st) {

@@ -469,6 +469,9 @@ struct ShardWork {
   unsigned long long *run_hl = nullptr, *rcnt = nullptr, *rfl = nullptr, *rsgrp = nullptr;
   int32_t* Rp1 = nullptr;
   unsigned rgroups = 1;
+  unsigned long long* racc = nullptr;  // RLE split on runs: [Rcap][5] exact (g, h) per run (scan records)
+  unsigned long long* rcar = nullptr;  //   their exclusive segmented prefixes (fp64 carries)
+  unsigned long long* rsg5 = nullptr;  //   scan scratch
   uint32_t* enc_cnt = nullptr;   // RLE split ablation: runs per next-level chunk
   uint32_t* enc_bits = nullptr;  //   and the next level's segment-start bitmap
   // fused dense levels: plans of two levels, per-tile records / carries / side bits
@@ -665,6 +668,10 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     const char* fe = getenv("GBDT_FUSED");
     fused = fused && fe && fe[0] != '0';
   }
+  // RLE shards without missing values find splits over the runs (levels.cu k_run_split);
+  // GBDT_RUNSPLIT=0 keeps the per-entry scan of the plain lists (A/B and cross-check)
+  bool runsplit = !ds.has_missing;
+  if (const char* rse = getenv("GBDT_RUNSPLIT")) runsplit = runsplit && rse[0] != '0';
 
   // ---------------------------------------------------------------- per-shard state
   std::vector<ShardWork> sw(nloc);
@@ -748,6 +755,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         q.take<unsigned long long>(2 * (size_t)w.rgroups + 8);
         q.take<uint32_t>((size_t)C0 + 2);
         q.take<uint32_t>((size_t)sh.cap / 32 + 2);
+        q.take<unsigned long long>(5 * (size_t)Rcap); q.take<unsigned long long>(5 * (size_t)Rcap);
+        q.take<unsigned long long>(5 * (size_t)w.rgroups + 8);
       };
       Carve rp{nullptr};
       rz(rp);
@@ -765,6 +774,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       w.Rp1 = r.take<int32_t>(1); w.rsgrp = r.take<unsigned long long>(2 * (size_t)w.rgroups + 8);
       w.enc_cnt = r.take<uint32_t>((size_t)C0 + 2);
       w.enc_bits = r.take<uint32_t>((size_t)sh.cap / 32 + 2);
+      w.racc = r.take<unsigned long long>(5 * (size_t)Rcap); w.rcar = r.take<unsigned long long>(5 * (size_t)Rcap);
+      w.rsg5 = r.take<unsigned long long>(5 * (size_t)w.rgroups + 8);
     }
     if (fused && m > 0) {
       w.tiles = fused_tiles(n, m);
@@ -983,14 +994,24 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         A.segPG_out = w.segPG; A.segPH_out = w.segPH;
         // present totals per segment (needed for the missing direction), from the chunk pass
         A.segEnd = ds.has_missing ? w.segEnd : nullptr;
+        const bool rs = runsplit && sh.rle;
         kt.begin(GBDT_PHASE_K_CHUNK_AGG);
-        if (lvl > 0 && !ds.has_missing) LK.chunk_desc(A, w.groups, st);  // aggregates from the scatter
-        else LK.tile_prefix(A, hmode, /*gather=*/lvl == 0, w.groups, st);
+        if (rs) {
+          if (lvl == 0) LK.tile_prefix(A, hmode, /*gather=*/true, w.groups, st);  // the root g-list
+        } else if (lvl > 0 && !ds.has_missing) {
+          LK.chunk_desc(A, w.groups, st);  // aggregates from the scatter
+        } else {
+          LK.tile_prefix(A, hmode, /*gather=*/lvl == 0, w.groups, st);
+        }
         kt.end();
 
         kt.begin(GBDT_PHASE_K_SPLIT);
-        LK.short_split(A, w.level_sl(lvl), hmode, /*gather=*/lvl == 0, st);
-        LK.split_find(A, hmode, ds.has_missing, sh.rle, st);
+        if (rs) {
+          LK.run_split(A, hmode, w.racc, w.rcar, w.rsg5, w.rgroups, st);
+        } else {
+          LK.short_split(A, w.level_sl(lvl), hmode, /*gather=*/lvl == 0, st);
+          LK.split_find(A, hmode, ds.has_missing, sh.rle, st);
+        }
         kt.end();
         if (P.profile) {  // the level's list entries (byte model of the bench), off the timed kernels
           k_level_entries<<<(unsigned)std::min<int64_t>(ceil_div(sh.m, 256), sms * 4), 256, 0, st>>>(tb.col_len, sh.m, lent + lvl);
@@ -1118,7 +1139,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         PA.g_out = w.glist[(lvl + 1) & 1]; PA.h_out = w.hlist[(lvl + 1) & 1];
         PA.epochp = epoch;
         // without missing values the scatter accumulates the next level's chunk aggregates
-        PA.cagg_next = ds.has_missing ? nullptr : w.cagg;
+        PA.cagg_next = (ds.has_missing || (runsplit && sh.rle)) ? nullptr : w.cagg;
         PA.nxt = tn;
         PA.fx = fxs;
         PlanArgs PL;

@@ -199,11 +199,12 @@ def test_deterministic_across_runs():
 
 
 # ------------------------------------------------------------------ a8 RLE: direct split
-# The RLE path reads values from the runs and splits the runs themselves (no decompression in HBM);
-# it sees the same entry streams, so its trees and margins must be bit-identical to the plain
-# level-by-level path (GBDT_FUSED=0: dense data otherwise takes the fused pass of fused.cu, whose
-# sums associate differently; GBDT_SHORT=0: the same for the short-list path), and both match the
-# oracle.
+# The RLE path reads values from the runs and splits the runs themselves (no decompression in HBM).
+# With its per-entry scan (GBDT_RUNSPLIT=0) it sees the same entry streams as the plain lists, so
+# its trees and margins must be bit-identical to the plain level-by-level path (GBDT_FUSED=0: dense
+# data otherwise takes the fused pass of fused.cu, whose sums associate differently; GBDT_SHORT=0:
+# the same for the short-list path), and both match the oracle.  The split on runs (the default
+# for dense RLE data, k_run_split) is tested against the oracle below.
 @pytest.mark.parametrize("maker", [
     lambda: synth.c5(n=40000, T=3),
     lambda: synth.table1(),
@@ -215,6 +216,7 @@ def test_deterministic_across_runs():
 def test_rle_direct_split_bit_identical(maker, monkeypatch):
     p = maker()
     monkeypatch.setenv("GBDT_FUSED", "0")
+    monkeypatch.setenv("GBDT_RUNSPLIT", "0")
     # plain lists route short sparse attributes through the short path (levels.cu k_short_*), whose
     # prefix sums associate in list order; the RLE path keeps the chunk kernels throughout
     monkeypatch.setenv("GBDT_SHORT", "0")
@@ -234,10 +236,63 @@ def test_rle_c5_against_oracle():
 def test_rle_with_shards(k, monkeypatch):
     p = synth.c5(n=30000, T=2)
     monkeypatch.setenv("GBDT_FUSED", "0")
+    monkeypatch.setenv("GBDT_RUNSPLIT", "0")
     ref_model, ref_margin = _train(p)
     model, margin = _train(p, rle="on", n_shards=k)
     assert np.array_equal(model.nodes().view(np.uint8), ref_model.nodes().view(np.uint8))
     assert np.array_equal(margin, ref_margin)
+
+
+# ------------------------------------------------------------------ a4-a6 RLE: split on runs
+# Dense RLE data: every run's (G, H) is an exact fixed-point total of its chunk partials and the
+# candidates are the run ends, so the result is oracle-equal and independent of the sharding.
+# Cases: C5-shaped (<= 64 values), Table I, high cardinality (many runs per segment: the 32-run
+# steps and their carry), squared and logistic, depth 8 (more than 32 nodes: global records),
+# general labels (h gathered, hmode 2), C2-shaped (one-hot and integer columns).
+@pytest.mark.parametrize("maker", [
+    lambda: synth.c5(n=40000, T=3),
+    lambda: synth.table1(),
+    lambda: synth.random_small(8, n=9000, m=5, nan_frac=0.0, n_distinct=3000),
+    lambda: synth.random_small(81, n=7000, m=4, nan_frac=0.0, n_distinct=200, loss="logistic", d=8, T=2),
+    lambda: synth.c1(n=5000),
+    lambda: synth.c2(n=30000, T=3),
+])
+def test_rle_run_split_against_oracle(maker):
+    p = maker()
+    model, margin = _train(p, rle="on")
+    compare(p, model.nodes(), margin)
+
+
+def test_rle_run_split_general_labels():
+    """Logistic loss with labels outside {0, 1}: h is gathered per entry (hmode 2)."""
+    p = synth.c5(n=20000, T=2)
+    p.labels = (p.labels * 0.8 + 0.1).astype(np.float32)
+    model, margin = _train(p, rle="on")
+    compare(p, model.nodes(), margin)
+
+
+@pytest.mark.parametrize("k", [2, 4])
+def test_rle_run_split_shards_bit_identical(k):
+    p = synth.c5(n=30000, T=3)
+    ref_model, ref_margin = _train(p, rle="on")
+    model, margin = _train(p, rle="on", n_shards=k)
+    assert np.array_equal(model.nodes().view(np.uint8), ref_model.nodes().view(np.uint8))
+    assert np.array_equal(margin, ref_margin)
+    compare(p, model.nodes(), margin)
+
+
+def test_rle_run_split_equals_entry_scan_structure(monkeypatch):
+    """The split on runs and the per-entry scan of the same runs choose the same splits (their
+    sums associate differently, so weights agree to rounding)."""
+    p = synth.c5(n=50000, T=3)
+    model, margin = _train(p, rle="on")
+    monkeypatch.setenv("GBDT_RUNSPLIT", "0")
+    ref_model, ref_margin = _train(p, rle="on")
+    a, b = model.nodes(), ref_model.nodes()
+    for f in ("heap_id", "is_leaf", "attr", "default_left", "count", "split_value"):
+        assert np.array_equal(a[f], b[f]), f
+    np.testing.assert_allclose(a["weight"], b["weight"], rtol=1e-9, atol=1e-12)
+    np.testing.assert_allclose(margin, ref_margin, rtol=1e-9, atol=1e-12)
 
 
 def test_rle_export_matches_oracle_encoding():

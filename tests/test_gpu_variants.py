@@ -62,9 +62,11 @@ def test_rle_auto_decides_per_attribute(monkeypatch):
     groups = [(ds.info(s)["attr_begin"], ds.info(s)["attr_end"], ds.info(s)["runs"] > 0) for s in range(k)]
     assert groups == [(0, 1, True), (1, 3, False), (3, 5, True), (5, 6, False)], groups
     m_auto, y_auto = gbdt.train(ds, **{k2: v for k2, v in p.params.items()})
+    compare(p, m_auto.nodes(), y_auto)                       # RLE shards split on their runs
     monkeypatch.setenv("GBDT_FUSED", "0")
-    _same((m_auto, y_auto), gbdt.train_problem(p))           # trees as without RLE, bit for bit
-    compare(p, m_auto.nodes(), y_auto)
+    monkeypatch.setenv("GBDT_RUNSPLIT", "0")                 # per-entry scan of the runs:
+    m_scan = gbdt.train(ds, **{k2: v for k2, v in p.params.items()})
+    _same(m_scan, gbdt.train_problem(p))                     # trees as without RLE, bit for bit
 
 
 def test_rle_auto_uniform_decision_keeps_one_shard():
