@@ -244,7 +244,7 @@ struct LevelKernels {
   // a4-a6 with RLE and no missing values: run totals from the level's g-list, then the
   // split find over the runs (racc: [Rcap][5] exact fixed-point g, h per run as scan records,
   // rcar: their exclusive segmented prefixes, rsg: scan scratch of 5 * groups + 8 words)
-  void run_split(const SplitArgs& A, int hmode, unsigned long long* racc, unsigned long long* rcar,
+  void run_split(const SplitArgs& A, int hmode, bool root, unsigned long long* racc, unsigned long long* rcar,
                  unsigned long long* rsg, unsigned groups, cudaStream_t st);
   // RLE split ablation (Fig. 6): decompress a level's runs into its value list; compress
   // the next level's value list (per node segment) into its run tables

@@ -2683,11 +2683,16 @@ __global__ void __launch_bounds__(kThreads) k_run_agg(SplitArgs A, unsigned long
         p0[u] = M.p0;
         len[u] = (int)(M.p1 - M.p0);
         rb[u] = tb.run_chunk[cu];
-        one[u] = tb.run_pos[rb[u]] + tb.run_len[rb[u]] >= M.p1;
       }
+      // the g loads do not wait for the run lookup (a multi-run chunk wastes them)
       const double* gp = A.glist + p0[u] + lane;
 #pragma unroll
-      for (int k = 0; k < kItems; ++k) g[u][k] = (one[u] && 32 * k + lane < len[u]) ? __ldcs(gp + 32 * k) : 0.0;
+      for (int k = 0; k < kItems; ++k) g[u][k] = (32 * k + lane < len[u]) ? __ldcs(gp + 32 * k) : 0.0;
+    }
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      const int cu = c + u * nw;
+      if (cu < C) one[u] = tb.run_pos[rb[u]] + tb.run_len[rb[u]] >= p0[u] + len[u];
     }
 #pragma unroll
     for (int u = 0; u < 2; ++u) {
@@ -2714,6 +2719,79 @@ __global__ void __launch_bounds__(kThreads) k_run_agg(SplitArgs A, unsigned long
         fx_atomic_add(racc + 5ll * rb[u], to_fx(sg, Fg));
         fx_atomic_add(racc + 5ll * rb[u] + 2, to_fx(sh, Fh));
       }
+    }
+  }
+}
+
+// k_run_root: the root level of the split on runs, one warp per 256-entry chunk (lane l on entries
+// 8l .. 8l+7): g (and h) gathered by instance into the g-list (once per tree, L2 evict-last), and
+// the run totals of the single-run chunks as in k_run_agg; other chunks are listed for
+// k_run_agg_multi, which reads the g-list written here.
+template <int HMODE>
+__global__ void __launch_bounds__(kThreads) k_run_root(SplitArgs A, unsigned long long* __restrict__ racc) {
+  constexpr bool kH = HMODE == kHGather;
+  __shared__ TabCache tc;
+  const int lane = threadIdx.x & 31;
+  const int K = *A.t.Kp;
+  const int C = *A.t.tb.C;
+  if (K == 0) return;
+  tab_load(tc, A.t);
+  __syncthreads();
+  const Tables& tb = A.t.tb;
+  const int Fg = A.fx[0], Fh = A.fx[1];
+  const unsigned long long pol_keep = policy_evict_last();
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int c = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < C; c += nw) {
+    const ChunkMeta M = chunk_meta(tc, A.t, K, c);
+    const long long p1 = M.p1;
+    const long long base = M.p0 + (long long)lane * kItems;
+    const int rb = tb.run_chunk[c];
+    double g[kItems], h[kItems];
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) { g[k] = 0.0; h[k] = 0.0; }
+    if (base < p1) {
+      const int4 i0 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base));
+      const int4 i1 = __ldcs(reinterpret_cast<const int4*>(A.t.ins + base + 4));
+      const int id[kItems] = {i0.x, i0.y, i0.z, i0.w, i1.x, i1.y, i1.z, i1.w};
+#pragma unroll
+      for (int k = 0; k < kItems; ++k) {
+        if (base + k < p1) {
+          g[k] = ld_keep(A.g + id[k], pol_keep);
+          h[k] = kH ? ld_keep(A.h + id[k], pol_keep) : hess_of<HMODE>(g[k]);
+        }
+      }
+      if (base + kItems <= p1) {  // lists are padded to 4 entries only: never write past the chunk
+        double2* go = reinterpret_cast<double2*>(A.glist + base);
+#pragma unroll
+        for (int q = 0; q < kItems / 2; ++q) __stcs(go + q, make_double2(g[2 * q], g[2 * q + 1]));
+        if (kH) {
+          double2* ho = reinterpret_cast<double2*>(A.hlist + base);
+#pragma unroll
+          for (int q = 0; q < kItems / 2; ++q) __stcs(ho + q, make_double2(h[2 * q], h[2 * q + 1]));
+        }
+      } else {
+#pragma unroll
+        for (int k = 0; k < kItems; ++k)
+          if (base + k < p1) {
+            A.glist[base + k] = g[k];
+            if (kH) A.hlist[base + k] = h[k];
+          }
+      }
+    }
+    if (tb.run_pos[rb] + tb.run_len[rb] < p1) {  // several runs: k_run_agg_multi
+      if (lane == 0) A.genlist[atomicAdd(A.ngen, 1)] = c;
+      continue;
+    }
+    double sg = ((g[0] + g[1]) + (g[2] + g[3])) + ((g[4] + g[5]) + (g[6] + g[7]));
+    double sh = ((h[0] + h[1]) + (h[2] + h[3])) + ((h[4] + h[5]) + (h[6] + h[7]));
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+      sg = sg + __shfl_xor_sync(0xffffffffu, sg, o);
+      sh = sh + __shfl_xor_sync(0xffffffffu, sh, o);
+    }
+    if (lane == 0) {
+      fx_atomic_add(racc + 5ll * rb, to_fx(sg, Fg));
+      fx_atomic_add(racc + 5ll * rb + 2, to_fx(sh, Fh));
     }
   }
 }
@@ -3322,13 +3400,22 @@ void LevelKernels::rle_encode(const Tables& tn, int m, const int32_t* Knp, const
   count_launch(6);
 }
 
-void LevelKernels::run_split(const SplitArgs& A, int hmode, unsigned long long* racc, unsigned long long* rcar,
-                             unsigned long long* rsg, unsigned groups, cudaStream_t st) {
+void LevelKernels::run_split(const SplitArgs& A, int hmode, bool root, unsigned long long* racc,
+                             unsigned long long* rcar, unsigned long long* rsg, unsigned groups, cudaStream_t st) {
   k_run_init<<<(unsigned)(sms * 4), kThreads, 0, st>>>(A, racc);
   const unsigned ga = (unsigned)(sms * 8);
-  if (hmode == 0) { k_run_agg<0><<<ga, kThreads, 0, st>>>(A, racc); k_run_agg_multi<0><<<ga, kThreads, 0, st>>>(A, racc); }
-  else if (hmode == 1) { k_run_agg<1><<<ga, kThreads, 0, st>>>(A, racc); k_run_agg_multi<1><<<ga, kThreads, 0, st>>>(A, racc); }
-  else { k_run_agg<2><<<ga, kThreads, 0, st>>>(A, racc); k_run_agg_multi<2><<<ga, kThreads, 0, st>>>(A, racc); }
+  if (root) {  // the g-list is gathered here
+    if (hmode == 0) k_run_root<0><<<ga, kThreads, 0, st>>>(A, racc);
+    else if (hmode == 1) k_run_root<1><<<ga, kThreads, 0, st>>>(A, racc);
+    else k_run_root<2><<<ga, kThreads, 0, st>>>(A, racc);
+  } else {
+    if (hmode == 0) k_run_agg<0><<<ga, kThreads, 0, st>>>(A, racc);
+    else if (hmode == 1) k_run_agg<1><<<ga, kThreads, 0, st>>>(A, racc);
+    else k_run_agg<2><<<ga, kThreads, 0, st>>>(A, racc);
+  }
+  if (hmode == 0) k_run_agg_multi<0><<<ga, kThreads, 0, st>>>(A, racc);
+  else if (hmode == 1) k_run_agg_multi<1><<<ga, kThreads, 0, st>>>(A, racc);
+  else k_run_agg_multi<2><<<ga, kThreads, 0, st>>>(A, racc);
   GBDT_LAUNCH_CHECK();
   count_launch(3);
   launch_scan<true>(A.t.tb.R, racc, rsg, rcar, groups, st, A.fx);

@@ -997,7 +997,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         const bool rs = runsplit && sh.rle;
         kt.begin(GBDT_PHASE_K_CHUNK_AGG);
         if (rs) {
-          if (lvl == 0) LK.tile_prefix(A, hmode, /*gather=*/true, w.groups, st);  // the root g-list
+          // the split on runs gathers the root g-list itself (k_run_root)
         } else if (lvl > 0 && !ds.has_missing) {
           LK.chunk_desc(A, w.groups, st);  // aggregates from the scatter
         } else {
@@ -1007,7 +1007,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
 
         kt.begin(GBDT_PHASE_K_SPLIT);
         if (rs) {
-          LK.run_split(A, hmode, w.racc, w.rcar, w.rsg5, w.rgroups, st);
+          LK.run_split(A, hmode, /*root=*/lvl == 0, w.racc, w.rcar, w.rsg5, w.rgroups, st);
         } else {
           LK.short_split(A, w.level_sl(lvl), hmode, /*gather=*/lvl == 0, st);
           LK.split_find(A, hmode, ds.has_missing, sh.rle, st);
