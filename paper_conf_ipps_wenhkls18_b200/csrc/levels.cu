@@ -480,6 +480,8 @@ __global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
         d.vnext = vnx;
         A.desc[c] = d;
         fxv_store(A.cagg + 5ll * c, FXV{to_fx(lg, Fg), to_fx(lh, Fh), len, s0 == M.p0 ? 1 : 0}, M.reset);
+        // with missing values k_sf_gen takes every chunk but k_sf_short's: list them all
+        if (A.segEnd) A.genlist[atomicAdd(A.ngen, 1)] = c;
         if (A.segEnd && p1 == se) {  // the segment ends here: its present totals (see k_seg_totals)
           const long long s = M.sb + j0;
           A.segPG_out[s] = lg;
@@ -1555,8 +1557,9 @@ __global__ void __launch_bounds__(kThreads, GBDT_GEN_CTAS) k_sf_gen(SplitArgs A)
     for (int j = threadIdx.x; j < kWarps * kWarpK; j += blockDim.x) wgk[j / kWarpK][j % kWarpK] = 0ull;
   __syncthreads();
   const int nw = (gridDim.x * blockDim.x) >> 5;
-  // with missing values every chunk; else the chunks k_chunk_agg listed (they cross segments)
-  constexpr bool kAll = kMissing || kTotals;
+  // the chunks k_chunk_agg listed: with missing values every chunk of the general layout (the
+  // short ones are k_sf_short's), else those that cross segments; the totals pass takes all
+  constexpr bool kAll = kTotals;
   const int n = kAll ? nchunks(A.t.tb) : *A.ngen;
   // 32 chunks per warp step (lane l tests chunk bt + l * nbat); the short ones are k_sf_short's,
   // so they cost one descriptor word here instead of a dependent descriptor load each
