@@ -68,6 +68,8 @@ def parse():
     ap.add_argument("--rle", default="off")
     ap.add_argument("--rle-split", default="direct", choices=["direct", "decompress"],
                     help="RLE node split: direct (P:250, Fig. 7) or the decompression ablation (P:248, Fig. 6)")
+    ap.add_argument("--local-shards", type=int, default=int(os.environ.get("GBDT_LOCAL_SHARDS", "1")),
+                    help="attribute shards inside this process (1, 2, 4 or 8; they pipeline on streams)")
     ap.add_argument("--dense", action="store_true",
                     help="dense representation, absent values filled with 0 (P:116, P:405-413, SURVEY §8(f4))")
     ap.add_argument("--comm", default="nccl", choices=["nccl", "host"],
@@ -233,7 +235,8 @@ def main():
         comm = gbdt.comm_from_callbacks(local) if host_comm else gbdt.comm_from_torch(local)
     stream = torch.cuda.current_stream()
     ds = gbdt.load_csr(prob.indptr, prob.indices, prob.values, prob.labels, prob.m, rle=args.rle,
-                       stream=stream.cuda_stream, comm=comm, keep_rows=args.smartgd == "off", dense=args.dense)
+                       stream=stream.cuda_stream, comm=comm, keep_rows=args.smartgd == "off", dense=args.dense,
+                       n_shards=args.local_shards)
     info = ds.info(0)
     m_local = info["attr_end"] - info["attr_begin"]
     tp = dict(max_depth=d, lam=P["lam"], gamma=P["gamma"], eta=P["eta"], base_margin=P["base_margin"],
@@ -324,7 +327,7 @@ def main():
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         ds2 = gbdt.load_csr(hp, hi, hv, hl, prob.m, rle=args.rle, stream=stream.cuda_stream, comm=comm,
-                            keep_rows=args.smartgd == "off", dense=args.dense)
+                            keep_rows=args.smartgd == "off", dense=args.dense, n_shards=args.local_shards)
         model2, margin2 = gbdt.train(ds2, n_trees=args.steps, want_margin=True, **tp)
         torch.cuda.synchronize()
         te = time.perf_counter() - t0

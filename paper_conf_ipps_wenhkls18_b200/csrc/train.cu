@@ -884,6 +884,28 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
   }
   const double thr = P.gamma > 0 ? P.gamma : 0.0;
 
+  // Several local shards: their partitions and next-level split finds run pipelined on one stream
+  // each (profiling, the fused pass and the level-capture hook keep the sequential order;
+  // GBDT_PIPE=0 forces it)
+  bool pipe = nloc > 1 && !tm.on && !fused && cap_level < 0 && !custom;
+  if (const char* pe = getenv("GBDT_PIPE")) pipe = pipe && pe[0] != '0';
+  struct PipeRes {
+    std::vector<cudaStream_t> st;
+    std::vector<cudaEvent_t> ev;
+    ~PipeRes() {
+      for (auto e : ev) cudaEventDestroy(e);
+      for (auto x : st) cudaStreamDestroy(x);
+    }
+  } pres;
+  if (pipe) {
+    pres.st.resize(nloc, nullptr);
+    pres.ev.resize(1 + 2 * (size_t)nloc, nullptr);
+    for (auto& x : pres.st) GBDT_CUDA(cudaStreamCreateWithFlags(&x, cudaStreamNonBlocking));
+    for (auto& e : pres.ev) GBDT_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  }
+  cudaStream_t* pst = pres.st.data();
+  cudaEvent_t* pev = pres.ev.data();
+
   // One tree of Alg. 1 (every tree-dependent pointer is resolved on the device from tidx, so the
   // same launch sequence builds any tree): captured once into a CUDA graph and replayed T times
   // when nothing in it needs the host (no profiling events, no user-loss callback, no
@@ -914,6 +936,118 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
     count_launch(2);
     tm.end();
 
+    // split find of level L for local shard li on stream s (a3-a6)
+    auto split_shard = [&](int li, int L, cudaStream_t s) {
+      const int lvl = L;
+      NodeTab& cur = nt[L & 1];
+      cudaStream_t st = s;
+        Shard& sh = *ds.shards[li];
+        ShardWork& w = sw[li];
+        if (sh.m == 0) return;
+        const Tables tb = lvl == 0 ? w.root : w.tab[lvl & 1];
+        const float* val = lvl == 0 ? sh.val0.as<float>() : sh.valw[lvl & 1].as<float>();
+        const int32_t* ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
+        SplitArgs A;
+        A.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters, w.level_flag(lvl)};
+        A.desc = w.desc; A.rle = sh.rle ? 1 : 0; A.genlist = w.genlist; A.ngen = w.counters + 2;
+        A.g = gv; A.h = hv; A.nodes = cur; A.segPG = w.segPG; A.segPH = w.segPH; A.lam = P.lambda;
+        A.epochp = epoch; A.fx = fxs; A.rec = w.rec;
+        A.glist = w.glist[lvl & 1]; A.hlist = w.hlist[lvl & 1]; A.cagg = w.cagg; A.carry = w.carry;
+        A.sgrp = w.sgrp; A.nrec = w.nrec; A.gkey = w.gkey; A.shard = sh.index;
+        A.segPG_out = w.segPG; A.segPH_out = w.segPH;
+        // present totals per segment (needed for the missing direction, P:208), from the chunk pass
+        A.segEnd = ds.has_missing ? w.segEnd : nullptr;
+        const bool rs = runsplit && sh.rle;
+        kt.begin(GBDT_PHASE_K_CHUNK_AGG);
+        if (rs) {
+          // the split on runs gathers the root g-list itself (k_run_root)
+        } else if (lvl > 0 && !ds.has_missing) {
+          LK.chunk_desc(A, w.groups, st);  // aggregates from the scatter
+        } else {
+          LK.tile_prefix(A, hmode, /*gather=*/lvl == 0, w.groups, st);
+        }
+        kt.end();
+
+        kt.begin(GBDT_PHASE_K_SPLIT);
+        if (rs) {
+          LK.run_split(A, hmode, /*root=*/lvl == 0, w.racc, w.rcar, w.rsg5, w.rgroups, st);
+        } else {
+          LK.short_split(A, w.level_sl(lvl), hmode, /*gather=*/lvl == 0, st);
+          LK.split_find(A, hmode, ds.has_missing, sh.rle, st);
+        }
+        kt.end();
+        if (P.profile) {  // the level's list entries (byte model of the bench), off the timed kernels
+          k_level_entries<<<(unsigned)std::min<int64_t>(ceil_div(sh.m, 256), sms * 4), 256, 0, st>>>(tb.col_len, sh.m, lent + lvl);
+          GBDT_LAUNCH_CHECK();
+          count_launch();
+        }
+    };
+    // partition of level L for local shard li on stream s (a8); ev_count: recorded after the count
+    auto part_shard = [&](int li, int L, cudaStream_t s, cudaEvent_t ev_count) {
+      const int lvl = L;
+      NodeTab& cur = nt[L & 1];
+      NodeTab& nxt = nt[(L + 1) & 1];
+      const int Kl = 1 << L;
+      cudaStream_t st = s;
+      (void)cur;
+        Shard& sh = *ds.shards[li];
+        ShardWork& w = sw[li];
+        if (sh.m == 0) return;
+        const Tables tb = lvl == 0 ? w.root : w.tab[lvl & 1];
+        const Tables tn = w.tab[(lvl + 1) & 1];
+        const float* val = lvl == 0 ? sh.val0.as<float>() : sh.valw[lvl & 1].as<float>();
+        const int32_t* ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
+        if (ds.has_missing) {
+          const size_t Sl = (size_t)sh.m * Kl;
+          GBDT_CUDA(cudaMemsetAsync(w.segH, 0, Sl * 4, st));
+          GBDT_CUDA(cudaMemsetAsync(w.segL, 0, Sl * 4, st));
+        }
+        PartArgs PA;
+        PA.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters + 1, w.level_flag(lvl)};
+        const ShortList lsl = w.level_sl(lvl);
+        PA.side = side; PA.hbit = hbit; PA.cidx = cidx; PA.slist = w.slist; PA.segH = w.segH; PA.segL = w.segL;
+        PA.seg_pre = w.seg_pre; PA.out_hi = w.out_hi; PA.out_lo = w.out_lo;
+        PA.val_out = sh.valw[(lvl + 1) & 1].as<float>();
+        PA.ins_out = sh.insw[(lvl + 1) & 1].as<int32_t>();
+        PA.ccnt = w.ccnt; PA.cpre = w.cpre; PA.sgrp = w.sgrp;
+        PA.g_in = w.glist[lvl & 1]; PA.h_in = w.hlist[lvl & 1];
+        PA.g_out = w.glist[(lvl + 1) & 1]; PA.h_out = w.hlist[(lvl + 1) & 1];
+        PA.epochp = epoch;
+        // without missing values the scatter accumulates the next level's chunk aggregates
+        PA.cagg_next = (ds.has_missing || (runsplit && sh.rle)) ? nullptr : w.cagg;
+        PA.nxt = tn;
+        PA.fx = fxs;
+        PlanArgs PL;
+        PL.m = sh.m; PL.counted = ds.has_missing; PL.Kp = cur.K; PL.Knp = nxt.K; PL.cidx = cidx; PL.ncnt = nxt.cnt;
+        PL.segH = w.segH; PL.segL = w.segL; PL.seg_pre = w.seg_pre;
+        PL.out_hi = w.out_hi; PL.out_lo = w.out_lo; PL.len_tmp = w.len_tmp; PL.nxt = tn;
+        PL.el = w.pel; PL.egrp = w.pgrp; PL.egroups = w.pgroups; PL.mp1 = w.mp1; PL.sflag = w.level_flag(lvl + 1);
+        RunArgs RA;
+        if (sh.rle) {
+          RA.m = sh.m; RA.Kp = cur.K; RA.Knp = nxt.K; RA.cidx = cidx; RA.cur = tb; RA.nxt = tn;
+          RA.slist = w.slist; RA.cpre = w.cpre; RA.run_seg = w.run_seg; RA.run_hl = w.run_hl; RA.cnt = w.rcnt; RA.fl = w.rfl;
+          RA.Rp1 = w.Rp1; RA.sgrp = w.rsgrp; RA.groups = w.rgroups;
+        }
+        // RLE split ablation (gbdt_params.rle_decompress, P:248 Fig. 6): the runs are decompressed
+        // into the level's value list, the lists partitioned as plain ones, the children re-encoded
+        const bool dec = sh.rle && P.rle_decompress;
+        if (dec && lvl > 0) {
+          LK.rle_decompress(tb, sh.valw[lvl & 1].as<float>(), st);
+          PA.t.val = sh.valw[lvl & 1].as<float>();
+        }
+        kt.begin(GBDT_PHASE_K_COUNT);
+        LK.partition_count(PA, PL, ds.has_missing, w.groups, st, &lsl);
+        if (ev_count) GBDT_CUDA(cudaEventRecord(ev_count, st));  // the next shard's count may start
+        kt.end();
+        kt.begin(GBDT_PHASE_K_SCATTER);
+        if (PA.cagg_next)
+          GBDT_CUDA(cudaMemsetAsync(w.cagg, 0, sizeof(unsigned long long) * 5 * (size_t)std::max<int64_t>(sh.C0, 1), st));
+        LK.partition_scatter(PA, hmode, (sh.rle && !dec) ? &RA : nullptr, st, &lsl);
+        if (dec)
+          LK.rle_encode(tn, sh.m, nxt.K, sh.valw[(lvl + 1) & 1].as<float>(), w.enc_cnt, w.enc_bits,
+                        ((size_t)sh.cap / 32 + 2) * 4, st);
+        kt.end();
+    };
     for (int lvl = 0; lvl < d; ++lvl) {
       NodeTab& cur = nt[lvl & 1];
       NodeTab& nxt = nt[(lvl + 1) & 1];
@@ -968,7 +1102,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       }
       // fz: this level's node bests were found by the previous level's fused pass
       const bool fz = fused && lvl >= 1;
-      if (!fz) {
+      if (!fz && !(pipe && lvl > 0)) {
       tm.begin(GBDT_PHASE_DECIDE);
       k_level_begin<<<1, 1024, 0, st>>>(epoch, sw[0].counters, 0, nrec, nloc, cur.K, gkey, tkey, Kcap);
       GBDT_LAUNCH_CHECK();
@@ -978,46 +1112,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       }
       tm.begin(GBDT_PHASE_SPLIT_FIND);
       for (int li = 0; li < nloc && !fz; ++li) {
-        Shard& sh = *ds.shards[li];
-        ShardWork& w = sw[li];
-        if (sh.m == 0) continue;
-        const Tables tb = lvl == 0 ? w.root : w.tab[lvl & 1];
-        const float* val = lvl == 0 ? sh.val0.as<float>() : sh.valw[lvl & 1].as<float>();
-        const int32_t* ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
-        SplitArgs A;
-        A.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters, w.level_flag(lvl)};
-        A.desc = w.desc; A.rle = sh.rle ? 1 : 0; A.genlist = w.genlist; A.ngen = w.counters + 2;
-        A.g = gv; A.h = hv; A.nodes = cur; A.segPG = w.segPG; A.segPH = w.segPH; A.lam = P.lambda;
-        A.epochp = epoch; A.fx = fxs; A.rec = w.rec;
-        A.glist = w.glist[lvl & 1]; A.hlist = w.hlist[lvl & 1]; A.cagg = w.cagg; A.carry = w.carry;
-        A.sgrp = w.sgrp; A.nrec = w.nrec; A.gkey = w.gkey; A.shard = sh.index;
-        A.segPG_out = w.segPG; A.segPH_out = w.segPH;
-        // present totals per segment (needed for the missing direction, P:208), from the chunk pass
-        A.segEnd = ds.has_missing ? w.segEnd : nullptr;
-        const bool rs = runsplit && sh.rle;
-        kt.begin(GBDT_PHASE_K_CHUNK_AGG);
-        if (rs) {
-          // the split on runs gathers the root g-list itself (k_run_root)
-        } else if (lvl > 0 && !ds.has_missing) {
-          LK.chunk_desc(A, w.groups, st);  // aggregates from the scatter
-        } else {
-          LK.tile_prefix(A, hmode, /*gather=*/lvl == 0, w.groups, st);
-        }
-        kt.end();
-
-        kt.begin(GBDT_PHASE_K_SPLIT);
-        if (rs) {
-          LK.run_split(A, hmode, /*root=*/lvl == 0, w.racc, w.rcar, w.rsg5, w.rgroups, st);
-        } else {
-          LK.short_split(A, w.level_sl(lvl), hmode, /*gather=*/lvl == 0, st);
-          LK.split_find(A, hmode, ds.has_missing, sh.rle, st);
-        }
-        kt.end();
-        if (P.profile) {  // the level's list entries (byte model of the bench), off the timed kernels
-          k_level_entries<<<(unsigned)std::min<int64_t>(ceil_div(sh.m, 256), sms * 4), 256, 0, st>>>(tb.col_len, sh.m, lent + lvl);
-          GBDT_LAUNCH_CHECK();
-          count_launch();
-        }
+        if (pipe && lvl > 0) break;  // found by the pipelined partition of the previous level
+        split_shard(li, lvl, st);
       }
       tm.end();
       tm.begin(GBDT_PHASE_DECIDE);
@@ -1114,63 +1210,27 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         tm.end();
         continue;
       }
-      for (int li = 0; li < nloc; ++li) {
-        Shard& sh = *ds.shards[li];
-        ShardWork& w = sw[li];
-        if (sh.m == 0) continue;
-        const Tables tb = lvl == 0 ? w.root : w.tab[lvl & 1];
-        const Tables tn = w.tab[(lvl + 1) & 1];
-        const float* val = lvl == 0 ? sh.val0.as<float>() : sh.valw[lvl & 1].as<float>();
-        const int32_t* ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
-        if (ds.has_missing) {
-          const size_t Sl = (size_t)sh.m * Kl;
-          GBDT_CUDA(cudaMemsetAsync(w.segH, 0, Sl * 4, st));
-          GBDT_CUDA(cudaMemsetAsync(w.segL, 0, Sl * 4, st));
+      if (pipe) {
+        // Pipelined over the local shards (one stream each): shard li's partition of this level
+        // and its split find of the next; its count starts when shard li-1's count is done, so
+        // the L1TEX-bound count of one shard overlaps the DRAM-bound scatter and the issue-bound
+        // split find of the others.  The next level's begin runs first, on st.
+        k_level_begin<<<1, 1024, 0, st>>>(epoch, sw[0].counters, 0, nrec, nloc, nxt.K, gkey, tkey, Kcap);
+        GBDT_LAUNCH_CHECK();
+        count_launch();
+        for (int li = 0; li < nloc; ++li) GBDT_CUDA(cudaMemsetAsync(sw[li].counters, 0, 4 * sizeof(int), st));
+        GBDT_CUDA(cudaEventRecord(pev[0], st));
+        for (int li = 0; li < nloc; ++li) {
+          cudaStream_t ss = pst[li];
+          GBDT_CUDA(cudaStreamWaitEvent(ss, pev[0], 0));
+          if (li > 0) GBDT_CUDA(cudaStreamWaitEvent(ss, pev[1 + (li - 1)], 0));
+          part_shard(li, lvl, ss, pev[1 + li]);
+          split_shard(li, lvl + 1, ss);
+          GBDT_CUDA(cudaEventRecord(pev[1 + nloc + li], ss));
         }
-        PartArgs PA;
-        PA.t = TileArgs{val, ins, tb, sh.m, sh.a_begin, cur.K, w.counters + 1, w.level_flag(lvl)};
-        const ShortList lsl = w.level_sl(lvl);
-        PA.side = side; PA.hbit = hbit; PA.cidx = cidx; PA.slist = w.slist; PA.segH = w.segH; PA.segL = w.segL;
-        PA.seg_pre = w.seg_pre; PA.out_hi = w.out_hi; PA.out_lo = w.out_lo;
-        PA.val_out = sh.valw[(lvl + 1) & 1].as<float>();
-        PA.ins_out = sh.insw[(lvl + 1) & 1].as<int32_t>();
-        PA.ccnt = w.ccnt; PA.cpre = w.cpre; PA.sgrp = w.sgrp;
-        PA.g_in = w.glist[lvl & 1]; PA.h_in = w.hlist[lvl & 1];
-        PA.g_out = w.glist[(lvl + 1) & 1]; PA.h_out = w.hlist[(lvl + 1) & 1];
-        PA.epochp = epoch;
-        // without missing values the scatter accumulates the next level's chunk aggregates
-        PA.cagg_next = (ds.has_missing || (runsplit && sh.rle)) ? nullptr : w.cagg;
-        PA.nxt = tn;
-        PA.fx = fxs;
-        PlanArgs PL;
-        PL.m = sh.m; PL.counted = ds.has_missing; PL.Kp = cur.K; PL.Knp = nxt.K; PL.cidx = cidx; PL.ncnt = nxt.cnt;
-        PL.segH = w.segH; PL.segL = w.segL; PL.seg_pre = w.seg_pre;
-        PL.out_hi = w.out_hi; PL.out_lo = w.out_lo; PL.len_tmp = w.len_tmp; PL.nxt = tn;
-        PL.el = w.pel; PL.egrp = w.pgrp; PL.egroups = w.pgroups; PL.mp1 = w.mp1; PL.sflag = w.level_flag(lvl + 1);
-        RunArgs RA;
-        if (sh.rle) {
-          RA.m = sh.m; RA.Kp = cur.K; RA.Knp = nxt.K; RA.cidx = cidx; RA.cur = tb; RA.nxt = tn;
-          RA.slist = w.slist; RA.cpre = w.cpre; RA.run_seg = w.run_seg; RA.run_hl = w.run_hl; RA.cnt = w.rcnt; RA.fl = w.rfl;
-          RA.Rp1 = w.Rp1; RA.sgrp = w.rsgrp; RA.groups = w.rgroups;
-        }
-        // RLE split ablation (gbdt_params.rle_decompress, P:248 Fig. 6): the runs are decompressed
-        // into the level's value list, the lists partitioned as plain ones, the children re-encoded
-        const bool dec = sh.rle && P.rle_decompress;
-        if (dec && lvl > 0) {
-          LK.rle_decompress(tb, sh.valw[lvl & 1].as<float>(), st);
-          PA.t.val = sh.valw[lvl & 1].as<float>();
-        }
-        kt.begin(GBDT_PHASE_K_COUNT);
-        LK.partition_count(PA, PL, ds.has_missing, w.groups, st, &lsl);
-        kt.end();
-        kt.begin(GBDT_PHASE_K_SCATTER);
-        if (PA.cagg_next)
-          GBDT_CUDA(cudaMemsetAsync(w.cagg, 0, sizeof(unsigned long long) * 5 * (size_t)std::max<int64_t>(sh.C0, 1), st));
-        LK.partition_scatter(PA, hmode, (sh.rle && !dec) ? &RA : nullptr, st, &lsl);
-        if (dec)
-          LK.rle_encode(tn, sh.m, nxt.K, sh.valw[(lvl + 1) & 1].as<float>(), w.enc_cnt, w.enc_bits,
-                        ((size_t)sh.cap / 32 + 2) * 4, st);
-        kt.end();
+        for (int li = 0; li < nloc; ++li) GBDT_CUDA(cudaStreamWaitEvent(st, pev[1 + nloc + li], 0));
+      } else {
+        for (int li = 0; li < nloc; ++li) part_shard(li, lvl, st, nullptr);
       }
       tm.end();
     }
