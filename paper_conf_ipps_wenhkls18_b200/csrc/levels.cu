@@ -367,7 +367,10 @@ __device__ __forceinline__ void agg_short(const SplitArgs& A, const ChunkMeta& M
 // the chunk's g-list, read from the partition-carried g-list below -- and the chunk's segmented
 // aggregate (sum since its last segment head, fixed association) as an exact fixed-point value.
 template <int HMODE, bool kGather>
-__global__ void __launch_bounds__(kThreads) k_chunk_agg(SplitArgs A) {
+#ifndef GBDT_AGG_CTAS
+#define GBDT_AGG_CTAS 4  // <= 64 registers (~96 B of spills): C4a chunk pass 2.01 -> 1.78 ms/tree, C3/C2 unchanged
+#endif
+__global__ void __launch_bounds__(kThreads, GBDT_AGG_CTAS) k_chunk_agg(SplitArgs A) {
   __shared__ TabCache tc;
   const int lane = threadIdx.x & 31;
   const int K = *A.t.Kp;
@@ -1528,7 +1531,10 @@ __global__ void __launch_bounds__(kThreads) k_short_scatter(PartArgs A, ShortLis
 
 // ---------------------------------------------------------------------------- k_sf_gen
 #ifndef GBDT_GEN_CTAS
-#define GBDT_GEN_CTAS 2
+// 3 CTAs per SM (<= 85 registers; the missing-value variant does not spill): C4a split
+// 5.16 -> 4.11 ms/tree (the kernel stalls on fixed-latency dependencies and instruction fetch,
+// so more warps per SM pay), C4b 0.44 -> 0.47
+#define GBDT_GEN_CTAS 3
 #endif
 #ifndef GBDT_GEN_DYN
 #define GBDT_GEN_DYN 1  // dynamic claim of the chunk steps (missing values)
