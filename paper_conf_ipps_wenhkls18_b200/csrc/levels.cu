@@ -1250,7 +1250,10 @@ __device__ __forceinline__ void sf_short(const SplitArgs& A, NodeBest& B, unsign
 #define GBDT_SF_SHORT_KERNEL 1
 #endif
 template <int HMODE, bool kMissing, bool kRLE>
-__global__ void __launch_bounds__(kThreads) k_sf_short(SplitArgs A) {
+#ifndef GBDT_SFSHORT_CTAS
+#define GBDT_SFSHORT_CTAS 1
+#endif
+__global__ void __launch_bounds__(kThreads, GBDT_SFSHORT_CTAS) k_sf_short(SplitArgs A) {
   __shared__ NodeBest B;
   __shared__ unsigned long long wgk[kWarps][kWarpK];
   __shared__ Rec wrec[kWarps][kWarpK];
@@ -1347,7 +1350,10 @@ __device__ __forceinline__ SLane short_lane(const ShortList& S, const Tables& tb
 }
 
 template <int HMODE, bool kGather>
-__global__ void __launch_bounds__(kThreads) k_short_split(SplitArgs A, ShortList S) {
+#ifndef GBDT_SSPLIT_CTAS
+#define GBDT_SSPLIT_CTAS 1
+#endif
+__global__ void __launch_bounds__(kThreads, GBDT_SSPLIT_CTAS) k_short_split(SplitArgs A, ShortList S) {
   constexpr bool kH = HMODE == kHGather;
   __shared__ NodeBest B;
   __shared__ unsigned long long wgk[kWarps][kWarpK];
@@ -1885,7 +1891,10 @@ __device__ __forceinline__ void count_short(const PartArgs& A, const ChunkMeta& 
 #ifndef GBDT_COUNT_SHORT
 #define GBDT_COUNT_SHORT 1
 #endif
-__global__ void __launch_bounds__(kThreads) k_part_count(PartArgs A, int counted) {
+#ifndef GBDT_COUNT_CTAS
+#define GBDT_COUNT_CTAS 1
+#endif
+__global__ void __launch_bounds__(kThreads, GBDT_COUNT_CTAS) k_part_count(PartArgs A, int counted) {
   __shared__ TabCache tc;
   const int lane = threadIdx.x & 31;
   const int K = *A.t.Kp;
@@ -2663,7 +2672,10 @@ __global__ void __launch_bounds__(kThreads) k_run_init(SplitArgs A, unsigned lon
 // low-cardinality lists), two chunks in flight per warp: lane sums in item order, a butterfly, one
 // exact add per total.  Chunks holding several runs are listed (A.genlist) for k_run_agg_multi.
 template <int HMODE>
-__global__ void __launch_bounds__(kThreads) k_run_agg(SplitArgs A, unsigned long long* __restrict__ racc) {
+#ifndef GBDT_RUNAGG_CTAS
+#define GBDT_RUNAGG_CTAS 6  // C5 RLE split 2.42 -> 2.27 ms/tree
+#endif
+__global__ void __launch_bounds__(kThreads, GBDT_RUNAGG_CTAS) k_run_agg(SplitArgs A, unsigned long long* __restrict__ racc) {
   constexpr bool kH = HMODE == kHGather;
   __shared__ TabCache tc;
   const int lane = threadIdx.x & 31;
