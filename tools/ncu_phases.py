@@ -17,7 +17,8 @@ def short(name):
 
 def phase_of(name):
     n = short(name)
-    if n.startswith(("k_chunk_agg", "k_desc", "k_sf_", "k_seg_totals")) or n.startswith("k_scan") and "<1>" in n:
+    if n.startswith(("k_chunk_agg", "k_desc", "k_sf_", "k_seg_totals", "k_short_split", "k_run_root", "k_run_agg",
+                     "k_run_init", "k_run_split")) or n.startswith("k_scan") and "<1>" in n:
         return "split_find"
     if n.startswith(("k_part_", "k_plan_", "k_chunk_attr", "k_run_", "k_tile_agg", "k_tscan", "k_fused")) or \
             n.startswith("k_scan") and "<0>" in n:
