@@ -368,9 +368,10 @@ __device__ __forceinline__ void agg_short(const SplitArgs& A, const ChunkMeta& M
 // aggregate (sum since its last segment head, fixed association) as an exact fixed-point value.
 template <int HMODE, bool kGather>
 #ifndef GBDT_AGG_CTAS
-#define GBDT_AGG_CTAS 4  // <= 64 registers (~96 B of spills): C4a chunk pass 2.01 -> 1.78 ms/tree, C3/C2 unchanged
-#endif
-__global__ void __launch_bounds__(kThreads, GBDT_AGG_CTAS) k_chunk_agg(SplitArgs A) {
+#define GBDT_AGG_CTAS 4  // list-reading instantiation (missing values, below the root): <= 64 registers
+#endif                   // (~96 B of spills), C4a chunk pass 2.01 -> 1.78 ms/tree; the root gather stays at
+                         // 3 CTAs/SM (C3 root 3.33 vs 3.37 ms/tree at 4)
+__global__ void __launch_bounds__(kThreads, kGather ? 3 : GBDT_AGG_CTAS) k_chunk_agg(SplitArgs A) {
   __shared__ TabCache tc;
   const int lane = threadIdx.x & 31;
   const int K = *A.t.Kp;

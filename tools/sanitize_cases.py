@@ -1,4 +1,4 @@
-"""Small trainings covering every kernel family (dense, missing values, sparse short lists, RLE and
+"""Small trainings covering every kernel family (dense, missing values, sparse short lists, RLE (split on runs) and
 its decompression ablation, AUTO RLE, dense representation, loopback shards, deep trees,
 SmartGD-off, the fused dense pass, prediction), for compute-sanitizer runs."""
 import os
@@ -20,6 +20,12 @@ cases = [
     ("rle_auto", synth.c2(n=6000, T=2), {"rle": "auto"}),
     ("dense_repr", synth.c4(seed=12, n=800, m=200, density=0.05, T=2), {"dense": True}),
     ("fused", synth.c3(n=20000, T=2), {"_env": "GBDT_FUSED"}),
+    # round 2: the split on runs (multi-run chunks, shards pipelined on streams, depth 8)
+    ("rle_many_runs", synth.random_small(8, n=9000, m=5, nan_frac=0.0, n_distinct=3000), {"rle": "on"}),
+    ("rle_shards", synth.c5(n=20000, T=2), {"rle": "on", "n_shards": 2}),
+    ("rle_deep", synth.random_small(81, n=7000, m=4, nan_frac=0.0, n_distinct=200, loss="logistic", d=8, T=2),
+     {"rle": "on"}),
+    ("dense_shards", synth.c3(n=20000, T=2), {"n_shards": 4}),
 ]
 for name, p, kw in cases:
     env = kw.pop("_env", None)
