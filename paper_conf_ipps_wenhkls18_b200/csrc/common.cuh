@@ -183,9 +183,10 @@ enum { kHConst2 = 0, kHFromG = 1, kHGather = 2 };
 template <int HMODE>
 __device__ __forceinline__ double hess_of(double g) {
   if (HMODE == kHConst2) return 2.0;
-  // logistic, 0/1 labels: y = [g < 0] (g = p - y with p in [0,1]); q = g + y (K1)
-  const double q = g < 0.0 ? __dadd_rn(g, 1.0) : g;
-  const double hh = __dmul_rn(q, __dsub_rn(1.0, q));
+  // logistic, 0/1 labels: g = p - y with p in [0,1], so |g| is 1 - p (y = 1) or p (y = 0) and
+  // h = |g| (1 - |g|) = p (1 - p) (K1); |g| is an operand modifier, no select
+  const double a = fabs(g);
+  const double hh = __dmul_rn(a, __dsub_rn(1.0, a));
   // max(hh, 1e-16); hh is never NaN (q in [0, 1]), so a plain compare-select (no fmax NaN rules)
   double r;
   asm("{\n .reg .pred p;\n setp.lt.f64 p, %1, 0d3C9CD2B297D889BC;\n selp.f64 %0, 0d3C9CD2B297D889BC, %1, p;\n}"
