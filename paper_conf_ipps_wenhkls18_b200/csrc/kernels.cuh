@@ -79,6 +79,10 @@ struct SplitArgs {
   double* segPH_out;     //   + k_seg_totals
   int32_t* segEnd;       // [m*K] chunk holding the segment's last entry if the segment began in an
                          // earlier chunk, else -1; nullptr: no missing values
+  // the attributes not on the short path (k_seg_totals walks only their segments while the short
+  // path is active); nullptr: every attribute
+  const int32_t* longa = nullptr;
+  int nlong = 0;
 };
 
 struct PartArgs {

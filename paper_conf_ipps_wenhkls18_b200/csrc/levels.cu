@@ -3225,9 +3225,12 @@ __global__ void __launch_bounds__(kThreads) k_seg_totals(SplitArgs A) {
   const int K = *A.t.Kp;
   const long long S = (long long)A.t.m * K;
   const bool sp = A.t.sflag && K <= 32;  // the short path's segments sum their own totals
-  for (long long s = blockIdx.x * (long long)blockDim.x + threadIdx.x; s < S; s += (long long)gridDim.x * blockDim.x) {
+  const bool la = sp && A.longa;          // ... so only the other attributes' segments are walked
+  const long long N = la ? (long long)A.nlong * K : S;
+  for (long long t = blockIdx.x * (long long)blockDim.x + threadIdx.x; t < N; t += (long long)gridDim.x * blockDim.x) {
+    const long long s = la ? (long long)A.longa[t / K] * K + t % K : t;
     if (A.t.tb.seg_cnt[s] == 0) continue;
-    if (sp && A.t.sflag[s / K]) continue;
+    if (sp && !la && A.t.sflag[s / K]) continue;
     const int ce = A.segEnd[s];
     if (ce < 0) continue;
     const CarryD cx = carry_load(A.carry + 5ll * ce);

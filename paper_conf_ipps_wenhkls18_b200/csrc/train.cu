@@ -487,6 +487,8 @@ struct ShardWork {
   // chunk lists of the root and of the two level tables
   DBuf shortmem;
   ShortList sl;
+  int32_t* longa = nullptr;  // the attributes not on the short path
+  int nlong = 0;
   uint8_t* sflag = nullptr;
   uint8_t* jl[2] = {nullptr, nullptr};  // node index of each short-list entry, two levels
   // the level's short-path arguments (levels 0..kShortLevels-1, where K <= 32), else none
@@ -813,6 +815,9 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
       if (!attrs.empty()) {
         std::vector<uint8_t> flag((size_t)m, 0);
         for (int32_t a : attrs) flag[(size_t)a] = 1;
+        std::vector<int32_t> longa;  // the other attributes (k_seg_totals)
+        for (int a = 0; a < m; ++a)
+          if (!flag[(size_t)a]) longa.push_back(a);
         std::vector<int32_t> lc;  // root chunks of the other attributes (chunk_start as build_layout)
         lc.reserve((size_t)C0);
         int32_t cs = 0;
@@ -837,7 +842,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         auto zs = [&](Carve& z) {
           z.take<int32_t>(attrs.size()); z.take<uint8_t>((size_t)m); z.take<int32_t>((size_t)C0); z.take<int32_t>(4);
           z.take<int32_t>((size_t)C0); z.take<int32_t>((size_t)C0); z.take<int2>(batch.size());
-          z.take<uint8_t>((size_t)sh.cap); z.take<uint8_t>((size_t)sh.cap);
+          z.take<uint8_t>((size_t)sh.cap); z.take<uint8_t>((size_t)sh.cap); z.take<int32_t>(longa.size() + 1);
         };
         zs(zp);
         w.shortmem.alloc(zp.off + 1024, st);
@@ -851,6 +856,10 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         int2* d_batch = z.take<int2>(batch.size());
         w.jl[0] = z.take<uint8_t>((size_t)sh.cap);
         w.jl[1] = z.take<uint8_t>((size_t)sh.cap);
+        w.longa = z.take<int32_t>(longa.size() + 1);
+        w.nlong = (int)longa.size();
+        if (!longa.empty())
+          GBDT_CUDA(cudaMemcpyAsync(w.longa, longa.data(), 4 * longa.size(), cudaMemcpyHostToDevice, st));
         w.root.lc = rlc;
         w.root.nlc = nl;
         w.tab[0].nlc = nl + 1;
@@ -957,6 +966,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         A.segPG_out = w.segPG; A.segPH_out = w.segPH;
         // present totals per segment (needed for the missing direction), from the chunk pass
         A.segEnd = ds.has_missing ? w.segEnd : nullptr;
+        if (w.level_flag(lvl)) { A.longa = w.longa; A.nlong = w.nlong; }
         const bool rs = runsplit && sh.rle;
         kt.begin(GBDT_PHASE_K_CHUNK_AGG);
         if (rs) {
