@@ -164,67 +164,103 @@ __global__ void k_layout_scatter(int64_t N, int m, const unsigned long long* __r
   }
 }
 
-// RLE: one run per maximal group of equal values inside an attribute list.
-__global__ void k_run_heads(int m, const int64_t* __restrict__ col_start, const int64_t* __restrict__ col_len,
-                            const float* __restrict__ val, uint32_t* __restrict__ run_count) {
-  // one block per attribute
-  for (int a = blockIdx.x; a < m; a += gridDim.x) {
-    const int64_t s = col_start[a], L = col_len[a];
+// RLE: one run per maximal group of equal values inside an attribute list.  The lists are
+// cut into PIECES of at most kRunPiece entries of one attribute (host-built, int4: attribute, first
+// entry within the list, length, 0); one block per piece, so a few long attributes (C5: 18 lists of
+// 5 M entries) use the whole GPU.  A run head is an entry whose value differs from its predecessor
+// in the list (or the list's first entry).
+constexpr int kRunPiece = 16384;
+
+__device__ __forceinline__ bool run_head(const float* __restrict__ val, int64_t s, int64_t q) {
+  return q == 0 || val[s + q] != val[s + q - 1];
+}
+
+// heads per piece (and per attribute)
+__global__ void __launch_bounds__(256) k_run_heads(const int4* __restrict__ pieces, int np,
+                                                   const int64_t* __restrict__ col_start,
+                                                   const float* __restrict__ val, uint32_t* __restrict__ piece_cnt,
+                                                   uint32_t* __restrict__ run_count) {
+  __shared__ uint32_t ws[8];
+  for (int pi = blockIdx.x; pi < np; pi += gridDim.x) {
+    const int4 P = pieces[pi];
+    const int64_t s = col_start[P.x];
     uint32_t c = 0;
-    for (int64_t r = threadIdx.x; r < L; r += blockDim.x)
-      c += (r == 0 || val[s + r] != val[s + r - 1]) ? 1u : 0u;
+    for (int64_t q = P.y + threadIdx.x; q < (int64_t)P.y + P.z; q += blockDim.x) c += run_head(val, s, q) ? 1u : 0u;
     for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
-    __shared__ uint32_t ws[32];
     if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = c;
     __syncthreads();
     if (threadIdx.x == 0) {
       uint32_t t = 0;
-      for (int i = 0; i < (int)(blockDim.x >> 5); ++i) t += ws[i];
-      run_count[a] = t;
+      for (int i = 0; i < 8; ++i) t += ws[i];
+      piece_cnt[pi] = t;
+      if (run_count) atomicAdd(run_count + P.x, t);
     }
     __syncthreads();
   }
 }
 
-__global__ void k_run_fill(int m, const int64_t* __restrict__ col_start, const int64_t* __restrict__ col_len,
-                           const float* __restrict__ val, const int64_t* __restrict__ run_ptr,
-                           float* __restrict__ run_val, int32_t* __restrict__ run_len) {
-  // one warp per attribute walks its list serially in 32-wide chunks (load time only)
-  const int lane = threadIdx.x & 31;
-  for (int a = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5); a < m; a += gridDim.x * (blockDim.x / 32)) {
-    const int64_t s = col_start[a], L = col_len[a];
-    int64_t r = run_ptr[a] - 1;  // current run index (before the first head)
-    int64_t run_begin = 0;
-    for (int64_t base = 0; base < L; base += 32) {
-      const int64_t q = base + lane;
-      const bool head = q < L && (q == 0 || val[s + q] != val[s + q - 1]);
-      const unsigned hm = __ballot_sync(0xffffffffu, head);
-      // close runs: each head at q closes the previous run [run_begin, q)
-      unsigned mm = hm;
-      while (mm) {
-        const int l = __ffs(mm) - 1;
-        mm &= mm - 1;
-        const int64_t qh = base + l;
-        if (r >= run_ptr[a] && lane == 0) run_len[r] = (int32_t)(qh - run_begin);
-        ++r;
-        run_begin = qh;
-        if (lane == 0) run_val[r] = val[s + qh];
+// every head writes its run: value and list position (the run index = the piece's first run + the
+// heads before it in the piece, by a block scan per 256-entry tile)
+__global__ void __launch_bounds__(256) k_run_fill(const int4* __restrict__ pieces, int np,
+                                                  const int64_t* __restrict__ col_start, const float* __restrict__ val,
+                                                  const int64_t* __restrict__ piece_run, float* __restrict__ run_val,
+                                                  int64_t* __restrict__ run_pos) {
+  __shared__ uint32_t ws[8];
+  __shared__ int64_t base_s;
+  for (int pi = blockIdx.x; pi < np; pi += gridDim.x) {
+    const int4 P = pieces[pi];
+    const int64_t s = col_start[P.x];
+    if (threadIdx.x == 0) base_s = piece_run[pi];
+    __syncthreads();
+    int64_t base = base_s;
+    for (int64_t t0 = P.y; t0 < (int64_t)P.y + P.z; t0 += blockDim.x) {
+      const int64_t q = t0 + threadIdx.x;
+      const bool h = q < (int64_t)P.y + P.z && run_head(val, s, q);
+      const unsigned bm = __ballot_sync(0xffffffffu, h);
+      const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+      if (lane == 0) ws[w] = __popc(bm);
+      __syncthreads();
+      uint32_t before = 0, tot = 0;
+      for (int i = 0; i < 8; ++i) { before += i < w ? ws[i] : 0u; tot += ws[i]; }
+      if (h) {
+        const int64_t r = base + before + __popc(bm & ((1u << lane) - 1u));
+        run_val[r] = val[s + q];
+        run_pos[r] = s + q;
       }
+      base += tot;
+      __syncthreads();
     }
-    if (L > 0 && lane == 0) run_len[r] = (int32_t)(L - run_begin);
   }
 }
 
-// run positions in the padded list: prefix of the run lengths inside each attribute
-__global__ void k_run_pos(int m, const int64_t* __restrict__ col_start, const int64_t* __restrict__ run_ptr,
-                          const int32_t* __restrict__ run_len, int64_t* __restrict__ run_pos,
-                          int32_t* __restrict__ seg_run, int32_t* __restrict__ R) {
+// run lengths from the positions; the segment -> run table of the root (one segment per
+// attribute) and the run count
+__global__ void k_run_pos(int m, const int64_t* __restrict__ col_start, const int64_t* __restrict__ col_len,
+                          const int64_t* __restrict__ run_ptr, const int64_t* __restrict__ run_pos,
+                          int32_t* __restrict__ run_len, int32_t* __restrict__ seg_run, int32_t* __restrict__ R) {
+  const int64_t Rn = run_ptr[m];
   for (int a = blockIdx.x * blockDim.x + threadIdx.x; a <= m; a += gridDim.x * blockDim.x) {
     seg_run[a] = (int32_t)run_ptr[a];
-    if (a == m) { *R = (int32_t)run_ptr[m]; continue; }
-    int64_t p = col_start[a];
-    for (int64_t r = run_ptr[a]; r < run_ptr[a + 1]; ++r) { run_pos[r] = p; p += run_len[r]; }
+    if (a == m) *R = (int32_t)Rn;
   }
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < Rn; r += (int64_t)gridDim.x * blockDim.x) {
+    int lo = 0, hi = m - 1;  // attribute of run r: the largest a with run_ptr[a] <= r
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (run_ptr[mid] <= r) lo = mid; else hi = mid - 1;
+    }
+    const int64_t end = r + 1 < run_ptr[lo + 1] ? run_pos[r + 1] : col_start[lo] + col_len[lo];
+    run_len[r] = (int32_t)(end - run_pos[r]);
+  }
+}
+
+// pieces of the lists of a shard (host)
+static std::vector<int4> run_pieces(const Shard& sh) {
+  std::vector<int4> pc;
+  for (int a = 0; a < sh.m; ++a)
+    for (int64_t o = 0; o < sh.h_col_len[(size_t)a]; o += kRunPiece)
+      pc.push_back(make_int4(a, (int)o, (int)std::min<int64_t>(kRunPiece, sh.h_col_len[(size_t)a] - o), 0));
+  return pc;
 }
 
 __global__ void k_run_chunk_root(int m, Tables tb) {
@@ -295,10 +331,17 @@ void densify(int64_t n, int64_t m, const int64_t* d_indptr, const int32_t* d_idx
 std::vector<uint32_t> attribute_runs(const Shard& sh, cudaStream_t st, int sms) {
   std::vector<uint32_t> hc((size_t)std::max(sh.m, 0), 0u);
   if (sh.m == 0 || sh.nnz == 0) return hc;
-  DBuf cnt((size_t)sh.m * 4, st);
-  k_run_heads<<<(unsigned)std::min(sh.m, sms * 8), 256, 0, st>>>(sh.m, sh.root.col_start, sh.root.col_len,
-                                                               sh.val0.as<float>(), cnt.as<uint32_t>());
-  GBDT_LAUNCH_CHECK();
+  const std::vector<int4> pc = run_pieces(sh);
+  const int np = (int)pc.size();
+  DBuf cnt((size_t)sh.m * 4, st), dpc((size_t)std::max(np, 1) * 16, st), pcnt((size_t)std::max(np, 1) * 4, st);
+  GBDT_CUDA(cudaMemsetAsync(cnt.p, 0, (size_t)sh.m * 4, st));
+  if (np) {
+    GBDT_CUDA(cudaMemcpyAsync(dpc.p, pc.data(), (size_t)np * 16, cudaMemcpyHostToDevice, st));
+    k_run_heads<<<(unsigned)std::min(np, sms * 16), 256, 0, st>>>(dpc.as<int4>(), np, sh.root.col_start,
+                                                                 sh.val0.as<float>(), pcnt.as<uint32_t>(),
+                                                                 cnt.as<uint32_t>());
+    GBDT_LAUNCH_CHECK();
+  }
   GBDT_CUDA(cudaMemcpyAsync(hc.data(), cnt.p, (size_t)sh.m * 4, cudaMemcpyDeviceToHost, st));
   GBDT_CUDA(cudaStreamSynchronize(st));
   return hc;
@@ -431,12 +474,20 @@ void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices
 
     // ---- optional RLE of the sorted lists
     if (ds.rle != GBDT_RLE_OFF) {
-      DBuf cnt((size_t)m * 4, st);
-      k_run_heads<<<(unsigned)std::min(m, sms * 8), 256, 0, st>>>(m, sh.root.col_start, sh.root.col_len,
-                                                                 sh.val0.as<float>(), cnt.as<uint32_t>());
-      GBDT_LAUNCH_CHECK();
-      std::vector<uint32_t> hc(m);
+      const std::vector<int4> pc = run_pieces(sh);
+      const int np = (int)pc.size();
+      DBuf cnt((size_t)m * 4, st), dpc((size_t)std::max(np, 1) * 16, st), pcnt((size_t)std::max(np, 1) * 4, st);
+      GBDT_CUDA(cudaMemsetAsync(cnt.p, 0, (size_t)m * 4, st));
+      if (np) {
+        GBDT_CUDA(cudaMemcpyAsync(dpc.p, pc.data(), (size_t)np * 16, cudaMemcpyHostToDevice, st));
+        k_run_heads<<<(unsigned)std::min(np, sms * 16), 256, 0, st>>>(dpc.as<int4>(), np, sh.root.col_start,
+                                                                     sh.val0.as<float>(), pcnt.as<uint32_t>(),
+                                                                     cnt.as<uint32_t>());
+        GBDT_LAUNCH_CHECK();
+      }
+      std::vector<uint32_t> hc(m), hp((size_t)np);
       GBDT_CUDA(cudaMemcpyAsync(hc.data(), cnt.p, (size_t)m * 4, cudaMemcpyDeviceToHost, st));
+      if (np) GBDT_CUDA(cudaMemcpyAsync(hp.data(), pcnt.p, (size_t)np * 4, cudaMemcpyDeviceToHost, st));
       GBDT_CUDA(cudaStreamSynchronize(st));
       int64_t R = 0, entries = 0;
       for (int a = 0; a < m; ++a) { R += hc[a]; entries += sh.h_col_len[a]; }
@@ -445,23 +496,33 @@ void build_layout(Dataset& ds, const int64_t* d_indptr, const int32_t* d_indices
       if (ds.rle == GBDT_RLE_ON || ratio >= thr) {
         std::vector<int64_t> rp(m + 1, 0);
         for (int a = 0; a < m; ++a) rp[a + 1] = rp[a] + hc[a];
+        std::vector<int64_t> prun((size_t)std::max(np, 1), 0);  // first run of every piece
+        {
+          int64_t acc = 0;
+          for (int i = 0; i < np; ++i) { prun[(size_t)i] = acc; acc += hp[(size_t)i]; }
+        }
         sh.rle = true;
         sh.runs = R;
         sh.run_ptr.alloc((size_t)(m + 1) * 8, st);
         sh.run_val.alloc((size_t)std::max<int64_t>(R, 1) * 4 + 64, st);
         sh.run_len.alloc((size_t)std::max<int64_t>(R, 1) * 4 + 64, st);
-        GBDT_CUDA(cudaMemcpyAsync(sh.run_ptr.p, rp.data(), (size_t)(m + 1) * 8, cudaMemcpyHostToDevice, st));
-        k_run_fill<<<(unsigned)std::min<int64_t>(ceil_div(m, 8), (int64_t)sms * 8), 256, 0, st>>>(
-            m, sh.root.col_start, sh.root.col_len, sh.val0.as<float>(), sh.run_ptr.as<int64_t>(),
-            sh.run_val.as<float>(), sh.run_len.as<int32_t>());
-        GBDT_LAUNCH_CHECK();
         sh.run_pos.alloc((size_t)std::max<int64_t>(R, 1) * 8 + 64, st);
+        DBuf dprun((size_t)std::max(np, 1) * 8, st);
+        GBDT_CUDA(cudaMemcpyAsync(sh.run_ptr.p, rp.data(), (size_t)(m + 1) * 8, cudaMemcpyHostToDevice, st));
+        if (np) {
+          GBDT_CUDA(cudaMemcpyAsync(dprun.p, prun.data(), (size_t)np * 8, cudaMemcpyHostToDevice, st));
+          k_run_fill<<<(unsigned)std::min(np, sms * 16), 256, 0, st>>>(dpc.as<int4>(), np, sh.root.col_start,
+                                                                      sh.val0.as<float>(), dprun.as<int64_t>(),
+                                                                      sh.run_val.as<float>(), sh.run_pos.as<int64_t>());
+          GBDT_LAUNCH_CHECK();
+        }
         sh.run_seg.alloc((size_t)(m + 1) * 4 + 64, st);
         int32_t* Rdev = reinterpret_cast<int32_t*>(sh.run_seg.as<char>() + (size_t)(m + 1) * 4 + 16);
-        k_run_pos<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(m + 1, 256), (int64_t)sms * 4)), 256, 0, st>>>(
-            m, sh.root.col_start, sh.run_ptr.as<int64_t>(), sh.run_len.as<int32_t>(), sh.run_pos.as<int64_t>(),
-            sh.run_seg.as<int32_t>(), Rdev);
+        k_run_pos<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(std::max<int64_t>(R, m + 1), 256), (int64_t)sms * 8)), 256, 0, st>>>(
+            m, sh.root.col_start, sh.root.col_len, sh.run_ptr.as<int64_t>(), sh.run_pos.as<int64_t>(),
+            sh.run_len.as<int32_t>(), sh.run_seg.as<int32_t>(), Rdev);
         GBDT_LAUNCH_CHECK();
+        GBDT_CUDA(cudaStreamSynchronize(st));  // the host vectors (pieces, piece runs) outlive the copies
         sh.root.seg_run = sh.run_seg.as<int32_t>();
         sh.root.run_val = sh.run_val.as<float>();
         sh.root.run_len = sh.run_len.as<int32_t>();
