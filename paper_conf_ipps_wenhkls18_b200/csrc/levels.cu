@@ -3212,6 +3212,13 @@ void launch_short(const SplitArgs& A, bool missing, bool rle, unsigned grid, cud
 template <bool kFx>
 void launch_scan(const int32_t* Cp, unsigned long long* in, unsigned long long* gbuf, unsigned long long* out,
                  unsigned groups, cudaStream_t st, const int32_t* fx = nullptr) {
+  if (groups == 1) {  // one group (e.g. the plan's scan over the attributes): its carry is zero --
+    // gbuf is never written when a buffer's bound is one group, and it starts zeroed
+    k_scan3<kFx><<<1, kThreads, 0, st>>>(Cp, in, gbuf, out, fx);
+    GBDT_LAUNCH_CHECK();
+    count_launch(1);
+    return;
+  }
   k_scan1<kFx><<<groups, kThreads, 0, st>>>(Cp, in, gbuf);
   k_scan2<kFx><<<1, kScan2Threads, 0, st>>>(Cp, gbuf);
   k_scan3<kFx><<<groups, kThreads, 0, st>>>(Cp, in, gbuf, out, fx);
