@@ -2706,10 +2706,16 @@ __global__ void __launch_bounds__(kThreads, GBDT_RUNAGG_CTAS) k_run_agg(SplitArg
         len[u] = (int)(M.p1 - M.p0);
         rb[u] = tb.run_chunk[cu];
       }
-      // the g loads do not wait for the run lookup (a multi-run chunk wastes them)
+      // the g loads do not wait for the run lookup (a multi-run chunk wastes them); full chunks
+      // (nearly all) without per-item predicates
       const double* gp = A.glist + p0[u] + lane;
+      if (len[u] == kChunk) {
 #pragma unroll
-      for (int k = 0; k < kItems; ++k) g[u][k] = (32 * k + lane < len[u]) ? __ldcs(gp + 32 * k) : 0.0;
+        for (int k = 0; k < kItems; ++k) g[u][k] = __ldcs(gp + 32 * k);
+      } else {
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) g[u][k] = (32 * k + lane < len[u]) ? __ldcs(gp + 32 * k) : 0.0;
+      }
     }
 #pragma unroll
     for (int u = 0; u < 2; ++u) {
@@ -2725,22 +2731,29 @@ __global__ void __launch_bounds__(kThreads, GBDT_RUNAGG_CTAS) k_run_agg(SplitArg
         continue;
       }
       double sg = 0.0, sh = 0.0;
+      if (len[u] == kChunk) {
 #pragma unroll
-      for (int k = 0; k < kItems; ++k) {
-        const bool in = 32 * k + lane < len[u];
-        const double hk = in ? (kH ? __ldcs(A.hlist + p0[u] + 32 * k + lane) : hess_of<HMODE>(g[u][k])) : 0.0;
-        sg = sg + g[u][k];
-        sh = sh + hk;
+        for (int k = 0; k < kItems; ++k) {
+          const double hk = kH ? __ldcs(A.hlist + p0[u] + 32 * k + lane) : hess_of<HMODE>(g[u][k]);
+          sg = sg + g[u][k];
+          sh = sh + hk;
+        }
+      } else {
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+          const bool in = 32 * k + lane < len[u];
+          const double hk = in ? (kH ? __ldcs(A.hlist + p0[u] + 32 * k + lane) : hess_of<HMODE>(g[u][k])) : 0.0;
+          sg = sg + g[u][k];
+          sh = sh + hk;
+        }
       }
 #pragma unroll
       for (int o = 16; o; o >>= 1) {
         sg = sg + __shfl_xor_sync(0xffffffffu, sg, o);
         sh = sh + __shfl_xor_sync(0xffffffffu, sh, o);
       }
-      if (lane == 0) {
-        fx_atomic_add(racc + 5ll * rb[u], to_fx(sg, Fg));
-        fx_atomic_add(racc + 5ll * rb[u] + 2, to_fx(sh, Fh));
-      }
+      // g and h totals converted and added by two lanes at once
+      if (lane < 2) fx_atomic_add(racc + 5ll * rb[u] + 2 * lane, to_fx(lane ? sh : sg, lane ? Fh : Fg));
     }
   }
 }
