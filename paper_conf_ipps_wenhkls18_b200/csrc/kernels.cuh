@@ -36,6 +36,17 @@ struct ShortList {
   int nb = 0;
   const uint8_t* jl = nullptr;     // per list entry: its node j at this level (nullptr: root, j = 0)
   uint8_t* jl_out = nullptr;       // the next level's, written by the scatter (nullptr: not needed)
+  // In-place mode (trees of depth <= 6): the short lists are never partitioned.  They stay in the
+  // root layout (cs0 / cl0, the root values, g in gsh / hsh at root positions), every entry keeps
+  // its node index in jl (0xff: its node became a leaf), updated in place by k_short_update, and
+  // the split find sorts a list's lanes by node (stable: the partitioned order) before its scans.
+  int inplace = 0;
+  const int64_t* cs0 = nullptr;
+  const int64_t* cl0 = nullptr;
+  const float* val0 = nullptr;
+  const int32_t* ins0 = nullptr;
+  double* gsh = nullptr;
+  double* hsh = nullptr;
 };
 
 

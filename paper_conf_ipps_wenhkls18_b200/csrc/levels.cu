@@ -1336,10 +1336,37 @@ __device__ __forceinline__ SLane short_lane(const ShortList& S, const Tables& tb
   L.a = sub < (b.y & 0xffff) ? S.attrs[b.x + sub] : -1;
   long long len = 0;
   L.p0 = 0;
-  if (L.a >= 0) { L.p0 = tb.col_start[L.a]; len = tb.col_len[L.a]; }
+  if (L.a >= 0) {
+    L.p0 = S.inplace ? S.cs0[L.a] : tb.col_start[L.a];
+    len = S.inplace ? S.cl0[L.a] : tb.col_len[L.a];
+  }
   L.valid = e < len;
   L.p = L.p0 + e;
   L.j = (L.valid && S.jl) ? (int)S.jl[L.p] : 0;
+  if (S.inplace && S.jl) {
+    // in-place lists: the group's lanes sorted by node, stably (= the partitioned list), the
+    // entries of nodes that became leaves (0xff) and the lanes past the list at the end
+    const int key = (L.valid && L.j != 0xff) ? L.j : 63;
+    unsigned m = L.gm;
+    int less = 0;
+#pragma unroll
+    for (int bt = 5; bt >= 0; --bt) {
+      const unsigned bal = __ballot_sync(0xffffffffu, (key >> bt) & 1);
+      if ((key >> bt) & 1) { less += __popc(m & ~bal); m &= bal; } else { m &= ~bal; }
+    }
+    const int dest = sub * W + less + __popc(m & ((1u << lane) - 1u));
+    unsigned cand = 0xffffffffu;  // the lane whose entry lands on this lane
+#pragma unroll
+    for (int bt = 0; bt < 5; ++bt) {
+      const unsigned bal = __ballot_sync(0xffffffffu, (dest >> bt) & 1);
+      cand &= ((lane >> bt) & 1) ? bal : ~bal;
+    }
+    const int src = __ffs(cand) - 1;
+    const int ks = __shfl_sync(0xffffffffu, key, src);
+    L.valid = ks != 63;
+    L.j = L.valid ? ks : 0;
+    L.p = L.p0 + (src & (W - 1));
+  }
   const int jp = __shfl_up_sync(0xffffffffu, L.j, 1);
   L.hm = __ballot_sync(0xffffffffu, L.valid && (e == 0 || jp != L.j));
   const unsigned vm = __ballot_sync(0xffffffffu, L.valid) & L.gm;
@@ -1375,16 +1402,19 @@ __global__ void __launch_bounds__(kThreads, GBDT_SSPLIT_CTAS) k_short_split(Spli
     float v = 0.f;
     double g = 0.0, h = 0.0;
     if (L.valid) {
-      v = __ldcs(A.t.val + L.p);
+      // in-place lists: root values and the short lists' own g-list, at root positions
+      double* const gl = S.inplace ? S.gsh : A.glist;
+      double* const hl = S.inplace ? S.hsh : A.hlist;
+      v = __ldcs((S.inplace ? S.val0 : A.t.val) + L.p);
       if (kGather) {
-        const int id = __ldcs(A.t.ins + L.p);
+        const int id = __ldcs((S.inplace ? S.ins0 : A.t.ins) + L.p);
         g = ld_keep(A.g + id, pol_keep);
         h = kH ? ld_keep(A.h + id, pol_keep) : hess_of<HMODE>(g);
-        __stcs(A.glist + L.p, g);
-        if (kH) __stcs(A.hlist + L.p, h);
+        __stcs(gl + L.p, g);
+        if (kH) __stcs(hl + L.p, h);
       } else {
-        g = __ldcs(A.glist + L.p);
-        h = kH ? __ldcs(A.hlist + L.p) : hess_of<HMODE>(g);
+        g = __ldcs(gl + L.p);
+        h = kH ? __ldcs(hl + L.p) : hess_of<HMODE>(g);
       }
     }
     // segmented inclusive scan (k_sf_short's association)
@@ -1433,6 +1463,7 @@ __global__ void __launch_bounds__(kThreads, GBDT_SSPLIT_CTAS) k_short_split(Spli
     const double wg = __shfl_sync(0xffffffffu, ig, q), wh = __shfl_sync(0xffffffffu, ih, q);
     const int wd = __shfl_sync(0xffffffffu, bd, q);
     const float wv = __shfl_sync(0xffffffffu, v, q);
+    const long long wp = __shfl_sync(0xffffffffu, L.p, q);  // (in-place lists: lanes are sorted)
     Rec r;
     unsigned long long gk = 0ull;
     if (post) {
@@ -1443,7 +1474,7 @@ __global__ void __launch_bounds__(kThreads, GBDT_SSPLIT_CTAS) k_short_split(Spli
       r.node = L.j;
       r.epoch = epoch;
       r.shard = A.shard;
-      r.pos = L.p + (q - lane);
+      r.pos = wp;
       if (wd) {
         r.GL = wg + (nv.G - PG);
         r.HL = wh + (nv.H - PH);
@@ -1477,6 +1508,28 @@ __global__ void __launch_bounds__(kThreads, GBDT_SSPLIT_CTAS) k_short_split(Spli
       A.rec[gs] = wrec[bw][jj];
       atomicMax(A.gkey + jj, wgk[bw][jj]);
     }
+  }
+}
+
+// In-place short lists (ShortList::inplace): the partition only moves every entry's node index to
+// its child's (0xff when its node became a leaf); the lists themselves stay where they are
+__global__ void __launch_bounds__(kThreads) k_short_update(PartArgs A, ShortList S) {
+  const int K = *A.t.Kp;
+  if (K == 0 || K > kWarpK || S.nb == 0) return;
+  const int lane = threadIdx.x & 31;
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int bi = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; bi < S.nb; bi += nw) {
+    const int2 b = S.batch[bi];
+    const int lw = b.y >> 16, W = 1 << lw, sub = lane >> lw, e = lane & (W - 1);
+    if (sub >= (b.y & 0xffff)) continue;
+    const int a = S.attrs[b.x + sub];
+    if (e >= S.cl0[a]) continue;
+    const long long p = S.cs0[a] + e;
+    const int j = S.jl ? (int)S.jl[p] : 0;
+    if (j == 0xff) continue;
+    const uint8_t sd = __ldg(A.side + __ldcs(S.ins0 + p));
+    const int c = A.cidx[j];
+    S.jl_out[p] = (sd == 0 || c < 0) ? (uint8_t)0xff : (uint8_t)(sd == 1 ? c : c + 1);
   }
 }
 
@@ -3359,7 +3412,7 @@ void LevelKernels::partition_count(const PartArgs& A, const PlanArgs& P, bool co
   else k_part_count_dense<<<grid_count_dense, kThreads, 0, st>>>(A);
   GBDT_LAUNCH_CHECK();
   count_launch();
-  if (sl && sl->nb) {
+  if (sl && sl->nb && !sl->inplace) {  // (in-place lists have no segments to count)
     k_short_count<<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);
     GBDT_LAUNCH_CHECK();
     count_launch();
@@ -3382,7 +3435,11 @@ void launch_scatter(const LevelKernels& L, const PartArgs& A, cudaStream_t st) {
 
 void LevelKernels::partition_scatter(const PartArgs& A, int hmode, const RunArgs* rle, cudaStream_t st,
                                      const ShortList* sl) {
-  if (sl && sl->nb) {
+  if (sl && sl->nb && sl->inplace) {
+    k_short_update<<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);
+    GBDT_LAUNCH_CHECK();
+    count_launch();
+  } else if (sl && sl->nb) {
     if (hmode == 0) k_short_scatter<0><<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);
     else if (hmode == 1) k_short_scatter<1><<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);
     else k_short_scatter<2><<<(unsigned)(sms * 8), kThreads, 0, st>>>(A, *sl);

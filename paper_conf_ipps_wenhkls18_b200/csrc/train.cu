@@ -368,12 +368,29 @@ __global__ void k_decide(DecideArgs A) {
 // ============================================================================ a7: node map
 __global__ void k_mark(const int32_t* __restrict__ Kp, const int32_t* __restrict__ cidx,
                        const Rec* __restrict__ winner, int shard, int a_base, Tables tb,
-                       const int32_t* __restrict__ ins, uint32_t* __restrict__ bits) {
+                       const int32_t* __restrict__ ins, uint32_t* __restrict__ bits,
+                       const uint8_t* __restrict__ sflag, ShortList S) {
   const int K = *Kp;
   const int j = blockIdx.y;
   if (j >= K || cidx[j] < 0) return;
   const Rec& w = winner[j];
   if (w.shard != shard) return;
+  if (S.inplace && S.jl && sflag && sflag[w.attr - a_base]) {
+    // an in-place short list (not partitioned): node j's entries are those carrying j, in value
+    // order; the high side is every one up to the winner's position (root positions)
+    if (blockIdx.x != 0) return;
+    const int a = w.attr - a_base;
+    const long long p0 = S.cs0[a], L = S.cl0[a];
+    for (long long q = threadIdx.x; q < L; q += blockDim.x) {
+      const long long p = p0 + q;
+      if ((int)S.jl[p] != j) continue;
+      if ((int)(p <= w.pos) != w.dir) {
+        const int i = S.ins0[p];
+        atomicOr(bits + (i >> 5), 1u << (i & 31));
+      }
+    }
+    return;
+  }
   const long long s = (long long)(w.attr - a_base) * K + j;
   const long long s0 = tb.seg_start[s], n = tb.seg_cnt[s];
   const int defhi = w.dir;
@@ -513,10 +530,16 @@ struct ShardWork {
   int nlong = 0;
   uint8_t* sflag = nullptr;
   uint8_t* jl[2] = {nullptr, nullptr};  // node index of each short-list entry, two levels
+  DBuf shortg;                           // in-place mode: the short lists' g (h) lists
   // the level's short-path arguments (levels 0..kShortLevels-1, where K <= 32), else none
   ShortList level_sl(int lvl) const {
     ShortList r = sl;
-    if (lvl >= kShortLevels) { r.n = 0; r.nb = 0; return r; }
+    if (lvl >= kShortLevels) { r.n = 0; r.nb = 0; r.inplace = 0; return r; }
+    if (sl.inplace) {  // one node-index list, updated in place
+      r.jl = lvl == 0 ? nullptr : jl[0];
+      r.jl_out = jl[0];
+      return r;
+    }
     r.jl = lvl == 0 ? nullptr : jl[lvl & 1];
     r.jl_out = lvl + 1 < kShortLevels ? jl[(lvl + 1) & 1] : nullptr;
     return r;
@@ -896,6 +919,20 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         w.sl.n = (int)attrs.size();
         w.sl.batch = d_batch;
         w.sl.nb = (int)batch.size();
+        // in-place short lists when every level of the tree is on the short path (depth <= 6):
+        // no partition of them at all (GBDT_SHORT_INPLACE=0: partitioned like the other lists)
+        bool inplace = d <= kShortLevels && cap_level < 0 && !sh.rle;
+        if (const char* e = getenv("GBDT_SHORT_INPLACE")) inplace = inplace && e[0] != '0';
+        if (inplace) {
+          w.shortg.alloc((size_t)sh.cap * 8 * (hmode == kHGather ? 2 : 1) + 64, st);
+          w.sl.inplace = 1;
+          w.sl.cs0 = w.root.col_start;
+          w.sl.cl0 = w.root.col_len;
+          w.sl.val0 = sh.val0.as<float>();
+          w.sl.ins0 = sh.ins0.as<int32_t>();
+          w.sl.gsh = w.shortg.as<double>();
+          w.sl.hsh = hmode == kHGather ? w.shortg.as<double>() + sh.cap : nullptr;
+        }
       }
     }
     w.nrec = nrec + li;
@@ -1189,7 +1226,8 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         const Tables tb = lvl == 0 ? sw[li].root : sw[li].tab[lvl & 1];
         const int32_t* ins = lvl == 0 ? sh.ins0.as<int32_t>() : sh.insw[lvl & 1].as<int32_t>();
         dim3 grid((unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256 * (int64_t)Kl), (int64_t)sms * 4)), (unsigned)Kl);
-        k_mark<<<grid, 256, 0, st>>>(cur.K, cidx, winner, sh.index, sh.a_begin, tb, ins, bits);
+        k_mark<<<grid, 256, 0, st>>>(cur.K, cidx, winner, sh.index, sh.a_begin, tb, ins, bits,
+                                     sw[li].level_flag(lvl), sw[li].level_sl(lvl));
         GBDT_LAUNCH_CHECK();
         count_launch();
       }

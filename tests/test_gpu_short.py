@@ -1,4 +1,4 @@
-"""Short-list path (levels.cu k_short_split / k_short_count / k_short_scatter) on the GPU (-m gpu).
+"""Short-list path (levels.cu k_short_split / k_short_count / k_short_scatter / k_short_update) on the GPU (-m gpu).
 
 Sparse attributes whose root list has at most 32 entries are split and partitioned a lane per entry,
 32/W lists per warp, at levels 0-5; the chunk kernels take the other attributes.  The path keeps the
@@ -86,3 +86,21 @@ def test_short_path_shards(monkeypatch):
     _same(ref, ref_margin, model, margin)
     one, one_margin = gbdt.train_problem(p)
     _same(one, one_margin, model, margin)
+
+
+# In-place short lists (depth <= 6, the default there): never partitioned, node index per entry
+# updated in place, lanes sorted by node before the scans -- bit-identical to the partitioned short
+# lists (GBDT_SHORT_INPLACE=0), including new leaves (0xff entries), shards and every gradient mode.
+@pytest.mark.parametrize("name,maker,kw", [
+    ("logistic", lambda: synth.c4(seed=21, n=2000, m=2500, density=0.01, T=3), {}),
+    ("squared-gamma", lambda: synth.c4(seed=22, n=3000, m=3000, density=0.01, T=3), {"loss": "squared", "gamma": 0.5}),
+    ("h-gathered", lambda: _fractional_labels(synth.c4(seed=23, n=1500, m=2000, density=0.01, T=2)), {}),
+    ("shards", lambda: synth.c4(seed=24, n=2000, m=2500, density=0.01, T=2), {"n_shards": 4}),
+])
+def test_short_inplace_equals_partitioned(monkeypatch, name, maker, kw):
+    p = maker()
+    monkeypatch.setenv("GBDT_SHORT_INPLACE", "0")
+    ref, ref_margin = gbdt.train_problem(p, **kw)
+    monkeypatch.setenv("GBDT_SHORT_INPLACE", "1")
+    model, margin = gbdt.train_problem(p, **kw)
+    _same(ref, ref_margin, model, margin)
