@@ -143,6 +143,7 @@ struct PlanArgs {
   const int32_t* mp1;     // m + 1 (device)
   Tables nxt;
   const uint8_t* sflag = nullptr;  // short-path attributes: left out of nxt.lc when K' <= 32
+  int inplace = 0;                 // in-place short lists: their child lists are empty, no segments
 };
 
 struct RunArgs {

@@ -2168,7 +2168,9 @@ __global__ void __launch_bounds__(kThreads) k_plan_attr(PlanArgs A) {
   const int nw = (gridDim.x * blockDim.x) >> 5;
   for (int a0 = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * per; a0 <= m; a0 += nw * per) {
     const int a = a0 + sub;
-    const bool act = a < m;
+    // in-place short lists take no room in the level buffers and have no segments
+    const bool skip = a < m && A.inplace && A.sflag && A.sflag[a];
+    const bool act = a < m && !skip;
     if (a == m && jj == 0) { A.el[2ll * m] = 0ull; A.el[2ll * m + 1] = 0ull; }
     unsigned long long pre = 0;
     long long L = 0;
@@ -2202,7 +2204,7 @@ __global__ void __launch_bounds__(kThreads) k_plan_attr(PlanArgs A) {
       for (int o = G >> 1; o; o >>= 1) l += __shfl_xor_sync(0xffffffffu, l, o, G);
       L += l;
     }
-    if (act && jj == 0) {
+    if ((act || skip) && jj == 0) {
       A.nxt.col_len[a] = L;
       A.el[2ll * a] = (unsigned long long)((L + 3) & ~3ll) | ((unsigned long long)((L + kChunk - 1) / kChunk) << 32);
       A.el[2ll * a + 1] = 0ull;
@@ -2217,7 +2219,7 @@ __global__ void __launch_bounds__(kThreads) k_plan_seg(PlanArgs A) {
   const int nw = (gridDim.x * blockDim.x) >> 5;
   for (int a0 = ((blockIdx.x * blockDim.x + threadIdx.x) >> 5) * per; a0 <= m; a0 += nw * per) {
     const int a = a0 + sub;
-    const bool act = a < m;
+    const bool act = a < m && !(A.inplace && A.sflag && A.sflag[a]);  // (in-place short lists: no segments)
     long long cs = 0;
     if (a <= m) {
       const unsigned long long ex = A.el[2ll * a];

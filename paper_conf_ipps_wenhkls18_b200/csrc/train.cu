@@ -1091,6 +1091,7 @@ void train(Dataset& ds, const gbdt_params& P, Model& model, double* margin_out) 
         PL.segH = w.segH; PL.segL = w.segL; PL.seg_pre = w.seg_pre;
         PL.out_hi = w.out_hi; PL.out_lo = w.out_lo; PL.len_tmp = w.len_tmp; PL.nxt = tn;
         PL.el = w.pel; PL.egrp = w.pgrp; PL.egroups = w.pgroups; PL.mp1 = w.mp1; PL.sflag = w.level_flag(lvl + 1);
+        PL.inplace = w.sl.inplace;
         RunArgs RA;
         if (sh.rle) {
           RA.m = sh.m; RA.Kp = cur.K; RA.Knp = nxt.K; RA.cidx = cidx; RA.cur = tb; RA.nxt = tn;
