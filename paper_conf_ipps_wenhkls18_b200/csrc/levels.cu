@@ -1379,7 +1379,7 @@ __device__ __forceinline__ SLane short_lane(const ShortList& S, const Tables& tb
 
 template <int HMODE, bool kGather>
 #ifndef GBDT_SSPLIT_CTAS
-#define GBDT_SSPLIT_CTAS 1
+#define GBDT_SSPLIT_CTAS 4  // <= 64 registers: C4a split 4.92 -> 4.21 ms/tree
 #endif
 __global__ void __launch_bounds__(kThreads, GBDT_SSPLIT_CTAS) k_short_split(SplitArgs A, ShortList S) {
   constexpr bool kH = HMODE == kHGather;
