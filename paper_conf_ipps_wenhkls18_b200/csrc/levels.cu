@@ -2050,7 +2050,10 @@ __device__ __forceinline__ unsigned ld_keep_u32(const uint32_t* p, unsigned long
   asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
   return v;
 }
-__global__ void __launch_bounds__(kThreads) k_part_count_dense(PartArgs A) {
+#ifndef GBDT_CDENSE_CTAS
+#define GBDT_CDENSE_CTAS 1
+#endif
+__global__ void __launch_bounds__(kThreads, GBDT_CDENSE_CTAS) k_part_count_dense(PartArgs A) {
   __shared__ TabCache tc;
   const int lane = threadIdx.x & 31;
   const int K = *A.t.Kp;
@@ -2818,7 +2821,10 @@ __global__ void __launch_bounds__(kThreads, GBDT_RUNAGG_CTAS) k_run_agg(SplitArg
 // the run totals of the single-run chunks as in k_run_agg; other chunks are listed for
 // k_run_agg_multi, which reads the g-list written here.
 template <int HMODE>
-__global__ void __launch_bounds__(kThreads) k_run_root(SplitArgs A, unsigned long long* __restrict__ racc) {
+#ifndef GBDT_RUNROOT_CTAS
+#define GBDT_RUNROOT_CTAS 1
+#endif
+__global__ void __launch_bounds__(kThreads, GBDT_RUNROOT_CTAS) k_run_root(SplitArgs A, unsigned long long* __restrict__ racc) {
   constexpr bool kH = HMODE == kHGather;
   __shared__ TabCache tc;
   const int lane = threadIdx.x & 31;
