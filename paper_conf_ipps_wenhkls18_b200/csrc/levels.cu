@@ -1252,9 +1252,14 @@ __device__ __forceinline__ void sf_short(const SplitArgs& A, NodeBest& B, unsign
 #endif
 template <int HMODE, bool kMissing, bool kRLE>
 #ifndef GBDT_SFSHORT_CTAS
-#define GBDT_SFSHORT_CTAS 1
+#define GBDT_SFSHORT_CTAS 0  // 0: the compiler's choice (a minimum of 1 CTA/SM would let it take more registers)
 #endif
-__global__ void __launch_bounds__(kThreads, GBDT_SFSHORT_CTAS) k_sf_short(SplitArgs A) {
+#if GBDT_SFSHORT_CTAS > 0
+#define LB_GBDT_SFSHORT_CTAS __launch_bounds__(kThreads, GBDT_SFSHORT_CTAS)
+#else
+#define LB_GBDT_SFSHORT_CTAS __launch_bounds__(kThreads)
+#endif
+__global__ void LB_GBDT_SFSHORT_CTAS k_sf_short(SplitArgs A) {
   __shared__ NodeBest B;
   __shared__ unsigned long long wgk[kWarps][kWarpK];
   __shared__ Rec wrec[kWarps][kWarpK];
@@ -1946,9 +1951,14 @@ __device__ __forceinline__ void count_short(const PartArgs& A, const ChunkMeta& 
 #define GBDT_COUNT_SHORT 1
 #endif
 #ifndef GBDT_COUNT_CTAS
-#define GBDT_COUNT_CTAS 1
+#define GBDT_COUNT_CTAS 0  // 0: the compiler's choice (a minimum of 1 CTA/SM would let it take more registers)
 #endif
-__global__ void __launch_bounds__(kThreads, GBDT_COUNT_CTAS) k_part_count(PartArgs A, int counted) {
+#if GBDT_COUNT_CTAS > 0
+#define LB_GBDT_COUNT_CTAS __launch_bounds__(kThreads, GBDT_COUNT_CTAS)
+#else
+#define LB_GBDT_COUNT_CTAS __launch_bounds__(kThreads)
+#endif
+__global__ void LB_GBDT_COUNT_CTAS k_part_count(PartArgs A, int counted) {
   __shared__ TabCache tc;
   const int lane = threadIdx.x & 31;
   const int K = *A.t.Kp;
@@ -2051,9 +2061,14 @@ __device__ __forceinline__ unsigned ld_keep_u32(const uint32_t* p, unsigned long
   return v;
 }
 #ifndef GBDT_CDENSE_CTAS
-#define GBDT_CDENSE_CTAS 1
+#define GBDT_CDENSE_CTAS 0  // 0: the compiler's choice (a minimum of 1 CTA/SM would let it take more registers)
 #endif
-__global__ void __launch_bounds__(kThreads, GBDT_CDENSE_CTAS) k_part_count_dense(PartArgs A) {
+#if GBDT_CDENSE_CTAS > 0
+#define LB_GBDT_CDENSE_CTAS __launch_bounds__(kThreads, GBDT_CDENSE_CTAS)
+#else
+#define LB_GBDT_CDENSE_CTAS __launch_bounds__(kThreads)
+#endif
+__global__ void LB_GBDT_CDENSE_CTAS k_part_count_dense(PartArgs A) {
   __shared__ TabCache tc;
   const int lane = threadIdx.x & 31;
   const int K = *A.t.Kp;
@@ -2822,9 +2837,14 @@ __global__ void __launch_bounds__(kThreads, GBDT_RUNAGG_CTAS) k_run_agg(SplitArg
 // k_run_agg_multi, which reads the g-list written here.
 template <int HMODE>
 #ifndef GBDT_RUNROOT_CTAS
-#define GBDT_RUNROOT_CTAS 1
+#define GBDT_RUNROOT_CTAS 0  // 0: the compiler's choice (a minimum of 1 CTA/SM would let it take more registers)
 #endif
-__global__ void __launch_bounds__(kThreads, GBDT_RUNROOT_CTAS) k_run_root(SplitArgs A, unsigned long long* __restrict__ racc) {
+#if GBDT_RUNROOT_CTAS > 0
+#define LB_GBDT_RUNROOT_CTAS __launch_bounds__(kThreads, GBDT_RUNROOT_CTAS)
+#else
+#define LB_GBDT_RUNROOT_CTAS __launch_bounds__(kThreads)
+#endif
+__global__ void LB_GBDT_RUNROOT_CTAS k_run_root(SplitArgs A, unsigned long long* __restrict__ racc) {
   constexpr bool kH = HMODE == kHGather;
   __shared__ TabCache tc;
   const int lane = threadIdx.x & 31;
